@@ -1,0 +1,176 @@
+/*
+ * sptrsv.h -- C ABI of the B200-native CapelliniSpTRSV hot path.
+ *
+ * Operation (sec.1; Alg.1): solve L x = b for x,
+ * L an n x n sparse LOWER-triangular matrix in CSR form, b and x dense fp64:
+ *     x_i = (b_i - sum_{j<i, L_ij stored} L_ij * x_j) / L_ii ,  i = 0..n-1.
+ * Method (Alg.5 "Writing-First CapelliniSpTRSV"): no level
+ * preprocessing; one GPU thread per component x_i in original row order, which
+ * busy-waits on per-component ready flags of its dependencies, accumulates the
+ * partial sum, then publishes x_i.  Rows whose 32-row group has a high mean
+ * nnz/row are solved one WARP per row instead (the thread/warp hybrid the paper
+ * proposes in sec.4.4; warp kernel = Alg.3).
+ *
+ * All functions are host functions and thread-compatible (one handle must not
+ * be used from two host threads at once).  Pointers documented "device" must
+ * be device pointers valid on the CURRENT CUDA device (e.g. a torch tensor's
+ * data_ptr()); "host" pointers are ordinary host memory.  Streams are passed as
+ * sptrsv_stream_t, which is a cudaStream_t (NULL = the legacy default stream).
+ * No torch or CUDA types appear in this header.
+ *
+ * Return value: every function returns SPTRSV_OK (0) or a negative
+ * sptrsv_status.  sptrsv_strerror() maps a status to a static string.
+ */
+#ifndef SPTRSV_H_
+#define SPTRSV_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SPTRSV_ABI_VERSION 1
+
+typedef struct sptrsv_handle_s *sptrsv_handle_t;
+typedef void *sptrsv_stream_t; /* cudaStream_t */
+
+typedef enum sptrsv_status {
+    SPTRSV_OK = 0,
+    SPTRSV_ERR_INVALID_ARG = -1,  /* null pointer, n < 0, bad option value ...             */
+    SPTRSV_ERR_NOT_LOWER = -2,    /* a stored column j > i                                  */
+    SPTRSV_ERR_MISSING_DIAG = -3, /* empty row, or the last stored column of row i != i     */
+    SPTRSV_ERR_ZERO_DIAG = -4,    /* L_ii == 0                                              */
+    SPTRSV_ERR_UNSORTED = -5,     /* columns of a row not strictly increasing (dup/unsorted) */
+    SPTRSV_ERR_BAD_ROWPTR = -6,   /* rowptr[0] != 0, decreasing, or entry beyond rowptr[n]  */
+    SPTRSV_ERR_BAD_COL = -7,      /* a column index < 0                                     */
+    SPTRSV_ERR_TOO_LARGE = -8,    /* n > 2^31 - 2 (int32 CSR)                  */
+    SPTRSV_ERR_CUDA = -9,         /* a CUDA runtime call failed (launch, copy, ...)         */
+    SPTRSV_ERR_ALLOC = -10,       /* device / pinned allocation failed                      */
+    SPTRSV_ERR_TIMEOUT = -11      /* watchdog: a solve spun past SPTRSV_OPT_SPIN_LIMIT      */
+} sptrsv_status;
+
+/* Options (sptrsv_set_option / sptrsv_get_option).  None changes the result
+ * beyond fp64 summation order (warp mode sums lane-strided partials). */
+typedef enum sptrsv_option {
+    SPTRSV_OPT_MODE = 1,           /* 0 AUTO (default), 1 THREAD (every row thread-level,
+                                      Alg.5), 2 WARP (every row warp-level, Alg.3).
+                                      Setting it re-plans (synchronous).                    */
+    SPTRSV_OPT_WARP_THRESHOLD = 2, /* AUTO: a 32-row group goes warp-level when its mean
+                                      nnz/row exceeds this (default 16; sec.4.4, DESIGN G10).
+                                      Setting it re-plans (synchronous).                    */
+    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 128, 256 (default), 512, 1024        */
+    SPTRSV_OPT_BACKOFF_MIN_NS = 4, /* __nanosleep after a pass where no lane progressed     */
+    SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
+    SPTRSV_OPT_SPIN_LIMIT = 6,     /* watchdog: idle passes per warp before TIMEOUT (0=off) */
+    SPTRSV_OPT_L2_WINDOW = 7,      /* 1: cudaAccessPolicyWindow persisting over the flags   */
+    SPTRSV_OPT_STAGE_SMEM = 8      /* 1 (default): thread-level warps stage their CSR slice
+                                      in shared memory with coalesced loads                 */
+} sptrsv_option;
+
+typedef struct sptrsv_info {
+    int32_t n;
+    int32_t n_thread_groups;  /* 32-row groups solved thread-level                       */
+    int64_t nnz;              /* rowptr[n]                                                */
+    int32_t n_warp_rows;      /* rows solved warp-level                                   */
+    int32_t n_tasks;          /* warp tasks per solve = n_thread_groups + n_warp_rows     */
+    int32_t max_row_nnz;      /* longest row (incl. diagonal)                             */
+    int32_t device;           /* CUDA ordinal the handle is bound to                      */
+    float analyse_ms;         /* wall time of sptrsv_analyse_csr (Table 1 analogue)        */
+    uint32_t solves;          /* solves enqueued through this handle                      */
+} sptrsv_info;
+
+/*
+ * sptrsv_analyse_csr -- O(nnz) setup; the paper's "MALLOC(get_value, m)"
+ * (Alg.5 l.1) plus the nnz-per-row pass the hybrid needs
+ * (sec.4.4).  No level analysis, no reordering, no format
+ * conversion.
+ *   n       number of rows/columns, 0 <= n <= 2^31 - 2.
+ *   rowptr  device, int32[n+1]; rowptr[0] = 0, nondecreasing; nnz = rowptr[n].
+ *   colidx  device, int32[nnz]; per row strictly increasing, all <= i, and the
+ *           diagonal (column i) stored LAST (Alg.1 l.5).
+ *   val     device, double[nnz]; val[rowptr[i+1]-1] = L_ii != 0.
+ *   out     host; receives the new handle (NULL on error).
+ * Ownership: rowptr/colidx/val are BORROWED -- the caller keeps them alive and
+ * unmodified until sptrsv_destroy.  The handle owns its workspace (flags,
+ * in-degrees, task list, solve state).
+ * Synchronous: runs on the legacy default stream and blocks until done; the
+ * caller must have completed any writes to the CSR arrays.  Malformed input
+ * returns the error of the lowest offending row (codes above) -- it never
+ * reaches the spin loop, where it could hang.  Binds the handle to the
+ * current device.
+ */
+int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
+                       const double *val, sptrsv_handle_t *out);
+
+/*
+ * sptrsv_solve -- one solve L x = b (Alg.5), enqueued on
+ * `stream`; asynchronous, never synchronises the host.  Exactly ONE kernel
+ * launch (the per-solve flag reset of Alg.5 l.2 is an epoch bump done inside
+ * the kernel), so it is CUDA-graph capturable.
+ *   b  device, double[n], read-only.   x  device, double[n], fully overwritten.
+ *   b and x must not alias.  Solves through one handle are ordered on one
+ *   stream; concurrent solves with the same handle on different streams are
+ *   undefined (shared flags).  Distinct handles are independent.
+ * Returns launch errors only; a watchdog timeout is reported by sptrsv_check.
+ */
+int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream);
+
+/*
+ * sptrsv_solve_host -- end-to-end convenience: copies b (host) to handle-owned
+ * device staging, solves, copies x back to host, and synchronises `stream`.
+ * b_host/x_host: host double[n] (pinned memory gives full PCIe bandwidth).
+ */
+int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host,
+                      sptrsv_stream_t stream);
+
+/* sptrsv_destroy -- frees the handle's workspace (synchronises the device
+ * first).  NULL is a no-op. */
+int sptrsv_destroy(sptrsv_handle_t h);
+
+int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value);
+int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value);
+
+/* sptrsv_info -- sizes, plan and timing of the handle (host struct). */
+int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out);
+
+/* sptrsv_get_indegree -- copies the in-degrees computed by analyse
+ * (indeg[i] = number of stored off-diagonals of row i = dependencies of x_i,
+ * PAPER.md:67-69) into device int32[n] `out_dev`, async on `stream`. */
+int sptrsv_get_indegree(sptrsv_handle_t h, int32_t *out_dev, sptrsv_stream_t stream);
+
+/*
+ * sptrsv_levels -- diagnostic, not part of the solve: the level of every
+ * component (level[i] = 0 without dependencies, else 1 + max
+ * level of its dependencies) computed on the GPU with the same
+ * synchronization-free flag protocol, plus the level-set histogram (Table 6
+ * beta = n / nlevels).
+ *   level_dev   device int32[n] or NULL.   counts_dev  device int32[n] or NULL;
+ *   counts_dev[l] = components in level l for l < nlevels (entries >= nlevels
+ *   are zero).  nlevels_host: host int32, receives max level + 1.
+ * Synchronises `stream`.
+ */
+int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev,
+                  int32_t *nlevels_host, sptrsv_stream_t stream);
+
+/* sptrsv_check -- synchronises `stream`, returns SPTRSV_ERR_TIMEOUT if the
+ * watchdog fired in any solve since the last check (and clears it), else OK. */
+int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream);
+
+/*
+ * sptrsv_flag_latency -- diagnostic microbenchmark on the current device: two
+ * CTAs ping-pong `iters` times through the publish/consume pair the solve uses
+ * and report the mean one-way hop in nanoseconds (t_hop of the critical-path
+ * latency bound).  protocol: 0 = st.release flag / ld.acquire poll
+ * + relaxed x load (the solve's protocol), 1 = relaxed poll + fence.acq_rel,
+ * 2 = value-as-flag (x polled directly; ablation only).  Synchronous.
+ */
+int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop);
+
+const char *sptrsv_strerror(int status);
+int sptrsv_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPTRSV_H_ */

@@ -1,0 +1,168 @@
+"""B200-native CapelliniSpTRSV: synchronization-free fp64 sparse lower-triangular solve.
+
+Thin Python layer over the C ABI in ``include/sptrsv.h`` (``libsptrsv.so``).
+PyTorch supplies device memory and streams only; every step of the solve is a
+hand-written sm_100a kernel.  Paper: Su et al., ICPP '20.
+
+    import torch, paper_conf_icpp_suz0hw0w20_b200 as cap
+    L = cap.analyse(rowptr, colidx, val)      # torch CUDA tensors, int32/int32/float64
+    L.solve(b, x)                             # async on the current stream
+"""
+from __future__ import annotations
+
+import ctypes
+
+from . import _lib
+from ._lib import (MODE_AUTO, MODE_THREAD, MODE_WARP, OPT_BACKOFF_MAX_NS, OPT_BACKOFF_MIN_NS,
+                   OPT_CTA_THREADS, OPT_L2_WINDOW, OPT_MODE, OPT_SPIN_LIMIT, OPT_STAGE_SMEM,
+                   OPT_WARP_THRESHOLD, SptrsvError, check)
+
+__all__ = ["analyse", "Handle", "SptrsvError", "flag_latency", "MODE_AUTO", "MODE_THREAD",
+           "MODE_WARP", "lib"]
+
+lib = _lib.lib
+
+
+def _stream_ptr(stream) -> int | None:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def _need(t, dtype, n, name):
+    import torch
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if n is not None and t.numel() != n:
+        raise ValueError(f"{name} must have {n} elements, got {t.numel()}")
+
+
+class Handle:
+    """An analysed matrix (``sptrsv_analyse_csr``).  Keeps the CSR tensors alive."""
+
+    def __init__(self, rowptr, colidx, val):
+        import torch
+        _need(rowptr, torch.int32, None, "rowptr")
+        n = rowptr.numel() - 1
+        if n < 0:
+            raise ValueError("rowptr must have n+1 >= 1 entries")
+        _need(colidx, torch.int32, None, "colidx")
+        _need(val, torch.float64, colidx.numel(), "val")
+        if not (rowptr.device == colidx.device == val.device):
+            raise ValueError("CSR tensors must live on one device")
+        self.device = rowptr.device
+        self.n = n
+        self._keep = (rowptr, colidx, val)
+        self._h = ctypes.c_void_p()
+        with torch.cuda.device(self.device):
+            torch.cuda.current_stream().synchronize()  # analyse runs on the legacy default stream
+            check(lib.sptrsv_analyse_csr(n, rowptr.data_ptr(), colidx.data_ptr() if colidx.numel() else None,
+                                         val.data_ptr() if val.numel() else None, ctypes.byref(self._h)),
+                  "sptrsv_analyse_csr")
+
+    # -- solve -------------------------------------------------------------------------
+    def solve(self, b, x=None, stream=None):
+        """x <- L^{-1} b (fp64, device tensors), enqueued on ``stream`` (default: current)."""
+        import torch
+        _need(b, torch.float64, self.n, "b")
+        if x is None:
+            x = torch.empty_like(b)
+        _need(x, torch.float64, self.n, "x")
+        if self.n:
+            check(lib.sptrsv_solve(self._h, b.data_ptr(), x.data_ptr(), _stream_ptr(stream)), "sptrsv_solve")
+        return x
+
+    def solve_host(self, b_host, x_host, stream=None):
+        """End to end from host buffers (numpy float64 or pinned CPU tensors); synchronous."""
+        import numpy as np
+        import torch
+
+        def ptr(a):
+            if isinstance(a, np.ndarray):
+                assert a.dtype == np.float64 and a.flags.c_contiguous and a.size == self.n
+                return a.ctypes.data
+            assert isinstance(a, torch.Tensor) and a.device.type == "cpu" and a.dtype == torch.float64
+            assert a.is_contiguous() and a.numel() == self.n
+            return a.data_ptr()
+        with torch.cuda.device(self.device):
+            check(lib.sptrsv_solve_host(self._h, ptr(b_host), ptr(x_host), _stream_ptr(stream)),
+                  "sptrsv_solve_host")
+        return x_host
+
+    def check(self, stream=None):
+        """Synchronise and raise SptrsvError(ERR_TIMEOUT) if the watchdog fired."""
+        check(lib.sptrsv_check(self._h, _stream_ptr(stream)), "sptrsv_check")
+
+    # -- diagnostics ---------------------------------------------------------------------
+    def indegree(self, stream=None):
+        import torch
+        out = torch.empty(self.n, dtype=torch.int32, device=self.device)
+        check(lib.sptrsv_get_indegree(self._h, out.data_ptr() if self.n else None, _stream_ptr(stream)),
+              "sptrsv_get_indegree")
+        return out
+
+    def levels(self, stream=None):
+        """(level[n] int32, nlevels, counts[nlevels] int32) computed on the GPU."""
+        import torch
+        lv = torch.empty(self.n, dtype=torch.int32, device=self.device)
+        counts = torch.empty(self.n, dtype=torch.int32, device=self.device)
+        nl = ctypes.c_int32(0)
+        if self.n:
+            check(lib.sptrsv_levels(self._h, lv.data_ptr(), counts.data_ptr(), ctypes.byref(nl),
+                                    _stream_ptr(stream)), "sptrsv_levels")
+        return lv, int(nl.value), counts[: nl.value]
+
+    def info(self) -> dict:
+        inf = _lib.sptrsv_info()
+        check(lib.sptrsv_get_info(self._h, ctypes.byref(inf)), "sptrsv_get_info")
+        return {f: getattr(inf, f) for f, _ in inf._fields_}
+
+    def set_option(self, key: int, value: int) -> None:
+        check(lib.sptrsv_set_option(self._h, key, int(value)), "sptrsv_set_option")
+
+    def get_option(self, key: int) -> int:
+        v = ctypes.c_int64(0)
+        check(lib.sptrsv_get_option(self._h, key, ctypes.byref(v)), "sptrsv_get_option")
+        return int(v.value)
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.sptrsv_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+
+def analyse(rowptr, colidx, val, **options) -> Handle:
+    """``sptrsv_analyse_csr`` + options (mode=, warp_threshold=, cta_threads=, ...)."""
+    h = Handle(rowptr, colidx, val)
+    keys = {"mode": OPT_MODE, "warp_threshold": OPT_WARP_THRESHOLD, "cta_threads": OPT_CTA_THREADS,
+            "backoff_min_ns": OPT_BACKOFF_MIN_NS, "backoff_max_ns": OPT_BACKOFF_MAX_NS,
+            "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM}
+    for k, v in options.items():
+        h.set_option(keys[k], v)
+    return h
+
+
+def flag_latency(iters: int = 20000, protocol: int = 0) -> float:
+    """Mean one-way flag hop (ns) between two CTAs on the current device (sptrsv_flag_latency)."""
+    v = ctypes.c_double(0.0)
+    check(lib.sptrsv_flag_latency(iters, protocol, ctypes.byref(v)), "sptrsv_flag_latency")
+    return float(v.value)

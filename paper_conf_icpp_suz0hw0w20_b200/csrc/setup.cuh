@@ -1,0 +1,137 @@
+// setup.cuh -- O(nnz) analyse kernels (SURVEY/DESIGN row a1).
+//
+//   k_validate   per-row CSR checks (the shape Alg.1 assumes: PAPER.md:72,
+//                :89-91), in-degree, longest row
+//   k_plan_count per 32-row group: thread- or warp-level (sec.4.4,
+//                PAPER.md:329-335) -> tasks per group, block totals
+//   k_plan_write block-local exclusive scan + host-scanned block offsets ->
+//                the row-ordered task list
+// None of this is level analysis: it reads each row once, in row order.
+#pragma once
+#include <cstdint>
+
+namespace sptrsv_dev {
+
+enum : int {  // same numbering as sptrsv_status (negated)
+    E_NOT_LOWER = 2, E_MISSING_DIAG = 3, E_ZERO_DIAG = 4, E_UNSORTED = 5, E_BAD_ROWPTR = 6, E_BAD_COL = 7
+};
+
+// status: 64-bit min over (row << 8 | code) -> the lowest offending row wins,
+// which is the row-ordered error the oracle reports too.
+__global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ rowptr,
+                                                  const int32_t *__restrict__ colidx,
+                                                  const double *__restrict__ val, int32_t n,
+                                                  int64_t nnz, int32_t *indeg,
+                                                  unsigned long long *status, int32_t *max_row) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    int len = 0;
+    if (i < n) {
+        const int64_t s = rowptr[i], e = rowptr[i + 1];
+        int code = 0;
+        if (s < 0 || e < s || e > nnz) {
+            code = E_BAD_ROWPTR;
+        } else if (e == s) {
+            code = E_MISSING_DIAG;
+        } else {
+            int prev = -1;
+            for (int64_t j = s; j < e; ++j) {
+                const int c = colidx[j];
+                if (c < 0) { code = E_BAD_COL; break; }
+                if (c > i) { code = E_NOT_LOWER; break; }
+                if (j > s && c <= prev) { code = E_UNSORTED; break; }
+                prev = c;
+            }
+            if (!code) {
+                if (colidx[e - 1] != i) code = E_MISSING_DIAG;
+                else if (val[e - 1] == 0.0) code = E_ZERO_DIAG;
+            }
+        }
+        if (code) atomicMin(status, ((unsigned long long)i << 8) | (unsigned long long)code);
+        len = code ? 0 : (int)(e - s);
+        indeg[i] = code ? 0 : (int)(e - s - 1);
+    }
+    for (int off = 16; off > 0; off >>= 1) len = max(len, __shfl_xor_sync(0xffffffffu, len, off));
+    if ((threadIdx.x & 31) == 0 && len > 0) atomicMax(max_row, len);
+}
+
+// mode: 0 auto, 1 all thread-level, 2 all warp-level.
+// A group of `rows` rows goes warp-level in auto mode when its nnz (diagonals
+// included) exceeds threshold * rows, i.e. mean nnz/row > threshold.
+__device__ __forceinline__ int group_tasks(const int32_t *rowptr, int32_t n, int g, int mode,
+                                           int threshold, bool *is_warp) {
+    const int r0 = g * 32;
+    const int rows = min(32, n - r0);
+    const long long gnnz = (long long)rowptr[r0 + rows] - rowptr[r0];
+    const bool w = (mode == 2) || (mode == 0 && gnnz > (long long)threshold * rows);
+    *is_warp = w;
+    return w ? rows : 1;
+}
+
+__device__ __forceinline__ int block_exclusive_scan(int v, int *s_warp, int *total) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    int inc = v;
+    for (int off = 1; off < 32; off <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, inc, off);
+        if (lane >= off) inc += t;
+    }
+    if (lane == 31) s_warp[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+        const int nw = blockDim.x >> 5;
+        int w = lane < nw ? s_warp[lane] : 0;
+        int wi = w;
+        for (int off = 1; off < 32; off <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, wi, off);
+            if (lane >= off) wi += t;
+        }
+        if (lane < nw) s_warp[lane] = wi - w;
+        if (lane == nw - 1) s_warp[32] = wi;
+    }
+    __syncthreads();
+    *total = s_warp[32];
+    const int r = s_warp[warp] + inc - v;
+    __syncthreads();
+    return r;
+}
+
+__global__ void __launch_bounds__(1024) k_plan_count(const int32_t *__restrict__ rowptr, int32_t n,
+                                                     int32_t ngroups, int mode, int threshold,
+                                                     int32_t *blk_tasks, int32_t *blk_tgroups) {
+    __shared__ int s_warp[33];
+    const int g = blockIdx.x * blockDim.x + threadIdx.x;
+    int t = 0, tg = 0;
+    if (g < ngroups) {
+        bool w;
+        t = group_tasks(rowptr, n, g, mode, threshold, &w);
+        tg = w ? 0 : 1;
+    }
+    int tot_t, tot_g;
+    block_exclusive_scan(t, s_warp, &tot_t);
+    block_exclusive_scan(tg, s_warp, &tot_g);
+    if (threadIdx.x == 0) {
+        blk_tasks[blockIdx.x] = tot_t;
+        blk_tgroups[blockIdx.x] = tot_g;
+    }
+}
+
+__global__ void __launch_bounds__(1024) k_plan_write(const int32_t *__restrict__ rowptr, int32_t n,
+                                                     int32_t ngroups, int mode, int threshold,
+                                                     const int32_t *__restrict__ blk_offset,
+                                                     int32_t *tasks) {
+    __shared__ int s_warp[33];
+    const int g = blockIdx.x * blockDim.x + threadIdx.x;
+    int t = 0;
+    bool w = false;
+    if (g < ngroups) t = group_tasks(rowptr, n, g, mode, threshold, &w);
+    int tot;
+    const int off = block_exclusive_scan(t, s_warp, &tot) + blk_offset[blockIdx.x];
+    if (g < ngroups) {
+        if (w) {
+            for (int k = 0; k < t; ++k) tasks[off + k] = ~(g * 32 + k);  // warp task: row
+        } else {
+            tasks[off] = g * 32;  // thread task: first row of the group
+        }
+    }
+}
+
+}  // namespace sptrsv_dev

@@ -1,0 +1,555 @@
+// sptrsv.cu -- host side of the C ABI declared in include/sptrsv.h.
+//
+// Torch-free: raw device pointers and cudaStream_t only.  Built as
+// libsptrsv.so for sm_100a (see paper_conf_icpp_suz0hw0w20_b200/build.py).
+#include <cuda_runtime.h>
+
+#include <chrono>
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "setup.cuh"
+#include "solve.cuh"
+#include "sptrsv.h"
+
+using namespace sptrsv_dev;
+
+namespace {
+
+constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
+
+struct Workspace {
+    uint32_t *flags = nullptr;     // n
+    int32_t *indeg = nullptr;      // n
+    int32_t *tasks = nullptr;      // n_tasks (PLAN_LIST only)
+    SolveState *st = nullptr;      // 1
+    uint32_t *lvl = nullptr;       // n (levels diagnostic, lazy)
+    double *b_stage = nullptr;     // n (solve_host, lazy)
+    double *x_stage = nullptr;     // n (solve_host, lazy)
+};
+
+}  // namespace
+
+struct sptrsv_handle_s {
+    int device = 0;
+    int32_t n = 0;
+    int64_t nnz = 0;
+    const int32_t *rowptr = nullptr;
+    const int32_t *colidx = nullptr;
+    const double *val = nullptr;
+    Workspace ws;
+    // plan
+    int plan = PLAN_THREAD;
+    int32_t n_tasks = 0;
+    int32_t n_tasks_cap = 0;
+    int32_t n_thread_groups = 0;
+    int32_t n_warp_rows = 0;
+    int32_t max_row = 0;
+    // options
+    int mode = 0;
+    int threshold = 16;
+    int cta_threads = 256;
+    uint32_t backoff_min = 0;
+    uint32_t backoff_max = 256;
+    uint32_t spin_limit = 1u << 24;
+    int l2_window = 0;
+    int stage = 1;
+    // bookkeeping
+    uint32_t solves = 0;
+    uint32_t since_reset = 0;
+    float analyse_ms = 0.f;
+};
+
+#define CK(call)                                        \
+    do {                                                \
+        if ((call) != cudaSuccess) {                    \
+            (void)cudaGetLastError();                   \
+            return SPTRSV_ERR_CUDA;                     \
+        }                                               \
+    } while (0)
+
+namespace {
+
+size_t stage_smem_bytes(int cta_threads) {
+    return (size_t)(cta_threads / 32) * kStageCap * (sizeof(double) + sizeof(int32_t));
+}
+
+int set_kernel_attrs() {
+    static int done = 0;
+    static int rc = SPTRSV_OK;
+    if (done) return rc;
+    const int maxb = (int)stage_smem_bytes(1024);
+    if (cudaFuncSetAttribute(k_solve<PLAN_THREAD>, cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) != cudaSuccess ||
+        cudaFuncSetAttribute(k_solve<PLAN_WARP>, cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) != cudaSuccess ||
+        cudaFuncSetAttribute(k_solve<PLAN_LIST>, cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) != cudaSuccess) {
+        (void)cudaGetLastError();
+        rc = SPTRSV_ERR_CUDA;
+    }
+    done = 1;
+    return rc;
+}
+
+void free_ws(Workspace &w) {
+    cudaFree(w.flags);
+    cudaFree(w.indeg);
+    cudaFree(w.tasks);
+    cudaFree(w.st);
+    cudaFree(w.lvl);
+    cudaFree(w.b_stage);
+    cudaFree(w.x_stage);
+    w = Workspace();
+}
+
+// Build the row-ordered task list for the current mode/threshold (synchronous).
+int build_plan(sptrsv_handle_s *h) {
+    const int32_t n = h->n;
+    const int32_t ngroups = (n + 31) / 32;
+    if (ngroups == 0) {
+        h->n_tasks = 0;
+        h->n_thread_groups = 0;
+        h->n_warp_rows = 0;
+        h->plan = PLAN_THREAD;
+        return SPTRSV_OK;
+    }
+    const int nb = (ngroups + 1023) / 1024;
+    int32_t *d_bt = nullptr, *d_bg = nullptr, *d_off = nullptr;
+    std::vector<int32_t> bt(nb), bg(nb), off(nb);
+    int rc = SPTRSV_OK;
+    do {
+        if (cudaMalloc(&d_bt, sizeof(int32_t) * nb) != cudaSuccess ||
+            cudaMalloc(&d_bg, sizeof(int32_t) * nb) != cudaSuccess ||
+            cudaMalloc(&d_off, sizeof(int32_t) * nb) != cudaSuccess) {
+            rc = SPTRSV_ERR_ALLOC;
+            break;
+        }
+        k_plan_count<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_bt, d_bg);
+        if (cudaGetLastError() != cudaSuccess ||
+            cudaMemcpy(bt.data(), d_bt, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(bg.data(), d_bg, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        int64_t tot = 0, tg = 0;
+        for (int b = 0; b < nb; ++b) {
+            off[b] = (int32_t)tot;
+            tot += bt[b];
+            tg += bg[b];
+        }
+        h->n_tasks = (int32_t)tot;
+        h->n_thread_groups = (int32_t)tg;
+        h->n_warp_rows = (int32_t)(tot - tg);  // every warp-level group contributes one task per row
+        if (tg == ngroups) {
+            h->plan = PLAN_THREAD;  // implicit mapping: task t = rows [32t, 32t+32)
+        } else if (tg == 0) {
+            h->plan = PLAN_WARP;    // implicit mapping: task t = row t
+        } else {
+            h->plan = PLAN_LIST;
+            if (h->n_tasks > h->n_tasks_cap) {
+                cudaFree(h->ws.tasks);
+                h->ws.tasks = nullptr;
+                if (cudaMalloc(&h->ws.tasks, sizeof(int32_t) * (size_t)h->n_tasks) != cudaSuccess) {
+                    h->n_tasks_cap = 0;
+                    rc = SPTRSV_ERR_ALLOC;
+                    break;
+                }
+                h->n_tasks_cap = h->n_tasks;
+            }
+            if (cudaMemcpy(d_off, off.data(), sizeof(int32_t) * nb, cudaMemcpyHostToDevice) != cudaSuccess) {
+                rc = SPTRSV_ERR_CUDA;
+                break;
+            }
+            k_plan_write<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_off, h->ws.tasks);
+            if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
+                rc = SPTRSV_ERR_CUDA;
+                break;
+            }
+        }
+    } while (0);
+    if (rc != SPTRSV_OK) (void)cudaGetLastError();
+    cudaFree(d_bt);
+    cudaFree(d_bg);
+    cudaFree(d_off);
+    return rc;
+}
+
+int reset_state(sptrsv_handle_s *h, cudaStream_t s) {
+    // flags := 0, epoch := 0x01010101 (any nonzero value works), counters := 0
+    CK(cudaMemsetAsync(h->ws.flags, 0, sizeof(uint32_t) * (size_t)(h->n > 0 ? h->n : 1), s));
+    CK(cudaMemsetAsync(h->ws.st, 0, sizeof(SolveState), s));
+    CK(cudaMemsetAsync(&h->ws.st->epoch.v, 1, sizeof(uint32_t), s));
+    h->since_reset = 0;
+    return SPTRSV_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int sptrsv_abi_version(void) { return SPTRSV_ABI_VERSION; }
+
+const char *sptrsv_strerror(int status) {
+    switch (status) {
+        case SPTRSV_OK: return "ok";
+        case SPTRSV_ERR_INVALID_ARG: return "invalid argument";
+        case SPTRSV_ERR_NOT_LOWER: return "entry above the diagonal (column > row)";
+        case SPTRSV_ERR_MISSING_DIAG: return "row without a diagonal as its last entry";
+        case SPTRSV_ERR_ZERO_DIAG: return "zero diagonal";
+        case SPTRSV_ERR_UNSORTED: return "columns not strictly increasing (unsorted or duplicate)";
+        case SPTRSV_ERR_BAD_ROWPTR: return "malformed rowptr";
+        case SPTRSV_ERR_BAD_COL: return "negative column index";
+        case SPTRSV_ERR_TOO_LARGE: return "matrix too large for int32 CSR";
+        case SPTRSV_ERR_CUDA: return "CUDA runtime error";
+        case SPTRSV_ERR_ALLOC: return "allocation failed";
+        case SPTRSV_ERR_TIMEOUT: return "watchdog timeout in solve";
+        default: return "unknown status";
+    }
+}
+
+int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
+                       sptrsv_handle_t *out) {
+    const auto t0 = std::chrono::steady_clock::now();
+    if (!out) return SPTRSV_ERR_INVALID_ARG;
+    *out = nullptr;
+    if (n < 0) return SPTRSV_ERR_INVALID_ARG;
+    if (n > 0x7FFFFFFE) return SPTRSV_ERR_TOO_LARGE;
+    if (!rowptr || (n > 0 && (!colidx || !val))) return SPTRSV_ERR_INVALID_ARG;
+    int rc = set_kernel_attrs();
+    if (rc) return rc;
+    auto *h = new (std::nothrow) sptrsv_handle_s();
+    if (!h) return SPTRSV_ERR_ALLOC;
+    if (cudaGetDevice(&h->device) != cudaSuccess) {
+        delete h;
+        return SPTRSV_ERR_CUDA;
+    }
+    h->n = n;
+    h->rowptr = rowptr;
+    h->colidx = colidx;
+    h->val = val;
+    unsigned long long *d_status = nullptr;
+    int32_t *d_maxrow = nullptr;
+    do {
+        int32_t ends[2] = {0, 0};
+        if (cudaMemcpy(&ends[0], rowptr, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(&ends[1], rowptr + n, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        if (ends[0] != 0 || ends[1] < 0) {
+            rc = SPTRSV_ERR_BAD_ROWPTR;
+            break;
+        }
+        h->nnz = ends[1];
+        const size_t nn = (size_t)(n > 0 ? n : 1);
+        if (cudaMalloc(&h->ws.flags, sizeof(uint32_t) * nn) != cudaSuccess ||
+            cudaMalloc(&h->ws.indeg, sizeof(int32_t) * nn) != cudaSuccess ||
+            cudaMalloc(&h->ws.st, sizeof(SolveState)) != cudaSuccess ||
+            cudaMalloc(&d_status, sizeof(unsigned long long)) != cudaSuccess ||
+            cudaMalloc(&d_maxrow, sizeof(int32_t)) != cudaSuccess) {
+            rc = SPTRSV_ERR_ALLOC;
+            break;
+        }
+        if (cudaMemset(d_status, 0xff, sizeof(unsigned long long)) != cudaSuccess ||
+            cudaMemset(d_maxrow, 0, sizeof(int32_t)) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        if (n > 0) {
+            k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->nnz, h->ws.indeg, d_status,
+                                                 d_maxrow);
+            if (cudaGetLastError() != cudaSuccess) {
+                rc = SPTRSV_ERR_CUDA;
+                break;
+            }
+        }
+        unsigned long long status = 0;
+        if (cudaMemcpy(&status, d_status, sizeof(status), cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(&h->max_row, d_maxrow, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        if (status != ~0ull) {
+            rc = -(int)(status & 0xff);
+            break;
+        }
+        rc = build_plan(h);
+        if (rc) break;
+        rc = reset_state(h, 0);
+        if (rc) break;
+        if (cudaDeviceSynchronize() != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+    } while (0);
+    cudaFree(d_status);
+    cudaFree(d_maxrow);
+    if (rc != SPTRSV_OK) {
+        (void)cudaGetLastError();
+        free_ws(h->ws);
+        delete h;
+        return rc;
+    }
+    h->analyse_ms =
+        std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = h;
+    return SPTRSV_OK;
+}
+
+int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream) {
+    if (!h) return SPTRSV_ERR_INVALID_ARG;
+    if (h->n == 0) return SPTRSV_OK;
+    if (!b || !x || b == x) return SPTRSV_ERR_INVALID_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (h->since_reset >= kEpochResetAt) {
+        int rc = reset_state(h, s);
+        if (rc) return rc;
+    }
+    SolveParams p;
+    p.rowptr = h->rowptr;
+    p.colidx = h->colidx;
+    p.val = h->val;
+    p.b = b;
+    p.x = x;
+    p.flags = h->ws.flags;
+    p.tasks = h->ws.tasks;
+    p.st = h->ws.st;
+    p.n = h->n;
+    p.n_tasks = h->n_tasks;
+    p.backoff_min = h->backoff_min;
+    p.backoff_max = h->backoff_max;
+    p.spin_limit = h->spin_limit;
+    p.stage = h->stage;
+    const int warps = h->cta_threads / 32;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
+    cfg.blockDim = dim3((unsigned)h->cta_threads);
+    cfg.dynamicSmemBytes = h->stage && h->plan != PLAN_WARP ? stage_smem_bytes(h->cta_threads) : 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    cfg.numAttrs = 0;
+    if (h->l2_window) {
+        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[0].val.accessPolicyWindow.base_ptr = h->ws.flags;
+        attr[0].val.accessPolicyWindow.num_bytes = sizeof(uint32_t) * (size_t)h->n;
+        attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
+        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+    }
+    cudaError_t e;
+    switch (h->plan) {
+        case PLAN_THREAD: e = cudaLaunchKernelEx(&cfg, k_solve<PLAN_THREAD>, p); break;
+        case PLAN_WARP: e = cudaLaunchKernelEx(&cfg, k_solve<PLAN_WARP>, p); break;
+        default: e = cudaLaunchKernelEx(&cfg, k_solve<PLAN_LIST>, p); break;
+    }
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_CUDA;
+    }
+    h->solves++;
+    h->since_reset++;
+    return SPTRSV_OK;
+}
+
+int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, sptrsv_stream_t stream) {
+    if (!h) return SPTRSV_ERR_INVALID_ARG;
+    if (h->n == 0) return SPTRSV_OK;
+    if (!b_host || !x_host) return SPTRSV_ERR_INVALID_ARG;
+    const size_t bytes = sizeof(double) * (size_t)h->n;
+    if (!h->ws.b_stage) {
+        if (cudaMalloc(&h->ws.b_stage, bytes) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_ALLOC;
+        }
+    }
+    if (!h->ws.x_stage) {
+        if (cudaMalloc(&h->ws.x_stage, bytes) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_ALLOC;
+        }
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
+    int rc = sptrsv_solve(h, h->ws.b_stage, h->ws.x_stage, stream);
+    if (rc) return rc;
+    CK(cudaMemcpyAsync(x_host, h->ws.x_stage, bytes, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    return SPTRSV_OK;
+}
+
+int sptrsv_destroy(sptrsv_handle_t h) {
+    if (!h) return SPTRSV_OK;
+    int prev = 0;
+    cudaGetDevice(&prev);
+    cudaSetDevice(h->device);
+    cudaDeviceSynchronize();
+    free_ws(h->ws);
+    cudaSetDevice(prev);
+    delete h;
+    return SPTRSV_OK;
+}
+
+int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
+    if (!h) return SPTRSV_ERR_INVALID_ARG;
+    switch (key) {
+        case SPTRSV_OPT_MODE:
+            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
+            h->mode = (int)value;
+            return build_plan(h);
+        case SPTRSV_OPT_WARP_THRESHOLD:
+            if (value < 0 || value > (1 << 30)) return SPTRSV_ERR_INVALID_ARG;
+            h->threshold = (int)value;
+            return build_plan(h);
+        case SPTRSV_OPT_CTA_THREADS:
+            if (value != 128 && value != 256 && value != 512 && value != 1024) return SPTRSV_ERR_INVALID_ARG;
+            h->cta_threads = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_BACKOFF_MIN_NS:
+            if (value < 0 || value > 1000000) return SPTRSV_ERR_INVALID_ARG;
+            h->backoff_min = (uint32_t)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_BACKOFF_MAX_NS:
+            if (value < 0 || value > 1000000) return SPTRSV_ERR_INVALID_ARG;
+            h->backoff_max = (uint32_t)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_SPIN_LIMIT:
+            if (value < 0 || value > 0xFFFFFFFFll) return SPTRSV_ERR_INVALID_ARG;
+            h->spin_limit = (uint32_t)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_L2_WINDOW: {
+            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            if (value) {
+                cudaDeviceProp prop;
+                CK(cudaGetDeviceProperties(&prop, h->device));
+                size_t want = sizeof(uint32_t) * (size_t)h->n;
+                if (want > (size_t)prop.persistingL2CacheMaxSize) want = prop.persistingL2CacheMaxSize;
+                size_t cur = 0;
+                CK(cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize));
+                if (cur < want) CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+            }
+            h->l2_window = (int)value;
+            return SPTRSV_OK;
+        }
+        case SPTRSV_OPT_STAGE_SMEM:
+            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            h->stage = (int)value;
+            return SPTRSV_OK;
+        default:
+            return SPTRSV_ERR_INVALID_ARG;
+    }
+}
+
+int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
+    if (!h || !value) return SPTRSV_ERR_INVALID_ARG;
+    switch (key) {
+        case SPTRSV_OPT_MODE: *value = h->mode; return SPTRSV_OK;
+        case SPTRSV_OPT_WARP_THRESHOLD: *value = h->threshold; return SPTRSV_OK;
+        case SPTRSV_OPT_CTA_THREADS: *value = h->cta_threads; return SPTRSV_OK;
+        case SPTRSV_OPT_BACKOFF_MIN_NS: *value = h->backoff_min; return SPTRSV_OK;
+        case SPTRSV_OPT_BACKOFF_MAX_NS: *value = h->backoff_max; return SPTRSV_OK;
+        case SPTRSV_OPT_SPIN_LIMIT: *value = h->spin_limit; return SPTRSV_OK;
+        case SPTRSV_OPT_L2_WINDOW: *value = h->l2_window; return SPTRSV_OK;
+        case SPTRSV_OPT_STAGE_SMEM: *value = h->stage; return SPTRSV_OK;
+        default: return SPTRSV_ERR_INVALID_ARG;
+    }
+}
+
+int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
+    if (!h || !out) return SPTRSV_ERR_INVALID_ARG;
+    out->n = h->n;
+    out->nnz = h->nnz;
+    out->n_thread_groups = h->n_thread_groups;
+    out->n_warp_rows = h->n_warp_rows;
+    out->n_tasks = h->n_tasks;
+    out->max_row_nnz = h->max_row;
+    out->device = h->device;
+    out->analyse_ms = h->analyse_ms;
+    out->solves = h->solves;
+    return SPTRSV_OK;
+}
+
+int sptrsv_get_indegree(sptrsv_handle_t h, int32_t *out_dev, sptrsv_stream_t stream) {
+    if (!h || (!out_dev && h->n > 0)) return SPTRSV_ERR_INVALID_ARG;
+    if (h->n == 0) return SPTRSV_OK;
+    CK(cudaMemcpyAsync(out_dev, h->ws.indeg, sizeof(int32_t) * (size_t)h->n, cudaMemcpyDeviceToDevice,
+                       (cudaStream_t)stream));
+    return SPTRSV_OK;
+}
+
+int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev, int32_t *nlevels_host,
+                  sptrsv_stream_t stream) {
+    if (!h || !nlevels_host) return SPTRSV_ERR_INVALID_ARG;
+    *nlevels_host = 0;
+    if (h->n == 0) return SPTRSV_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t n = (size_t)h->n;
+    if (!h->ws.lvl) {
+        if (cudaMalloc(&h->ws.lvl, sizeof(uint32_t) * (n + 1)) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_ALLOC;
+        }
+    }
+    int32_t *d_nlev = reinterpret_cast<int32_t *>(h->ws.lvl + n);
+    CK(cudaMemsetAsync(h->ws.lvl, 0, sizeof(uint32_t) * (n + 1), s));
+    CK(cudaMemsetAsync(&h->ws.st->lticket.v, 0, sizeof(uint32_t), s));
+    if (counts_dev) CK(cudaMemsetAsync(counts_dev, 0, sizeof(int32_t) * n, s));
+    const int groups = (h->n + 31) / 32;
+    k_levels<<<(groups + 7) / 8, 256, 0, s>>>(h->rowptr, h->colidx, h->ws.lvl, h->ws.st, h->n);
+    CK(cudaGetLastError());
+    k_level_finish<<<(h->n + 255) / 256, 256, 0, s>>>(h->ws.lvl, level_dev, counts_dev, d_nlev, h->n);
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(nlevels_host, d_nlev, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    return SPTRSV_OK;
+}
+
+int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
+    if (!h) return SPTRSV_ERR_INVALID_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(cudaStreamSynchronize(s));
+    uint32_t err = 0;
+    CK(cudaMemcpy(&err, &h->ws.st->error.v, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+    if (err) {
+        CK(cudaMemset(&h->ws.st->error.v, 0, sizeof(uint32_t)));
+        return SPTRSV_ERR_TIMEOUT;
+    }
+    return SPTRSV_OK;
+}
+
+int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop) {
+    if (iters <= 0 || protocol < 0 || protocol > 2 || !ns_per_hop) return SPTRSV_ERR_INVALID_ARG;
+    uint32_t *flags = nullptr;
+    double *xs = nullptr, *sink = nullptr;
+    unsigned long long *ns = nullptr;
+    int rc = SPTRSV_OK;
+    do {
+        if (cudaMalloc(&flags, 256) != cudaSuccess || cudaMalloc(&xs, 256) != cudaSuccess ||
+            cudaMalloc(&sink, 16) != cudaSuccess || cudaMalloc(&ns, 8) != cudaSuccess) {
+            rc = SPTRSV_ERR_ALLOC;
+            break;
+        }
+        if (cudaMemset(flags, 0, 256) != cudaSuccess || cudaMemset(xs, 0, 256) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        k_pingpong<<<2, 32>>>(flags, xs, iters, protocol, ns, sink);
+        unsigned long long t = 0;
+        if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess ||
+            cudaMemcpy(&t, ns, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        *ns_per_hop = (double)t / (2.0 * iters);
+    } while (0);
+    (void)cudaGetLastError();
+    cudaFree(flags);
+    cudaFree(xs);
+    cudaFree(sink);
+    cudaFree(ns);
+    return rc;
+}
+
+}  // extern "C"

@@ -1,0 +1,72 @@
+"""CPU-side checks of the boundary: the C-ABI library builds, loads without a GPU and
+exports every function include/sptrsv.h declares; the binding's marshalling tables
+match the header.  No compute calls (no GPU here)."""
+import os
+import re
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "sptrsv.h")
+
+
+def _declared():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(sptrsv_[a-z_]+)\s*\(", src)))
+
+
+@pytest.fixture(scope="module")
+def libpath():
+    from paper_conf_icpp_suz0hw0w20_b200 import build
+    return build.build()
+
+
+def test_header_declares_the_north_star_entry_points():
+    d = _declared()
+    for name in ("sptrsv_analyse_csr", "sptrsv_solve", "sptrsv_destroy"):
+        assert name in d
+
+
+def test_library_exports_every_declared_symbol(libpath):
+    out = subprocess.run(["nm", "-D", "--defined-only", libpath], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT\s+(sptrsv_[a-z_]+)\b", out))
+    missing = [f for f in _declared() if f not in exported]
+    assert not missing, missing
+
+
+def test_binding_covers_header_and_loads(libpath):
+    import paper_conf_icpp_suz0hw0w20_b200._lib as L
+    assert sorted(L.EXPORTS) == _declared()
+    assert L.lib.sptrsv_abi_version() == 1
+    assert L.lib.sptrsv_strerror(-3).decode().startswith("row without a diagonal")
+    # argument validation happens before any CUDA call
+    assert L.lib.sptrsv_analyse_csr(-1, None, None, None, None) == L.ERR_INVALID_ARG
+    assert L.lib.sptrsv_solve(None, None, None, None) == L.ERR_INVALID_ARG
+    assert L.lib.sptrsv_destroy(None) == L.OK
+
+
+def test_status_codes_match_oracle_numbering():
+    import oracle
+    import paper_conf_icpp_suz0hw0w20_b200._lib as L
+    for name in ("NOT_LOWER", "MISSING_DIAG", "ZERO_DIAG", "BAD_ROWPTR", "BAD_COL"):
+        assert getattr(oracle, name) == getattr(L, "ERR_" + name)
+    assert oracle.UNSORTED == L.ERR_UNSORTED
+
+
+def test_kernels_are_sm100a_sass(libpath):
+    out = subprocess.run(["cuobjdump", "--list-elf", libpath], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    sass = subprocess.run(["cuobjdump", "-sass", libpath], capture_output=True, text=True).stdout
+    # the flag protocol: acquire polls (strong GPU loads + L1 invalidate), release publishes
+    assert "LDG.E.STRONG.GPU" in sass and "CCTL.IVALL" in sass and "NANOSLEEP" in sass
+
+
+def test_product_package_never_imports_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icpp_suz0hw0w20_b200")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                txt = open(os.path.join(dp, f)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt and "oracle.c" not in txt, f

@@ -1,0 +1,238 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bars:
+* thread-level rows: BIT-EXACT vs oracle.solve (same row order, separately rounded
+  mul/add, IEEE division -- Alg.1 arithmetic);
+* warp-level rows (lane-strided partial sums + butterfly, Alg.3): max componentwise
+  relative error <= 1e-12 (north_star tolerance; DESIGN.md derives the bound);
+* exact-integer systems, diagonal and bidiagonal closed forms: bit-exact in every mode;
+* integer outputs (in-degrees, levels, level counts, nlevels): bit-exact.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-12
+
+
+@pytest.fixture(scope="module")
+def cap():
+    import paper_conf_icpp_suz0hw0w20_b200 as cap
+    return cap
+
+
+def dev_csr(s):
+    d = torch.device("cuda:0")
+    return (torch.from_numpy(s.rowptr).to(d), torch.from_numpy(s.colidx).to(d),
+            torch.from_numpy(s.val).to(d), torch.from_numpy(s.b).to(d))
+
+
+def gpu_solve(cap, s, mode=0, poison=True, **opt):
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v, mode=mode, **opt) as h:
+        x = torch.full_like(b, float("nan")) if poison else torch.empty_like(b)
+        h.solve(b, x)
+        h.check()
+        info = h.info()
+        return x.cpu().numpy(), info
+
+
+def relerr(a, ref):
+    return float(np.max(np.abs(a - ref) / np.maximum(np.abs(ref), 1e-300))) if ref.size else 0.0
+
+
+MODES = [0, 1, 2]
+
+
+# ------------------------------------------------------------------ small, many tiles + ragged tails
+
+@pytest.mark.parametrize("n", [1, 2, 31, 32, 33, 63, 65, 257, 1000, 4099])
+@pytest.mark.parametrize("mode", MODES)
+def test_random_small_sizes(cap, n, mode):
+    s = synth.gen_random_lower(n, 4, seed=n)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    x, info = gpu_solve(cap, s, mode)
+    if mode == 1:
+        assert np.array_equal(x, ref)
+    else:
+        assert relerr(x, ref) <= TOL
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_c1_config(cap, mode):
+    s = synth.gen_c1()
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    x, info = gpu_solve(cap, s, mode)
+    assert info["nnz"] == 3994
+    if mode in (0, 1):  # c1 has ~4 nnz/row: auto picks thread level everywhere
+        assert np.array_equal(x, ref)
+        assert info["n_warp_rows"] == (0 if mode == 0 else 0)
+    else:
+        assert relerr(x, ref) <= TOL
+
+
+def test_dense_lower_rows_up_to_500(cap):
+    s = synth.gen_dense_lower(500)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    for mode in MODES:
+        x, _ = gpu_solve(cap, s, mode)
+        assert relerr(x, ref) <= TOL, mode
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_closed_forms_bit_exact(cap, mode):
+    d = synth.gen_diag(10_001)
+    x, _ = gpu_solve(cap, d, mode)
+    assert np.array_equal(x, d.b / d.val)
+    c = synth.gen_chain(3000)
+    x, _ = gpu_solve(cap, c, mode)
+    want = np.array([1.0 - 2.0 ** -(i + 1) if i <= 52 else 1.0 for i in range(3000)])
+    assert np.array_equal(x, want)
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("gen", ["c1", "c2s", "c2is", "c4s", "dense"])
+def test_exact_integer_systems_bit_exact(cap, mode, gen):
+    base = {"c1": lambda: synth.gen_c1(), "c2s": lambda: synth.gen_c2(n=50_000),
+            "c2is": lambda: synth.gen_c2i(n=50_000), "c4s": lambda: synth.gen_c4(n=20_000, nlevels=100),
+            "dense": lambda: synth.gen_dense_lower(200)}[gen]()
+    s = synth.integerize(base)
+    x, _ = gpu_solve(cap, s, mode)
+    assert np.array_equal(x, s.x_true)
+
+
+# ------------------------------------------------------------------ protocol stress
+
+@pytest.mark.parametrize("cta", [128, 256, 512, 1024])
+@pytest.mark.parametrize("stage", [0, 1])
+def test_interleaved_levels_stress(cap, cta, stage):
+    """c2i: half the dependencies inside the same warp (Challenge 1)."""
+    s = synth.gen_c2i(n=200_000)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    x, _ = gpu_solve(cap, s, 0, cta_threads=cta, stage_smem=stage)
+    assert np.array_equal(x, ref)
+
+
+def test_back_to_back_solves_and_epoch(cap):
+    """Several solves with different b through one handle (epoch flags must reset)."""
+    s = synth.gen_c2(n=100_000)
+    rp, ci, v, _ = dev_csr(s)
+    rng = np.random.default_rng(0)
+    with cap.analyse(rp, ci, v) as h:
+        for it in range(20):
+            bb = rng.uniform(-1, 1, s.n)
+            x = torch.full((s.n,), float("nan"), dtype=torch.float64, device="cuda:0")
+            h.solve(torch.from_numpy(bb).cuda(), x)
+            h.check()
+            assert np.array_equal(x.cpu().numpy(), oracle.solve(s.rowptr, s.colidx, s.val, bb)), it
+        assert h.info()["solves"] == 20
+
+
+def test_many_solves_on_side_stream_and_graph_capture(cap):
+    s = synth.gen_c1()
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        st = torch.cuda.Stream()
+        x = torch.empty_like(b)
+        with torch.cuda.stream(st):
+            for _ in range(200):
+                h.solve(b, x)
+        h.check(st)
+        assert np.array_equal(x.cpu().numpy(), ref)
+        # CUDA graph: the solve is one kernel whose epoch lives on the device
+        g = torch.cuda.CUDAGraph()
+        x2 = torch.empty_like(b)
+        with torch.cuda.stream(st):
+            h.solve(b, x2, stream=st)  # warm
+            st.synchronize()
+            with torch.cuda.graph(g, stream=st):
+                h.solve(b, x2, stream=st)
+        for _ in range(5):
+            x2.fill_(float("nan"))
+            g.replay()
+            torch.cuda.synchronize()
+            assert np.array_equal(x2.cpu().numpy(), ref)
+
+
+def test_solve_host_e2e(cap):
+    s = synth.gen_c2(n=100_000)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, _ = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        bh = torch.from_numpy(s.b).pin_memory()
+        xh = torch.empty(s.n, dtype=torch.float64).pin_memory()
+        h.solve_host(bh, xh)
+        assert np.array_equal(xh.numpy(), ref)
+
+
+def test_empty_matrix(cap):
+    d = torch.device("cuda:0")
+    rp = torch.zeros(1, dtype=torch.int32, device=d)
+    e = torch.zeros(0, dtype=torch.int32, device=d)
+    ev = torch.zeros(0, dtype=torch.float64, device=d)
+    with cap.analyse(rp, e, ev) as h:
+        x = h.solve(torch.zeros(0, dtype=torch.float64, device=d))
+        assert x.numel() == 0
+        assert h.levels()[1] == 0
+
+
+# ------------------------------------------------------------------ validation (same codes as oracle)
+
+CASES = [
+    ([0, 1, 3], [0, 1, 1], [1, 1, 1]),
+    ([0, 2, 3], [0, 1, 1], [1, 1, 1]),
+    ([0, 1, 3], [0, 1, 0], [1, 1, 1]),
+    ([0, 1, 2], [0, 0], [1, 1]),
+    ([0, 1, 1], [0], [1]),
+    ([0, 1, 3], [0, 0, 1], [1, 1, 0]),
+    ([1, 1, 3], [0, 0, 1], [1, 1, 1]),
+    ([0, 1, 0, 3], [0, 0, 1], [1, 1, 1]),
+    ([0, 1, 3], [0, -1, 1], [1, 1, 1]),
+    ([0, 1, 3, 5, 6], [0, 0, 1, 1, 9, 3], [1, 1, 1, 1, 1, 1]),
+]
+
+
+@pytest.mark.parametrize("case", range(len(CASES)))
+def test_validation_codes_match_oracle(cap, case):
+    rp, ci, v = CASES[case]
+    code, _ = oracle.validate(np.array(rp, np.int32), np.array(ci, np.int32), np.array(v, float))
+    assert code != 0
+    d = torch.device("cuda:0")
+    with pytest.raises(cap.SptrsvError) as e:
+        cap.analyse(torch.tensor(rp, dtype=torch.int32, device=d), torch.tensor(ci, dtype=torch.int32, device=d),
+                    torch.tensor(v, dtype=torch.float64, device=d))
+    assert e.value.status == code
+
+
+# ------------------------------------------------------------------ integer diagnostics
+
+@pytest.mark.parametrize("gen", ["c1", "c2s", "c2is", "grid", "c4s", "chain", "fig2"])
+def test_indegree_and_levels_bit_exact(cap, gen):
+    if gen == "fig2":
+        rp_, ci_ = synth.gen_fig2_pattern()
+        s = synth.from_pattern("fig2", rp_, ci_, np.random.default_rng(0))
+    else:
+        s = {"c1": lambda: synth.gen_c1(), "c2s": lambda: synth.gen_c2(n=100_000),
+             "c2is": lambda: synth.gen_c2i(n=100_000), "grid": lambda: synth.gen_grid(300),
+             "c4s": lambda: synth.gen_c4(n=50_000, nlevels=250), "chain": lambda: synth.gen_chain(20_000)}[gen]()
+    rp, ci, v, _ = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        assert np.array_equal(h.indegree().cpu().numpy(), oracle.indegree(s.rowptr, s.colidx))
+        lv, nl, counts = h.levels()
+        olv = oracle.levels_bfs(s.rowptr, s.colidx)
+        onl, ocounts = oracle.level_counts(olv)
+        assert np.array_equal(lv.cpu().numpy(), olv)
+        assert nl == onl
+        assert np.array_equal(counts.cpu().numpy(), ocounts)
+
+
+def test_flag_latency_runs(cap):
+    for proto in (0, 1, 2):
+        t = cap.flag_latency(2000, proto)
+        assert 10.0 < t < 100_000.0
