@@ -1,0 +1,368 @@
+#!/usr/bin/env python
+"""Benchmark: SpTRSV GFLOPS (2*nnz / solve time, fp64) and % of HBM roofline on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl cuda|reference]
+
+One step = one solve L x = b (the whole hot path: a single k_solve launch) of the
+config's synthetic system, inputs resident in HBM.  N=1 workload = BASELINE.json
+configs[1] ("c2": n=1e6, ~3 nnz/row, 10 levels x 1e5).  Under torchrun (N>1) every
+rank solves its own independent system of the same shape (seed + rank): weak
+scaling, no data-path collective; NCCL is used only for the
+barrier and the max-over-ranks of the timed region.  ``--config c5`` instead shards
+the 8 fixed C5 systems over the ranks (strong scaling).
+
+The oracle (oracle/, the plain CPU implementation) is used here only for the
+cpu_baseline leg and for --impl reference, as the task rules allow.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "SpTRSV GFLOPS (2*nnz/solve time, fp64)"
+UNIT = "GFLOPS"
+WORKLOADS = {
+    "c1": "random lower-triangular CSR n=1000, ~4 nnz/row, diagonally dominant, fp64, single RHS",
+    "c2": "n=1,000,000, ~3 nnz/row (2.8 nnz/row), 10 levels x 100,000 components (warp-underutilisation regime)",
+    "c3": "lower factor of a 2D 5-point grid 2048x2048 (n=4,194,304, 4095 anti-diagonal levels)",
+    "c4": "n=1,000,000, ~64 nnz/row, 1000 levels x 1000 (warp-per-row regime)",
+    "c5": "batch of 8 independent n=2,000,000 low-nnz systems (10 levels x 200,000) sharded over ranks",
+    "chain": "bidiagonal chain n=100,000 (pure dependency chain)",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="c2", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="cuda", choices=["cuda", "reference"])
+    ap.add_argument("--mode", type=int, default=0, help="0 auto, 1 thread, 2 warp")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0, help="cpu_baseline sample budget")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu: no clocks/e2e/cpu legs")
+    ap.add_argument("--opt", action="append", default=[], help="extra handle option key=value")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ workload
+
+def systems_for_rank(config: str, rank: int, world: int):
+    import synth
+    if config == "c5":
+        return [synth.gen_c5(s) for s in range(8) if s % world == rank]
+    if config == "c2":
+        return [synth.gen_c2(seed=2 + rank)]
+    if config == "c3":
+        return [synth.gen_c3(seed=3 + rank)]
+    if config == "c4":
+        return [synth.gen_c4(seed=4 + rank)]
+    if config == "c1":
+        return [synth.gen_c1(seed=1 + rank)]
+    if config == "chain":
+        return [synth.gen_chain()]
+    raise ValueError(config)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy bandwidth)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(config: str):
+    """Per-launch dram read+write bytes of k_solve from the committed ncu --set full capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        if config in d:
+            return d[config]
+    return None
+
+
+# ------------------------------------------------------------------ clocks (nvidia-smi during the timed region)
+
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap,clocks_event_reasons.hw_power_brake_slowdown")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *exc):
+        if self.proc:
+            time.sleep(0.15)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap", "hw_power_brake"]
+        reasons = sorted({names[k] for r in self.rows for k in range(5) if r[2 + k].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------------ reference arm (the CPU oracle)
+
+def run_reference(args, rank, world):
+    import oracle
+    if rank != 0:
+        return
+    systems = systems_for_rank(args.config, 0, 1)
+    if args.config == "c5":
+        systems = systems  # all 8 on the host
+    for _ in range(args.warmup):
+        for s in systems:
+            oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        for s in systems:
+            oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        times.append(time.perf_counter() - t0)
+    nnz = sum(s.nnz for s in systems)
+    tot = float(np.sum(times))
+    value = 2.0 * nnz * args.steps / tot / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "weak" if args.config != "c5" else "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {WORKLOADS[args.config]}", "n": int(sum(s.n for s in systems)),
+                   "nnz": int(nnz)},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": f"{len(systems)} full system(s) per step, {args.steps} steps, single-thread C "
+                                   f"oracle (Alg. 1), host {os.cpu_count()} cores"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(systems, budget_s):
+    import oracle
+    s = systems[0]
+    reps, t0 = 0, time.perf_counter()
+    oracle.solve(s.rowptr, s.colidx, s.val, s.b)  # warm
+    t0 = time.perf_counter()
+    while True:
+        oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s or reps >= 2000:
+            break
+    return {"value": 2.0 * s.nnz * reps / el / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{reps} repeated full solves of the rank-0 system ({s.name}, n={s.n}, nnz={s.nnz}) in "
+                      f"{el:.1f}s, single-thread C oracle (Alg. 1, gcc -O2); host has {os.cpu_count()} cores"}
+
+
+# ------------------------------------------------------------------ the CUDA arm
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import torch
+    import paper_conf_icpp_suz0hw0w20_b200 as cap
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+
+    systems = systems_for_rank(args.config, rank, world)
+    opts = {"mode": args.mode}
+    for kv in args.opt:
+        k, v = kv.split("=")
+        opts[k] = int(v)
+    handles, bufs = [], []
+    for s in systems:
+        rp, ci, v, b = (torch.from_numpy(a).to(dev) for a in (s.rowptr, s.colidx, s.val, s.b))
+        h = cap.analyse(rp, ci, v, **opts)
+        x = torch.empty_like(b)
+        handles.append(h)
+        bufs.append((rp, ci, v, b, x))
+    stream = torch.cuda.current_stream(dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)  # > 126 MB L2
+
+    def step(i):
+        for h, (_, _, _, b, x) in zip(handles, bufs):
+            h.solve(b, x, stream=stream)
+
+    for i in range(args.warmup):
+        flush.zero_()
+        step(i)
+    for h in handles:
+        h.check(stream)
+
+    # ---- timed region: K steps, barrier + synchronize on both sides; L2 flushed between steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    sampler = ClockSampler(local) if not args.profile else None
+    if sampler:
+        sampler.__enter__()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        flush.zero_()
+        ev[i][0].record(stream)
+        step(i)
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    if sampler:
+        sampler.__exit__(None, None, None)
+    for h in handles:
+        h.check(stream)
+    step_ms = np.array([a.elapsed_time(b) for a, b in ev])
+    tot_s = float(step_ms.sum()) * 1e-3
+    if dist:
+        t = torch.tensor([tot_s], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot_s = float(t.item())
+    nnz_rank = sum(s.nnz for s in systems)
+    nnz_all = nnz_rank
+    if dist:
+        t = torch.tensor([nnz_rank], device=dev, dtype=torch.float64)
+        dist.all_reduce(t)
+        nnz_all = float(t.item())
+    value = 2.0 * nnz_all * args.steps / tot_s / 1e9
+    kernel_s = float(np.median(step_ms)) * 1e-3 / max(1, len(systems))
+
+    # ---- roofline of the dominant (only) kernel, k_solve
+    peak, peak_src = peaks()
+    alg_bytes = systems[0].alg_bytes()
+    achieved = alg_bytes / kernel_s / 1e9
+    roof = {"bound": "hbm", "kernel": "k_solve", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 5), "traffic": ncu_traffic(args.config),
+            "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src,
+            "alg_bytes_formula": "4(n+1) + 12*nnz + 8n (b) + 8n (x) + 4n (flags)"}
+
+    # ---- critical-path latency bound: (levels - 1) * t_hop
+    import synth  # noqa: F401
+    lat = None
+    if not args.profile:
+        levels = {"c1": None, "c2": 10, "c3": 4095, "c4": 1000, "c5": 10, "chain": systems[0].n}[args.config]
+        if levels is None:
+            lv, levels, _ = handles[0].levels(stream)
+        t_hop = cap.flag_latency(20000, 0)
+        lat = {"levels": int(levels), "t_hop_ns": round(t_hop, 1),
+               "bound_us": round((levels - 1) * t_hop * 1e-3, 2),
+               "frac": round((levels - 1) * t_hop * 1e-9 / kernel_s, 4)}
+
+    # ---- e2e: through the C-ABI host-buffer call, H2D + solve + D2H inside the timed region
+    e2e = None
+    if not args.no_e2e and not args.profile:
+        hb = [torch.from_numpy(s.b).pin_memory() for s in systems]
+        hx = [torch.empty(s.n, dtype=torch.float64).pin_memory() for s in systems]
+        for h, b_, x_ in zip(handles, hb, hx):
+            h.solve_host(b_, x_, stream=stream)
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e_ms = []
+        for i in range(args.steps):
+            flush.zero_()
+            a, bb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            for h, b_, x_ in zip(handles, hb, hx):
+                h.solve_host(b_, x_, stream=stream)
+            bb.record(stream)
+            bb.synchronize()
+            e_ms.append(a.elapsed_time(bb))
+        torch.cuda.synchronize()
+        et = float(np.sum(e_ms)) * 1e-3
+        if dist:
+            dist.barrier()
+            t = torch.tensor([et], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            et = float(t.item())
+        ok = all(np.array_equal(x_.numpy(), x.cpu().numpy()) for x_, (_, _, _, _, x) in zip(hx, bufs))
+        e2e = {"value": 2.0 * nnz_all * args.steps / et / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": int(sum(8 * s.n for s in systems)),
+               "d2h_bytes_per_step": int(sum(8 * s.n for s in systems)),
+               "matches_device_path": bool(ok)}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
+        cpu = cpu_baseline(systems, args.cpu_seconds)
+
+    if rank == 0:
+        info = handles[0].info()
+        line = {
+            "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot_s / args.steps * 1e3, 5),
+            "higher_is_better": True, "scaling": "strong" if args.config == "c5" else "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config}: {WORKLOADS[args.config]}",
+                       "n": systems[0].n, "nnz": systems[0].nnz, "systems_per_rank": len(systems),
+                       "mode": {0: "auto", 1: "thread", 2: "warp"}[args.mode],
+                       "plan": {"thread_groups": info["n_thread_groups"], "warp_rows": info["n_warp_rows"]},
+                       "analyse_ms": round(info["analyse_ms"], 3),
+                       "l2": "flushed between timed steps (256 MiB write, outside the per-step events)",
+                       "parallelism": f"replicas x{world}" if args.config != "c5" else f"systems sharded over {world}",
+                       "options": opts},
+            "roofline": roof,
+            "latency_bound": lat,
+            "e2e": e2e,
+            "gpu_launches": args.steps * len(systems),
+            "cpu_baseline": cpu,
+            "clocks": sampler.summary() if sampler else None,
+        }
+        print(json.dumps(line), flush=True)
+    for h in handles:
+        h.close()
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

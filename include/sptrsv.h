@@ -64,8 +64,15 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
     SPTRSV_OPT_SPIN_LIMIT = 6,     /* watchdog: idle passes per warp before TIMEOUT (0=off) */
     SPTRSV_OPT_L2_WINDOW = 7,      /* 1: cudaAccessPolicyWindow persisting over the flags   */
-    SPTRSV_OPT_STAGE_SMEM = 8      /* 1 (default): thread-level warps stage their CSR slice
+    SPTRSV_OPT_STAGE_SMEM = 8,     /* 1 (default): thread-level warps stage their CSR slice
                                       in shared memory with coalesced loads                 */
+    SPTRSV_OPT_PROTOCOL = 9,       /* cross-CTA ready protocol: 0 FLAGS (default) = uint32
+                                      epoch flags, st.release.gpu / ld.acquire.gpu (Alg.5
+                                      l.15-16 + DESIGN G6); 1 FUSED = 16-byte record per
+                                      component, each 8-byte half = epoch<<32 | half of x_i,
+                                      no fences                     */
+    SPTRSV_OPT_LOCAL = 10          /* 1 (default): dependencies produced inside the same CTA
+                                      are read from a shared-memory copy of x               */
 } sptrsv_option;
 
 typedef struct sptrsv_info {
@@ -163,9 +170,13 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream);
  * and report the mean one-way hop in nanoseconds (t_hop of the critical-path
  * latency bound).  protocol: 0 = st.release flag / ld.acquire poll
  * + relaxed x load (the solve's protocol), 1 = relaxed poll + fence.acq_rel,
- * 2 = value-as-flag (x polled directly; ablation only).  Synchronous.
+ * 2 = value-as-flag (x polled directly; ablation only); single-CTA probes:
+ * 3 = dependent ld.relaxed.gpu chain (ns per L2 round trip), 4 = st x +
+ * st.release flag pairs (ns per publish).  sm_mhz (host, may be NULL)
+ * receives the SM clock seen during the probe (clock64 / globaltimer).
+ * Synchronous.
  */
-int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop);
+int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop, double *sm_mhz);
 
 const char *sptrsv_strerror(int status);
 int sptrsv_abi_version(void);

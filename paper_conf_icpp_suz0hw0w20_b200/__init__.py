@@ -14,11 +14,11 @@ import ctypes
 
 from . import _lib
 from ._lib import (MODE_AUTO, MODE_THREAD, MODE_WARP, OPT_BACKOFF_MAX_NS, OPT_BACKOFF_MIN_NS,
-                   OPT_CTA_THREADS, OPT_L2_WINDOW, OPT_MODE, OPT_SPIN_LIMIT, OPT_STAGE_SMEM,
-                   OPT_WARP_THRESHOLD, SptrsvError, check)
+                   OPT_CTA_THREADS, OPT_L2_WINDOW, OPT_LOCAL, OPT_MODE, OPT_PROTOCOL, OPT_SPIN_LIMIT,
+                   OPT_STAGE_SMEM, OPT_WARP_THRESHOLD, PROTO_FLAGS, PROTO_FUSED, SptrsvError, check)
 
 __all__ = ["analyse", "Handle", "SptrsvError", "flag_latency", "MODE_AUTO", "MODE_THREAD",
-           "MODE_WARP", "lib"]
+           "MODE_WARP", "PROTO_FLAGS", "PROTO_FUSED", "lib"]
 
 lib = _lib.lib
 
@@ -155,14 +155,16 @@ def analyse(rowptr, colidx, val, **options) -> Handle:
     h = Handle(rowptr, colidx, val)
     keys = {"mode": OPT_MODE, "warp_threshold": OPT_WARP_THRESHOLD, "cta_threads": OPT_CTA_THREADS,
             "backoff_min_ns": OPT_BACKOFF_MIN_NS, "backoff_max_ns": OPT_BACKOFF_MAX_NS,
-            "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM}
+            "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
+            "protocol": OPT_PROTOCOL, "local": OPT_LOCAL}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h
 
 
-def flag_latency(iters: int = 20000, protocol: int = 0) -> float:
-    """Mean one-way flag hop (ns) between two CTAs on the current device (sptrsv_flag_latency)."""
-    v = ctypes.c_double(0.0)
-    check(lib.sptrsv_flag_latency(iters, protocol, ctypes.byref(v)), "sptrsv_flag_latency")
-    return float(v.value)
+def flag_latency(iters: int = 20000, protocol: int = 0, with_clock: bool = False):
+    """Mean one-way flag hop (ns) between two CTAs on the current device (sptrsv_flag_latency).
+    protocol 0 = the solve's release/acquire pair; see include/sptrsv.h for 1-4."""
+    v, mhz = ctypes.c_double(0.0), ctypes.c_double(0.0)
+    check(lib.sptrsv_flag_latency(iters, protocol, ctypes.byref(v), ctypes.byref(mhz)), "sptrsv_flag_latency")
+    return (float(v.value), float(mhz.value)) if with_clock else float(v.value)

@@ -41,6 +41,9 @@ OPT_BACKOFF_MAX_NS = 5
 OPT_SPIN_LIMIT = 6
 OPT_L2_WINDOW = 7
 OPT_STAGE_SMEM = 8
+OPT_PROTOCOL = 9
+OPT_LOCAL = 10
+PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
 
 
@@ -73,7 +76,8 @@ EXPORTS = {
     "sptrsv_get_indegree": (ctypes.c_int, [_h, _p, _p]),
     "sptrsv_levels": (ctypes.c_int, [_h, _p, _p, ctypes.POINTER(_i32), _p]),
     "sptrsv_check": (ctypes.c_int, [_h, _p]),
-    "sptrsv_flag_latency": (ctypes.c_int, [_i32, _i32, ctypes.POINTER(ctypes.c_double)]),
+    "sptrsv_flag_latency": (ctypes.c_int, [_i32, _i32, ctypes.POINTER(ctypes.c_double),
+                                           ctypes.POINTER(ctypes.c_double)]),
     "sptrsv_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "sptrsv_abi_version": (ctypes.c_int, []),
 }

@@ -1,0 +1,155 @@
+// diag.cuh -- diagnostics outside the timed solve: GPU level analysis (SURVEY
+// row a10) and the flag-hop microbenchmark (t_hop of the latency bound).
+#pragma once
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "solve.cuh"
+
+namespace sptrsv_dev {
+
+// ---------------------------------------------------------------- levels (diagnostic)
+//
+// lvl[i] = level(i) + 1 once known, 0 before.  The value IS the
+// message, so a relaxed poll suffices (no second location is read).
+// level(i) = max over dependencies of lvl[j] (= 1 + level(j)), 0 without any.
+__global__ void __launch_bounds__(256) k_levels(const int32_t *__restrict__ rowptr,
+                                                const int32_t *__restrict__ colidx, uint32_t *lvl,
+                                                SolveState *st, int32_t n) {
+    __shared__ uint32_t s_blk;
+    if (threadIdx.x == 0) s_blk = atomicAdd(&st->lticket.v, 1u);
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int r0 = ((int)s_blk * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32;
+    if (r0 >= n) return;
+    const int i = r0 + lane;
+    const bool act = i < n;
+    int j = 0, jd = 0;
+    if (act) {
+        j = rowptr[i];
+        jd = rowptr[i + 1] - 1;
+    }
+    uint32_t cur = 0;
+    bool done = !act;
+    uint32_t backoff = 0;
+    while (true) {
+        bool prog = false;
+        if (!done) {
+            const int m = min(kU, jd - j);
+            uint32_t f[kU];
+#pragma unroll
+            for (int k = 0; k < kU; ++k) f[k] = (k < m) ? ld_relaxed_u32(lvl + colidx[j + k]) : 0u;
+            int q = 0;
+#pragma unroll
+            for (int k = 0; k < kU; ++k)
+                if (q == k && k < m && f[k] != 0u) {
+                    q = k + 1;
+                    cur = max(cur, f[k]);
+                }
+            j += q;
+            prog = q > 0;
+            if (j == jd) {
+                st_relaxed_u32(lvl + i, cur + 1u);
+                done = true;
+                prog = true;
+            }
+        }
+        if (!__ballot_sync(FULL, !done)) break;
+        if (__ballot_sync(FULL, prog)) {
+            backoff = 0;
+        } else {
+            if (backoff) nanosleep_ns(backoff);
+            backoff = backoff ? min(backoff * 2u, 1024u) : 32u;
+        }
+    }
+}
+
+__global__ void k_level_finish(const uint32_t *__restrict__ lvl, int32_t *level_out,
+                               int32_t *counts, int32_t *nlevels, int32_t n) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    const bool act = i < n;
+    const int lv = act ? (int)lvl[i] - 1 : -1;
+    if (act && level_out) level_out[i] = lv;
+    // warp-aggregated histogram: lanes with the same level add once
+    const unsigned am = __ballot_sync(FULL, act);
+    if (act) {
+        const unsigned peers = __match_any_sync(am, lv);
+        if (counts && (__ffs(peers) - 1) == (threadIdx.x & 31)) atomicAdd(counts + lv, __popc(peers));
+    }
+    int mx = lv;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) mx = max(mx, __shfl_xor_sync(FULL, mx, off));
+    if ((threadIdx.x & 31) == 0 && mx >= 0) atomicMax(nlevels, mx + 1);
+}
+
+// ---------------------------------------------------------------- flag-hop microbenchmark
+//
+// Two single-thread CTAs (normally on different SMs) bounce `iters` messages.
+// Each message = an x value + its flag, published and consumed exactly as the
+// solve does it (protocol 0), or with relaxed polls + fence.acq_rel (1), or
+// value-as-flag (2).  Single-CTA probes: 3 = dependent ld.relaxed.gpu chain
+// (L2 round trip), 4 = st x + st.release flag pairs (publish cost).
+// out[0] = elapsed ns on CTA 0, out[1] = elapsed SM cycles on CTA 0.
+__global__ void k_pingpong(uint32_t *flags, double *xs, int iters, int protocol,
+                           unsigned long long *out, double *sink) {
+    if (threadIdx.x != 0) return;
+    const int me = blockIdx.x;
+    uint32_t *myf = flags + me * 32;
+    uint32_t *of = flags + (1 - me) * 32;
+    double *myx = xs + me * 16;
+    double *ox = xs + (1 - me) * 16;
+    double acc = 0.0;
+    const uint64_t t0 = globaltimer_ns();
+    const long long c0 = clock64();
+    if (protocol >= 3) {
+        if (me == 0) {
+            if (protocol == 3) {
+                uint32_t v = 0;
+                for (int k = 0; k < iters; ++k) v = ld_relaxed_u32(flags + 64 + (v & 1u));
+                acc = v;
+            } else {
+                for (int k = 1; k <= iters; ++k) {
+                    myx[0] = (double)k;
+                    st_release_u32(myf, (uint32_t)k);
+                }
+            }
+        }
+    } else {
+        for (int k = 1; k <= iters; ++k) {
+            const bool send_first = (me == 0);
+            for (int phase = 0; phase < 2; ++phase) {
+                const bool send = (phase == 0) == send_first;
+                if (send) {
+                    if (protocol == 2) {
+                        st_relaxed_f64(myx, (double)k);
+                    } else {
+                        myx[0] = (double)k;
+                        st_release_u32(myf, (uint32_t)k);
+                    }
+                } else {
+                    if (protocol == 0) {
+                        while (ld_acquire_u32(of) != (uint32_t)k) {}
+                        acc += ld_relaxed_f64(ox);
+                    } else if (protocol == 1) {
+                        while (ld_relaxed_u32(of) != (uint32_t)k) {}
+                        fence_acq_rel_gpu();
+                        acc += ld_relaxed_f64(ox);
+                    } else {
+                        double v;
+                        while ((v = ld_relaxed_f64(ox)) != (double)k) {}
+                        acc += v;
+                    }
+                }
+            }
+        }
+    }
+    const long long c1 = clock64();
+    const uint64_t t1 = globaltimer_ns();
+    if (me == 0) {
+        out[0] = t1 - t0;
+        out[1] = (unsigned long long)(c1 - c0);
+    }
+    sink[me] = acc;
+}
+
+}  // namespace sptrsv_dev

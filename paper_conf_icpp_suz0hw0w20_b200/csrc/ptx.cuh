@@ -42,6 +42,18 @@ __device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long
     return v;
 }
 
+// 16-byte vector accesses: each 8-byte element is single-copy atomic (the
+// PROTO_FUSED record relies on exactly that, never on 16-byte atomicity).
+__device__ __forceinline__ void ld_relaxed_v2_u64(const unsigned long long *p, unsigned long long &a,
+                                                  unsigned long long &b) {
+    asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+
+__device__ __forceinline__ void st_relaxed_v2_u64(unsigned long long *p, unsigned long long a,
+                                                  unsigned long long b) {
+    asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+
 __device__ __forceinline__ void st_release_u32(uint32_t *p, uint32_t v) {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -70,16 +82,18 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     return pol;
 }
 
+// volatile: the compiler must not speculate these loads out of a guarding
+// branch or ternary (a hoisted val[jd] with jd = -1 on an idle lane faults).
 __device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p, uint64_t pol) {
     int32_t v;
-    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
                  : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
 
 __device__ __forceinline__ double ld_stream_f64(const double *p, uint64_t pol) {
     double v;
-    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;"
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;"
                  : "=d"(v) : "l"(p), "l"(pol));
     return v;
 }

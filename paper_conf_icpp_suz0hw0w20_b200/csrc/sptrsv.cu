@@ -11,6 +11,7 @@
 #include <new>
 #include <vector>
 
+#include "diag.cuh"
 #include "setup.cuh"
 #include "solve.cuh"
 #include "sptrsv.h"
@@ -22,7 +23,8 @@ namespace {
 constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
 
 struct Workspace {
-    uint32_t *flags = nullptr;     // n
+    uint32_t *flags = nullptr;     // n      (PROTO_FLAGS)
+    unsigned long long *rec = nullptr;  // 2n (PROTO_FUSED, lazy)
     int32_t *indeg = nullptr;      // n
     int32_t *tasks = nullptr;      // n_tasks (PLAN_LIST only)
     SolveState *st = nullptr;      // 1
@@ -57,6 +59,8 @@ struct sptrsv_handle_s {
     uint32_t spin_limit = 1u << 24;
     int l2_window = 0;
     int stage = 1;
+    int proto = PROTO_FLAGS;
+    int local = 1;
     // bookkeeping
     uint32_t solves = 0;
     uint32_t since_reset = 0;
@@ -73,27 +77,41 @@ struct sptrsv_handle_s {
 
 namespace {
 
-size_t stage_smem_bytes(int cta_threads) {
-    return (size_t)(cta_threads / 32) * kStageCap * (sizeof(double) + sizeof(int32_t));
+// dynamic smem: x copy [warps*32] doubles, then (if staging) [warps][kStageCap] doubles + ints
+size_t solve_smem_bytes(int cta_threads, int stage) {
+    const size_t w = (size_t)(cta_threads / 32);
+    return w * 32 * sizeof(double) + (stage ? w * kStageCap * (sizeof(double) + sizeof(int32_t)) : 0);
+}
+
+typedef void (*solve_fn)(SolveParams);
+solve_fn solve_kernel(int plan, int proto) {
+    static const solve_fn tab[3][2] = {
+        {k_solve<PLAN_THREAD, PROTO_FLAGS>, k_solve<PLAN_THREAD, PROTO_FUSED>},
+        {k_solve<PLAN_WARP, PROTO_FLAGS>, k_solve<PLAN_WARP, PROTO_FUSED>},
+        {k_solve<PLAN_LIST, PROTO_FLAGS>, k_solve<PLAN_LIST, PROTO_FUSED>},
+    };
+    return tab[plan][proto];
 }
 
 int set_kernel_attrs() {
     static int done = 0;
     static int rc = SPTRSV_OK;
     if (done) return rc;
-    const int maxb = (int)stage_smem_bytes(1024);
-    if (cudaFuncSetAttribute(k_solve<PLAN_THREAD>, cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) != cudaSuccess ||
-        cudaFuncSetAttribute(k_solve<PLAN_WARP>, cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) != cudaSuccess ||
-        cudaFuncSetAttribute(k_solve<PLAN_LIST>, cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) != cudaSuccess) {
-        (void)cudaGetLastError();
-        rc = SPTRSV_ERR_CUDA;
-    }
+    const int maxb = (int)solve_smem_bytes(1024, 1);
+    for (int pl = 0; pl < 3; ++pl)
+        for (int pr = 0; pr < 2; ++pr)
+            if (cudaFuncSetAttribute(solve_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) !=
+                cudaSuccess) {
+                (void)cudaGetLastError();
+                rc = SPTRSV_ERR_CUDA;
+            }
     done = 1;
     return rc;
 }
 
 void free_ws(Workspace &w) {
     cudaFree(w.flags);
+    cudaFree(w.rec);
     cudaFree(w.indeg);
     cudaFree(w.tasks);
     cudaFree(w.st);
@@ -176,8 +194,9 @@ int build_plan(sptrsv_handle_s *h) {
 }
 
 int reset_state(sptrsv_handle_s *h, cudaStream_t s) {
-    // flags := 0, epoch := 0x01010101 (any nonzero value works), counters := 0
+    // flags / records := 0, epoch := 0x01010101 (any nonzero value works), counters := 0
     CK(cudaMemsetAsync(h->ws.flags, 0, sizeof(uint32_t) * (size_t)(h->n > 0 ? h->n : 1), s));
+    if (h->ws.rec) CK(cudaMemsetAsync(h->ws.rec, 0, 16 * (size_t)(h->n > 0 ? h->n : 1), s));
     CK(cudaMemsetAsync(h->ws.st, 0, sizeof(SolveState), s));
     CK(cudaMemsetAsync(&h->ws.st->epoch.v, 1, sizeof(uint32_t), s));
     h->since_reset = 0;
@@ -313,6 +332,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.b = b;
     p.x = x;
     p.flags = h->ws.flags;
+    p.rec = h->ws.rec;
     p.tasks = h->ws.tasks;
     p.st = h->ws.st;
     p.n = h->n;
@@ -321,11 +341,12 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.backoff_max = h->backoff_max;
     p.spin_limit = h->spin_limit;
     p.stage = h->stage;
+    p.local = h->local;
     const int warps = h->cta_threads / 32;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
     cfg.blockDim = dim3((unsigned)h->cta_threads);
-    cfg.dynamicSmemBytes = h->stage && h->plan != PLAN_WARP ? stage_smem_bytes(h->cta_threads) : 0;
+    cfg.dynamicSmemBytes = solve_smem_bytes(h->cta_threads, h->stage && h->plan != PLAN_WARP);
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
     cfg.numAttrs = 0;
@@ -339,12 +360,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
         cfg.attrs = attr;
         cfg.numAttrs = 1;
     }
-    cudaError_t e;
-    switch (h->plan) {
-        case PLAN_THREAD: e = cudaLaunchKernelEx(&cfg, k_solve<PLAN_THREAD>, p); break;
-        case PLAN_WARP: e = cudaLaunchKernelEx(&cfg, k_solve<PLAN_WARP>, p); break;
-        default: e = cudaLaunchKernelEx(&cfg, k_solve<PLAN_LIST>, p); break;
-    }
+    const cudaError_t e = cudaLaunchKernelEx(&cfg, solve_kernel(h->plan, h->proto), p);
     if (e != cudaSuccess) {
         (void)cudaGetLastError();
         return SPTRSV_ERR_CUDA;
@@ -437,6 +453,22 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->stage = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_PROTOCOL:
+            if (value != PROTO_FLAGS && value != PROTO_FUSED) return SPTRSV_ERR_INVALID_ARG;
+            if (value == PROTO_FUSED && !h->ws.rec && h->n > 0) {
+                // records are epoch-tagged like the flags: zeroed once, valid for any later epoch
+                if (cudaMalloc(&h->ws.rec, 16 * (size_t)h->n) != cudaSuccess) {
+                    (void)cudaGetLastError();
+                    return SPTRSV_ERR_ALLOC;
+                }
+                CK(cudaMemset(h->ws.rec, 0, 16 * (size_t)h->n));
+            }
+            h->proto = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_LOCAL:
+            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            h->local = (int)value;
+            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -453,6 +485,8 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_SPIN_LIMIT: *value = h->spin_limit; return SPTRSV_OK;
         case SPTRSV_OPT_L2_WINDOW: *value = h->l2_window; return SPTRSV_OK;
         case SPTRSV_OPT_STAGE_SMEM: *value = h->stage; return SPTRSV_OK;
+        case SPTRSV_OPT_PROTOCOL: *value = h->proto; return SPTRSV_OK;
+        case SPTRSV_OPT_LOCAL: *value = h->local; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }
@@ -519,15 +553,15 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
     return SPTRSV_OK;
 }
 
-int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop) {
-    if (iters <= 0 || protocol < 0 || protocol > 2 || !ns_per_hop) return SPTRSV_ERR_INVALID_ARG;
+int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop, double *sm_mhz) {
+    if (iters <= 0 || protocol < 0 || protocol > 4 || !ns_per_hop) return SPTRSV_ERR_INVALID_ARG;
     uint32_t *flags = nullptr;
     double *xs = nullptr, *sink = nullptr;
     unsigned long long *ns = nullptr;
     int rc = SPTRSV_OK;
     do {
         if (cudaMalloc(&flags, 256) != cudaSuccess || cudaMalloc(&xs, 256) != cudaSuccess ||
-            cudaMalloc(&sink, 16) != cudaSuccess || cudaMalloc(&ns, 8) != cudaSuccess) {
+            cudaMalloc(&sink, 16) != cudaSuccess || cudaMalloc(&ns, 16) != cudaSuccess) {
             rc = SPTRSV_ERR_ALLOC;
             break;
         }
@@ -536,13 +570,15 @@ int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop) {
             break;
         }
         k_pingpong<<<2, 32>>>(flags, xs, iters, protocol, ns, sink);
-        unsigned long long t = 0;
+        unsigned long long t[2] = {0, 0};
         if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess ||
-            cudaMemcpy(&t, ns, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            cudaMemcpy(t, ns, 16, cudaMemcpyDeviceToHost) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
-        *ns_per_hop = (double)t / (2.0 * iters);
+        // hops: 2 per iteration for the ping-pong protocols, 1 per iteration for the probes
+        *ns_per_hop = (double)t[0] / ((protocol >= 3 ? 1.0 : 2.0) * iters);
+        if (sm_mhz) *sm_mhz = t[0] ? (double)t[1] / (double)t[0] * 1e3 : 0.0;
     } while (0);
     (void)cudaGetLastError();
     cudaFree(flags);

@@ -27,28 +27,31 @@ def _run(s, **opt):
         return x1, x.cpu().numpy(), h.info()
 
 
-def test_c2_full():
+@pytest.mark.parametrize("proto", [0, 1])
+def test_c2_full(proto):
     s = synth.gen_c2()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x1, x2, info = _run(s)
+    x1, x2, info = _run(s, protocol=proto)
     assert info["n_warp_rows"] == 0  # 2.8 nnz/row -> thread level everywhere
     assert np.array_equal(x1, ref) and np.array_equal(x2, ref)
 
 
-def test_c3_full_ones_and_random():
+@pytest.mark.parametrize("proto", [0, 1])
+def test_c3_full_ones_and_random(proto):
     s = synth.gen_c3(ones=True)
-    x1, x2, _ = _run(s)
+    x1, x2, _ = _run(s, protocol=proto)
     assert np.array_equal(x1, np.ones(s.n)) and np.array_equal(x2, np.ones(s.n))
     s = synth.gen_c3()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x1, _, _ = _run(s)
+    x1, _, _ = _run(s, protocol=proto)
     assert np.array_equal(x1, ref)
 
 
-def test_c4_full_auto_picks_warp():
+@pytest.mark.parametrize("proto", [0, 1])
+def test_c4_full_auto_picks_warp(proto):
     s = synth.gen_c4()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x1, x2, info = _run(s)
+    x1, x2, info = _run(s, protocol=proto)
     assert info["n_thread_groups"] <= 32  # only the diagonal-only level-0 groups stay thread level
     err = np.max(np.abs(x1 - ref) / np.abs(ref))
     assert err <= TOL, err
@@ -62,8 +65,9 @@ def test_c5_system_full():
     assert np.array_equal(x1, ref)
 
 
-def test_chain_full_closed_form():
+@pytest.mark.parametrize("proto", [0, 1])
+def test_chain_full_closed_form(proto):
     s = synth.gen_chain()
-    x1, _, _ = _run(s)
+    x1, _, _ = _run(s, protocol=proto)
     want = np.array([1.0 - 2.0 ** -(i + 1) if i <= 52 else 1.0 for i in range(s.n)])
     assert np.array_equal(x1, want)

@@ -47,16 +47,19 @@ def relerr(a, ref):
 
 
 MODES = [0, 1, 2]
+PROTOS = [0, 1]  # 0 FLAGS (release/acquire), 1 FUSED (epoch-tagged value records)
 
 
 # ------------------------------------------------------------------ small, many tiles + ragged tails
 
 @pytest.mark.parametrize("n", [1, 2, 31, 32, 33, 63, 65, 257, 1000, 4099])
 @pytest.mark.parametrize("mode", MODES)
-def test_random_small_sizes(cap, n, mode):
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("local", [0, 1])
+def test_random_small_sizes(cap, n, mode, proto, local):
     s = synth.gen_random_lower(n, 4, seed=n)
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x, info = gpu_solve(cap, s, mode)
+    x, info = gpu_solve(cap, s, mode, protocol=proto, local=local)
     if mode == 1:
         assert np.array_equal(x, ref)
     else:
@@ -96,13 +99,14 @@ def test_closed_forms_bit_exact(cap, mode):
 
 
 @pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("gen", ["c1", "c2s", "c2is", "c4s", "dense"])
-def test_exact_integer_systems_bit_exact(cap, mode, gen):
+def test_exact_integer_systems_bit_exact(cap, mode, proto, gen):
     base = {"c1": lambda: synth.gen_c1(), "c2s": lambda: synth.gen_c2(n=50_000),
             "c2is": lambda: synth.gen_c2i(n=50_000), "c4s": lambda: synth.gen_c4(n=20_000, nlevels=100),
             "dense": lambda: synth.gen_dense_lower(200)}[gen]()
     s = synth.integerize(base)
-    x, _ = gpu_solve(cap, s, mode)
+    x, _ = gpu_solve(cap, s, mode, protocol=proto)
     assert np.array_equal(x, s.x_true)
 
 
@@ -110,20 +114,23 @@ def test_exact_integer_systems_bit_exact(cap, mode, gen):
 
 @pytest.mark.parametrize("cta", [128, 256, 512, 1024])
 @pytest.mark.parametrize("stage", [0, 1])
-def test_interleaved_levels_stress(cap, cta, stage):
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("local", [0, 1])
+def test_interleaved_levels_stress(cap, cta, stage, proto, local):
     """c2i: half the dependencies inside the same warp (Challenge 1)."""
     s = synth.gen_c2i(n=200_000)
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x, _ = gpu_solve(cap, s, 0, cta_threads=cta, stage_smem=stage)
+    x, _ = gpu_solve(cap, s, 0, cta_threads=cta, stage_smem=stage, protocol=proto, local=local)
     assert np.array_equal(x, ref)
 
 
-def test_back_to_back_solves_and_epoch(cap):
+@pytest.mark.parametrize("proto", PROTOS)
+def test_back_to_back_solves_and_epoch(cap, proto):
     """Several solves with different b through one handle (epoch flags must reset)."""
     s = synth.gen_c2(n=100_000)
     rp, ci, v, _ = dev_csr(s)
     rng = np.random.default_rng(0)
-    with cap.analyse(rp, ci, v) as h:
+    with cap.analyse(rp, ci, v, protocol=proto) as h:
         for it in range(20):
             bb = rng.uniform(-1, 1, s.n)
             x = torch.full((s.n,), float("nan"), dtype=torch.float64, device="cuda:0")
@@ -133,11 +140,12 @@ def test_back_to_back_solves_and_epoch(cap):
         assert h.info()["solves"] == 20
 
 
-def test_many_solves_on_side_stream_and_graph_capture(cap):
+@pytest.mark.parametrize("proto", PROTOS)
+def test_many_solves_on_side_stream_and_graph_capture(cap, proto):
     s = synth.gen_c1()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     rp, ci, v, b = dev_csr(s)
-    with cap.analyse(rp, ci, v) as h:
+    with cap.analyse(rp, ci, v, protocol=proto) as h:
         st = torch.cuda.Stream()
         x = torch.empty_like(b)
         with torch.cuda.stream(st):
@@ -232,7 +240,20 @@ def test_indegree_and_levels_bit_exact(cap, gen):
         assert np.array_equal(counts.cpu().numpy(), ocounts)
 
 
+def test_protocol_switch_on_one_handle(cap):
+    s = synth.gen_c2i(n=50_000)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        for proto in (0, 1, 0, 1):
+            h.set_option(cap.OPT_PROTOCOL, proto)
+            x = torch.full_like(b, float("nan"))
+            h.solve(b, x)
+            h.check()
+            assert np.array_equal(x.cpu().numpy(), ref)
+
+
 def test_flag_latency_runs(cap):
-    for proto in (0, 1, 2):
+    for proto in (0, 1, 2, 3, 4):
         t = cap.flag_latency(2000, proto)
         assert 10.0 < t < 100_000.0
