@@ -160,6 +160,11 @@ int sptrsv_get_indegree(sptrsv_handle_t h, int32_t *out_dev, sptrsv_stream_t str
 int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev,
                   int32_t *nlevels_host, sptrsv_stream_t stream);
 
+/* sptrsv_set_trace -- diagnostic: while trace_dev (device uint64[n]) is set,
+ * every solve writes the %globaltimer (ns) at which x_i was published into
+ * trace_dev[i] -- the critical path, row by row.  NULL turns it off. */
+int sptrsv_set_trace(sptrsv_handle_t h, uint64_t *trace_dev);
+
 /* sptrsv_check -- synchronises `stream`, returns SPTRSV_ERR_TIMEOUT if the
  * watchdog fired in any solve since the last check (and clears it), else OK. */
 int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream);

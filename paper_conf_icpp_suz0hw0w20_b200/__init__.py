@@ -119,6 +119,18 @@ class Handle:
                                     _stream_ptr(stream)), "sptrsv_levels")
         return lv, int(nl.value), counts[: nl.value]
 
+    def trace(self, b, x=None, stream=None):
+        """Diagnostic solve that records the publish time (ns, %globaltimer) of every x_i."""
+        import torch
+        tr = torch.zeros(self.n, dtype=torch.int64, device=self.device)
+        check(lib.sptrsv_set_trace(self._h, tr.data_ptr()), "sptrsv_set_trace")
+        try:
+            x = self.solve(b, x, stream)
+            self.check(stream)
+        finally:
+            check(lib.sptrsv_set_trace(self._h, None), "sptrsv_set_trace")
+        return x, tr
+
     def info(self) -> dict:
         inf = _lib.sptrsv_info()
         check(lib.sptrsv_get_info(self._h, ctypes.byref(inf)), "sptrsv_get_info")

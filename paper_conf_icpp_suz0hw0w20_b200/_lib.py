@@ -76,6 +76,7 @@ EXPORTS = {
     "sptrsv_get_indegree": (ctypes.c_int, [_h, _p, _p]),
     "sptrsv_levels": (ctypes.c_int, [_h, _p, _p, ctypes.POINTER(_i32), _p]),
     "sptrsv_check": (ctypes.c_int, [_h, _p]),
+    "sptrsv_set_trace": (ctypes.c_int, [_h, _p]),
     "sptrsv_flag_latency": (ctypes.c_int, [_i32, _i32, ctypes.POINTER(ctypes.c_double),
                                            ctypes.POINTER(ctypes.c_double)]),
     "sptrsv_strerror": (ctypes.c_char_p, [ctypes.c_int]),

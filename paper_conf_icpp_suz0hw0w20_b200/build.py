@@ -1,6 +1,7 @@
 """Build libsptrsv.so in-tree for sm_100a (nvcc; no JIT cache, no torch extension).
 
-    python -m paper_conf_icpp_suz0hw0w20_b200.build          # or __graft_entry__.build()
+    python paper_conf_icpp_suz0hw0w20_b200/build.py          # or __graft_entry__.build()
+(run it by path: importing the package loads the library this script builds)
 """
 from __future__ import annotations
 

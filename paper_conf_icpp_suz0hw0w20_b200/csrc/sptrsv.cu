@@ -54,13 +54,14 @@ struct sptrsv_handle_s {
     int mode = 0;
     int threshold = 16;
     int cta_threads = 256;
-    uint32_t backoff_min = 0;
-    uint32_t backoff_max = 256;
+    uint32_t backoff_min = 32;
+    uint32_t backoff_max = 512;
     uint32_t spin_limit = 1u << 24;
     int l2_window = 0;
     int stage = 1;
     int proto = PROTO_FLAGS;
     int local = 1;
+    unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
     uint32_t since_reset = 0;
@@ -342,6 +343,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.spin_limit = h->spin_limit;
     p.stage = h->stage;
     p.local = h->local;
+    p.trace = h->trace;
     const int warps = h->cta_threads / 32;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
@@ -537,6 +539,12 @@ int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev, in
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(nlevels_host, d_nlev, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    return SPTRSV_OK;
+}
+
+int sptrsv_set_trace(sptrsv_handle_t h, uint64_t *trace_dev) {
+    if (!h) return SPTRSV_ERR_INVALID_ARG;
+    h->trace = reinterpret_cast<unsigned long long *>(trace_dev);
     return SPTRSV_OK;
 }
 

@@ -19,8 +19,8 @@ def _declared():
 
 @pytest.fixture(scope="module")
 def libpath():
-    from paper_conf_icpp_suz0hw0w20_b200 import build
-    return build.build()
+    import __graft_entry__
+    return __graft_entry__._load_builder().build()
 
 
 def test_header_declares_the_north_star_entry_points():
