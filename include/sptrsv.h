@@ -177,7 +177,8 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream);
  * + relaxed x load (the solve's protocol), 1 = relaxed poll + fence.acq_rel,
  * 2 = value-as-flag (x polled directly; ablation only); single-CTA probes:
  * 3 = dependent ld.relaxed.gpu chain (ns per L2 round trip), 4 = st x +
- * st.release flag pairs (ns per publish).  sm_mhz (host, may be NULL)
+ * st.release flag pairs (ns per publish), 5 = dependent fp64 IEEE divisions,
+ * 6 = dependent DFMA, 7 = shared-memory store->load round trip.  sm_mhz (host, may be NULL)
  * receives the SM clock seen during the probe (clock64 / globaltimer).
  * Synchronous.
  */

@@ -103,7 +103,23 @@ __global__ void k_pingpong(uint32_t *flags, double *xs, int iters, int protocol,
     const long long c0 = clock64();
     if (protocol >= 3) {
         if (me == 0) {
-            if (protocol == 3) {
+            if (protocol == 5) {  // dependent IEEE fp64 divisions
+                double v = 1.5, d = 1.0000001;
+                for (int k = 0; k < iters; ++k) v = __ddiv_rn(v + 1.0, d);
+                acc = v;
+            } else if (protocol == 6) {  // dependent DFMA chain
+                double v = 1.5;
+                for (int k = 0; k < iters; ++k) v = fma(v, 0.999999, 1e-7);
+                acc = v;
+            } else if (protocol == 7) {  // shared-memory store -> volatile load round trip
+                __shared__ unsigned long long sm[64];
+                unsigned long long v = 0;
+                for (int k = 0; k < iters; ++k) {
+                    asm volatile("st.volatile.shared.u64 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(sm + (v & 1))), "l"(v + 1) : "memory");
+                    asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"((unsigned)__cvta_generic_to_shared(sm + (v & 1))) : "memory");
+                }
+                acc = (double)v;
+            } else if (protocol == 3) {
                 uint32_t v = 0;
                 for (int k = 0; k < iters; ++k) v = ld_relaxed_u32(flags + 64 + (v & 1u));
                 acc = v;

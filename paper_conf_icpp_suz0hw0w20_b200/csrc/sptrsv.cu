@@ -562,7 +562,7 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
 }
 
 int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop, double *sm_mhz) {
-    if (iters <= 0 || protocol < 0 || protocol > 4 || !ns_per_hop) return SPTRSV_ERR_INVALID_ARG;
+    if (iters <= 0 || protocol < 0 || protocol > 7 || !ns_per_hop) return SPTRSV_ERR_INVALID_ARG;
     uint32_t *flags = nullptr;
     double *xs = nullptr, *sink = nullptr;
     unsigned long long *ns = nullptr;

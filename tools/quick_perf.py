@@ -9,7 +9,7 @@ PEAK = 6539.9e9
 cfgs = sys.argv[1].split(",") if len(sys.argv) > 1 else ["c1", "c2", "c3", "c4", "chain"]
 opts = json.loads(sys.argv[2]) if len(sys.argv) > 2 else {}
 flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
-for p in (0, 1, 2, 3, 4):
+for p in (0, 1, 2, 3, 4, 5, 6, 7):
     print("flag_latency proto", p, "%.1f ns @ %.0f MHz" % cap.flag_latency(20000, p, True), flush=True)
 for name in cfgs:
     s = synth.make(name)
