@@ -54,8 +54,8 @@ struct sptrsv_handle_s {
     int mode = 0;
     int threshold = 16;
     int cta_threads = 256;
-    uint32_t backoff_min = 32;
-    uint32_t backoff_max = 512;
+    uint32_t backoff_min = 0;
+    uint32_t backoff_max = 256;
     uint32_t spin_limit = 1u << 24;
     int l2_window = 0;
     int stage = 1;

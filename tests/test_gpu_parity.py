@@ -98,6 +98,32 @@ def test_closed_forms_bit_exact(cap, mode):
     assert np.array_equal(x, want)
 
 
+@pytest.mark.parametrize("mode", [1, 2])
+def test_division_bit_exact_wide_range(cap, mode):
+    """x_i = b_i / d_i over the whole double range + specials: the kernel's divide (Markstein
+    step + exactness test, __ddiv_rn fallback) must equal IEEE division bit for bit."""
+    rng = np.random.default_rng(123)
+    n = 1 << 21
+    def wide(m):
+        e = rng.integers(-1060, 1030, size=m)
+        return np.ldexp(rng.uniform(1.0, 2.0, size=m), e) * rng.choice([-1.0, 1.0], size=m)
+    d, b = wide(n), wide(n)
+    k = n // 4  # a quarter in the common range (fast path)
+    d[:k] = rng.uniform(0.5, 4.0, size=k)
+    b[:k] = rng.uniform(-3.0, 3.0, size=k)
+    sp = np.array([0.0, -0.0, np.inf, -np.inf, np.nan, 5e-324, -5e-324, 2.2250738585072014e-308,
+                   1.7976931348623157e308, 1.0, -1.0, 3.0])
+    b[k:k + sp.size * sp.size] = np.repeat(sp, sp.size)
+    d[k:k + sp.size * sp.size] = np.tile(sp, sp.size)
+    d[d == 0.0] = 1.0  # a zero diagonal is rejected by analyse
+    with np.errstate(all="ignore"):
+        want = b / d
+    s = synth.CSRSystem("div", n, np.arange(n + 1, dtype=np.int32), np.arange(n, dtype=np.int32), d, b, None, {})
+    x, _ = gpu_solve(cap, s, mode)
+    same = (x.view(np.int64) == want.view(np.int64)) | (np.isnan(x) & np.isnan(want))
+    assert same.all(), (np.nonzero(~same)[0][:10], x[~same][:5], want[~same][:5])
+
+
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("gen", ["c1", "c2s", "c2is", "c4s", "dense"])
