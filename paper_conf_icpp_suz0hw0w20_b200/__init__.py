@@ -168,7 +168,9 @@ def analyse(rowptr, colidx, val, **options) -> Handle:
     keys = {"mode": OPT_MODE, "warp_threshold": OPT_WARP_THRESHOLD, "cta_threads": OPT_CTA_THREADS,
             "backoff_min_ns": OPT_BACKOFF_MIN_NS, "backoff_max_ns": OPT_BACKOFF_MAX_NS,
             "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
-            "protocol": OPT_PROTOCOL, "local": OPT_LOCAL}
+            "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
+            "pipe_stages": _lib.OPT_PIPE_STAGES, "pipe_batch": _lib.OPT_PIPE_BATCH,
+            "pipe_entries": _lib.OPT_PIPE_ENTRIES}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

@@ -43,6 +43,11 @@ OPT_L2_WINDOW = 7
 OPT_STAGE_SMEM = 8
 OPT_PROTOCOL = 9
 OPT_LOCAL = 10
+OPT_ENGINE = 11
+OPT_PIPE_STAGES = 12
+OPT_PIPE_BATCH = 13
+OPT_PIPE_ENTRIES = 14
+ENGINE_ONESHOT, ENGINE_PIPE = 0, 1
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
 

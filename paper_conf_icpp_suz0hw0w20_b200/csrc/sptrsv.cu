@@ -14,6 +14,7 @@
 #include "diag.cuh"
 #include "setup.cuh"
 #include "solve.cuh"
+#include "solve_pipe.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -61,6 +62,12 @@ struct sptrsv_handle_s {
     int stage = 1;
     int proto = PROTO_FLAGS;
     int local = 1;
+    int engine = 1;         // 0 one-shot (k_solve), 1 pipelined (k_solve_pipe)
+    int pipe_stages = 3;
+    int pipe_batch = 2;
+    int pipe_entries = 0;   // 0 = 4 per row of a round
+    int grid_cache_key = -1;
+    int grid_cache = 0;
     unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
@@ -94,18 +101,55 @@ solve_fn solve_kernel(int plan, int proto) {
     return tab[plan][proto];
 }
 
+typedef void (*pipe_fn)(SolveParams, PipeGeom);
+pipe_fn pipe_kernel(int plan, int proto) {
+    static const pipe_fn tab[3][2] = {
+        {k_solve_pipe<PLAN_THREAD, PROTO_FLAGS>, k_solve_pipe<PLAN_THREAD, PROTO_FUSED>},
+        {k_solve_pipe<PLAN_WARP, PROTO_FLAGS>, k_solve_pipe<PLAN_WARP, PROTO_FUSED>},
+        {k_solve_pipe<PLAN_LIST, PROTO_FLAGS>, k_solve_pipe<PLAN_LIST, PROTO_FUSED>},
+    };
+    return tab[plan][proto];
+}
+
+int round16(int b) { return (b + 15) & ~15; }
+
+PipeGeom pipe_geom(const sptrsv_handle_s *h) {
+    PipeGeom g;
+    g.W = h->cta_threads / 32 - 1;
+    g.S = h->pipe_stages;
+    g.B = h->pipe_batch;
+    g.RB = 32 * g.W;
+    g.E = h->pipe_entries > 0 ? h->pipe_entries : 4 * g.RB;
+    int off = 64;  // StageHdr
+    g.off_rp = off;
+    off += round16(4 * (g.RB + 1) + 32);
+    g.off_b = off;
+    off += round16(8 * g.RB + 32);
+    g.off_col = off;
+    off += round16(4 * g.E + 32);
+    g.off_val = off;
+    off += round16(8 * g.E + 32);
+    g.off_xc = off;
+    off += round16(8 * g.RB);
+    g.stage_bytes = round16(off);
+    return g;
+}
+
 int set_kernel_attrs() {
     static int done = 0;
     static int rc = SPTRSV_OK;
     if (done) return rc;
     const int maxb = (int)solve_smem_bytes(1024, 1);
     for (int pl = 0; pl < 3; ++pl)
-        for (int pr = 0; pr < 2; ++pr)
+        for (int pr = 0; pr < 2; ++pr) {
             if (cudaFuncSetAttribute(solve_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) !=
-                cudaSuccess) {
+                    cudaSuccess ||
+                cudaFuncSetAttribute(pipe_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     227 * 1024) != cudaSuccess) {
                 (void)cudaGetLastError();
                 rc = SPTRSV_ERR_CUDA;
             }
+        }
     done = 1;
     return rc;
 }
@@ -344,6 +388,41 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.stage = h->stage;
     p.local = h->local;
     p.trace = h->trace;
+    p.nnz = h->nnz;
+    const bool aligned = ((((uintptr_t)h->rowptr) | ((uintptr_t)h->colidx) | ((uintptr_t)h->val) | ((uintptr_t)b)) & 15) == 0;
+    if (h->engine == 1 && aligned && h->cta_threads >= 64) {
+        const PipeGeom g = pipe_geom(h);
+        const size_t smem = (size_t)g.S * g.stage_bytes;
+        const int key = (h->plan * 2 + h->proto) * 4096 + h->cta_threads + (int)(smem >> 4) * 8192;
+        if (key != h->grid_cache_key) {
+            int per_sm = 0, sms = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pipe_kernel(h->plan, h->proto),
+                                                              h->cta_threads, smem) != cudaSuccess ||
+                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device) != cudaSuccess) {
+                (void)cudaGetLastError();
+                return SPTRSV_ERR_CUDA;
+            }
+            if (per_sm < 1) return SPTRSV_ERR_INVALID_ARG;  // ring does not fit: fewer stages / threads
+            h->grid_cache = per_sm * sms;
+            h->grid_cache_key = key;
+        }
+        const int rounds = (h->n_tasks + g.W - 1) / g.W;
+        const int grid = rounds < h->grid_cache ? (rounds > 0 ? rounds : 1) : h->grid_cache;
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)grid);
+        cfg.blockDim = dim3((unsigned)h->cta_threads);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = s;
+        cfg.numAttrs = 0;
+        const cudaError_t e = cudaLaunchKernelEx(&cfg, pipe_kernel(h->plan, h->proto), p, g);
+        if (e != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_CUDA;
+        }
+        h->solves++;
+        h->since_reset++;
+        return SPTRSV_OK;
+    }
     const int warps = h->cta_threads / 32;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
@@ -471,6 +550,22 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->local = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_ENGINE:
+            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            h->engine = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_PIPE_STAGES:
+            if (value < 2 || value > 8) return SPTRSV_ERR_INVALID_ARG;
+            h->pipe_stages = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_PIPE_BATCH:
+            if (value < 1 || value > 32) return SPTRSV_ERR_INVALID_ARG;
+            h->pipe_batch = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_PIPE_ENTRIES:
+            if (value < 0 || value > (1 << 16)) return SPTRSV_ERR_INVALID_ARG;
+            h->pipe_entries = (int)value;
+            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -489,6 +584,10 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_STAGE_SMEM: *value = h->stage; return SPTRSV_OK;
         case SPTRSV_OPT_PROTOCOL: *value = h->proto; return SPTRSV_OK;
         case SPTRSV_OPT_LOCAL: *value = h->local; return SPTRSV_OK;
+        case SPTRSV_OPT_ENGINE: *value = h->engine; return SPTRSV_OK;
+        case SPTRSV_OPT_PIPE_STAGES: *value = h->pipe_stages; return SPTRSV_OK;
+        case SPTRSV_OPT_PIPE_BATCH: *value = h->pipe_batch; return SPTRSV_OK;
+        case SPTRSV_OPT_PIPE_ENTRIES: *value = h->pipe_entries; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }

@@ -48,6 +48,7 @@ def relerr(a, ref):
 
 MODES = [0, 1, 2]
 PROTOS = [0, 1]  # 0 FLAGS (release/acquire), 1 FUSED (epoch-tagged value records)
+ENGINES = [0, 1]  # 0 one-shot k_solve, 1 pipelined k_solve_pipe (TMA ring + loader warp)
 
 
 # ------------------------------------------------------------------ small, many tiles + ragged tails
@@ -56,10 +57,11 @@ PROTOS = [0, 1]  # 0 FLAGS (release/acquire), 1 FUSED (epoch-tagged value record
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("local", [0, 1])
-def test_random_small_sizes(cap, n, mode, proto, local):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_random_small_sizes(cap, n, mode, proto, local, engine):
     s = synth.gen_random_lower(n, 4, seed=n)
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x, info = gpu_solve(cap, s, mode, protocol=proto, local=local)
+    x, info = gpu_solve(cap, s, mode, protocol=proto, local=local, engine=engine)
     if mode == 1:
         assert np.array_equal(x, ref)
     else:
@@ -126,13 +128,14 @@ def test_division_bit_exact_wide_range(cap, mode):
 
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("engine", ENGINES)
 @pytest.mark.parametrize("gen", ["c1", "c2s", "c2is", "c4s", "dense"])
-def test_exact_integer_systems_bit_exact(cap, mode, proto, gen):
+def test_exact_integer_systems_bit_exact(cap, mode, proto, engine, gen):
     base = {"c1": lambda: synth.gen_c1(), "c2s": lambda: synth.gen_c2(n=50_000),
             "c2is": lambda: synth.gen_c2i(n=50_000), "c4s": lambda: synth.gen_c4(n=20_000, nlevels=100),
             "dense": lambda: synth.gen_dense_lower(200)}[gen]()
     s = synth.integerize(base)
-    x, _ = gpu_solve(cap, s, mode, protocol=proto)
+    x, _ = gpu_solve(cap, s, mode, protocol=proto, engine=engine)
     assert np.array_equal(x, s.x_true)
 
 
@@ -142,21 +145,23 @@ def test_exact_integer_systems_bit_exact(cap, mode, proto, gen):
 @pytest.mark.parametrize("stage", [0, 1])
 @pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("local", [0, 1])
-def test_interleaved_levels_stress(cap, cta, stage, proto, local):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_interleaved_levels_stress(cap, cta, stage, proto, local, engine):
     """c2i: half the dependencies inside the same warp (Challenge 1)."""
     s = synth.gen_c2i(n=200_000)
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x, _ = gpu_solve(cap, s, 0, cta_threads=cta, stage_smem=stage, protocol=proto, local=local)
+    x, _ = gpu_solve(cap, s, 0, cta_threads=cta, stage_smem=stage, protocol=proto, local=local, engine=engine)
     assert np.array_equal(x, ref)
 
 
 @pytest.mark.parametrize("proto", PROTOS)
-def test_back_to_back_solves_and_epoch(cap, proto):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_back_to_back_solves_and_epoch(cap, proto, engine):
     """Several solves with different b through one handle (epoch flags must reset)."""
     s = synth.gen_c2(n=100_000)
     rp, ci, v, _ = dev_csr(s)
     rng = np.random.default_rng(0)
-    with cap.analyse(rp, ci, v, protocol=proto) as h:
+    with cap.analyse(rp, ci, v, protocol=proto, engine=engine) as h:
         for it in range(20):
             bb = rng.uniform(-1, 1, s.n)
             x = torch.full((s.n,), float("nan"), dtype=torch.float64, device="cuda:0")
@@ -167,11 +172,12 @@ def test_back_to_back_solves_and_epoch(cap, proto):
 
 
 @pytest.mark.parametrize("proto", PROTOS)
-def test_many_solves_on_side_stream_and_graph_capture(cap, proto):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_many_solves_on_side_stream_and_graph_capture(cap, proto, engine):
     s = synth.gen_c1()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     rp, ci, v, b = dev_csr(s)
-    with cap.analyse(rp, ci, v, protocol=proto) as h:
+    with cap.analyse(rp, ci, v, protocol=proto, engine=engine) as h:
         st = torch.cuda.Stream()
         x = torch.empty_like(b)
         with torch.cuda.stream(st):
@@ -264,6 +270,35 @@ def test_indegree_and_levels_bit_exact(cap, gen):
         assert np.array_equal(lv.cpu().numpy(), olv)
         assert nl == onl
         assert np.array_equal(counts.cpu().numpy(), ocounts)
+
+
+@pytest.mark.parametrize("stages,batch,entries,cta", [(2, 1, 0, 64), (3, 2, 0, 256), (4, 4, 64, 256),
+                                                      (8, 32, 0, 1024), (2, 3, 100, 512)])
+def test_pipe_geometry_variants(cap, stages, batch, entries, cta):
+    """Ring depth, ticket batch, stage capacity (tiny -> direct global reads) and CTA size."""
+    for gen in (lambda: synth.gen_c2i(n=60_000), lambda: synth.gen_c4(n=8_000, nlevels=40),
+                lambda: synth.gen_random_lower(5000, 6, seed=9)):
+        s = gen()
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        for proto in PROTOS:
+            x, _ = gpu_solve(cap, s, 0, engine=1, pipe_stages=stages, pipe_batch=batch, pipe_entries=entries,
+                             cta_threads=cta, protocol=proto)
+            assert relerr(x, ref) <= TOL
+
+
+def test_pipe_unaligned_b_falls_back(cap):
+    """b at an 8-byte (not 16-byte) offset: the TMA ring needs 16-byte alignment -> one-shot engine."""
+    s = synth.gen_c2(n=20_000)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, _ = dev_csr(s)
+    store = torch.zeros(s.n + 1, dtype=torch.float64, device="cuda:0")
+    store[1:] = torch.from_numpy(s.b).cuda()
+    b_off = store[1:]
+    with cap.analyse(rp, ci, v, engine=1) as h:
+        x = torch.full_like(b_off, float("nan"))
+        h.solve(b_off, x)
+        h.check()
+        assert np.array_equal(x.cpu().numpy(), ref)
 
 
 def test_protocol_switch_on_one_handle(cap):
