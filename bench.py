@@ -54,6 +54,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--profile", action="store_true", help="short run for ncu: no clocks/e2e/cpu legs")
     ap.add_argument("--opt", action="append", default=[], help="extra handle option key=value")
+    ap.add_argument("--no-flags-leg", action="store_true", help="skip the FLAGS-protocol comparison leg")
     return ap.parse_args()
 
 
@@ -61,16 +62,17 @@ def parse():
 
 def systems_for_rank(config: str, rank: int, world: int):
     import synth
+    from paper_conf_icpp_suz0hw0w20_b200.batch import replica_seed, shard
     if config == "c5":
-        return [synth.gen_c5(s) for s in range(8) if s % world == rank]
+        return [synth.gen_c5(s) for s in shard(8, rank, world)]
     if config == "c2":
-        return [synth.gen_c2(seed=2 + rank)]
+        return [synth.gen_c2(seed=replica_seed(2, rank))]
     if config == "c3":
-        return [synth.gen_c3(seed=3 + rank)]
+        return [synth.gen_c3(seed=replica_seed(3, rank))]
     if config == "c4":
-        return [synth.gen_c4(seed=4 + rank)]
+        return [synth.gen_c4(seed=replica_seed(4, rank))]
     if config == "c1":
-        return [synth.gen_c1(seed=1 + rank)]
+        return [synth.gen_c1(seed=replica_seed(1, rank))]
     if config == "chain":
         return [synth.gen_chain()]
     raise ValueError(config)
@@ -218,7 +220,7 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     systems = systems_for_rank(args.config, rank, world)
-    opts = {"mode": args.mode}
+    opts = {"mode": args.mode, "protocol": 1}
     for kv in args.opt:
         k, v = kv.split("=")
         opts[k] = int(v)
@@ -277,6 +279,36 @@ def main():
     value = 2.0 * nnz_all * args.steps / tot_s / 1e9
     kernel_s = float(np.median(step_ms)) * 1e-3 / max(1, len(systems))
 
+    # ---- comparison leg: the release/acquire FLAGS protocol (north_star's literal protocol)
+    flags_leg = None
+    if not args.no_flags_leg and not args.profile and opts.get("protocol", 1) != 0:
+        for h in handles:
+            h.set_option(cap.OPT_PROTOCOL, 0)
+        for i in range(args.warmup):
+            flush.zero_()
+            step(i)
+        ev2 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            flush.zero_()
+            ev2[i][0].record(stream)
+            step(i)
+            ev2[i][1].record(stream)
+        torch.cuda.synchronize()
+        for h in handles:
+            h.check(stream)
+            h.set_option(cap.OPT_PROTOCOL, opts.get("protocol", 1))
+        ft = float(np.sum([a.elapsed_time(b) for a, b in ev2])) * 1e-3
+        if dist:
+            t = torch.tensor([ft], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ft = float(t.item())
+        flags_leg = {"protocol": "flags (st.release.gpu / ld.acquire.gpu epoch flags)",
+                     "value": round(2.0 * nnz_all * args.steps / ft / 1e9, 3), "unit": UNIT,
+                     "ms_per_step": round(ft / args.steps * 1e3, 5)}
+
     # ---- roofline of the dominant (only) kernel, k_solve
     peak, peak_src = peaks()
     alg_bytes = systems[0].alg_bytes()
@@ -293,7 +325,10 @@ def main():
         levels = {"c1": None, "c2": 10, "c3": 4095, "c4": 1000, "c5": 10, "chain": systems[0].n}[args.config]
         if levels is None:
             lv, levels, _ = handles[0].levels(stream)
-        t_hop = cap.flag_latency(20000, 0)
+        # one-way hop of the protocol in use: FLAGS = st.release/ld.acquire pair + x load (probe 0),
+        # FUSED = value-carrying relaxed store / poll (probe 2); median of 3 probes
+        probe = 0 if opts.get("protocol", 1) == 0 else 2
+        t_hop = float(np.median([cap.flag_latency(20000, probe) for _ in range(3)]))
         lat = {"levels": int(levels), "t_hop_ns": round(t_hop, 1),
                "bound_us": round((levels - 1) * t_hop * 1e-3, 2),
                "frac": round((levels - 1) * t_hop * 1e-9 / kernel_s, 4)}
@@ -350,6 +385,9 @@ def main():
                        "l2": "flushed between timed steps (256 MiB write, outside the per-step events)",
                        "parallelism": f"replicas x{world}" if args.config != "c5" else f"systems sharded over {world}",
                        "options": opts},
+            "protocol": {1: "fused (epoch-tagged 16-byte value records, no fences)",
+                         0: "flags (st.release.gpu / ld.acquire.gpu)"}[opts.get("protocol", 1)],
+            "flags_protocol_leg": flags_leg,
             "roofline": roof,
             "latency_bound": lat,
             "e2e": e2e,

@@ -59,7 +59,7 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_WARP_THRESHOLD = 2, /* AUTO: a 32-row group goes warp-level when its mean
                                       nnz/row exceeds this (default 16; sec.4.4, DESIGN G10).
                                       Setting it re-plans (synchronous).                    */
-    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 128, 256 (default), 512, 1024; the
+    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 64, 128, 256 (default), 512, 1024; the
                                       PIPE engine uses one of the warps as its loader       */
     SPTRSV_OPT_BACKOFF_MIN_NS = 4, /* __nanosleep after a pass where no lane progressed     */
     SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
@@ -67,20 +67,20 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_L2_WINDOW = 7,      /* 1: cudaAccessPolicyWindow persisting over the flags   */
     SPTRSV_OPT_STAGE_SMEM = 8,     /* 1 (default): thread-level warps stage their CSR slice
                                       in shared memory with coalesced loads                 */
-    SPTRSV_OPT_PROTOCOL = 9,       /* cross-CTA ready protocol: 0 FLAGS (default) = uint32
-                                      epoch flags, st.release.gpu / ld.acquire.gpu (Alg.5
-                                      l.15-16 + DESIGN G6); 1 FUSED = 16-byte record per
-                                      component, each 8-byte half = epoch<<32 | half of x_i,
-                                      no fences                     */
+    SPTRSV_OPT_PROTOCOL = 9,       /* cross-CTA ready protocol: 0 FLAGS = uint32 epoch flags,
+                                      st.release.gpu / ld.acquire.gpu (Alg.5 l.15-16 + DESIGN
+                                      G6); 1 FUSED (default) = 16-byte record per component,
+                                      each 8-byte half = epoch<<32 | half of x_i, no fences
+                                                                     */
     SPTRSV_OPT_LOCAL = 10,         /* 1 (default): dependencies produced inside the same CTA
                                       are read from a shared-memory copy of x               */
-    SPTRSV_OPT_ENGINE = 11,        /* 1 (default) PIPE: persistent CTAs, a loader warp streams
-                                      rounds of rows into a shared-memory ring by TMA bulk
-                                      copy; 0 ONE-SHOT: one CTA per row range, ticketed.
-                                      PIPE needs 16-byte aligned rowptr/colidx/val/b and
-                                      falls back to ONE-SHOT otherwise                      */
+    SPTRSV_OPT_ENGINE = 11,        /* 0 (default) ONE-SHOT: one CTA per row range, ticketed;
+                                      1 PIPE: persistent CTAs, a loader warp streams rounds
+                                      of rows into a shared-memory ring by TMA bulk copy.
+                                      PIPE needs 16-byte aligned rowptr/colidx/val/b and a
+                                      ring that fits; it falls back to ONE-SHOT otherwise   */
     SPTRSV_OPT_PIPE_STAGES = 12,   /* PIPE ring depth, 2..8 (default 3)                     */
-    SPTRSV_OPT_PIPE_BATCH = 13,    /* PIPE rounds taken per ticket, 1..32 (default 2)       */
+    SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
     SPTRSV_OPT_PIPE_ENTRIES = 14   /* PIPE colidx/val entries per stage (0 = 4 per row)     */
 } sptrsv_option;
 

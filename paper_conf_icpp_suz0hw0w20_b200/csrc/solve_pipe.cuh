@@ -94,94 +94,114 @@ __device__ __forceinline__ int round_row(const SolveParams &p, int t) {
 }
 
 // ---------------------------------------------------------------- loader warp
+//
+// Rounds are taken one ticket at a time (consecutive rounds go to different
+// CTAs, so a CTA never queues a round behind its own predecessor), with a
+// two-round lookahead so the ticket atomic and the rowptr bounds of the next
+// rounds are in flight while the current one is staged:
+//   iteration k: ticket for round k+2 issued, bounds for round k+1 issued,
+//                round k staged (its bounds arrived during iteration k-1).
+struct RoundInfo {
+    int t0, t1, r0, r1, e0, e1;
+    bool valid;
+};
+
+template <int PLAN>
+__device__ __forceinline__ RoundInfo round_info(const SolveParams &p, const PipeGeom &g, unsigned q, uint64_t pol) {
+    RoundInfo ri;
+    const long long t0l = (long long)q * g.W;
+    ri.valid = t0l < p.n_tasks;
+    ri.t0 = ri.valid ? (int)t0l : 0;
+    ri.t1 = ri.valid ? min(p.n_tasks, ri.t0 + g.W) : 0;
+    ri.r0 = ri.valid ? round_row<PLAN>(p, ri.t0) : 0;
+    ri.r1 = ri.valid ? round_row<PLAN>(p, ri.t1) : 0;
+    ri.e0 = ri.valid ? ld_stream_i32(p.rowptr + ri.r0, pol) : 0;
+    ri.e1 = ri.valid ? ld_stream_i32(p.rowptr + ri.r1, pol) : 0;
+    return ri;
+}
+
 template <int PLAN>
 __device__ void pipe_loader(const SolveParams &p, const PipeGeom &g, unsigned char *ring, unsigned full0,
                             unsigned empty0, int lane, uint64_t pol) {
     const unsigned ring_s = smem_u32(ring);
-    int k = 0;
-    bool more = true;
-    while (more) {
-        // ---- a batch of B consecutive rounds from the ticket (lane l describes round q0+l)
-        unsigned q0 = 0;
-        if (lane == 0) q0 = atomicAdd(&p.st->ticket.v, (unsigned)g.B);
-        q0 = __shfl_sync(FULL, q0, 0);
-        const int q = (int)q0 + lane;
-        const long long t0l = (long long)q * g.W;
-        int t0 = 0, t1 = 0, r0 = p.n, r1 = p.n, e0 = 0, e1 = 0;
-        const bool valid = lane < g.B && t0l < p.n_tasks;
-        if (valid) {
-            t0 = (int)t0l;
-            t1 = min(p.n_tasks, t0 + g.W);
-            r0 = round_row<PLAN>(p, t0);
-            r1 = round_row<PLAN>(p, t1);
-            e0 = ld_stream_i32(p.rowptr + r0, pol);
-            e1 = ld_stream_i32(p.rowptr + r1, pol);
+    // lookahead state lives in lane 0 (the other lanes only help with tails / xc init)
+    unsigned q_cur = 0, q_next = 0, q_next2 = 0;
+    RoundInfo ri_next;
+    if (lane == 0) {
+        q_cur = atomicAdd(&p.st->ticket.v, 1u);
+        q_next = atomicAdd(&p.st->ticket.v, 1u);
+    }
+    RoundInfo ri = {};
+    if (lane == 0) ri = round_info<PLAN>(p, g, q_cur, pol);
+    for (int k = 0;; ++k) {
+        if (lane == 0) {
+            q_next2 = atomicAdd(&p.st->ticket.v, 1u);       // result used two iterations later
+            ri_next = round_info<PLAN>(p, g, q_next, pol);   // loads used next iteration
         }
-        for (int jb = 0; jb < g.B; ++jb, ++k) {
-            const int s = k % g.S;
-            const unsigned full = full0 + 8u * s, empty = empty0 + 8u * s;
-            unsigned char *st = ring + (size_t)s * g.stage_bytes;
-            const unsigned st_s = ring_s + (unsigned)s * g.stage_bytes;
-            if (k >= g.S) {  // wait until the compute warps released this stage
-                const unsigned par = (unsigned)((k / g.S) - 1) & 1u;
-                unsigned spins = 0;
-                while (!mbar_try_wait(empty, par)) {
-                    if ((++spins & 1023u) == 0 && ld_relaxed_u32(&p.st->abort.v)) return;
-                }
+        const int s = k % g.S;
+        const unsigned full = full0 + 8u * s, empty = empty0 + 8u * s;
+        unsigned char *st = ring + (size_t)s * g.stage_bytes;
+        const unsigned st_s = ring_s + (unsigned)s * g.stage_bytes;
+        if (k >= g.S) {  // wait until the compute warps released this stage
+            const unsigned par = (unsigned)((k / g.S) - 1) & 1u;
+            unsigned spins = 0;
+            while (!mbar_try_wait(empty, par)) {
+                if ((++spins & 1023u) == 0 && ld_relaxed_u32(&p.st->abort.v)) return;
             }
-            const bool v = __shfl_sync(FULL, valid, jb);
-            StageHdr *h = reinterpret_cast<StageHdr *>(st);
-            if (!v) {  // end of work: an empty stage with q = -1
-                if (lane == 0) {
-                    h->q = -1;
-                    mbar_arrive_expect_tx(full, 0);
-                }
-                more = false;
-                break;
+        }
+        StageHdr *h = reinterpret_cast<StageHdr *>(st);
+        const bool v = __shfl_sync(FULL, ri.valid, 0);
+        if (!v) {  // end of work: an empty stage with q = -1
+            if (lane == 0) {
+                h->q = -1;
+                mbar_arrive_expect_tx(full, 0);
             }
-            const int R0 = __shfl_sync(FULL, r0, jb), R1 = __shfl_sync(FULL, r1, jb);
-            const int T0 = __shfl_sync(FULL, t0, jb), T1 = __shfl_sync(FULL, t1, jb);
-            const int E0 = __shfl_sync(FULL, e0, jb), E1 = __shfl_sync(FULL, e1, jb);
-            const bool staged = (E1 - E0) <= g.E;
-            // x copy of the round := sentinel (dependencies inside the round poll it)
-            unsigned long long *xc = reinterpret_cast<unsigned long long *>(st + g.off_xc);
-            for (int r = lane; r < R1 - R0; r += 32) xc[r] = kSentinel;
-            unsigned tx = 0;
-            // tails first (plain stores), then one arrive.expect_tx, then the bulk copies
-            const int rp_off = stage_span<4>(p.rowptr, R0, R1 + 1, (long long)p.n + 1, st_s + g.off_rp, &tx, lane,
-                                             true, false, full, pol);
-            const int b_off = stage_span<8>(p.b, R0, R1, p.n, st_s + g.off_b, &tx, lane, true, false, full, pol);
-            int c_off = 0, v_off = 0;
-            const long long nnz = p.nnz;
+            return;
+        }
+        const int R0 = __shfl_sync(FULL, ri.r0, 0), R1 = __shfl_sync(FULL, ri.r1, 0);
+        const int E0 = __shfl_sync(FULL, ri.e0, 0), E1 = __shfl_sync(FULL, ri.e1, 0);
+        const bool staged = (E1 - E0) <= g.E;
+        // x copy of the round := sentinel (dependencies inside the round poll it)
+        unsigned long long *xc = reinterpret_cast<unsigned long long *>(st + g.off_xc);
+        for (int r = lane; r < R1 - R0; r += 32) xc[r] = kSentinel;
+        unsigned tx = 0;
+        // tails first (plain stores), then one arrive.expect_tx, then the bulk copies
+        const long long nnz = p.nnz;
+        const int rp_off = stage_span<4>(p.rowptr, R0, R1 + 1, (long long)p.n + 1, st_s + g.off_rp, &tx, lane,
+                                         true, false, full, pol);
+        const int b_off = stage_span<8>(p.b, R0, R1, p.n, st_s + g.off_b, &tx, lane, true, false, full, pol);
+        int c_off = 0, v_off = 0;
+        if (staged) {
+            c_off = stage_span<4>(p.colidx, E0, E1, nnz, st_s + g.off_col, &tx, lane, true, false, full, pol);
+            v_off = stage_span<8>(p.val, E0, E1, nnz, st_s + g.off_val, &tx, lane, true, false, full, pol);
+        }
+        if (lane == 0) {
+            h->q = (int)q_cur;
+            h->t0 = ri.t0;
+            h->t1 = ri.t1;
+            h->r0 = R0;
+            h->r1 = R1;
+            h->rp_off = rp_off;
+            h->b_off = b_off;
+            h->c_off = c_off;
+            h->v_off = v_off;
+            h->staged = staged;
+        }
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive_expect_tx(full, tx);
+            stage_span<4>(p.rowptr, R0, R1 + 1, (long long)p.n + 1, st_s + g.off_rp, nullptr, 0, false, true,
+                          full, pol);
+            stage_span<8>(p.b, R0, R1, p.n, st_s + g.off_b, nullptr, 0, false, true, full, pol);
             if (staged) {
-                c_off = stage_span<4>(p.colidx, E0, E1, nnz, st_s + g.off_col, &tx, lane, true, false, full, pol);
-                v_off = stage_span<8>(p.val, E0, E1, nnz, st_s + g.off_val, &tx, lane, true, false, full, pol);
+                stage_span<4>(p.colidx, E0, E1, nnz, st_s + g.off_col, nullptr, 0, false, true, full, pol);
+                stage_span<8>(p.val, E0, E1, nnz, st_s + g.off_val, nullptr, 0, false, true, full, pol);
             }
-            if (lane == 0) {
-                h->q = (int)q0 + jb;
-                h->t0 = T0;
-                h->t1 = T1;
-                h->r0 = R0;
-                h->r1 = R1;
-                h->rp_off = rp_off;
-                h->b_off = b_off;
-                h->c_off = c_off;
-                h->v_off = v_off;
-                h->staged = staged;
-            }
-            __syncwarp();
-            if (lane == 0) {
-                mbar_arrive_expect_tx(full, tx);
-                stage_span<4>(p.rowptr, R0, R1 + 1, (long long)p.n + 1, st_s + g.off_rp, nullptr, 0, false, true,
-                              full, pol);
-                stage_span<8>(p.b, R0, R1, p.n, st_s + g.off_b, nullptr, 0, false, true, full, pol);
-                if (staged) {
-                    stage_span<4>(p.colidx, E0, E1, nnz, st_s + g.off_col, nullptr, 0, false, true, full, pol);
-                    stage_span<8>(p.val, E0, E1, nnz, st_s + g.off_val, nullptr, 0, false, true, full, pol);
-                }
-            }
-            __syncwarp();
+            q_cur = q_next;
+            q_next = q_next2;
+            ri = ri_next;
         }
+        __syncwarp();
     }
 }
 
@@ -208,9 +228,9 @@ __device__ bool pipe_compute(const SolveParams &p, const PipeGeom &g, unsigned c
         if (t < h->t1) {
             const int32_t *rp = reinterpret_cast<const int32_t *>(st + g.off_rp) - h->rp_off;
             const double *bb = reinterpret_cast<const double *>(st + g.off_b) - h->b_off;
-            const int32_t *sc = reinterpret_cast<const int32_t *>(st + g.off_col) - h->c_off;
-            const double *sv = reinterpret_cast<const double *>(st + g.off_val) - h->v_off;
-            const bool staged = h->staged != 0;
+            // one code path: generic pointers to the staged slice, or to global memory
+            const int32_t *cp = h->staged ? reinterpret_cast<const int32_t *>(st + g.off_col) - h->c_off : p.colidx;
+            const double *vp = h->staged ? reinterpret_cast<const double *>(st + g.off_val) - h->v_off : p.val;
             Cta cta;
             cta.xc = reinterpret_cast<unsigned long long *>(const_cast<unsigned char *>(st) + g.off_xc);
             cta.xc_s = ring_s + (unsigned)s * g.stage_bytes + g.off_xc;
@@ -219,6 +239,8 @@ __device__ bool pipe_compute(const SolveParams &p, const PipeGeom &g, unsigned c
             int tv = t;
             if (PLAN == PLAN_LIST) tv = __ldg(p.tasks + t);
             const bool thread_level = (PLAN == PLAN_THREAD) || (PLAN == PLAN_LIST && tv >= 0);
+            auto col_at = [&](int jj) -> int { return cp[jj]; };
+            auto val_at = [&](int jj) -> double { return vp[jj]; };
             if (thread_level) {
                 const int r0 = (PLAN == PLAN_THREAD) ? t * 32 : tv;
                 const int rows = min(32, p.n - r0);
@@ -227,26 +249,11 @@ __device__ bool pipe_compute(const SolveParams &p, const PipeGeom &g, unsigned c
                 const int rs = act ? rp[i] : 0;
                 const int re = act ? rp[i + 1] : 1;
                 const double bi = act ? bb[i] : 0.0;
-                if (staged)
-                    ok = thread_rows<PROTO>(p, cta, i, act, rs, re, bi, epoch, lane,
-                                            [&](int jj) -> int { return sc[jj]; },
-                                            [&](int jj) -> double { return sv[jj]; });
-                else
-                    ok = thread_rows<PROTO>(p, cta, i, act, rs, re, bi, epoch, lane,
-                                            [&](int jj) -> int { return ld_stream_i32(p.colidx + jj, pol); },
-                                            [&](int jj) -> double { return ld_stream_f64(p.val + jj, pol); });
+                ok = thread_rows<PROTO>(p, cta, i, act, rs, re, bi, epoch, lane, col_at, val_at);
             } else {
                 const int i = (PLAN == PLAN_WARP) ? t : ~tv;
                 const int rs = rp[i], re = rp[i + 1];
-                const double bi = bb[i];
-                if (staged)
-                    ok = warp_row<PROTO>(p, cta, i, rs, re, bi, sv[re - 1], epoch, lane,
-                                         [&](int jj) -> int { return sc[jj]; },
-                                         [&](int jj) -> double { return sv[jj]; });
-                else
-                    ok = warp_row<PROTO>(p, cta, i, rs, re, bi, ld_stream_f64(p.val + re - 1, pol), epoch, lane,
-                                         [&](int jj) -> int { return ld_stream_i32(p.colidx + jj, pol); },
-                                         [&](int jj) -> double { return ld_stream_f64(p.val + jj, pol); });
+                ok = warp_row<PROTO>(p, cta, i, rs, re, bb[i], vp[re - 1], epoch, lane, col_at, val_at);
             }
         }
         __syncwarp();

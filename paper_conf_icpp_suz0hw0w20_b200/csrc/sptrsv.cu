@@ -60,11 +60,11 @@ struct sptrsv_handle_s {
     uint32_t spin_limit = 1u << 24;
     int l2_window = 0;
     int stage = 1;
-    int proto = PROTO_FLAGS;
+    int proto = PROTO_FUSED;
     int local = 1;
-    int engine = 1;         // 0 one-shot (k_solve), 1 pipelined (k_solve_pipe)
+    int engine = 0;         // 0 one-shot (k_solve), 1 pipelined (k_solve_pipe)
     int pipe_stages = 3;
-    int pipe_batch = 2;
+    int pipe_batch = 1;  // (kept for the ABI; the loader takes one round per ticket)
     int pipe_entries = 0;   // 0 = 4 per row of a round
     int grid_cache_key = -1;
     int grid_cache = 0;
@@ -112,6 +112,7 @@ pipe_fn pipe_kernel(int plan, int proto) {
 }
 
 int round16(int b) { return (b + 15) & ~15; }
+constexpr int kPipeMaxSmem = 200 * 1024;  // ring bytes per CTA, at most (227 KB minus static smem and slack)
 
 PipeGeom pipe_geom(const sptrsv_handle_s *h) {
     PipeGeom g;
@@ -145,7 +146,7 @@ int set_kernel_attrs() {
             if (cudaFuncSetAttribute(solve_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) !=
                     cudaSuccess ||
                 cudaFuncSetAttribute(pipe_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     227 * 1024) != cudaSuccess) {
+                                     kPipeMaxSmem) != cudaSuccess) {
                 (void)cudaGetLastError();
                 rc = SPTRSV_ERR_CUDA;
             }
@@ -308,6 +309,7 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
         h->nnz = ends[1];
         const size_t nn = (size_t)(n > 0 ? n : 1);
         if (cudaMalloc(&h->ws.flags, sizeof(uint32_t) * nn) != cudaSuccess ||
+            (h->proto == PROTO_FUSED && cudaMalloc(&h->ws.rec, 16 * nn) != cudaSuccess) ||
             cudaMalloc(&h->ws.indeg, sizeof(int32_t) * nn) != cudaSuccess ||
             cudaMalloc(&h->ws.st, sizeof(SolveState)) != cudaSuccess ||
             cudaMalloc(&d_status, sizeof(unsigned long long)) != cudaSuccess ||
@@ -393,6 +395,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     if (h->engine == 1 && aligned && h->cta_threads >= 64) {
         const PipeGeom g = pipe_geom(h);
         const size_t smem = (size_t)g.S * g.stage_bytes;
+        if (smem > (size_t)kPipeMaxSmem) goto oneshot;  // ring does not fit: run the one-shot engine
         const int key = (h->plan * 2 + h->proto) * 4096 + h->cta_threads + (int)(smem >> 4) * 8192;
         if (key != h->grid_cache_key) {
             int per_sm = 0, sms = 0;
@@ -402,10 +405,10 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
                 (void)cudaGetLastError();
                 return SPTRSV_ERR_CUDA;
             }
-            if (per_sm < 1) return SPTRSV_ERR_INVALID_ARG;  // ring does not fit: fewer stages / threads
             h->grid_cache = per_sm * sms;
             h->grid_cache_key = key;
         }
+        if (h->grid_cache < 1) goto oneshot;  // not even one CTA fits: one-shot engine
         const int rounds = (h->n_tasks + g.W - 1) / g.W;
         const int grid = rounds < h->grid_cache ? (rounds > 0 ? rounds : 1) : h->grid_cache;
         cudaLaunchConfig_t cfg = {};
@@ -423,6 +426,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
         h->since_reset++;
         return SPTRSV_OK;
     }
+oneshot:
     const int warps = h->cta_threads / 32;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
@@ -501,7 +505,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->threshold = (int)value;
             return build_plan(h);
         case SPTRSV_OPT_CTA_THREADS:
-            if (value != 128 && value != 256 && value != 512 && value != 1024) return SPTRSV_ERR_INVALID_ARG;
+            if (value != 64 && value != 128 && value != 256 && value != 512 && value != 1024) return SPTRSV_ERR_INVALID_ARG;
             h->cta_threads = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_BACKOFF_MIN_NS:

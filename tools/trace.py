@@ -45,3 +45,10 @@ if name == "chain":
     out["sum_us"] = {"inwarp": float(dt[inwarp].sum()) / 1e3, "warp_b": float(dt[warp_b].sum()) / 1e3,
                      "cta_b": float(dt[cta_b].sum()) / 1e3}
 print(json.dumps(out))
+if name == "c3":
+    g = 2048
+    T = t.reshape(g, g)
+    row_start = T.min(axis=1); row_end = T.max(axis=1)
+    print(json.dumps({"c3_row_start_us": [round(float(row_start[r]) / 1e3, 1) for r in range(0, g, 128)],
+                      "c3_row_end_us": [round(float(row_end[r]) / 1e3, 1) for r in range(0, g, 128)],
+                      "row0_cells_us": [round(float(T[0, c]) / 1e3, 2) for c in range(0, 2048, 128)]}))
