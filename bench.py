@@ -381,6 +381,8 @@ def main():
                        "n": systems[0].n, "nnz": systems[0].nnz, "systems_per_rank": len(systems),
                        "mode": {0: "auto", 1: "thread", 2: "warp"}[args.mode],
                        "plan": {"thread_groups": info["n_thread_groups"], "warp_rows": info["n_warp_rows"]},
+                       "engine": {0: "one-shot (staged, in-CTA x copy)", 1: "pipe (TMA ring)", 2: "dyn",
+                                  3: "lean", 4: "dyn-static"}.get(info["engine"], str(info["engine"])),
                        "analyse_ms": round(info["analyse_ms"], 3),
                        "l2": "flushed between timed steps (256 MiB write, outside the per-step events)",
                        "parallelism": f"replicas x{world}" if args.config != "c5" else f"systems sharded over {world}",

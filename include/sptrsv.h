@@ -74,14 +74,27 @@ typedef enum sptrsv_option {
                                                                      */
     SPTRSV_OPT_LOCAL = 10,         /* 1 (default): dependencies produced inside the same CTA
                                       are read from a shared-memory copy of x               */
-    SPTRSV_OPT_ENGINE = 11,        /* 0 (default) ONE-SHOT: one CTA per row range, ticketed;
+    SPTRSV_OPT_ENGINE = 11,        /* 5 (default) AUTO: LEAN for all-thread-level plans whose
+                                      dependencies are mostly far (< 1/4 within 256 rows),
+                                      else ONE-SHOT.  0 ONE-SHOT: one CTA per row range,
+                                      ticketed, smem-staged, in-CTA x copy;
                                       1 PIPE: persistent CTAs, a loader warp streams rounds
                                       of rows into a shared-memory ring by TMA bulk copy.
                                       PIPE needs 16-byte aligned rowptr/colidx/val/b and a
-                                      ring that fits; it falls back to ONE-SHOT otherwise   */
+                                      ring that fits; it falls back to ONE-SHOT otherwise.
+                                      2 DYN: persistent warps, every lane slot takes the next
+                                      row as soon as its row is published (all-thread-level
+                                      plans; ROWS_PER_LANE = slots per lane, 1/2/4).
+                                      3 LEAN: minimal-latency one-shot kernel for
+                                      all-thread-level plans (no staging, speculative rows).
+                                      4 DYN-STATIC: DYN with static round-robin 32-row units
+                                      (no ticket), launched cooperatively                  */
     SPTRSV_OPT_PIPE_STAGES = 12,   /* PIPE ring depth, 2..8 (default 3)                     */
     SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
-    SPTRSV_OPT_PIPE_ENTRIES = 14   /* PIPE colidx/val entries per stage (0 = 4 per row)     */
+    SPTRSV_OPT_PIPE_ENTRIES = 14,  /* PIPE colidx/val entries per stage (0 = 4 per row)     */
+    SPTRSV_OPT_ROWS_PER_LANE = 15  /* K = 1..4 thread-level rows per lane (lane owns rows
+                                      r0+lane+32k); applies to all-thread-level plans on
+                                      the ONE-SHOT engine with CTAs of <= 256 threads      */
 } sptrsv_option;
 
 typedef struct sptrsv_info {
@@ -94,6 +107,8 @@ typedef struct sptrsv_info {
     int32_t device;           /* CUDA ordinal the handle is bound to                      */
     float analyse_ms;         /* wall time of sptrsv_analyse_csr (Table 1 analogue)        */
     uint32_t solves;          /* solves enqueued through this handle                      */
+    int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
+    int32_t engine;           /* engine the next solve uses (AUTO resolved)                */
 } sptrsv_info;
 
 /*
@@ -169,9 +184,12 @@ int sptrsv_get_indegree(sptrsv_handle_t h, int32_t *out_dev, sptrsv_stream_t str
 int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev,
                   int32_t *nlevels_host, sptrsv_stream_t stream);
 
-/* sptrsv_set_trace -- diagnostic: while trace_dev (device uint64[n]) is set,
+/* sptrsv_set_trace -- diagnostic: while trace_dev (device uint64[3n]) is set,
  * every solve writes the %globaltimer (ns) at which x_i was published into
- * trace_dev[i] -- the critical path, row by row.  NULL turns it off. */
+ * trace_dev[i], and for thread-level rows the time row i consumed its last
+ * dependency into trace_dev[n + i] and the time its solve loop started (data
+ * loaded) into trace_dev[2n + i] -- the critical path, row by row.  NULL turns
+ * it off. */
 int sptrsv_set_trace(sptrsv_handle_t h, uint64_t *trace_dev);
 
 /* sptrsv_check -- synchronises `stream`, returns SPTRSV_ERR_TIMEOUT if the

@@ -120,9 +120,12 @@ class Handle:
         return lv, int(nl.value), counts[: nl.value]
 
     def trace(self, b, x=None, stream=None):
-        """Diagnostic solve that records the publish time (ns, %globaltimer) of every x_i."""
+        """Diagnostic solve: (x, trace) with trace[:n] = publish time (ns, %globaltimer) of each
+        x_i, trace[n:2n] = when (thread-level) row i consumed its last dependency (0 = none) and
+        trace[2n:] = when its solve loop started (0 = not recorded)."""
         import torch
-        tr = torch.zeros(self.n, dtype=torch.int64, device=self.device)
+        tr = torch.zeros(3 * self.n + 3, dtype=torch.int64, device=self.device)
+        tr[3 * self.n] = (1 << 63) - 1
         check(lib.sptrsv_set_trace(self._h, tr.data_ptr()), "sptrsv_set_trace")
         try:
             x = self.solve(b, x, stream)
@@ -170,7 +173,7 @@ def analyse(rowptr, colidx, val, **options) -> Handle:
             "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
             "pipe_stages": _lib.OPT_PIPE_STAGES, "pipe_batch": _lib.OPT_PIPE_BATCH,
-            "pipe_entries": _lib.OPT_PIPE_ENTRIES}
+            "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

@@ -47,7 +47,8 @@ OPT_ENGINE = 11
 OPT_PIPE_STAGES = 12
 OPT_PIPE_BATCH = 13
 OPT_PIPE_ENTRIES = 14
-ENGINE_ONESHOT, ENGINE_PIPE = 0, 1
+OPT_ROWS_PER_LANE = 15
+ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
 
@@ -63,6 +64,8 @@ class sptrsv_info(ctypes.Structure):
         ("device", ctypes.c_int32),
         ("analyse_ms", ctypes.c_float),
         ("solves", ctypes.c_uint32),
+        ("near_deps", ctypes.c_int64),
+        ("engine", ctypes.c_int32),
     ]
 
 

@@ -18,13 +18,18 @@ enum : int {  // same numbering as sptrsv_status (negated)
 
 // status: 64-bit min over (row << 8 | code) -> the lowest offending row wins,
 // which is the row-ordered error the oracle reports too.
+// Also counts "near" dependencies (i - col < 256: produced within about one CTA of
+// rows) -- the statistic ENGINE_AUTO uses to choose between the shared-memory
+// local resolution of the staged engine and the lean engine.
 __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ rowptr,
                                                   const int32_t *__restrict__ colidx,
                                                   const double *__restrict__ val, int32_t n,
                                                   int64_t nnz, int32_t *indeg,
-                                                  unsigned long long *status, int32_t *max_row) {
+                                                  unsigned long long *status, int32_t *max_row,
+                                                  unsigned long long *near_deps) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     int len = 0;
+    unsigned near = 0;
     if (i < n) {
         const int64_t s = rowptr[i], e = rowptr[i + 1];
         int code = 0;
@@ -39,6 +44,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
                 if (c < 0) { code = E_BAD_COL; break; }
                 if (c > i) { code = E_NOT_LOWER; break; }
                 if (j > s && c <= prev) { code = E_UNSORTED; break; }
+                if (c < i && i - c < 256) ++near;
                 prev = c;
             }
             if (!code) {
@@ -50,8 +56,12 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
         len = code ? 0 : (int)(e - s);
         indeg[i] = code ? 0 : (int)(e - s - 1);
     }
-    for (int off = 16; off > 0; off >>= 1) len = max(len, __shfl_xor_sync(0xffffffffu, len, off));
+    for (int off = 16; off > 0; off >>= 1) {
+        len = max(len, __shfl_xor_sync(0xffffffffu, len, off));
+        near += __shfl_xor_sync(0xffffffffu, near, off);
+    }
     if ((threadIdx.x & 31) == 0 && len > 0) atomicMax(max_row, len);
+    if ((threadIdx.x & 31) == 0 && near) atomicAdd(near_deps, (unsigned long long)near);
 }
 
 // mode: 0 auto, 1 all thread-level, 2 all warp-level.

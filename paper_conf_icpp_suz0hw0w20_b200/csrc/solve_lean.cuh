@@ -1,0 +1,138 @@
+// solve_lean.cuh -- ENGINE_LEAN: the minimal-latency one-shot kernel for
+// all-thread-level plans (short rows, the paper's target regime PAPER.md:188-192).
+//
+// Alg.5 with everything that is not the method trimmed off
+// the per-CTA critical path, because for rows of 2-4 entries the method's own
+// work is a few instructions and the solve is bound by how fast rows ENTER the
+// machine (measured: a 1M-row diagonal solve, no dependencies at all, took 26 us
+// in the staged engine vs a 14 us streaming floor):
+//   * the CTA ticket (forward progress, solve.cuh cta_ticket) is overlapped
+//     with a SPECULATIVE load of the rows the CTA gets when its ticket equals
+//     blockIdx.x (the common case; otherwise the rows are re-loaded);
+//   * no shared-memory staging and no in-CTA x copy: each lane loads its row's
+//     bounds, b_i, L_ii and first two entries straight into registers;
+//   * small register footprint (higher occupancy = more rows in flight).
+// The poll / consume / publish protocol (FLAGS or FUSED), the verified division
+// and the lean wait are the shared ones from solve.cuh.
+#pragma once
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "solve.cuh"
+
+namespace sptrsv_dev {
+
+constexpr int kLeanCta = 256;
+
+template <int PROTO>
+__global__ void __launch_bounds__(kLeanCta, 5) k_solve_lean(SolveParams p) {
+    __shared__ uint32_t s_blk, s_epoch;
+    const int tid = threadIdx.x;
+    const int lane = tid & 31;
+    const uint64_t pol = policy_evict_first();
+    // ---- speculative first-level loads for logical block == blockIdx.x
+    int i = (int)blockIdx.x * kLeanCta + tid;
+    int rs = 0, re = 1;
+    double bi = 0.0;
+    if (i < p.n) {
+        rs = ld_stream_i32(p.rowptr + i, pol);
+        re = ld_stream_i32(p.rowptr + i + 1, pol);
+        bi = ld_stream_f64(p.b + i, pol);
+    }
+    if (tid == 0) {
+        if (p.trace) {
+            atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
+            atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
+        }
+        cta_ticket(p, s_blk, s_epoch);
+    }
+    __syncthreads();
+    const uint32_t epoch = s_epoch;
+    if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
+        i = (int)s_blk * kLeanCta + tid;
+        rs = 0, re = 1, bi = 0.0;
+        if (i < p.n) {
+            rs = ld_stream_i32(p.rowptr + i, pol);
+            re = ld_stream_i32(p.rowptr + i + 1, pol);
+            bi = ld_stream_f64(p.b + i, pol);
+        }
+    }
+    const bool act = i < p.n;
+    const int jd = re - 1;
+    int j = rs;
+    // ---- second-level loads: L_ii and the next two dependencies
+    double dv = act ? ld_stream_f64(p.val + jd, pol) : 1.0;
+    int nc = (act && j < jd) ? ld_stream_i32(p.colidx + j, pol) : -1;
+    double nv = (act && j < jd) ? ld_stream_f64(p.val + j, pol) : 0.0;
+    int nc2 = (act && j + 1 < jd) ? ld_stream_i32(p.colidx + j + 1, pol) : -1;
+    Diag dg;
+    dg.init(dv);
+    double ls = 0.0;
+    bool done = !act;
+    Cta nocta;
+    nocta.R0 = nocta.R1 = 0;
+    nocta.xc = nullptr;
+    nocta.xc_s = 0;
+    SolveParams pp = p;
+    pp.local = 0;
+    uint32_t backoff = p.backoff_min, idle = 0;
+    // advance past a consumed dependency: the 2nd becomes the next, prefetch the 3rd
+    auto advance = [&]() {
+        ++j;
+        nc = nc2;
+        nv = (nc >= 0) ? ld_stream_f64(p.val + j, pol) : 0.0;
+        nc2 = (j + 1 < jd) ? ld_stream_i32(p.colidx + j + 1, pol) : -1;
+    };
+    while (true) {
+        bool prog = false;
+        if (!done) {
+            if (nc < 0) {  // reached the diagonal (Alg.5 l.12-16)
+                publish<PROTO>(pp, nocta, i, dg.div(__dsub_rn(bi, ls)), epoch);
+                done = true;
+                prog = true;
+            } else {
+                // poll the next two dependencies together, consume the ready prefix in row order
+                unsigned long long a0, a1, c0 = 0, c1 = 0;
+                poll1<PROTO>(pp, nc, a0, a1);
+                const int cc2 = nc2;
+                if (cc2 >= 0) poll1<PROTO>(pp, cc2, c0, c1);
+                if (ready1<PROTO>(a0, a1, epoch)) {
+                    if (p.trace) p.trace[p.n + i] = globaltimer_ns();
+                    ls = __dadd_rn(ls, __dmul_rn(nv, value1<PROTO>(pp, nc, a0, a1)));
+                    advance();
+                    prog = true;
+                    if (cc2 >= 0 && ready1<PROTO>(c0, c1, epoch)) {
+                        ls = __dadd_rn(ls, __dmul_rn(nv, value1<PROTO>(pp, cc2, c0, c1)));
+                        advance();
+                    }
+                    if (nc < 0) {
+                        publish<PROTO>(pp, nocta, i, dg.div(__dsub_rn(bi, ls)), epoch);
+                        done = true;
+                    }
+                }
+            }
+        }
+        if (!__ballot_sync(FULL, !done)) break;
+        if (__ballot_sync(FULL, prog)) {
+            backoff = p.backoff_min;
+            idle = 0;
+            continue;
+        }
+        if (backoff) nanosleep_ns(backoff);
+        backoff = min(max(backoff * 2u, 32u), p.backoff_max);
+        if ((++idle & 63u) == 0) {
+            uint32_t ab = 0;
+            if (lane == 0) {
+                if (p.spin_limit && idle >= p.spin_limit) {
+                    atomicCAS(&p.st->error.v, 0u, 1u);
+                    st_relaxed_u32(&p.st->abort.v, 1u);
+                }
+                ab = ld_relaxed_u32(&p.st->abort.v);
+            }
+            if (__shfl_sync(FULL, ab, 0)) break;
+        }
+    }
+    if (p.trace && lane == 0) atomicMax(&p.trace[3 * (size_t)p.n + 1], globaltimer_ns());  // last warp exit
+}
+
+}  // namespace sptrsv_dev

@@ -95,12 +95,18 @@ __device__ __forceinline__ int round_row(const SolveParams &p, int t) {
 
 // ---------------------------------------------------------------- loader warp
 //
-// Rounds are taken one ticket at a time (consecutive rounds go to different
-// CTAs, so a CTA never queues a round behind its own predecessor), with a
-// two-round lookahead so the ticket atomic and the rowptr bounds of the next
-// rounds are in flight while the current one is staged:
-//   iteration k: ticket for round k+2 issued, bounds for round k+1 issued,
-//                round k staged (its bounds arrived during iteration k-1).
+// Rounds are taken one ticket at a time (consecutive rounds land in different
+// CTAs, so a CTA never queues a round behind its own predecessor) with a deep
+// lane-parallel lookahead so that neither the ticket atomic nor the dependent
+// rowptr loads of a round are ever waited for:
+//   lane k % kLA holds the round consumed at iteration k; right after staging it
+//   the lane takes the ticket of the round it will stage kLA iterations later,
+//   and kD iterations after that it issues that round's rowptr bounds loads.
+// Tickets taken later are larger, and each lane's rounds are staged in ticket
+// order, so the CTA stages its rounds in increasing order (forward progress).
+constexpr int kLA = 12;
+constexpr int kLD = 4;
+
 struct RoundInfo {
     int t0, t1, r0, r1, e0, e1;
     bool valid;
@@ -122,22 +128,18 @@ __device__ __forceinline__ RoundInfo round_info(const SolveParams &p, const Pipe
 
 template <int PLAN>
 __device__ void pipe_loader(const SolveParams &p, const PipeGeom &g, unsigned char *ring, unsigned full0,
-                            unsigned empty0, int lane, uint64_t pol) {
+                            unsigned empty0, int lane, uint64_t pol, uint32_t *wt) {
     const unsigned ring_s = smem_u32(ring);
-    // lookahead state lives in lane 0 (the other lanes only help with tails / xc init)
-    unsigned q_cur = 0, q_next = 0, q_next2 = 0;
-    RoundInfo ri_next;
-    if (lane == 0) {
-        q_cur = atomicAdd(&p.st->ticket.v, 1u);
-        q_next = atomicAdd(&p.st->ticket.v, 1u);
-    }
+    unsigned tq = 0;
     RoundInfo ri = {};
-    if (lane == 0) ri = round_info<PLAN>(p, g, q_cur, pol);
+    // prologue: tickets for the first kLA rounds (in lane order), then their bounds
+    for (int j = 0; j < kLA; ++j) {
+        if (lane == j) tq = atomicAdd(wt, 1u);
+        __syncwarp();
+    }
+    if (lane < kLA) ri = round_info<PLAN>(p, g, tq, pol);
     for (int k = 0;; ++k) {
-        if (lane == 0) {
-            q_next2 = atomicAdd(&p.st->ticket.v, 1u);       // result used two iterations later
-            ri_next = round_info<PLAN>(p, g, q_next, pol);   // loads used next iteration
-        }
+        const int c = k % kLA;
         const int s = k % g.S;
         const unsigned full = full0 + 8u * s, empty = empty0 + 8u * s;
         unsigned char *st = ring + (size_t)s * g.stage_bytes;
@@ -150,7 +152,7 @@ __device__ void pipe_loader(const SolveParams &p, const PipeGeom &g, unsigned ch
             }
         }
         StageHdr *h = reinterpret_cast<StageHdr *>(st);
-        const bool v = __shfl_sync(FULL, ri.valid, 0);
+        const bool v = __shfl_sync(FULL, ri.valid, c);
         if (!v) {  // end of work: an empty stage with q = -1
             if (lane == 0) {
                 h->q = -1;
@@ -158,8 +160,14 @@ __device__ void pipe_loader(const SolveParams &p, const PipeGeom &g, unsigned ch
             }
             return;
         }
-        const int R0 = __shfl_sync(FULL, ri.r0, 0), R1 = __shfl_sync(FULL, ri.r1, 0);
-        const int E0 = __shfl_sync(FULL, ri.e0, 0), E1 = __shfl_sync(FULL, ri.e1, 0);
+        const int R0 = __shfl_sync(FULL, ri.r0, c), R1 = __shfl_sync(FULL, ri.r1, c);
+        const int T0 = __shfl_sync(FULL, ri.t0, c), T1 = __shfl_sync(FULL, ri.t1, c);
+        const int E0 = __shfl_sync(FULL, ri.e0, c), E1 = __shfl_sync(FULL, ri.e1, c);
+        const unsigned Q = __shfl_sync(FULL, tq, c);
+        // lookahead upkeep: lane c takes the ticket of its next round; the lane that took a
+        // ticket kLD iterations ago issues that round's bounds loads
+        if (lane == c) tq = atomicAdd(wt, 1u);
+        if (k >= kLD && lane == (k - kLD) % kLA) ri = round_info<PLAN>(p, g, tq, pol);
         const bool staged = (E1 - E0) <= g.E;
         // x copy of the round := sentinel (dependencies inside the round poll it)
         unsigned long long *xc = reinterpret_cast<unsigned long long *>(st + g.off_xc);
@@ -176,9 +184,9 @@ __device__ void pipe_loader(const SolveParams &p, const PipeGeom &g, unsigned ch
             v_off = stage_span<8>(p.val, E0, E1, nnz, st_s + g.off_val, &tx, lane, true, false, full, pol);
         }
         if (lane == 0) {
-            h->q = (int)q_cur;
-            h->t0 = ri.t0;
-            h->t1 = ri.t1;
+            h->q = (int)Q;
+            h->t0 = T0;
+            h->t1 = T1;
             h->r0 = R0;
             h->r1 = R1;
             h->rp_off = rp_off;
@@ -197,9 +205,6 @@ __device__ void pipe_loader(const SolveParams &p, const PipeGeom &g, unsigned ch
                 stage_span<4>(p.colidx, E0, E1, nnz, st_s + g.off_col, nullptr, 0, false, true, full, pol);
                 stage_span<8>(p.val, E0, E1, nnz, st_s + g.off_val, nullptr, 0, false, true, full, pol);
             }
-            q_cur = q_next;
-            q_next = q_next2;
-            ri = ri_next;
         }
         __syncwarp();
     }
@@ -266,7 +271,7 @@ template <int PLAN, int PROTO>
 __global__ void __launch_bounds__(1024) k_solve_pipe(SolveParams p, PipeGeom g) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ __align__(8) unsigned long long bars[2 * 8];  // full[S], empty[S] (S <= 8)
-    __shared__ uint32_t s_epoch;
+    __shared__ uint32_t s_epoch, s_blk;
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
     const unsigned full0 = smem_u32(&bars[0]), empty0 = smem_u32(&bars[8]);
@@ -276,27 +281,16 @@ __global__ void __launch_bounds__(1024) k_solve_pipe(SolveParams p, PipeGeom g) 
             mbar_init(empty0 + 8u * s, (unsigned)g.W);
         }
         fence_mbar_init();
-        s_epoch = ld_relaxed_u32(&p.st->epoch.v);
+        cta_ticket(p, s_blk, s_epoch);
+        p.st->wtick[(s_epoch + 1u) & 1u].v = 0;  // the next solve's work counter
     }
     __syncthreads();
     const uint32_t epoch = s_epoch;
     const uint64_t pol = policy_evict_first();
     if (warp == g.W)
-        pipe_loader<PLAN>(p, g, smem, full0, empty0, lane, pol);
+        pipe_loader<PLAN>(p, g, smem, full0, empty0, lane, pol, &p.st->wtick[epoch & 1u].v);
     else
         pipe_compute<PLAN, PROTO>(p, g, smem, full0, empty0, warp, lane, epoch, pol);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        const uint32_t prev = atomicAdd(&p.st->done.v, 1u);
-        if (prev == gridDim.x - 1) {
-            p.st->done.v = 0;
-            p.st->ticket.v = 0;
-            p.st->abort.v = 0;
-            p.st->epoch.v = epoch + 1;
-            __threadfence();
-        }
-    }
 }
 
 }  // namespace sptrsv_dev

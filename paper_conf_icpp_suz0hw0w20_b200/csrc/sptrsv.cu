@@ -15,6 +15,9 @@
 #include "setup.cuh"
 #include "solve.cuh"
 #include "solve_pipe.cuh"
+#include "solve_k.cuh"
+#include "solve_dyn.cuh"
+#include "solve_lean.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -51,6 +54,7 @@ struct sptrsv_handle_s {
     int32_t n_thread_groups = 0;
     int32_t n_warp_rows = 0;
     int32_t max_row = 0;
+    int64_t near_deps = 0;  // dependencies within 256 rows (analyse statistic for ENGINE_AUTO)
     // options
     int mode = 0;
     int threshold = 16;
@@ -62,12 +66,14 @@ struct sptrsv_handle_s {
     int stage = 1;
     int proto = PROTO_FUSED;
     int local = 1;
-    int engine = 0;         // 0 one-shot (k_solve), 1 pipelined (k_solve_pipe)
+    int engine = 5;         // 5 AUTO; 0 one-shot, 1 pipe, 2 dyn, 3 lean, 4 dyn-static
     int pipe_stages = 3;
     int pipe_batch = 1;  // (kept for the ABI; the loader takes one round per ticket)
     int pipe_entries = 0;   // 0 = 4 per row of a round
+    int rows_per_lane = 1;  // K: thread-level rows per lane (all-thread plans, one-shot engine)
     int grid_cache_key = -1;
     int grid_cache = 0;
+    int launch_key = -1;  // configuration of the last launch (see sptrsv_solve)
     unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
@@ -99,6 +105,28 @@ solve_fn solve_kernel(int plan, int proto) {
         {k_solve<PLAN_LIST, PROTO_FLAGS>, k_solve<PLAN_LIST, PROTO_FUSED>},
     };
     return tab[plan][proto];
+}
+
+solve_fn solve_k_kernel(int proto, int K) {
+    if (K == 2) return proto ? k_solve_k<PROTO_FUSED, 2> : k_solve_k<PROTO_FLAGS, 2>;
+    if (K == 3) return proto ? k_solve_k<PROTO_FUSED, 3> : k_solve_k<PROTO_FLAGS, 3>;
+    return proto ? k_solve_k<PROTO_FUSED, 4> : k_solve_k<PROTO_FLAGS, 4>;
+}
+
+solve_fn solve_dyn_kernel(int proto, int K, bool stat) {
+    if (stat) {
+        if (K == 2) return proto ? k_solve_dyn<PROTO_FUSED, 2, true> : k_solve_dyn<PROTO_FLAGS, 2, true>;
+        if (K == 4) return proto ? k_solve_dyn<PROTO_FUSED, 4, true> : k_solve_dyn<PROTO_FLAGS, 4, true>;
+        return proto ? k_solve_dyn<PROTO_FUSED, 1, true> : k_solve_dyn<PROTO_FLAGS, 1, true>;
+    }
+    if (K == 2) return proto ? k_solve_dyn<PROTO_FUSED, 2, false> : k_solve_dyn<PROTO_FLAGS, 2, false>;
+    if (K == 4) return proto ? k_solve_dyn<PROTO_FUSED, 4, false> : k_solve_dyn<PROTO_FLAGS, 4, false>;
+    return proto ? k_solve_dyn<PROTO_FUSED, 1, false> : k_solve_dyn<PROTO_FLAGS, 1, false>;
+}
+
+size_t solve_k_smem_bytes(int cta_threads, int K) {
+    const size_t w = (size_t)(cta_threads / 32);
+    return w * 32 * K * sizeof(double) + w * (size_t)k_warp_smem_bytes(K);
 }
 
 typedef void (*pipe_fn)(SolveParams, PipeGeom);
@@ -151,6 +179,13 @@ int set_kernel_attrs() {
                 rc = SPTRSV_ERR_CUDA;
             }
         }
+    for (int pr = 0; pr < 2; ++pr)
+        for (int K = 2; K <= 4; ++K)
+            if (cudaFuncSetAttribute(solve_k_kernel(pr, K), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)solve_k_smem_bytes(256, K)) != cudaSuccess) {
+                (void)cudaGetLastError();
+                rc = SPTRSV_ERR_CUDA;
+            }
     done = 1;
     return rc;
 }
@@ -240,11 +275,10 @@ int build_plan(sptrsv_handle_s *h) {
 }
 
 int reset_state(sptrsv_handle_s *h, cudaStream_t s) {
-    // flags / records := 0, epoch := 0x01010101 (any nonzero value works), counters := 0
+    // flags / records := 0 (no epoch matches), counters := 0; the next solve has epoch 1
     CK(cudaMemsetAsync(h->ws.flags, 0, sizeof(uint32_t) * (size_t)(h->n > 0 ? h->n : 1), s));
     if (h->ws.rec) CK(cudaMemsetAsync(h->ws.rec, 0, 16 * (size_t)(h->n > 0 ? h->n : 1), s));
     CK(cudaMemsetAsync(h->ws.st, 0, sizeof(SolveState), s));
-    CK(cudaMemsetAsync(&h->ws.st->epoch.v, 1, sizeof(uint32_t), s));
     h->since_reset = 0;
     return SPTRSV_OK;
 }
@@ -293,7 +327,7 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
     h->rowptr = rowptr;
     h->colidx = colidx;
     h->val = val;
-    unsigned long long *d_status = nullptr;
+    unsigned long long *d_status = nullptr, *d_near = nullptr;
     int32_t *d_maxrow = nullptr;
     do {
         int32_t ends[2] = {0, 0};
@@ -313,18 +347,20 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
             cudaMalloc(&h->ws.indeg, sizeof(int32_t) * nn) != cudaSuccess ||
             cudaMalloc(&h->ws.st, sizeof(SolveState)) != cudaSuccess ||
             cudaMalloc(&d_status, sizeof(unsigned long long)) != cudaSuccess ||
-            cudaMalloc(&d_maxrow, sizeof(int32_t)) != cudaSuccess) {
+            cudaMalloc(&d_maxrow, sizeof(int32_t)) != cudaSuccess ||
+            cudaMalloc(&d_near, sizeof(unsigned long long)) != cudaSuccess) {
             rc = SPTRSV_ERR_ALLOC;
             break;
         }
         if (cudaMemset(d_status, 0xff, sizeof(unsigned long long)) != cudaSuccess ||
-            cudaMemset(d_maxrow, 0, sizeof(int32_t)) != cudaSuccess) {
+            cudaMemset(d_maxrow, 0, sizeof(int32_t)) != cudaSuccess ||
+            cudaMemset(d_near, 0, sizeof(unsigned long long)) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
         if (n > 0) {
             k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->nnz, h->ws.indeg, d_status,
-                                                 d_maxrow);
+                                                 d_maxrow, d_near);
             if (cudaGetLastError() != cudaSuccess) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
@@ -332,7 +368,8 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
         }
         unsigned long long status = 0;
         if (cudaMemcpy(&status, d_status, sizeof(status), cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(&h->max_row, d_maxrow, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+            cudaMemcpy(&h->max_row, d_maxrow, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(&h->near_deps, d_near, sizeof(int64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
@@ -351,6 +388,7 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
     } while (0);
     cudaFree(d_status);
     cudaFree(d_maxrow);
+    cudaFree(d_near);
     if (rc != SPTRSV_OK) {
         (void)cudaGetLastError();
         free_ws(h->ws);
@@ -363,14 +401,152 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
     return SPTRSV_OK;
 }
 
+namespace {
+
+// One solve launch: which kernel, its geometry, and how it is parameterised.
+struct Launch {
+    const void *fn = nullptr;
+    int kind = 0;  // 0 SolveParams only, 1 SolveParams + PipeGeom
+    bool coop = false;  // cooperative launch (co-residency guaranteed)
+    dim3 grid, block;
+    size_t smem = 0;
+    PipeGeom geom;
+    int key = 0;  // configuration identity (the epoch arithmetic needs a fixed grid per key)
+};
+
+int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem, int key, int *out) {
+    if (key != h->grid_cache_key) {
+        int per_sm = 0, sms = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem) != cudaSuccess ||
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_CUDA;
+        }
+        h->grid_cache = per_sm * sms;
+        h->grid_cache_key = key;
+    }
+    *out = h->grid_cache;
+    return SPTRSV_OK;
+}
+
+// ENGINE_AUTO: all-thread-level plans go to the LEAN engine unless a quarter or
+// more of the dependencies are "near" (within 256 rows: chains, grid wavefronts),
+// where the staged one-shot engine's shared-memory local resolution wins; plans
+// with warp-level rows use the staged one-shot engine.  (Round-1 B200 sweeps,
+// DESIGN.md section 8.)
+int resolve_engine(const sptrsv_handle_s *h) {
+    if (h->engine != 5) return h->engine;
+    const long long offdiag = h->nnz - h->n;
+    if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_deps < offdiag)) return 3;
+    return 0;
+}
+
+int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
+    const int cta = h->cta_threads;
+    const int engine = resolve_engine(h);
+    // ---- ENGINE_PIPE: persistent, loader warp + TMA ring
+    if (engine == 1 && aligned && cta >= 64) {
+        const PipeGeom g = pipe_geom(h);
+        const size_t smem = (size_t)g.S * g.stage_bytes;
+        if (smem <= (size_t)kPipeMaxSmem) {
+            const void *fn = (const void *)pipe_kernel(h->plan, h->proto);
+            const int key = 1000000 + (h->plan * 2 + h->proto) * 100000 + cta * 16 + g.S;
+            int cap = 0;
+            int rc = occupancy_grid(h, fn, cta, smem, key, &cap);
+            if (rc) return rc;
+            if (cap >= 1) {
+                const int rounds = (h->n_tasks + g.W - 1) / g.W;
+                L->fn = fn;
+                L->kind = 1;
+                L->grid = dim3((unsigned)(rounds < cap ? (rounds > 0 ? rounds : 1) : cap));
+                L->block = dim3((unsigned)cta);
+                L->smem = smem;
+                L->geom = g;
+                L->key = key ^ (int)L->grid.x * 7919;
+                return SPTRSV_OK;
+            }
+        }
+    }
+    // ---- ENGINE_DYN: persistent, lane slots refilled row by row
+    if ((engine == 2 || engine == 4) && h->plan == PLAN_THREAD && cta <= 256) {
+        const int K = h->rows_per_lane == 3 ? 2 : h->rows_per_lane;
+        const bool stat = engine == 4;
+        const void *fn = (const void *)solve_dyn_kernel(h->proto, K, stat);
+        const size_t smem = (size_t)(cta / 32) * kDynWarpSmem;
+        const int key = 2000000 + h->proto * 100000 + K * 10000 + cta + (stat ? 500 : 0);
+        int cap = 0;
+        int rc = occupancy_grid(h, fn, cta, smem, key, &cap);
+        if (rc) return rc;
+        if (cap >= 1) {
+            long long grid = cap;
+            const long long need = stat ? ((long long)h->n + kDynSub * (cta / 32) - 1) / (kDynSub * (cta / 32))
+                                        : ((long long)h->n + kDynCtaChunk - 1) / kDynCtaChunk;
+            if (grid > need) grid = need;
+            L->fn = fn;
+            L->kind = 0;
+            L->coop = stat;
+            L->grid = dim3((unsigned)(grid > 0 ? grid : 1));
+            L->block = dim3((unsigned)cta);
+            L->smem = smem;
+            L->key = key ^ (int)L->grid.x * 7919;
+            return SPTRSV_OK;
+        }
+    }
+    // ---- ENGINE_LEAN: minimal one-shot kernel for all-thread-level plans
+    if (engine == 3 && h->plan == PLAN_THREAD) {
+        L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED> : (const void *)k_solve_lean<PROTO_FLAGS>;
+        L->kind = 0;
+        L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
+        L->block = dim3((unsigned)kLeanCta);
+        L->smem = 0;
+        L->key = 5000000 + h->proto * 100000;
+        L->key ^= (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
+    // ---- ONE-SHOT, K rows per lane
+    if (h->plan == PLAN_THREAD && h->rows_per_lane > 1 && cta <= 256) {
+        const int K = h->rows_per_lane;
+        const long long rows_per_cta = (long long)(cta / 32) * 32 * K;
+        L->fn = (const void *)solve_k_kernel(h->proto, K);
+        L->kind = 0;
+        L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
+        L->block = dim3((unsigned)cta);
+        L->smem = solve_k_smem_bytes(cta, K);
+        L->key = 3000000 + h->proto * 100000 + K * 10000 + cta;
+        L->key ^= (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
+    // ---- ONE-SHOT (default)
+    const int warps = cta / 32;
+    L->fn = (const void *)solve_kernel(h->plan, h->proto);
+    L->kind = 0;
+    L->grid = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
+    L->block = dim3((unsigned)cta);
+    L->smem = solve_smem_bytes(cta, h->stage && h->plan != PLAN_WARP);
+    L->key = 4000000 + (h->plan * 2 + h->proto) * 100000 + cta;
+    L->key ^= (int)L->grid.x * 7919;
+    return SPTRSV_OK;
+}
+
+}  // namespace
+
 int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!b || !x || b == x) return SPTRSV_ERR_INVALID_ARG;
     cudaStream_t s = (cudaStream_t)stream;
-    if (h->since_reset >= kEpochResetAt) {
-        int rc = reset_state(h, s);
+    const bool aligned =
+        ((((uintptr_t)h->rowptr) | ((uintptr_t)h->colidx) | ((uintptr_t)h->val) | ((uintptr_t)b)) & 15) == 0;
+    Launch L;
+    int rc = plan_launch(h, aligned, &L);
+    if (rc) return rc;
+    // The epoch of a solve is derived on the device from the start ticket and the
+    // grid size (solve.cuh SolveState); a new launch configuration, or an epoch
+    // about to wrap, re-zeroes the flags / records and the counters first.
+    if (L.key != h->launch_key || h->since_reset >= kEpochResetAt) {
+        rc = reset_state(h, s);
         if (rc) return rc;
+        h->launch_key = L.key;
     }
     SolveParams p;
     p.rowptr = h->rowptr;
@@ -382,70 +558,52 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.rec = h->ws.rec;
     p.tasks = h->ws.tasks;
     p.st = h->ws.st;
+    p.nnz = h->nnz;
     p.n = h->n;
     p.n_tasks = h->n_tasks;
+    p.epoch0 = 1;
+    p.grid = L.grid.x;
     p.backoff_min = h->backoff_min;
     p.backoff_max = h->backoff_max;
     p.spin_limit = h->spin_limit;
     p.stage = h->stage;
     p.local = h->local;
     p.trace = h->trace;
-    p.nnz = h->nnz;
-    const bool aligned = ((((uintptr_t)h->rowptr) | ((uintptr_t)h->colidx) | ((uintptr_t)h->val) | ((uintptr_t)b)) & 15) == 0;
-    if (h->engine == 1 && aligned && h->cta_threads >= 64) {
-        const PipeGeom g = pipe_geom(h);
-        const size_t smem = (size_t)g.S * g.stage_bytes;
-        if (smem > (size_t)kPipeMaxSmem) goto oneshot;  // ring does not fit: run the one-shot engine
-        const int key = (h->plan * 2 + h->proto) * 4096 + h->cta_threads + (int)(smem >> 4) * 8192;
-        if (key != h->grid_cache_key) {
-            int per_sm = 0, sms = 0;
-            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pipe_kernel(h->plan, h->proto),
-                                                              h->cta_threads, smem) != cudaSuccess ||
-                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device) != cudaSuccess) {
-                (void)cudaGetLastError();
-                return SPTRSV_ERR_CUDA;
-            }
-            h->grid_cache = per_sm * sms;
-            h->grid_cache_key = key;
-        }
-        if (h->grid_cache < 1) goto oneshot;  // not even one CTA fits: one-shot engine
-        const int rounds = (h->n_tasks + g.W - 1) / g.W;
-        const int grid = rounds < h->grid_cache ? (rounds > 0 ? rounds : 1) : h->grid_cache;
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3((unsigned)grid);
-        cfg.blockDim = dim3((unsigned)h->cta_threads);
-        cfg.dynamicSmemBytes = smem;
-        cfg.stream = s;
-        cfg.numAttrs = 0;
-        const cudaError_t e = cudaLaunchKernelEx(&cfg, pipe_kernel(h->plan, h->proto), p, g);
-        if (e != cudaSuccess) {
-            (void)cudaGetLastError();
-            return SPTRSV_ERR_CUDA;
-        }
-        h->solves++;
-        h->since_reset++;
-        return SPTRSV_OK;
-    }
-oneshot:
-    const int warps = h->cta_threads / 32;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
-    cfg.blockDim = dim3((unsigned)h->cta_threads);
-    cfg.dynamicSmemBytes = solve_smem_bytes(h->cta_threads, h->stage && h->plan != PLAN_WARP);
+    cfg.gridDim = L.grid;
+    cfg.blockDim = L.block;
+    cfg.dynamicSmemBytes = L.smem;
     cfg.stream = s;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     cfg.numAttrs = 0;
-    if (h->l2_window) {
-        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-        attr[0].val.accessPolicyWindow.base_ptr = h->ws.flags;
-        attr[0].val.accessPolicyWindow.num_bytes = sizeof(uint32_t) * (size_t)h->n;
-        attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
-        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
+    cfg.attrs = attr;
+    if (L.coop) {
+        attr[cfg.numAttrs].id = cudaLaunchAttributeCooperative;
+        attr[cfg.numAttrs].val.cooperative = 1;
+        cfg.numAttrs++;
     }
-    const cudaError_t e = cudaLaunchKernelEx(&cfg, solve_kernel(h->plan, h->proto), p);
+    if (h->l2_window && h->proto == PROTO_FLAGS) {
+        cudaLaunchAttribute &a = attr[cfg.numAttrs++];
+        a.id = cudaLaunchAttributeAccessPolicyWindow;
+        a.val.accessPolicyWindow.base_ptr = h->ws.flags;
+        a.val.accessPolicyWindow.num_bytes = sizeof(uint32_t) * (size_t)h->n;
+        a.val.accessPolicyWindow.hitRatio = 1.0f;
+        a.val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        a.val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    } else if (h->l2_window && h->ws.rec) {
+        cudaLaunchAttribute &a = attr[cfg.numAttrs++];
+        a.id = cudaLaunchAttributeAccessPolicyWindow;
+        a.val.accessPolicyWindow.base_ptr = h->ws.rec;
+        a.val.accessPolicyWindow.num_bytes = 16 * (size_t)h->n;
+        a.val.accessPolicyWindow.hitRatio = 1.0f;
+        a.val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        a.val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    }
+    cudaError_t e;
+    if (L.kind == 1)
+        e = cudaLaunchKernelEx(&cfg, (void (*)(SolveParams, PipeGeom))L.fn, p, L.geom);
+    else
+        e = cudaLaunchKernelEx(&cfg, (void (*)(SolveParams))L.fn, p);
     if (e != cudaSuccess) {
         (void)cudaGetLastError();
         return SPTRSV_ERR_CUDA;
@@ -555,7 +713,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->local = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
-            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 5) return SPTRSV_ERR_INVALID_ARG;
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_STAGES:
@@ -569,6 +727,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
         case SPTRSV_OPT_PIPE_ENTRIES:
             if (value < 0 || value > (1 << 16)) return SPTRSV_ERR_INVALID_ARG;
             h->pipe_entries = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_ROWS_PER_LANE:
+            if (value < 1 || value > 4) return SPTRSV_ERR_INVALID_ARG;
+            h->rows_per_lane = (int)value;
             return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
@@ -592,6 +754,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_PIPE_STAGES: *value = h->pipe_stages; return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_BATCH: *value = h->pipe_batch; return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_ENTRIES: *value = h->pipe_entries; return SPTRSV_OK;
+        case SPTRSV_OPT_ROWS_PER_LANE: *value = h->rows_per_lane; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }
@@ -607,6 +770,8 @@ int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
     out->device = h->device;
     out->analyse_ms = h->analyse_ms;
     out->solves = h->solves;
+    out->near_deps = h->near_deps;
+    out->engine = resolve_engine(h);
     return SPTRSV_OK;
 }
 
@@ -659,6 +824,8 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
     CK(cudaMemcpy(&err, &h->ws.st->error.v, sizeof(uint32_t), cudaMemcpyDeviceToHost));
     if (err) {
         CK(cudaMemset(&h->ws.st->error.v, 0, sizeof(uint32_t)));
+        CK(cudaMemset(&h->ws.st->abort.v, 0, sizeof(uint32_t)));
+        h->launch_key = -1;  // flags of the aborted solve are partial: re-zero before the next one
         return SPTRSV_ERR_TIMEOUT;
     }
     return SPTRSV_OK;

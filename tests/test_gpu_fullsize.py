@@ -27,23 +27,24 @@ def _run(s, **opt):
         return x1, x.cpu().numpy(), h.info()
 
 
-@pytest.mark.parametrize("proto", [0, 1])
-def test_c2_full(proto):
+@pytest.mark.parametrize("proto,K,engine", [(0, 1, 0), (1, 1, 0), (1, 2, 0), (1, 4, 0), (1, 1, 2), (1, 2, 2),
+                                             (0, 2, 2)])
+def test_c2_full(proto, K, engine):
     s = synth.gen_c2()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x1, x2, info = _run(s, protocol=proto)
+    x1, x2, info = _run(s, protocol=proto, rows_per_lane=K, engine=engine)
     assert info["n_warp_rows"] == 0  # 2.8 nnz/row -> thread level everywhere
     assert np.array_equal(x1, ref) and np.array_equal(x2, ref)
 
 
-@pytest.mark.parametrize("proto", [0, 1])
-def test_c3_full_ones_and_random(proto):
+@pytest.mark.parametrize("proto,K", [(0, 1), (1, 1), (1, 4)])
+def test_c3_full_ones_and_random(proto, K):
     s = synth.gen_c3(ones=True)
-    x1, x2, _ = _run(s, protocol=proto)
+    x1, x2, _ = _run(s, protocol=proto, rows_per_lane=K)
     assert np.array_equal(x1, np.ones(s.n)) and np.array_equal(x2, np.ones(s.n))
     s = synth.gen_c3()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    x1, _, _ = _run(s, protocol=proto)
+    x1, _, _ = _run(s, protocol=proto, rows_per_lane=K)
     assert np.array_equal(x1, ref)
 
 

@@ -286,6 +286,75 @@ def test_pipe_geometry_variants(cap, stages, batch, entries, cta):
             assert relerr(x, ref) <= TOL
 
 
+@pytest.mark.parametrize("K", [2, 3, 4])
+@pytest.mark.parametrize("proto", PROTOS)
+def test_rows_per_lane(cap, K, proto):
+    """K thread-level rows per lane (coarsened Writing-First): bit-exact like K = 1."""
+    for n in (1, 31, 33, 200, 4099):
+        s = synth.gen_random_lower(n, 4, seed=n + 7)
+        x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K)
+        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
+    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=100_000), lambda: synth.gen_grid(300),
+                lambda: synth.gen_chain(20_000), lambda: synth.gen_dense_lower(120)):
+        s = gen()
+        for local, cta in ((1, 256), (0, 256), (1, 128), (1, 64)):
+            x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K, local=local, cta_threads=cta)
+            assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), (s.name, local, cta)
+    si = synth.integerize(synth.gen_c2i(n=50_000))
+    x, _ = gpu_solve(cap, si, 1, protocol=proto, rows_per_lane=K)
+    assert np.array_equal(x, si.x_true)
+
+
+@pytest.mark.parametrize("K", [1, 2, 4])
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("engine", [2, 4])
+def test_dyn_engine(cap, K, proto, engine):
+    """ENGINE_DYN (rows re-assigned to lane slots as they finish): bit-exact like the others."""
+    for n in (1, 31, 33, 129, 200, 4099):
+        s = synth.gen_random_lower(n, 4, seed=n + 11)
+        x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K, engine=engine)
+        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
+    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=300_000), lambda: synth.gen_grid(200),
+                lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100)):
+        s = gen()
+        for cta in (256, 64):
+            x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K, engine=engine, cta_threads=cta)
+            assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), (s.name, cta)
+    si = synth.integerize(synth.gen_c2i(n=50_000))
+    x, _ = gpu_solve(cap, si, 1, protocol=proto, rows_per_lane=K, engine=engine)
+    assert np.array_equal(x, si.x_true)
+
+
+@pytest.mark.parametrize("proto", PROTOS)
+def test_lean_engine(cap, proto):
+    """ENGINE_LEAN (no staging, speculative rows): bit-exact like the others."""
+    for n in (1, 31, 33, 255, 257, 4099):
+        s = synth.gen_random_lower(n, 4, seed=n + 13)
+        x, _ = gpu_solve(cap, s, 1, protocol=proto, engine=3)
+        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
+    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=300_000), lambda: synth.gen_grid(200),
+                lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100), lambda: synth.gen_diag(70_001)):
+        s = gen()
+        x, _ = gpu_solve(cap, s, 1, protocol=proto, engine=3)
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        assert np.array_equal(x, ref), s.name
+    si = synth.integerize(synth.gen_c2i(n=50_000))
+    x, _ = gpu_solve(cap, si, 1, protocol=proto, engine=3)
+    assert np.array_equal(x, si.x_true)
+
+
+def test_engine_auto_choice(cap):
+    """ENGINE_AUTO: far dependencies -> LEAN (3); chains / grid wavefronts -> staged one-shot (0)."""
+    for gen, want in ((lambda: synth.gen_c2(n=100_000), 3), (lambda: synth.gen_grid(100), 0),
+                      (lambda: synth.gen_chain(3000), 0), (lambda: synth.gen_diag(5000), 3),
+                      (lambda: synth.gen_c4(n=5000, nlevels=50), 0)):
+        s = gen()
+        x, info = gpu_solve(cap, s)
+        assert info["engine"] == want, (s.name, info)
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        assert relerr(x, ref) <= TOL
+
+
 def test_pipe_unaligned_b_falls_back(cap):
     """b at an 8-byte (not 16-byte) offset: the TMA ring needs 16-byte alignment -> one-shot engine."""
     s = synth.gen_c2(n=20_000)

@@ -17,8 +17,15 @@ for _ in range(3):
     h.solve(b, x)
 h.check()
 x, tr = h.trace(b, x)
-t = tr.cpu().numpy().astype(np.int64)
-t = t - t.min()
+tt = tr.cpu().numpy().astype(np.int64)
+t0 = tt[: s.n].min()
+if tt.size >= 3 * s.n + 3 and tt[3 * s.n + 1] > 0:
+    print(json.dumps({"kernel_entry_to_first_publish_us": round((t0 - tt[3 * s.n]) / 1e3, 2),
+                      "last_publish_to_last_exit_us": round((tt[3 * s.n + 1] - tt[: s.n].max()) / 1e3, 2),
+                      "ctas": int(tt[3 * s.n + 2])}))
+t = tt[: s.n] - t0
+seen = np.where(tt[s.n:2 * s.n] > 0, tt[s.n:2 * s.n] - t0, -1)
+start = np.where(tt[2 * s.n:3 * s.n] > 0, tt[2 * s.n:3 * s.n] - t0, -1)
 lv = oracle.levels_dp(s.rowptr, s.colidx)
 nl = int(lv.max()) + 1
 # completion time of each level = max publish time of its rows
@@ -52,3 +59,25 @@ if name == "c3":
     print(json.dumps({"c3_row_start_us": [round(float(row_start[r]) / 1e3, 1) for r in range(0, g, 128)],
                       "c3_row_end_us": [round(float(row_end[r]) / 1e3, 1) for r in range(0, g, 128)],
                       "row0_cells_us": [round(float(T[0, c]) / 1e3, 2) for c in range(0, 2048, 128)]}))
+# ---- reaction time: publish(i) - max publish(dependencies of i), per row (the hop under load)
+rp, ci = s.rowptr.astype(np.int64), s.colidx.astype(np.int64)
+rows = np.repeat(np.arange(s.n), np.diff(rp))
+off = ci != rows
+dep_t = np.zeros(s.n, np.int64)
+np.maximum.at(dep_t, rows[off], t[ci[off]])
+has = np.bincount(rows[off], minlength=s.n) > 0
+react = (t - dep_t)[has]
+sv = seen[has]
+okm = sv >= 0
+vis = (sv - dep_t[has])[okm]       # dependency published -> seen ready by the consumer
+proc = (t[has] - sv)[okm]          # seen ready -> consumer published
+st_h = start[has]
+wait_before_start = (st_h - dep_t[has])[st_h >= 0]  # > 0: the consumer started after its dep was published
+print(json.dumps({"consumer_started_after_dep_frac": round(float((wait_before_start > 0).mean()), 3) if wait_before_start.size else None,
+                  "start_minus_dep_ns_p10_50_90": [int(np.percentile(wait_before_start, q)) for q in (10, 50, 90)] if wait_before_start.size else None,
+                  "row_start_us_by_decile": [round(float(np.percentile(start[start >= 0], q)) / 1e3, 2) for q in range(0, 101, 10)] if (start >= 0).any() else None}))
+print(json.dumps({"visibility_ns_p10_50_90": [int(np.percentile(vis, q)) for q in (10, 50, 90)] if okm.any() else None,
+                  "seen_to_publish_ns_p10_50_90": [int(np.percentile(proc, q)) for q in (10, 50, 90)] if okm.any() else None}))
+print(json.dumps({"react_ns_p10_50_90_99": [int(np.percentile(react, q)) for q in (10, 50, 90, 99)],
+                  "nodep_publish_us_p10_50_90_max": [round(float(np.percentile(t[~has], q)) / 1e3, 2) for q in (10, 50, 90, 100)] if (~has).any() else None,
+                  "frac_react_gt_2us": round(float((react > 2000).mean()), 4)}))
