@@ -383,6 +383,7 @@ def main():
                        "plan": {"thread_groups": info["n_thread_groups"], "warp_rows": info["n_warp_rows"]},
                        "engine": {0: "one-shot (staged, in-CTA x copy)", 1: "pipe (TMA ring)", 2: "dyn",
                                   3: "lean", 4: "dyn-static"}.get(info["engine"], str(info["engine"])),
+                       "cta_threads": info["cta_threads"], "rows_per_lane": info["rows_per_lane"],
                        "analyse_ms": round(info["analyse_ms"], 3),
                        "l2": "flushed between timed steps (256 MiB write, outside the per-step events)",
                        "parallelism": f"replicas x{world}" if args.config != "c5" else f"systems sharded over {world}",

@@ -59,8 +59,9 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_WARP_THRESHOLD = 2, /* AUTO: a 32-row group goes warp-level when its mean
                                       nnz/row exceeds this (default 16; sec.4.4, DESIGN G10).
                                       Setting it re-plans (synchronous).                    */
-    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 64, 128, 256 (default), 512, 1024; the
-                                      PIPE engine uses one of the warps as its loader       */
+    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 64, 128, 256, 512, 1024, or 0 (default)
+                                      = the engine's measured best; the PIPE engine uses one
+                                      of the warps as its loader                            */
     SPTRSV_OPT_BACKOFF_MIN_NS = 4, /* __nanosleep after a pass where no lane progressed     */
     SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
     SPTRSV_OPT_SPIN_LIMIT = 6,     /* watchdog: idle passes per warp before TIMEOUT (0=off) */
@@ -93,8 +94,9 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
     SPTRSV_OPT_PIPE_ENTRIES = 14,  /* PIPE colidx/val entries per stage (0 = 4 per row)     */
     SPTRSV_OPT_ROWS_PER_LANE = 15  /* K = 1..4 thread-level rows per lane (lane owns rows
-                                      r0+lane+32k); applies to all-thread-level plans on
-                                      the ONE-SHOT engine with CTAs of <= 256 threads      */
+                                      r0+lane+32k), or 0 (default) = the engine's measured
+                                      best; applies to all-thread-level plans on the
+                                      ONE-SHOT engine with CTAs of <= 256 threads          */
 } sptrsv_option;
 
 typedef struct sptrsv_info {
@@ -109,6 +111,8 @@ typedef struct sptrsv_info {
     uint32_t solves;          /* solves enqueued through this handle                      */
     int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
     int32_t engine;           /* engine the next solve uses (AUTO resolved)                */
+    int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
+    int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
 } sptrsv_info;
 
 /*

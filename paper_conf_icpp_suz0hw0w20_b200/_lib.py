@@ -66,6 +66,8 @@ class sptrsv_info(ctypes.Structure):
         ("solves", ctypes.c_uint32),
         ("near_deps", ctypes.c_int64),
         ("engine", ctypes.c_int32),
+        ("cta_threads", ctypes.c_int32),
+        ("rows_per_lane", ctypes.c_int32),
     ]
 
 

@@ -58,7 +58,7 @@ struct sptrsv_handle_s {
     // options
     int mode = 0;
     int threshold = 16;
-    int cta_threads = 256;
+    int cta_threads = 0;    // 0 = per-engine default (see effective_geometry)
     uint32_t backoff_min = 0;
     uint32_t backoff_max = 256;
     uint32_t spin_limit = 1u << 24;
@@ -70,7 +70,7 @@ struct sptrsv_handle_s {
     int pipe_stages = 3;
     int pipe_batch = 1;  // (kept for the ABI; the loader takes one round per ticket)
     int pipe_entries = 0;   // 0 = 4 per row of a round
-    int rows_per_lane = 1;  // K: thread-level rows per lane (all-thread plans, one-shot engine)
+    int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
     int grid_cache_key = -1;
     int grid_cache = 0;
     int launch_key = -1;  // configuration of the last launch (see sptrsv_solve)
@@ -142,9 +142,9 @@ pipe_fn pipe_kernel(int plan, int proto) {
 int round16(int b) { return (b + 15) & ~15; }
 constexpr int kPipeMaxSmem = 200 * 1024;  // ring bytes per CTA, at most (227 KB minus static smem and slack)
 
-PipeGeom pipe_geom(const sptrsv_handle_s *h) {
+PipeGeom pipe_geom(const sptrsv_handle_s *h, int cta) {
     PipeGeom g;
-    g.W = h->cta_threads / 32 - 1;
+    g.W = cta / 32 - 1;
     g.S = h->pipe_stages;
     g.B = h->pipe_batch;
     g.RB = 32 * g.W;
@@ -441,12 +441,32 @@ int resolve_engine(const sptrsv_handle_s *h) {
     return 0;
 }
 
+// CTA size and rows per lane actually used: the user's values, else the
+// per-engine defaults measured best on B200 in round 1:
+// staged one-shot on near-dependency thread-level plans (grid wavefronts,
+// chains): 2 rows per lane in 128-thread CTAs; on plans with warp-level rows:
+// 64-thread CTAs; everything else 256 threads, 1 row per lane.
+void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) {
+    int c = 256, k = 1;
+    if (engine == 0) {
+        if (h->plan == PLAN_THREAD && h->nnz > h->n && 4 * h->near_deps >= h->nnz - h->n) {
+            c = 128;
+            k = 2;
+        } else if (h->plan != PLAN_THREAD) {
+            c = 64;
+        }
+    }
+    *cta = h->cta_threads ? h->cta_threads : c;
+    *K = h->rows_per_lane ? h->rows_per_lane : k;
+}
+
 int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
-    const int cta = h->cta_threads;
     const int engine = resolve_engine(h);
+    int cta = 256, Kq = 1;
+    effective_geometry(h, engine, &cta, &Kq);
     // ---- ENGINE_PIPE: persistent, loader warp + TMA ring
     if (engine == 1 && aligned && cta >= 64) {
-        const PipeGeom g = pipe_geom(h);
+        const PipeGeom g = pipe_geom(h, cta);
         const size_t smem = (size_t)g.S * g.stage_bytes;
         if (smem <= (size_t)kPipeMaxSmem) {
             const void *fn = (const void *)pipe_kernel(h->plan, h->proto);
@@ -469,7 +489,7 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
     }
     // ---- ENGINE_DYN: persistent, lane slots refilled row by row
     if ((engine == 2 || engine == 4) && h->plan == PLAN_THREAD && cta <= 256) {
-        const int K = h->rows_per_lane == 3 ? 2 : h->rows_per_lane;
+        const int K = Kq == 3 ? 2 : Kq;
         const bool stat = engine == 4;
         const void *fn = (const void *)solve_dyn_kernel(h->proto, K, stat);
         const size_t smem = (size_t)(cta / 32) * kDynWarpSmem;
@@ -504,8 +524,8 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
         return SPTRSV_OK;
     }
     // ---- ONE-SHOT, K rows per lane
-    if (h->plan == PLAN_THREAD && h->rows_per_lane > 1 && cta <= 256) {
-        const int K = h->rows_per_lane;
+    if (engine == 0 && h->plan == PLAN_THREAD && Kq > 1 && cta <= 256) {
+        const int K = Kq;
         const long long rows_per_cta = (long long)(cta / 32) * 32 * K;
         L->fn = (const void *)solve_k_kernel(h->proto, K);
         L->kind = 0;
@@ -663,7 +683,8 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->threshold = (int)value;
             return build_plan(h);
         case SPTRSV_OPT_CTA_THREADS:
-            if (value != 64 && value != 128 && value != 256 && value != 512 && value != 1024) return SPTRSV_ERR_INVALID_ARG;
+            if (value != 0 && value != 64 && value != 128 && value != 256 && value != 512 && value != 1024)
+                return SPTRSV_ERR_INVALID_ARG;
             h->cta_threads = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_BACKOFF_MIN_NS:
@@ -729,7 +750,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->pipe_entries = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE:
-            if (value < 1 || value > 4) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 4) return SPTRSV_ERR_INVALID_ARG;
             h->rows_per_lane = (int)value;
             return SPTRSV_OK;
         default:
@@ -772,6 +793,7 @@ int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
     out->solves = h->solves;
     out->near_deps = h->near_deps;
     out->engine = resolve_engine(h);
+    effective_geometry(h, out->engine, &out->cta_threads, &out->rows_per_lane);
     return SPTRSV_OK;
 }
 

@@ -345,12 +345,12 @@ def test_lean_engine(cap, proto):
 
 def test_engine_auto_choice(cap):
     """ENGINE_AUTO: far dependencies -> LEAN (3); chains / grid wavefronts -> staged one-shot (0)."""
-    for gen, want in ((lambda: synth.gen_c2(n=100_000), 3), (lambda: synth.gen_grid(100), 0),
-                      (lambda: synth.gen_chain(3000), 0), (lambda: synth.gen_diag(5000), 3),
-                      (lambda: synth.gen_c4(n=5000, nlevels=50), 0)):
+    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 0, 128, 2),
+                              (lambda: synth.gen_chain(3000), 0, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
+                              (lambda: synth.gen_c4(n=5000, nlevels=50), 0, 64, 1)):
         s = gen()
         x, info = gpu_solve(cap, s)
-        assert info["engine"] == want, (s.name, info)
+        assert (info["engine"], info["cta_threads"], info["rows_per_lane"]) == (want, cta, K), (s.name, info)
         ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
         assert relerr(x, ref) <= TOL
 
