@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--profile", action="store_true", help="short run for ncu: no clocks/e2e/cpu legs")
     ap.add_argument("--opt", action="append", default=[], help="extra handle option key=value")
     ap.add_argument("--no-flags-leg", action="store_true", help="skip the FLAGS-protocol comparison leg")
+    ap.add_argument("--nrhs", type=int, default=8, help="right-hand sides of the multi-RHS leg (0 = skip)")
     return ap.parse_args()
 
 
@@ -309,6 +310,41 @@ def main():
                      "value": round(2.0 * nnz_all * args.steps / ft / 1e9, 3), "unit": UNIT,
                      "ms_per_step": round(ft / args.steps * 1e3, 5)}
 
+    # ---- multi-RHS leg: sptrsv_solve_multi with nrhs right-hand sides, same timing rules
+    multi_leg = None
+    if args.nrhs > 0 and not args.profile:
+        Bs = [torch.from_numpy(np.ascontiguousarray(np.repeat(s.b[:, None], args.nrhs, axis=1)
+                                                    * (1.0 + np.arange(args.nrhs)[None, :]))).to(dev)
+              for s in systems]
+        Xs = [torch.empty_like(B) for B in Bs]
+        for i in range(args.warmup):
+            flush.zero_()
+            for h, B, X in zip(handles, Bs, Xs):
+                h.solve_multi(B, X, stream=stream)
+        ev3 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            flush.zero_()
+            ev3[i][0].record(stream)
+            for h, B, X in zip(handles, Bs, Xs):
+                h.solve_multi(B, X, stream=stream)
+            ev3[i][1].record(stream)
+        torch.cuda.synchronize()
+        for h in handles:
+            h.check(stream)
+        mt = float(np.sum([a.elapsed_time(b) for a, b in ev3])) * 1e-3
+        if dist:
+            t = torch.tensor([mt], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            mt = float(t.item())
+        ok = bool(torch.equal(Xs[0][:, 0], bufs[0][4]))  # column 0 = the single-RHS solve of b
+        multi_leg = {"nrhs": args.nrhs, "value": round(2.0 * nnz_all * args.nrhs * args.steps / mt / 1e9, 3),
+                     "unit": UNIT, "ms_per_step": round(mt / args.steps * 1e3, 5),
+                     "column0_matches_single_rhs": ok,
+                     "layout": "row-major B[i*nrhs + r], r-th column = (r+1) * b"}
+
     # ---- roofline of the dominant (only) kernel, k_solve
     peak, peak_src = peaks()
     alg_bytes = systems[0].alg_bytes()
@@ -391,6 +427,7 @@ def main():
             "protocol": {1: "fused (epoch-tagged 16-byte value records, no fences)",
                          0: "flags (st.release.gpu / ld.acquire.gpu)"}[opts.get("protocol", 1)],
             "flags_protocol_leg": flags_leg,
+            "multi_rhs_leg": multi_leg,
             "roofline": roof,
             "latency_bound": lat,
             "e2e": e2e,

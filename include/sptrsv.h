@@ -152,6 +152,18 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
 int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream);
 
 /*
+ * sptrsv_solve_multi -- L X = B for nrhs right-hand sides at once (SURVEY row
+ * f1; "multiple right-hand sides [21]"): one dependency hop per
+ * row serves all nrhs solves.  Row-major: B[i*ldb + r], X[i*ldx + r],
+ * 1 <= nrhs <= 32, ldb, ldx >= nrhs; B and X device, must not alias.  Same
+ * protocol option and options as sptrsv_solve; asynchronous, one launch.
+ * Each component (i, r) has its own ready word, so the handle keeps
+ * n * nrhs of them (allocated on first use).
+ */
+int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nrhs, int64_t ldb, int64_t ldx,
+                       sptrsv_stream_t stream);
+
+/*
  * sptrsv_solve_host -- end-to-end convenience: copies b (host) to handle-owned
  * device staging, solves, copies x back to host, and synchronises `stream`.
  * b_host/x_host: host double[n] (pinned memory gives full PCIe bandwidth).

@@ -11,6 +11,7 @@ What is here (each function cites the passage it follows):
 
 * :func:`validate`      -- the CSR shape Alg. 1 assumes
 * :func:`solve`         -- Algorithm 1, sequential forward substitution
+* :func:`solve_multi`   -- Algorithm 1 per column of B (multiple right-hand sides)
 * :func:`indegree`      -- dependencies per component
 * :func:`levels_dp`     -- level of each component, row-order recurrence
 * :func:`levels_bfs`    -- the same levels by Kahn's BFS (independent algorithm)
@@ -111,6 +112,16 @@ def solve(rowptr, colidx, val, b):
     if n > 0:
         _get().oracle_solve(n, rp, ci, v, bb, x)
     return x[:n]
+
+
+def solve_multi(rowptr, colidx, val, B):
+    """Multiple right-hand sides: Algorithm 1 applied to each
+    column of B (n x nrhs) independently -- the definition of X = L^{-1} B column by column."""
+    B = np.asarray(B, dtype=np.float64)
+    X = np.empty_like(B)
+    for r in range(B.shape[1]):
+        X[:, r] = solve(rowptr, colidx, val, np.ascontiguousarray(B[:, r]))
+    return X
 
 
 def indegree(rowptr, colidx):

@@ -79,6 +79,23 @@ class Handle:
             check(lib.sptrsv_solve(self._h, b.data_ptr(), x.data_ptr(), _stream_ptr(stream)), "sptrsv_solve")
         return x
 
+    def solve_multi(self, B, X=None, stream=None):
+        """X <- L^{-1} B for B of shape (n, nrhs) (row-major rows, nrhs <= 32), one launch."""
+        import torch
+        if not isinstance(B, torch.Tensor) or not B.is_cuda or B.dtype != torch.float64 or B.dim() != 2:
+            raise TypeError("B must be a 2-D float64 CUDA tensor")
+        if B.shape[0] != self.n or B.stride(1) != 1:
+            raise ValueError("B must be (n, nrhs) with unit column stride")
+        nrhs = B.shape[1]
+        if X is None:
+            X = torch.empty_like(B)
+        if X.shape != B.shape or X.stride(1) != 1 or X.dtype != torch.float64 or not X.is_cuda:
+            raise ValueError("X must match B")
+        if self.n and nrhs:
+            check(lib.sptrsv_solve_multi(self._h, B.data_ptr(), X.data_ptr(), nrhs, B.stride(0), X.stride(0),
+                                         _stream_ptr(stream)), "sptrsv_solve_multi")
+        return X
+
     def solve_host(self, b_host, x_host, stream=None):
         """End to end from host buffers (numpy float64 or pinned CPU tensors); synchronous."""
         import numpy as np

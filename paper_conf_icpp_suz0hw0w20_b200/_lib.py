@@ -79,6 +79,7 @@ EXPORTS = {
     "sptrsv_analyse_csr": (ctypes.c_int, [_i32, _p, _p, _p, ctypes.POINTER(_h)]),
     "sptrsv_solve": (ctypes.c_int, [_h, _p, _p, _p]),
     "sptrsv_solve_host": (ctypes.c_int, [_h, _p, _p, _p]),
+    "sptrsv_solve_multi": (ctypes.c_int, [_h, _p, _p, _i32, _i64, _i64, _p]),
     "sptrsv_destroy": (ctypes.c_int, [_h]),
     "sptrsv_set_option": (ctypes.c_int, [_h, ctypes.c_int, _i64]),
     "sptrsv_get_option": (ctypes.c_int, [_h, ctypes.c_int, ctypes.POINTER(_i64)]),

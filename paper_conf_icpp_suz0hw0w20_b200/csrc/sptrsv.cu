@@ -18,6 +18,7 @@
 #include "solve_k.cuh"
 #include "solve_dyn.cuh"
 #include "solve_lean.cuh"
+#include "solve_multi.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -34,6 +35,10 @@ struct Workspace {
     SolveState *st = nullptr;      // 1
     uint32_t *lvl = nullptr;       // n (levels diagnostic, lazy)
     double *b_stage = nullptr;     // n (solve_host, lazy)
+    SolveState *mst = nullptr;     // multi-RHS: own solve state (own epoch sequence)
+    uint32_t *mflags = nullptr;    // multi-RHS: n * mcap flags (FLAGS)
+    unsigned long long *mrec = nullptr;  // multi-RHS: n * mcap records (FUSED)
+    int64_t mcap = 0;              // right-hand sides the multi buffers hold
     double *x_stage = nullptr;     // n (solve_host, lazy)
 };
 
@@ -74,6 +79,8 @@ struct sptrsv_handle_s {
     int grid_cache_key = -1;
     int grid_cache = 0;
     int launch_key = -1;  // configuration of the last launch (see sptrsv_solve)
+    long long mlaunch_key = -1;  // same for sptrsv_solve_multi
+    uint32_t msince_reset = 0;
     unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
@@ -198,6 +205,9 @@ void free_ws(Workspace &w) {
     cudaFree(w.st);
     cudaFree(w.lvl);
     cudaFree(w.b_stage);
+    cudaFree(w.mst);
+    cudaFree(w.mflags);
+    cudaFree(w.mrec);
     cudaFree(w.x_stage);
     w = Workspace();
 }
@@ -633,6 +643,78 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     return SPTRSV_OK;
 }
 
+int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nrhs, int64_t ldb, int64_t ldx,
+                       sptrsv_stream_t stream) {
+    if (!h) return SPTRSV_ERR_INVALID_ARG;
+    if (nrhs < 1 || nrhs > 32 || ldb < nrhs || ldx < nrhs) return SPTRSV_ERR_INVALID_ARG;
+    if (h->n == 0) return SPTRSV_OK;
+    if (!B || !X || (const double *)X == B) return SPTRSV_ERR_INVALID_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t words = (size_t)h->n * (size_t)nrhs;
+    if (nrhs > h->ws.mcap) {  // (re)allocate the per-component ready words
+        cudaFree(h->ws.mflags);
+        cudaFree(h->ws.mrec);
+        h->ws.mflags = nullptr;
+        h->ws.mrec = nullptr;
+        if ((!h->ws.mst && cudaMalloc(&h->ws.mst, sizeof(SolveState)) != cudaSuccess) ||
+            cudaMalloc(&h->ws.mflags, 4 * words) != cudaSuccess || cudaMalloc(&h->ws.mrec, 16 * words) != cudaSuccess) {
+            (void)cudaGetLastError();
+            h->ws.mcap = 0;
+            return SPTRSV_ERR_ALLOC;
+        }
+        h->ws.mcap = nrhs;
+        h->mlaunch_key = -1;
+    }
+    int g = 1;
+    while (g < nrhs) g *= 2;
+    const int rows_per_cta = 256 / g;
+    const unsigned grid = (unsigned)((h->n + rows_per_cta - 1) / rows_per_cta);
+    const long long key = ((long long)grid << 8) | ((long long)nrhs << 1) | h->proto;
+    if (key != h->mlaunch_key || h->msince_reset >= kEpochResetAt) {
+        CK(cudaMemsetAsync(h->ws.mflags, 0, 4 * words, s));
+        CK(cudaMemsetAsync(h->ws.mrec, 0, 16 * words, s));
+        CK(cudaMemsetAsync(h->ws.mst, 0, sizeof(SolveState), s));
+        h->mlaunch_key = key;
+        h->msince_reset = 0;
+    }
+    SolveParams p = {};
+    p.rowptr = h->rowptr;
+    p.colidx = h->colidx;
+    p.val = h->val;
+    p.flags = h->ws.mflags;
+    p.rec = h->ws.mrec;
+    p.st = h->ws.mst;
+    p.nnz = h->nnz;
+    p.n = h->n;
+    p.n_tasks = h->n_tasks;
+    p.epoch0 = 1;
+    p.grid = grid;
+    p.backoff_min = h->backoff_min;
+    p.backoff_max = h->backoff_max;
+    p.spin_limit = h->spin_limit;
+    MultiParams m;
+    m.B = B;
+    m.X = X;
+    m.ldb = ldb;
+    m.ldx = ldx;
+    m.nrhs = nrhs;
+    m.g = g;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(256);
+    cfg.stream = s;
+    cfg.numAttrs = 0;
+    const cudaError_t e = h->proto ? cudaLaunchKernelEx(&cfg, k_solve_multi<PROTO_FUSED>, p, m)
+                                   : cudaLaunchKernelEx(&cfg, k_solve_multi<PROTO_FLAGS>, p, m);
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_CUDA;
+    }
+    h->solves++;
+    h->msince_reset++;
+    return SPTRSV_OK;
+}
+
 int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, sptrsv_stream_t stream) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
@@ -842,8 +924,16 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     cudaStream_t s = (cudaStream_t)stream;
     CK(cudaStreamSynchronize(s));
-    uint32_t err = 0;
+    uint32_t err = 0, merr = 0;
     CK(cudaMemcpy(&err, &h->ws.st->error.v, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+    if (h->ws.mst) {
+        CK(cudaMemcpy(&merr, &h->ws.mst->error.v, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+        if (merr) {
+            CK(cudaMemset(h->ws.mst, 0, sizeof(SolveState)));
+            h->mlaunch_key = -1;
+            return SPTRSV_ERR_TIMEOUT;
+        }
+    }
     if (err) {
         CK(cudaMemset(&h->ws.st->error.v, 0, sizeof(uint32_t)));
         CK(cudaMemset(&h->ws.st->abort.v, 0, sizeof(uint32_t)));

@@ -355,6 +355,33 @@ def test_engine_auto_choice(cap):
         assert relerr(x, ref) <= TOL
 
 
+@pytest.mark.parametrize("nrhs", [1, 2, 3, 4, 7, 8, 16, 32])
+@pytest.mark.parametrize("proto", PROTOS)
+def test_multi_rhs(cap, nrhs, proto):
+    """sptrsv_solve_multi (f1): every column bit-exact vs the oracle (thread-level arithmetic)."""
+    rng = np.random.default_rng(nrhs)
+    for gen in (lambda: synth.gen_random_lower(1001, 4, seed=5), lambda: synth.gen_c2i(n=60_000),
+                lambda: synth.gen_grid(64), lambda: synth.gen_c4(n=3000, nlevels=30)):
+        s = gen()
+        B = rng.uniform(-1, 1, (s.n, nrhs))
+        ref = oracle.solve_multi(s.rowptr, s.colidx, s.val, B)
+        rp, ci, v, _ = dev_csr(s)
+        with cap.analyse(rp, ci, v, protocol=proto) as h:
+            X = torch.full((s.n, nrhs), float("nan"), dtype=torch.float64, device="cuda:0")
+            h.solve_multi(torch.from_numpy(B).cuda(), X)
+            h.check()
+            assert np.array_equal(X.cpu().numpy(), ref), s.name
+            # padded leading dimensions, and a single solve in between (separate epochs)
+            Bp = torch.zeros((s.n, nrhs + 3), dtype=torch.float64, device="cuda:0")
+            Bp[:, :nrhs] = torch.from_numpy(B).cuda()
+            Xp = torch.full((s.n, nrhs + 5), float("nan"), dtype=torch.float64, device="cuda:0")
+            h.solve(torch.from_numpy(s.b).cuda())
+            h.solve_multi(Bp[:, :nrhs], Xp[:, :nrhs])
+            h.check()
+            assert np.array_equal(Xp[:, :nrhs].cpu().numpy(), ref)
+            assert torch.isnan(Xp[:, nrhs:]).all()
+
+
 def test_pipe_unaligned_b_falls_back(cap):
     """b at an 8-byte (not 16-byte) offset: the TMA ring needs 16-byte alignment -> one-shot engine."""
     s = synth.gen_c2(n=20_000)

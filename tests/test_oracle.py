@@ -134,6 +134,25 @@ def test_solve_componentwise_backward_error():
     assert np.max(r / denom) <= 2 * k * u / (1 - k * u)
 
 
+@pytest.mark.parametrize("n,nrhs", [(1, 1), (40, 3), (200, 8)])
+def test_solve_multi_matches_lapack(n, nrhs):
+    """Multi-RHS oracle vs LAPACK dtrtrs with a matrix right-hand side (one call, all columns)."""
+    s = synth.gen_dense_lower(n, seed=300 + n)
+    B = np.random.default_rng(n).uniform(-1, 1, (n, nrhs))
+    X = oracle.solve_multi(s.rowptr, s.colidx, s.val, B)
+    ref = scipy.linalg.solve_triangular(_dense(s), B, lower=True)
+    assert np.max(np.abs(X - ref)) / np.max(np.abs(ref)) <= 1e-13
+
+
+def test_solve_multi_integer_columns_bit_exact():
+    s = synth.integerize(synth.gen_c2(n=5000))
+    rng = np.random.default_rng(3)
+    XT = rng.integers(-8, 9, size=(s.n, 5)).astype(float)
+    A = scipy.sparse.csr_matrix((s.val, s.colidx, s.rowptr), shape=(s.n, s.n))
+    B = A @ XT
+    assert np.array_equal(oracle.solve_multi(s.rowptr, s.colidx, s.val, B), XT)
+
+
 def test_solve_empty():
     x = oracle.solve(np.zeros(1, np.int32), np.zeros(0, np.int32), np.zeros(0), np.zeros(0))
     assert x.shape == (0,)
