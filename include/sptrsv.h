@@ -93,10 +93,14 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_PIPE_STAGES = 12,   /* PIPE ring depth, 2..8 (default 3)                     */
     SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
     SPTRSV_OPT_PIPE_ENTRIES = 14,  /* PIPE colidx/val entries per stage (0 = 4 per row)     */
-    SPTRSV_OPT_ROWS_PER_LANE = 15  /* K = 1..4 thread-level rows per lane (lane owns rows
+    SPTRSV_OPT_ROWS_PER_LANE = 15, /* K = 1..4 thread-level rows per lane (lane owns rows
                                       r0+lane+32k), or 0 (default) = the engine's measured
                                       best; applies to all-thread-level plans on the
                                       ONE-SHOT engine with CTAs of <= 256 threads          */
+    SPTRSV_OPT_VARIANT = 16        /* ablation: 0 (default) product path; 3, 4, 5
+                                      = the paper's Alg.3 SyncFree (warp per row), Alg.4
+                                      Two-Phase, Alg.5 Writing-First with their printed
+                                      control flow (FLAGS protocol, solve_paper.cuh)        */
 } sptrsv_option;
 
 typedef struct sptrsv_info {

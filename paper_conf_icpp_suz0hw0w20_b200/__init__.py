@@ -190,7 +190,8 @@ def analyse(rowptr, colidx, val, **options) -> Handle:
             "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
             "pipe_stages": _lib.OPT_PIPE_STAGES, "pipe_batch": _lib.OPT_PIPE_BATCH,
-            "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE}
+            "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
+            "variant": _lib.OPT_VARIANT}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

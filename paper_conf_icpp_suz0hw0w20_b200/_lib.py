@@ -48,6 +48,7 @@ OPT_PIPE_STAGES = 12
 OPT_PIPE_BATCH = 13
 OPT_PIPE_ENTRIES = 14
 OPT_ROWS_PER_LANE = 15
+OPT_VARIANT = 16
 ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2

@@ -19,6 +19,7 @@
 #include "solve_dyn.cuh"
 #include "solve_lean.cuh"
 #include "solve_multi.cuh"
+#include "solve_paper.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -76,6 +77,7 @@ struct sptrsv_handle_s {
     int pipe_batch = 1;  // (kept for the ABI; the loader takes one round per ticket)
     int pipe_entries = 0;   // 0 = 4 per row of a round
     int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
+    int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
     int grid_cache_key = -1;
     int grid_cache = 0;
     int launch_key = -1;  // configuration of the last launch (see sptrsv_solve)
@@ -471,6 +473,21 @@ void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) 
 }
 
 int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
+    if (h->variant) {  // the paper's kernels, control flow as printed (solve_paper.cuh; ablation only)
+        L->kind = 0;
+        L->block = dim3(kPaperCta);
+        L->smem = 0;
+        if (h->variant == 3) {
+            L->fn = (const void *)k_paper_alg3;
+            L->grid = dim3((unsigned)((h->n + kPaperCta / 32 - 1) / (kPaperCta / 32)));
+        } else {
+            L->fn = h->variant == 4 ? (const void *)k_paper_alg4 : (const void *)k_paper_alg5;
+            L->grid = dim3((unsigned)((h->n + kPaperCta - 1) / kPaperCta));
+        }
+        L->key = 6000000 + h->variant * 100000;
+        L->key ^= (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
     const int engine = resolve_engine(h);
     int cta = 256, Kq = 1;
     effective_geometry(h, engine, &cta, &Kq);
@@ -835,6 +852,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value < 0 || value > 4) return SPTRSV_ERR_INVALID_ARG;
             h->rows_per_lane = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_VARIANT:
+            if (value != 0 && value != 3 && value != 4 && value != 5) return SPTRSV_ERR_INVALID_ARG;
+            h->variant = (int)value;
+            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -858,6 +879,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_PIPE_BATCH: *value = h->pipe_batch; return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_ENTRIES: *value = h->pipe_entries; return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE: *value = h->rows_per_lane; return SPTRSV_OK;
+        case SPTRSV_OPT_VARIANT: *value = h->variant; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }

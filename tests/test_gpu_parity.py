@@ -382,6 +382,21 @@ def test_multi_rhs(cap, nrhs, proto):
             assert torch.isnan(Xp[:, nrhs:]).all()
 
 
+@pytest.mark.parametrize("variant", [3, 4, 5])
+def test_paper_variants(cap, variant):
+    """The paper's Alg.3 / Alg.4 / Alg.5 kernels (ablation): same result -- thread-level ones
+    bit-exact (row order, unfused mul/add, IEEE division); Alg.3's tree sum within TOL."""
+    for gen in (lambda: synth.gen_random_lower(1000, 4, seed=3), lambda: synth.gen_c2i(n=50_000),
+                lambda: synth.gen_grid(64), lambda: synth.gen_c4(n=4000, nlevels=40), lambda: synth.gen_chain(2000)):
+        s = gen()
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        x, _ = gpu_solve(cap, s, 0, variant=variant)
+        if variant == 3:
+            assert relerr(x, ref) <= TOL, s.name
+        else:
+            assert np.array_equal(x, ref), s.name
+
+
 def test_pipe_unaligned_b_falls_back(cap):
     """b at an 8-byte (not 16-byte) offset: the TMA ring needs 16-byte alignment -> one-shot engine."""
     s = synth.gen_c2(n=20_000)

@@ -1,0 +1,85 @@
+"""SURVEY rows f2 + f3: the paper's kernels vs ours across parallel granularity delta, on B200.
+
+For synthetic leveled matrices spanning the paper's (n_level, nnz_row) plane (Fig.3/4/6,
+PAPER.md:216-220, :363, :393-397) it times
+  alg3  the paper's SyncFree, warp per row        (Alg.3)
+  alg4  the paper's Two-Phase CapelliniSpTRSV     (Alg.4)
+  alg5  the paper's Writing-First, literal         (Alg.5)
+  thread / warp / auto  this repo's product path with MODE_THREAD / MODE_WARP / AUTO
+and reports GFLOPS, delta (Eq.1, Table-6 reading), the paper's headline ratios
+(alg5/alg4 -- 28.9x on GTX 1080; alg5/alg3 -- 4.97x avg, Table 5) and the
+thread-vs-warp crossover that sets SPTRSV_OPT_WARP_THRESHOLD (f2, sec.4.4).
+
+usage: python tools/ablation.py [n] [out.jsonl]
+"""
+import json
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import oracle
+import synth
+import paper_conf_icpp_suz0hw0w20_b200 as cap
+
+n = int(sys.argv[1]) if len(sys.argv) > 1 else 200_000
+out = open(sys.argv[2], "w") if len(sys.argv) > 2 else None
+flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device="cuda")
+VARIANTS = {"alg3": dict(variant=3), "alg4": dict(variant=4), "alg5": dict(variant=5),
+            "thread": dict(mode=1, engine=0), "warp": dict(mode=2, engine=0), "auto": dict()}
+
+
+def timeit(h, b, x, reps=5, limit_s=20.0):
+    h.solve(b, x)
+    h.check()
+    ts, t_start = [], time.time()
+    for _ in range(reps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        h.solve(b, x)
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1) * 1e-3)
+        if time.time() - t_start > limit_s:
+            break
+    h.check()
+    return float(np.median(ts))
+
+
+rows = []
+for levels in (10, 100, 1000, 10000):
+    W = n // levels
+    for deps in (2, 4, 8, 16, 32, 64):
+        if deps - 1 >= W:
+            continue
+        s = synth.gen_leveled(n, levels, 1, deps - 1, 40 + levels + deps, f"lev{levels}_d{deps}")
+        d = torch.device("cuda")
+        rp, ci, v, b = (torch.from_numpy(a).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        nnz_row = s.nnz / s.n
+        rec = {"n": s.n, "levels": levels, "n_level": W, "nnz_row": round(nnz_row, 3),
+               "delta": round(oracle.parallel_granularity(W, nnz_row, "table6"), 4), "gflops": {}}
+        for name, opts in VARIANTS.items():
+            with cap.analyse(rp, ci, v, **opts) as h:
+                x = torch.empty_like(b)
+                t = timeit(h, b, x)
+                err = float(np.max(np.abs(x.cpu().numpy() - ref) / np.abs(ref)))
+                assert err <= 1e-12, (name, err)
+                rec["gflops"][name] = round(2 * s.nnz / t / 1e9, 3)
+        g = rec["gflops"]
+        rec["alg5_over_alg4"] = round(g["alg5"] / g["alg4"], 2)
+        rec["alg5_over_alg3"] = round(g["alg5"] / g["alg3"], 2)
+        rec["ours_over_alg5"] = round(g["auto"] / g["alg5"], 2)
+        rec["thread_over_warp"] = round(g["thread"] / g["warp"], 2)
+        print(json.dumps(rec), flush=True)
+        if out:
+            out.write(json.dumps(rec) + "\n")
+        rows.append(rec)
+        del rp, ci, v, b
+if out:
+    out.close()
