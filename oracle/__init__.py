@@ -12,6 +12,7 @@ What is here (each function cites the passage it follows):
 * :func:`validate`      -- the CSR shape Alg. 1 assumes
 * :func:`solve`         -- Algorithm 1, sequential forward substitution
 * :func:`solve_multi`   -- Algorithm 1 per column of B (multiple right-hand sides)
+* :func:`validate_tri` / :func:`solve_tri` -- upper / unit-diagonal forms (G25)
 * :func:`indegree`      -- dependencies per component
 * :func:`levels_dp`     -- level of each component, row-order recurrence
 * :func:`levels_bfs`    -- the same levels by Kahn's BFS (independent algorithm)
@@ -75,6 +76,11 @@ def _get():
         lib.oracle_levels_bfs.restype = ctypes.c_int32
         lib.oracle_level_counts.argtypes = [ctypes.c_int32, _i32p, _i32p]
         lib.oracle_level_counts.restype = ctypes.c_int32
+        lib.oracle_validate_tri.argtypes = [ctypes.c_int32, _i32p, _i32p, _f64p, ctypes.c_int64,
+                                            ctypes.c_int32, _i64p]
+        lib.oracle_validate_tri.restype = ctypes.c_int
+        lib.oracle_solve_tri.argtypes = [ctypes.c_int32, _i32p, _i32p, _f64p, ctypes.c_int32, _f64p, _f64p]
+        lib.oracle_solve_tri.restype = None
         _lib = lib
     return _lib
 
@@ -122,6 +128,41 @@ def solve_multi(rowptr, colidx, val, B):
     for r in range(B.shape[1]):
         X[:, r] = solve(rowptr, colidx, val, np.ascontiguousarray(B[:, r]))
     return X
+
+
+UPPER, UNIT_DIAG = 1, 2  # f4 flags (restated from oracle.c)
+
+
+def validate_tri(rowptr, colidx, val, flags):
+    """CSR rules for the four triangular forms (G25): lower / upper
+    (diagonal last / first), unit diagonal (diagonal not stored, rows may be empty)."""
+    rp, ci, v = _csr(rowptr, colidx, val)
+    n = rp.shape[0] - 1
+    bad = ctypes.c_int64(-1)
+    if v.shape[0] == 0:
+        v = np.zeros(1)
+    if ci.shape[0] == 0:
+        ci = np.zeros(1, dtype=np.int32)
+    code = _get().oracle_validate_tri(n, rp, ci, v, int(rp[-1]) if n >= 0 else 0, int(flags),
+                                      ctypes.byref(bad))
+    return int(code), int(bad.value)
+
+
+def solve_tri(rowptr, colidx, val, b, flags):
+    """Substitution for the four triangular forms (G25): Alg. 1
+     for lower, backward substitution (row order reversed, diagonal the first
+    stored entry) for UPPER; UNIT_DIAG drops the division.  flags=0 equals :func:`solve`."""
+    rp, ci, v = _csr(rowptr, colidx, val)
+    n = rp.shape[0] - 1
+    bb = np.ascontiguousarray(b, dtype=np.float64)
+    x = np.zeros(max(n, 1), dtype=np.float64)
+    if v.shape[0] == 0:
+        v = np.zeros(1)
+    if ci.shape[0] == 0:
+        ci = np.zeros(1, dtype=np.int32)
+    if n > 0:
+        _get().oracle_solve_tri(n, rp, ci, v, int(flags), bb, x)
+    return x[:n]
 
 
 def indegree(rowptr, colidx):

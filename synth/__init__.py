@@ -35,7 +35,7 @@ import numpy as np
 __all__ = [
     "CSRSystem", "gen_c1", "gen_c2", "gen_c2i", "gen_c3", "gen_grid", "gen_c4", "gen_c5",
     "gen_chain", "gen_diag", "gen_dense_lower", "gen_random_lower", "gen_leveled",
-    "gen_fig2_pattern", "integerize", "from_pattern", "CONFIGS", "make",
+    "gen_fig2_pattern", "integerize", "from_pattern", "to_upper", "to_unit", "CONFIGS", "make",
 ]
 
 
@@ -311,6 +311,46 @@ def integerize(sys: CSRSystem, seed: int = 11, lim: int = 8) -> CSRSystem:
     b = np.bincount(rows, weights=val * x_true[sys.colidx], minlength=n).astype(np.float64)
     return CSRSystem(sys.name + "_int", n, sys.rowptr, sys.colidx, val, b, x_true,
                      dict(sys.meta, integer=True))
+
+
+def to_upper(sys: CSRSystem) -> CSRSystem:
+    """the upper-triangular system U = P L P with P the reversal permutation
+    (U_ij = L_{n-1-i, n-1-j}); b and x_true reversed.  Row i of U is row n-1-i of L with
+    columns mapped c -> n-1-c and re-sorted ascending, so the diagonal comes FIRST.  Same
+    dependency DAG (reversed), same values, same nnz per row."""
+    n = sys.n
+    rp = sys.rowptr.astype(np.int64)
+    lens = np.diff(rp)[::-1]
+    rowptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(lens, out=rowptr[1:])
+    # the flattened entries of L reversed are exactly: row n-1 reversed, row n-2 reversed, ...
+    src = np.arange(sys.nnz - 1, -1, -1, dtype=np.int64)
+    colidx = (n - 1 - sys.colidx[src].astype(np.int64)).astype(np.int32)
+    val = sys.val[src].copy()
+    xt = None if sys.x_true is None else sys.x_true[::-1].copy()
+    return CSRSystem(sys.name + "_upper", n, rowptr.astype(np.int32), colidx, val, sys.b[::-1].copy(),
+                     xt, dict(sys.meta, upper=True))
+
+
+def to_unit(sys: CSRSystem, upper: bool = False) -> CSRSystem:
+    """the unit-diagonal system D^{-1} T (T = sys, D its diagonal) with the
+    diagonal NOT stored: every off-diagonal divided by its row's diagonal (the form an
+    incomplete factorisation produces), b = (I + N) @ x_true with N the stored entries.
+    ``upper`` says which side of each row holds the diagonal (first / last entry)."""
+    n = sys.n
+    rows = _rows_of(sys.rowptr)
+    is_diag = sys.colidx.astype(np.int64) == rows
+    d = np.ones(n)
+    d[rows[is_diag]] = sys.val[is_diag]
+    keep = ~is_diag
+    colidx = sys.colidx[keep].copy()
+    val = sys.val[keep] / d[rows[keep]]
+    rowptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(rows[keep], minlength=n), out=rowptr[1:])
+    xt = sys.x_true if sys.x_true is not None else np.ones(n)
+    b = xt + np.bincount(rows[keep], weights=val * xt[colidx], minlength=n)
+    return CSRSystem(sys.name + "_unit", n, rowptr.astype(np.int32), colidx, val, b.astype(np.float64),
+                     xt.copy(), dict(sys.meta, unit=True))
 
 
 CONFIGS = {
