@@ -151,7 +151,8 @@ def validate_tri(rowptr, colidx, val, flags):
 def solve_tri(rowptr, colidx, val, b, flags):
     """Substitution for the four triangular forms (G25): Alg. 1
      for lower, backward substitution (row order reversed, diagonal the first
-    stored entry) for UPPER; UNIT_DIAG drops the division.  flags=0 equals :func:`solve`."""
+    stored entry, off-diagonals summed in DESCENDING column order = earliest-solved first, the
+    mirror of Alg. 1) for UPPER; UNIT_DIAG drops the division.  flags=0 equals :func:`solve`."""
     rp, ci, v = _csr(rowptr, colidx, val)
     n = rp.shape[0] - 1
     bb = np.ascontiguousarray(b, dtype=np.float64)

@@ -128,6 +128,32 @@ def test_solve_tri_lower_is_algorithm1_bit_exact():
                           oracle.solve(s.rowptr, s.colidx, s.val, s.b))
 
 
+@pytest.mark.parametrize("gen", [lambda: synth.gen_random_lower(5000, 7, 12), lambda: synth.gen_c2(n=40_000),
+                                 lambda: synth.gen_grid(80)])
+def test_upper_is_mirror_of_algorithm1_bit_exact(gen):
+    """U = P L P (P the reversal): backward substitution on U IS Alg. 1 on L with b reversed,
+    operation for operation (G25's descending-column order), so the results agree bit-exactly
+    -- a pin through oracle.solve, which test_oracle.py ties to LAPACK / closed forms."""
+    s = gen()
+    u = synth.to_upper(s)
+    xl = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    xu = oracle.solve_tri(u.rowptr, u.colidx, u.val, u.b, U)
+    assert np.array_equal(xu, xl[::-1])
+
+
+def test_upper_sum_order_descending_column():
+    """Row 0 = [1 | 1, e, e] over columns (0 | 1, 2, 3), e = 1e-16, x1 = x2 = x3 = 1.  Descending
+    column: (e + e) + 1 = 1 + 2^-52; ascending: (1 + e) + e = 1.  Fixes G25's order, not just
+    the value."""
+    e = 1e-16
+    rp = np.array([0, 4, 5, 6, 7], np.int32)
+    ci = np.array([0, 1, 2, 3, 1, 2, 3], np.int32)
+    v = np.array([1.0, 1.0, e, e, 1.0, 1.0, 1.0])
+    x = oracle.solve_tri(rp, ci, v, np.array([0.0, 1.0, 1.0, 1.0]), U)
+    assert np.array_equal(x[1:], [1.0, 1.0, 1.0])
+    assert x[0] == -(1.0 + 2.0 ** -52)
+
+
 def test_upper_uses_first_entry_as_diagonal():
     """Row 0 = [U00=4, U01=2]; the diagonal is the FIRST entry: x1 = 3/5, x0 = (1 - 2*3/5)/4."""
     rp = np.array([0, 2, 3], np.int32)
