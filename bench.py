@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--profile", action="store_true", help="short run for ncu: no clocks/e2e/cpu legs")
     ap.add_argument("--opt", action="append", default=[], help="extra handle option key=value")
     ap.add_argument("--no-flags-leg", action="store_true", help="skip the FLAGS-protocol comparison leg")
+    ap.add_argument("--no-tri-leg", action="store_true", help="skip the upper / unit-diagonal (f4) leg")
     ap.add_argument("--nrhs", type=int, default=8, help="right-hand sides of the multi-RHS leg (0 = skip)")
     return ap.parse_args()
 
@@ -345,6 +346,60 @@ def main():
                      "column0_matches_single_rhs": ok,
                      "layout": "row-major B[i*nrhs + r], r-th column = (r+1) * b"}
 
+    # ---- triangular-forms leg: the same system as U = P L P (upper, backward
+    # substitution), as D^-1 L with implicit unit diagonal, and both; same timing rules
+    tri_leg = None
+    if not args.no_tri_leg and not args.profile:
+        import synth
+        tri_leg = {}
+        for name, up, un in (("upper", True, False), ("unit_lower", False, True), ("unit_upper", True, True)):
+            ts = []
+            for s in systems:
+                t = synth.to_upper(s) if up else s
+                t = synth.to_unit(t) if un else t
+                ts.append(t)
+            th, tb = [], []
+            for t in ts:
+                rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(dev) for a in (t.rowptr, t.colidx, t.val, t.b))
+                th.append(cap.analyse(rp, ci, v, upper=up, unit_diag=un, protocol=opts.get("protocol", 1)))
+                tb.append((rp, ci, v, b, torch.empty_like(b)))
+            for i in range(args.warmup):
+                flush.zero_()
+                for h, (_, _, _, b, x) in zip(th, tb):
+                    h.solve(b, x, stream=stream)
+            ev4 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                   for _ in range(args.steps)]
+            if dist:
+                dist.barrier()
+            torch.cuda.synchronize()
+            for i in range(args.steps):
+                flush.zero_()
+                ev4[i][0].record(stream)
+                for h, (_, _, _, b, x) in zip(th, tb):
+                    h.solve(b, x, stream=stream)
+                ev4[i][1].record(stream)
+            torch.cuda.synchronize()
+            for h in th:
+                h.check(stream)
+            tt = float(np.sum([a.elapsed_time(b) for a, b in ev4])) * 1e-3
+            if dist:
+                t_ = torch.tensor([tt], device=dev, dtype=torch.float64)
+                dist.all_reduce(t_, op=dist.ReduceOp.MAX)
+                tt = float(t_.item())
+            nnz_t = sum(t.nnz for t in ts)
+            if dist:
+                t_ = torch.tensor([nnz_t], device=dev, dtype=torch.float64)
+                dist.all_reduce(t_)
+                nnz_t = float(t_.item())
+            err = max(float(np.max(np.abs(x.cpu().numpy() - t.x_true) / np.abs(t.x_true)))
+                      for t, (_, _, _, _, x) in zip(ts, tb))
+            tri_leg[name] = {"value": round(2.0 * nnz_t * args.steps / tt / 1e9, 3), "unit": UNIT,
+                             "ms_per_step": round(tt / args.steps * 1e3, 5), "nnz": int(nnz_t),
+                             "max_rel_err_vs_x_true": err}
+            for h in th:
+                h.close()
+            del tb
+
     # ---- roofline of the dominant (only) kernel, k_solve
     peak, peak_src = peaks()
     alg_bytes = systems[0].alg_bytes()
@@ -428,6 +483,7 @@ def main():
                          0: "flags (st.release.gpu / ld.acquire.gpu)"}[opts.get("protocol", 1)],
             "flags_protocol_leg": flags_leg,
             "multi_rhs_leg": multi_leg,
+            "triangular_forms_leg": tri_leg,
             "roofline": roof,
             "latency_bound": lat,
             "e2e": e2e,

@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SPTRSV_ABI_VERSION 1
+#define SPTRSV_ABI_VERSION 2
 
 typedef struct sptrsv_handle_s *sptrsv_handle_t;
 typedef void *sptrsv_stream_t; /* cudaStream_t */
@@ -97,6 +97,8 @@ typedef enum sptrsv_option {
                                       r0+lane+32k), or 0 (default) = the engine's measured
                                       best; applies to all-thread-level plans on the
                                       ONE-SHOT engine with CTAs of <= 256 threads          */
+    SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5 (default), 6 or 8
+                                      resident 256-thread CTAs per SM                       */
     SPTRSV_OPT_VARIANT = 16        /* ablation: 0 (default) product path; 3, 4, 5
                                       = the paper's Alg.3 SyncFree (warp per row), Alg.4
                                       Two-Phase, Alg.5 Writing-First with their printed
@@ -141,6 +143,41 @@ typedef struct sptrsv_info {
  */
 int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
                        const double *val, sptrsv_handle_t *out);
+
+/* Triangular-form flags of sptrsv_analyse_csr_ex. */
+#define SPTRSV_TRI_UPPER 1     /* U x = b: entries j >= i, diagonal stored FIRST in each row */
+#define SPTRSV_TRI_UNIT_DIAG 2 /* diagonal implicitly 1 and NOT stored; rows may be empty    */
+
+/*
+ * sptrsv_analyse_csr_ex -- sptrsv_analyse_csr for the other triangular forms
+ * (the paper solves L x = b only, Alg.1 :82-92;
+ * DESIGN.md reading G25):
+ *   tri_flags = 0                      lower, diagonal last -- identical to
+ *                                      sptrsv_analyse_csr.
+ *   SPTRSV_TRI_UPPER                   upper: per row strictly increasing
+ *                                      columns, all >= i, column i FIRST,
+ *                                      val[rowptr[i]] = U_ii != 0; solved by
+ *                                      backward substitution
+ *                                      x_i = (b_i - sum_{j>i} U_ij x_j) / U_ii.
+ *   SPTRSV_TRI_UNIT_DIAG (| UPPER)     unit diagonal: no stored diagonal (a
+ *                                      stored column i is an error), all
+ *                                      entries strictly below (above) the
+ *                                      diagonal, x_i = b_i - sum_j T_ij x_j.
+ * Errors: other flag bits -> INVALID_ARG; an entry on the wrong side of the
+ * diagonal (or a stored diagonal under UNIT_DIAG) -> SPTRSV_ERR_NOT_LOWER; a
+ * missing / misplaced diagonal -> MISSING_DIAG; as sptrsv_analyse_csr
+ * otherwise (lowest offending row wins).  Same ownership and synchronisation
+ * as sptrsv_analyse_csr.
+ * A handle with tri_flags != 0 always runs the thread-level LEAN engine (upper
+ * rows are taken in reverse order behind the same start ticket, so the ticket
+ * order is a topological order); sptrsv_solve, sptrsv_solve_host,
+ * sptrsv_get_indegree and sptrsv_check work as for lower handles;
+ * sptrsv_solve_multi, sptrsv_levels, MODE = 2 (warp) and VARIANT != 0 return
+ * SPTRSV_ERR_INVALID_ARG.  Bit-exact with the fp64 substitution that sums each
+ * row's off-diagonals in stored order (one rounded multiply and add each).
+ */
+int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx,
+                          const double *val, int32_t tri_flags, sptrsv_handle_t *out);
 
 /*
  * sptrsv_solve -- one solve L x = b (Alg.5), enqueued on

@@ -45,9 +45,10 @@ def _need(t, dtype, n, name):
 
 
 class Handle:
-    """An analysed matrix (``sptrsv_analyse_csr``).  Keeps the CSR tensors alive."""
+    """An analysed matrix (``sptrsv_analyse_csr`` / ``sptrsv_analyse_csr_ex``).  Keeps the CSR
+    tensors alive.  ``upper`` / ``unit_diag`` select the f4 triangular forms (include/sptrsv.h)."""
 
-    def __init__(self, rowptr, colidx, val):
+    def __init__(self, rowptr, colidx, val, upper=False, unit_diag=False):
         import torch
         _need(rowptr, torch.int32, None, "rowptr")
         n = rowptr.numel() - 1
@@ -61,11 +62,13 @@ class Handle:
         self.n = n
         self._keep = (rowptr, colidx, val)
         self._h = ctypes.c_void_p()
+        self.tri = (_lib.TRI_UPPER if upper else 0) | (_lib.TRI_UNIT_DIAG if unit_diag else 0)
         with torch.cuda.device(self.device):
             torch.cuda.current_stream().synchronize()  # analyse runs on the legacy default stream
-            check(lib.sptrsv_analyse_csr(n, rowptr.data_ptr(), colidx.data_ptr() if colidx.numel() else None,
-                                         val.data_ptr() if val.numel() else None, ctypes.byref(self._h)),
-                  "sptrsv_analyse_csr")
+            check(lib.sptrsv_analyse_csr_ex(n, rowptr.data_ptr(), colidx.data_ptr() if colidx.numel() else None,
+                                            val.data_ptr() if val.numel() else None, self.tri,
+                                            ctypes.byref(self._h)),
+                  "sptrsv_analyse_csr_ex")
 
     # -- solve -------------------------------------------------------------------------
     def solve(self, b, x=None, stream=None):
@@ -182,16 +185,16 @@ class Handle:
         self.close()
 
 
-def analyse(rowptr, colidx, val, **options) -> Handle:
-    """``sptrsv_analyse_csr`` + options (mode=, warp_threshold=, cta_threads=, ...)."""
-    h = Handle(rowptr, colidx, val)
+def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Handle:
+    """``sptrsv_analyse_csr[_ex]`` + options (mode=, warp_threshold=, cta_threads=, ...)."""
+    h = Handle(rowptr, colidx, val, upper=upper, unit_diag=unit_diag)
     keys = {"mode": OPT_MODE, "warp_threshold": OPT_WARP_THRESHOLD, "cta_threads": OPT_CTA_THREADS,
             "backoff_min_ns": OPT_BACKOFF_MIN_NS, "backoff_max_ns": OPT_BACKOFF_MAX_NS,
             "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
             "pipe_stages": _lib.OPT_PIPE_STAGES, "pipe_batch": _lib.OPT_PIPE_BATCH,
             "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
-            "variant": _lib.OPT_VARIANT}
+            "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

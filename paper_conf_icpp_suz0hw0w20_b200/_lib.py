@@ -28,6 +28,10 @@ ERR_UNSORTED = -5
 ERR_BAD_ROWPTR = -6
 ERR_BAD_COL = -7
 ERR_TOO_LARGE = -8
+
+# triangular forms of sptrsv_analyse_csr_ex
+TRI_UPPER = 1
+TRI_UNIT_DIAG = 2
 ERR_CUDA = -9
 ERR_ALLOC = -10
 ERR_TIMEOUT = -11
@@ -49,6 +53,7 @@ OPT_PIPE_BATCH = 13
 OPT_PIPE_ENTRIES = 14
 OPT_ROWS_PER_LANE = 15
 OPT_VARIANT = 16
+OPT_LEAN_OCCUPANCY = 17
 ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
@@ -78,6 +83,7 @@ _i32, _i64 = ctypes.c_int32, ctypes.c_int64
 
 EXPORTS = {
     "sptrsv_analyse_csr": (ctypes.c_int, [_i32, _p, _p, _p, ctypes.POINTER(_h)]),
+    "sptrsv_analyse_csr_ex": (ctypes.c_int, [_i32, _p, _p, _p, _i32, ctypes.POINTER(_h)]),
     "sptrsv_solve": (ctypes.c_int, [_h, _p, _p, _p]),
     "sptrsv_solve_host": (ctypes.c_int, [_h, _p, _p, _p]),
     "sptrsv_solve_multi": (ctypes.c_int, [_h, _p, _p, _i32, _i64, _i64, _p]),

@@ -18,15 +18,18 @@ enum : int {  // same numbering as sptrsv_status (negated)
 
 // status: 64-bit min over (row << 8 | code) -> the lowest offending row wins,
 // which is the row-ordered error the oracle reports too.
-// Also counts "near" dependencies (i - col < 256: produced within about one CTA of
-// rows) -- the statistic ENGINE_AUTO uses to choose between the shared-memory
+// Also counts "near" dependencies (|i - col| < 256: produced within about one CTA
+// of rows) -- the statistic ENGINE_AUTO uses to choose between the shared-memory
 // local resolution of the staged engine and the lean engine.
+// tri: bit 0 UPPER (entries j >= i, diagonal FIRST), bit 1 UNIT
+// (diagonal implicit 1, not stored: entries strictly inside the triangle).
 __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ rowptr,
                                                   const int32_t *__restrict__ colidx,
                                                   const double *__restrict__ val, int32_t n,
                                                   int64_t nnz, int32_t *indeg,
                                                   unsigned long long *status, int32_t *max_row,
-                                                  unsigned long long *near_deps) {
+                                                  unsigned long long *near_deps, int tri) {
+    const bool upper = tri & 1, unit = tri & 2;
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     int len = 0;
     unsigned near = 0;
@@ -35,26 +38,28 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
         int code = 0;
         if (s < 0 || e < s || e > nnz) {
             code = E_BAD_ROWPTR;
-        } else if (e == s) {
+        } else if (e == s && !unit) {
             code = E_MISSING_DIAG;
         } else {
             int prev = -1;
             for (int64_t j = s; j < e; ++j) {
                 const int c = colidx[j];
-                if (c < 0) { code = E_BAD_COL; break; }
-                if (c > i) { code = E_NOT_LOWER; break; }
+                if (c < 0 || c >= n) { code = E_BAD_COL; break; }
+                // outside the triangle (for UNIT the diagonal itself is outside too)
+                if (upper ? (c < i || (unit && c == i)) : (c > i || (unit && c == i))) { code = E_NOT_LOWER; break; }
                 if (j > s && c <= prev) { code = E_UNSORTED; break; }
-                if (c < i && i - c < 256) ++near;
+                if (c != i && (c > i ? c - i : i - c) < 256) ++near;
                 prev = c;
             }
-            if (!code) {
-                if (colidx[e - 1] != i) code = E_MISSING_DIAG;
-                else if (val[e - 1] == 0.0) code = E_ZERO_DIAG;
+            if (!code && !unit) {
+                const int64_t jd = upper ? s : e - 1;  // diagonal: first (upper) / last (lower)
+                if (colidx[jd] != i) code = E_MISSING_DIAG;
+                else if (val[jd] == 0.0) code = E_ZERO_DIAG;
             }
         }
         if (code) atomicMin(status, ((unsigned long long)i << 8) | (unsigned long long)code);
         len = code ? 0 : (int)(e - s);
-        indeg[i] = code ? 0 : (int)(e - s - 1);
+        indeg[i] = code ? 0 : (int)(e - s - (unit ? 0 : 1));
     }
     for (int off = 16; off > 0; off >>= 1) {
         len = max(len, __shfl_xor_sync(0xffffffffu, len, off));

@@ -24,17 +24,22 @@ namespace sptrsv_dev {
 
 constexpr int kLeanCta = 256;
 
-template <int PROTO>
-__global__ void __launch_bounds__(kLeanCta, 5) k_solve_lean(SolveParams p) {
+// UPPER / UNIT: upper-triangular rows (diagonal first, dependencies
+// j > i) are taken in REVERSE order -- logical row r is row n-1-r, so the ticket
+// order is again a topological order; UNIT: the diagonal is implicitly 1 and
+// not stored.
+template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false>
+__global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint64_t pol = policy_evict_first();
     // ---- speculative first-level loads for logical block == blockIdx.x
     int i = (int)blockIdx.x * kLeanCta + tid;
+    if (UPPER) i = p.n - 1 - i;
     int rs = 0, re = 1;
     double bi = 0.0;
-    if (i < p.n) {
+    if (i >= 0 && i < p.n) {
         rs = ld_stream_i32(p.rowptr + i, pol);
         re = ld_stream_i32(p.rowptr + i + 1, pol);
         bi = ld_stream_f64(p.b + i, pol);
@@ -50,21 +55,28 @@ __global__ void __launch_bounds__(kLeanCta, 5) k_solve_lean(SolveParams p) {
     const uint32_t epoch = s_epoch;
     if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
         i = (int)s_blk * kLeanCta + tid;
+        if (UPPER) i = p.n - 1 - i;
         rs = 0, re = 1, bi = 0.0;
-        if (i < p.n) {
+        if (i >= 0 && i < p.n) {
             rs = ld_stream_i32(p.rowptr + i, pol);
             re = ld_stream_i32(p.rowptr + i + 1, pol);
             bi = ld_stream_f64(p.b + i, pol);
         }
     }
-    const bool act = i < p.n;
-    const int jd = re - 1;
-    int j = rs;
+    const bool act = i >= 0 && i < p.n;
+    // off-diagonal entries [lo, hi); the diagonal is last (lower), first (upper) or implicit
+    // (unit).  They are consumed earliest-solved first: ascending for lower (Alg.1 l.3-4),
+    // DESCENDING for upper (G25) -- the nearest, latest dependency is waited for last.
+    const int lo = (UPPER && !UNIT) ? rs + 1 : rs;
+    const int hi = (UPPER || UNIT) ? re : re - 1;
+    constexpr int dir = UPPER ? -1 : 1;
+    auto inr = [&](int k) { return UPPER ? k >= lo : k < hi; };
+    int j = UPPER ? hi - 1 : lo;
     // ---- second-level loads: L_ii and the next two dependencies
-    double dv = act ? ld_stream_f64(p.val + jd, pol) : 1.0;
-    int nc = (act && j < jd) ? ld_stream_i32(p.colidx + j, pol) : -1;
-    double nv = (act && j < jd) ? ld_stream_f64(p.val + j, pol) : 0.0;
-    int nc2 = (act && j + 1 < jd) ? ld_stream_i32(p.colidx + j + 1, pol) : -1;
+    double dv = (act && !UNIT) ? ld_stream_f64(p.val + (UPPER ? rs : re - 1), pol) : 1.0;
+    int nc = (act && inr(j)) ? ld_stream_i32(p.colidx + j, pol) : -1;
+    double nv = (act && inr(j)) ? ld_stream_f64(p.val + j, pol) : 0.0;
+    int nc2 = (act && inr(j + dir)) ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
     Diag dg;
     dg.init(dv);
     double ls = 0.0;
@@ -73,40 +85,39 @@ __global__ void __launch_bounds__(kLeanCta, 5) k_solve_lean(SolveParams p) {
     nocta.R0 = nocta.R1 = 0;
     nocta.xc = nullptr;
     nocta.xc_s = 0;
-    SolveParams pp = p;
-    pp.local = 0;
+    p.local = 0;  // no in-CTA x copy in this engine
     uint32_t backoff = p.backoff_min, idle = 0;
     // advance past a consumed dependency: the 2nd becomes the next, prefetch the 3rd
     auto advance = [&]() {
-        ++j;
+        j += dir;
         nc = nc2;
         nv = (nc >= 0) ? ld_stream_f64(p.val + j, pol) : 0.0;
-        nc2 = (j + 1 < jd) ? ld_stream_i32(p.colidx + j + 1, pol) : -1;
+        nc2 = inr(j + dir) ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
     };
     while (true) {
         bool prog = false;
         if (!done) {
             if (nc < 0) {  // reached the diagonal (Alg.5 l.12-16)
-                publish<PROTO>(pp, nocta, i, dg.div(__dsub_rn(bi, ls)), epoch);
+                publish<PROTO>(p, nocta, i, UNIT ? __dsub_rn(bi, ls) : dg.div(__dsub_rn(bi, ls)), epoch);
                 done = true;
                 prog = true;
             } else {
                 // poll the next two dependencies together, consume the ready prefix in row order
                 unsigned long long a0, a1, c0 = 0, c1 = 0;
-                poll1<PROTO>(pp, nc, a0, a1);
+                poll1<PROTO>(p, nc, a0, a1);
                 const int cc2 = nc2;
-                if (cc2 >= 0) poll1<PROTO>(pp, cc2, c0, c1);
+                if (cc2 >= 0) poll1<PROTO>(p, cc2, c0, c1);
                 if (ready1<PROTO>(a0, a1, epoch)) {
                     if (p.trace) p.trace[p.n + i] = globaltimer_ns();
-                    ls = __dadd_rn(ls, __dmul_rn(nv, value1<PROTO>(pp, nc, a0, a1)));
+                    ls = __dadd_rn(ls, __dmul_rn(nv, value1<PROTO>(p, nc, a0, a1)));
                     advance();
                     prog = true;
                     if (cc2 >= 0 && ready1<PROTO>(c0, c1, epoch)) {
-                        ls = __dadd_rn(ls, __dmul_rn(nv, value1<PROTO>(pp, cc2, c0, c1)));
+                        ls = __dadd_rn(ls, __dmul_rn(nv, value1<PROTO>(p, cc2, c0, c1)));
                         advance();
                     }
                     if (nc < 0) {
-                        publish<PROTO>(pp, nocta, i, dg.div(__dsub_rn(bi, ls)), epoch);
+                        publish<PROTO>(p, nocta, i, UNIT ? __dsub_rn(bi, ls) : dg.div(__dsub_rn(bi, ls)), epoch);
                         done = true;
                     }
                 }

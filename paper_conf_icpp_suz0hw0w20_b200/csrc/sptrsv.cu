@@ -78,6 +78,8 @@ struct sptrsv_handle_s {
     int pipe_entries = 0;   // 0 = 4 per row of a round
     int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
+    int lean_minb = 5;      // LEAN: minimum resident CTAs per SM the register budget targets
+    int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
     int grid_cache = 0;
     int launch_key = -1;  // configuration of the last launch (see sptrsv_solve)
@@ -321,12 +323,19 @@ const char *sptrsv_strerror(int status) {
 
 int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
                        sptrsv_handle_t *out) {
+    return sptrsv_analyse_csr_ex(n, rowptr, colidx, val, 0, out);
+}
+
+int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
+                          int32_t tri_flags, sptrsv_handle_t *out) {
     const auto t0 = std::chrono::steady_clock::now();
     if (!out) return SPTRSV_ERR_INVALID_ARG;
     *out = nullptr;
-    if (n < 0) return SPTRSV_ERR_INVALID_ARG;
+    if (n < 0 || (tri_flags & ~(SPTRSV_TRI_UPPER | SPTRSV_TRI_UNIT_DIAG))) return SPTRSV_ERR_INVALID_ARG;
     if (n > 0x7FFFFFFE) return SPTRSV_ERR_TOO_LARGE;
-    if (!rowptr || (n > 0 && (!colidx || !val))) return SPTRSV_ERR_INVALID_ARG;
+    // colidx / val may be NULL only when nnz == 0 (unit-diagonal identity), checked below
+    if (!rowptr || (n > 0 && !(tri_flags & SPTRSV_TRI_UNIT_DIAG) && (!colidx || !val)))
+        return SPTRSV_ERR_INVALID_ARG;
     int rc = set_kernel_attrs();
     if (rc) return rc;
     auto *h = new (std::nothrow) sptrsv_handle_s();
@@ -339,6 +348,8 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
     h->rowptr = rowptr;
     h->colidx = colidx;
     h->val = val;
+    h->tri = tri_flags;
+    if (tri_flags) h->mode = 1;  // f4 forms run on the thread-level LEAN engine only
     unsigned long long *d_status = nullptr, *d_near = nullptr;
     int32_t *d_maxrow = nullptr;
     do {
@@ -353,6 +364,10 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
             break;
         }
         h->nnz = ends[1];
+        if (h->nnz > 0 && (!colidx || !val)) {
+            rc = SPTRSV_ERR_INVALID_ARG;
+            break;
+        }
         const size_t nn = (size_t)(n > 0 ? n : 1);
         if (cudaMalloc(&h->ws.flags, sizeof(uint32_t) * nn) != cudaSuccess ||
             (h->proto == PROTO_FUSED && cudaMalloc(&h->ws.rec, 16 * nn) != cudaSuccess) ||
@@ -372,7 +387,7 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
         }
         if (n > 0) {
             k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->nnz, h->ws.indeg, d_status,
-                                                 d_maxrow, d_near);
+                                                 d_maxrow, d_near, tri_flags);
             if (cudaGetLastError() != cudaSuccess) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
@@ -447,6 +462,7 @@ int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem,
 // with warp-level rows use the staged one-shot engine.  (Round-1 B200 sweeps,
 // DESIGN.md section 8.)
 int resolve_engine(const sptrsv_handle_s *h) {
+    if (h->tri) return 3;  // upper / unit-diagonal handles: LEAN only
     if (h->engine != 5) return h->engine;
     const long long offdiag = h->nnz - h->n;
     if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_deps < offdiag)) return 3;
@@ -472,7 +488,28 @@ void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) 
     *K = h->rows_per_lane ? h->rows_per_lane : k;
 }
 
+typedef void (*lean_fn)(SolveParams);
+lean_fn lean_tri_kernel(int proto, int tri) {
+    static const lean_fn tab[4][2] = {
+        {k_solve_lean<PROTO_FLAGS, 5>, k_solve_lean<PROTO_FUSED, 5>},
+        {k_solve_lean<PROTO_FLAGS, 5, true, false>, k_solve_lean<PROTO_FUSED, 5, true, false>},
+        {k_solve_lean<PROTO_FLAGS, 5, false, true>, k_solve_lean<PROTO_FUSED, 5, false, true>},
+        {k_solve_lean<PROTO_FLAGS, 5, true, true>, k_solve_lean<PROTO_FUSED, 5, true, true>},
+    };
+    return tab[tri & 3][proto ? 1 : 0];
+}
+
 int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
+    if (h->tri) {  // f4: upper / unit-diagonal forms on the LEAN engine (solve_lean.cuh)
+        L->fn = (const void *)lean_tri_kernel(h->proto, h->tri);
+        L->kind = 0;
+        L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
+        L->block = dim3((unsigned)kLeanCta);
+        L->smem = 0;
+        L->key = 7000000 + h->proto * 100000 + h->tri * 10000;
+        L->key ^= (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
     if (h->variant) {  // the paper's kernels, control flow as printed (solve_paper.cuh; ablation only)
         L->kind = 0;
         L->block = dim3(kPaperCta);
@@ -541,12 +578,20 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
     }
     // ---- ENGINE_LEAN: minimal one-shot kernel for all-thread-level plans
     if (engine == 3 && h->plan == PLAN_THREAD) {
-        L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED> : (const void *)k_solve_lean<PROTO_FLAGS>;
+        // LEAN occupancy: minimum resident CTAs per SM = 5 (default), 6 or 8 (option rows_per_lane
+        // is not used by LEAN; lean_minb selects the register budget)
+        const int mb = h->lean_minb;
+        if (mb == 8)
+            L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED, 8> : (const void *)k_solve_lean<PROTO_FLAGS, 8>;
+        else if (mb == 6)
+            L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED, 6> : (const void *)k_solve_lean<PROTO_FLAGS, 6>;
+        else
+            L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED, 5> : (const void *)k_solve_lean<PROTO_FLAGS, 5>;
         L->kind = 0;
         L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
         L->block = dim3((unsigned)kLeanCta);
         L->smem = 0;
-        L->key = 5000000 + h->proto * 100000;
+        L->key = 5000000 + h->proto * 100000 + h->lean_minb * 1000;
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
@@ -663,7 +708,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
 int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nrhs, int64_t ldb, int64_t ldx,
                        sptrsv_stream_t stream) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
-    if (nrhs < 1 || nrhs > 32 || ldb < nrhs || ldx < nrhs) return SPTRSV_ERR_INVALID_ARG;
+    if (nrhs < 1 || nrhs > 32 || ldb < nrhs || ldx < nrhs || h->tri) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!B || !X || (const double *)X == B) return SPTRSV_ERR_INVALID_ARG;
     cudaStream_t s = (cudaStream_t)stream;
@@ -772,6 +817,11 @@ int sptrsv_destroy(sptrsv_handle_t h) {
 
 int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
+    if (h->tri) {  // f4 handles: thread-level LEAN only; the paper's variants are lower-only
+        if ((key == SPTRSV_OPT_MODE && value == 2) || (key == SPTRSV_OPT_VARIANT && value != 0))
+            return SPTRSV_ERR_INVALID_ARG;
+        if (key == SPTRSV_OPT_MODE) return (value < 0 || value > 2) ? SPTRSV_ERR_INVALID_ARG : SPTRSV_OK;
+    }
     switch (key) {
         case SPTRSV_OPT_MODE:
             if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
@@ -856,6 +906,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 3 && value != 4 && value != 5) return SPTRSV_ERR_INVALID_ARG;
             h->variant = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_LEAN_OCCUPANCY:
+            if (value != 5 && value != 6 && value != 8) return SPTRSV_ERR_INVALID_ARG;
+            h->lean_minb = (int)value;
+            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -880,6 +934,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_PIPE_ENTRIES: *value = h->pipe_entries; return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE: *value = h->rows_per_lane; return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT: *value = h->variant; return SPTRSV_OK;
+        case SPTRSV_OPT_LEAN_OCCUPANCY: *value = h->lean_minb; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }
@@ -911,7 +966,7 @@ int sptrsv_get_indegree(sptrsv_handle_t h, int32_t *out_dev, sptrsv_stream_t str
 
 int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev, int32_t *nlevels_host,
                   sptrsv_stream_t stream) {
-    if (!h || !nlevels_host) return SPTRSV_ERR_INVALID_ARG;
+    if (!h || !nlevels_host || h->tri) return SPTRSV_ERR_INVALID_ARG;
     *nlevels_host = 0;
     if (h->n == 0) return SPTRSV_OK;
     cudaStream_t s = (cudaStream_t)stream;
