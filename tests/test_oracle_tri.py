@@ -187,6 +187,7 @@ def test_validate_tri_codes():
     assert _case([0, 0], [], [], 4)[0] == oracle.INVALID_ARG
     # flags 0 agrees with the lower validator
     for rp, ci, v in (([0, 1, 3], [0, 0, 1], [1, 1, 1]), ([0, 2, 3], [0, 1, 1], [1, 1, 1]),
-                      ([0, 1, 3], [0, 0, 1], [1, 1, 0])):
+                      ([0, 1, 3], [0, 0, 1], [1, 1, 0]), ([0, 1, 3], [0, 0, 9], [1, 1, 1]),
+                      ([0, 1, 3], [0, -1, 1], [1, 1, 1])):
         assert _case(rp, ci, v, 0) == oracle.validate(np.array(rp, np.int32), np.array(ci, np.int32),
                                                       np.array(v, float))
