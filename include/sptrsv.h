@@ -77,7 +77,7 @@ typedef enum sptrsv_option {
                                       are read from a shared-memory copy of x               */
     SPTRSV_OPT_ENGINE = 11,        /* 5 (default) AUTO: LEAN for all-thread-level plans whose
                                       dependencies are mostly far (< 1/4 within 256 rows),
-                                      else ONE-SHOT.  0 ONE-SHOT: one CTA per row range,
+                                      HYBRID for plans with warp-level rows, else ONE-SHOT.  0 ONE-SHOT: one CTA per row range,
                                       ticketed, smem-staged, in-CTA x copy;
                                       1 PIPE: persistent CTAs, a loader warp streams rounds
                                       of rows into a shared-memory ring by TMA bulk copy.
@@ -89,7 +89,11 @@ typedef enum sptrsv_option {
                                       3 LEAN: minimal-latency one-shot kernel for
                                       all-thread-level plans (no staging, speculative rows).
                                       4 DYN-STATIC: DYN with static round-robin 32-row units
-                                      (no ticket), launched cooperatively                  */
+                                      (no ticket), launched cooperatively.
+                                      6 HYBRID: 64-thread CTAs, one task per warp -- a
+                                      warp-level row (Alg.3) or a 32-row thread group
+                                      (LEAN's per-lane loop), no staging / in-CTA copy;
+                                      all-thread-level plans run LEAN                        */
     SPTRSV_OPT_PIPE_STAGES = 12,   /* PIPE ring depth, 2..8 (default 3)                     */
     SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
     SPTRSV_OPT_PIPE_ENTRIES = 14,  /* PIPE colidx/val entries per stage (0 = 4 per row)     */
@@ -168,13 +172,18 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
  * missing / misplaced diagonal -> MISSING_DIAG; as sptrsv_analyse_csr
  * otherwise (lowest offending row wins).  Same ownership and synchronisation
  * as sptrsv_analyse_csr.
- * A handle with tri_flags != 0 always runs the thread-level LEAN engine (upper
- * rows are taken in reverse order behind the same start ticket, so the ticket
- * order is a topological order); sptrsv_solve, sptrsv_solve_host,
- * sptrsv_get_indegree and sptrsv_check work as for lower handles;
- * sptrsv_solve_multi, sptrsv_levels, MODE = 2 (warp) and VARIANT != 0 return
- * SPTRSV_ERR_INVALID_ARG.  Bit-exact with the fp64 substitution that sums each
- * row's off-diagonals in stored order (one rounded multiply and add each).
+ * A handle with tri_flags != 0 runs the thread-level LEAN engine, or -- when
+ * the plan is all warp-level (SPTRSV_OPT_MODE = 2, or AUTO with every 32-row
+ * group above the warp threshold) -- one warp per row (k_solve_tri_warp).
+ * Upper rows are taken in reverse order behind the same start ticket, so the
+ * ticket order is a topological order.  Each row's off-diagonals are summed
+ * earliest-solved first: ascending column (lower), descending column (upper).
+ * sptrsv_solve, sptrsv_solve_host, sptrsv_get_indegree, sptrsv_check and the
+ * options work as for lower handles (ENGINE is ignored);
+ * sptrsv_solve_multi, sptrsv_levels and VARIANT != 0 return
+ * SPTRSV_ERR_INVALID_ARG.  Thread-level rows are bit-exact with that fp64
+ * substitution (one rounded multiply and add each); warp rows are within the
+ * warp-mode bound, as for lower handles.  sptrsv_info.engine: 3 LEAN, 6 warp.
  */
 int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx,
                           const double *val, int32_t tri_flags, sptrsv_handle_t *out);

@@ -14,7 +14,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libsptrsv.so")
 SOURCES = [os.path.join(CSRC, f) for f in ("sptrsv.cu",)]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("solve.cuh", "solve_pipe.cuh", "solve_k.cuh", "solve_dyn.cuh", "solve_lean.cuh", "solve_multi.cuh", "solve_paper.cuh", "setup.cuh", "ptx.cuh", "diag.cuh")] + [
+DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("solve.cuh", "solve_pipe.cuh", "solve_k.cuh", "solve_dyn.cuh", "solve_lean.cuh", "solve_tri.cuh", "solve_multi.cuh", "solve_paper.cuh", "setup.cuh", "ptx.cuh", "diag.cuh")] + [
     os.path.join(ROOT, "include", "sptrsv.h")]
 
 NVCC_FLAGS = [

@@ -44,9 +44,10 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
             int prev = -1;
             for (int64_t j = s; j < e; ++j) {
                 const int c = colidx[j];
-                if (c < 0 || c >= n) { code = E_BAD_COL; break; }
+                if (c < 0) { code = E_BAD_COL; break; }
                 // outside the triangle (for UNIT the diagonal itself is outside too)
                 if (upper ? (c < i || (unit && c == i)) : (c > i || (unit && c == i))) { code = E_NOT_LOWER; break; }
+                if (c >= n) { code = E_BAD_COL; break; }  // upper only (lower has c <= i < n)
                 if (j > s && c <= prev) { code = E_UNSORTED; break; }
                 if (c != i && (c > i ? c - i : i - c) < 256) ++near;
                 prev = c;
@@ -72,11 +73,13 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
 // mode: 0 auto, 1 all thread-level, 2 all warp-level.
 // A group of `rows` rows goes warp-level in auto mode when its nnz (diagonals
 // included) exceeds threshold * rows, i.e. mean nnz/row > threshold.
+// rev (f4 UPPER): groups are over LOGICAL rows r -> row n-1-r (the solve order).
 __device__ __forceinline__ int group_tasks(const int32_t *rowptr, int32_t n, int g, int mode,
-                                           int threshold, bool *is_warp) {
+                                           int threshold, bool *is_warp, bool rev) {
     const int r0 = g * 32;
     const int rows = min(32, n - r0);
-    const long long gnnz = (long long)rowptr[r0 + rows] - rowptr[r0];
+    const long long gnnz = rev ? (long long)rowptr[n - r0] - rowptr[n - r0 - rows]
+                               : (long long)rowptr[r0 + rows] - rowptr[r0];
     const bool w = (mode == 2) || (mode == 0 && gnnz > (long long)threshold * rows);
     *is_warp = w;
     return w ? rows : 1;
@@ -111,13 +114,13 @@ __device__ __forceinline__ int block_exclusive_scan(int v, int *s_warp, int *tot
 
 __global__ void __launch_bounds__(1024) k_plan_count(const int32_t *__restrict__ rowptr, int32_t n,
                                                      int32_t ngroups, int mode, int threshold,
-                                                     int32_t *blk_tasks, int32_t *blk_tgroups) {
+                                                     int32_t *blk_tasks, int32_t *blk_tgroups, bool rev) {
     __shared__ int s_warp[33];
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
     int t = 0, tg = 0;
     if (g < ngroups) {
         bool w;
-        t = group_tasks(rowptr, n, g, mode, threshold, &w);
+        t = group_tasks(rowptr, n, g, mode, threshold, &w, rev);
         tg = w ? 0 : 1;
     }
     int tot_t, tot_g;
@@ -132,12 +135,12 @@ __global__ void __launch_bounds__(1024) k_plan_count(const int32_t *__restrict__
 __global__ void __launch_bounds__(1024) k_plan_write(const int32_t *__restrict__ rowptr, int32_t n,
                                                      int32_t ngroups, int mode, int threshold,
                                                      const int32_t *__restrict__ blk_offset,
-                                                     int32_t *tasks) {
+                                                     int32_t *tasks, bool rev) {
     __shared__ int s_warp[33];
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
     int t = 0;
     bool w = false;
-    if (g < ngroups) t = group_tasks(rowptr, n, g, mode, threshold, &w);
+    if (g < ngroups) t = group_tasks(rowptr, n, g, mode, threshold, &w, rev);
     int tot;
     const int off = block_exclusive_scan(t, s_warp, &tot) + blk_offset[blockIdx.x];
     if (g < ngroups) {

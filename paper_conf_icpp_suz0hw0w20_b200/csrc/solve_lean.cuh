@@ -24,46 +24,12 @@ namespace sptrsv_dev {
 
 constexpr int kLeanCta = 256;
 
-// UPPER / UNIT (SURVEY f4): upper-triangular rows (diagonal first, dependencies
-// j > i) are taken in REVERSE order -- logical row r is row n-1-r, so the ticket
-// order is again a topological order; UNIT: the diagonal is implicitly 1 and
-// not stored.
-template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false>
-__global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
-    __shared__ uint32_t s_blk, s_epoch;
-    const int tid = threadIdx.x;
-    const int lane = tid & 31;
-    const uint64_t pol = policy_evict_first();
-    // ---- speculative first-level loads for logical block == blockIdx.x
-    int i = (int)blockIdx.x * kLeanCta + tid;
-    if (UPPER) i = p.n - 1 - i;
-    int rs = 0, re = 1;
-    double bi = 0.0;
-    if (i >= 0 && i < p.n) {
-        rs = ld_stream_i32(p.rowptr + i, pol);
-        re = ld_stream_i32(p.rowptr + i + 1, pol);
-        bi = ld_stream_f64(p.b + i, pol);
-    }
-    if (tid == 0) {
-        if (p.trace) {
-            atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
-            atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
-        }
-        cta_ticket(p, s_blk, s_epoch);
-    }
-    __syncthreads();
-    const uint32_t epoch = s_epoch;
-    if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
-        i = (int)s_blk * kLeanCta + tid;
-        if (UPPER) i = p.n - 1 - i;
-        rs = 0, re = 1, bi = 0.0;
-        if (i >= 0 && i < p.n) {
-            rs = ld_stream_i32(p.rowptr + i, pol);
-            re = ld_stream_i32(p.rowptr + i + 1, pol);
-            bi = ld_stream_f64(p.b + i, pol);
-        }
-    }
-    const bool act = i >= 0 && i < p.n;
+// One warp, one row per lane (Alg.5 l.3-18): lane's row i (act: i is a real row), its
+// bounds [rs, re) and b_i already loaded.  Returns when every lane of the warp has
+// published, or on abort.  Shared by k_solve_lean and the f4 list kernel (solve_tri.cuh).
+template <int PROTO, bool UPPER, bool UNIT>
+__device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int rs, int re, double bi,
+                                          uint32_t epoch, int lane, uint64_t pol) {
     // off-diagonal entries [lo, hi); the diagonal is last (lower), first (upper) or implicit
     // (unit).  They are consumed earliest-solved first: ascending for lower (Alg.1 l.3-4),
     // DESCENDING for upper (G25) -- the nearest, latest dependency is waited for last.
@@ -143,6 +109,49 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
             if (__shfl_sync(FULL, ab, 0)) break;
         }
     }
+}
+
+// UPPER / UNIT (SURVEY f4): upper-triangular rows (diagonal first, dependencies
+// j > i) are taken in REVERSE order -- logical row r is row n-1-r, so the ticket
+// order is again a topological order; UNIT: the diagonal is implicitly 1 and
+// not stored.
+template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false>
+__global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
+    __shared__ uint32_t s_blk, s_epoch;
+    const int tid = threadIdx.x;
+    const int lane = tid & 31;
+    const uint64_t pol = policy_evict_first();
+    // ---- speculative first-level loads for logical block == blockIdx.x
+    int i = (int)blockIdx.x * kLeanCta + tid;
+    if (UPPER) i = p.n - 1 - i;
+    int rs = 0, re = 1;
+    double bi = 0.0;
+    if (i >= 0 && i < p.n) {
+        rs = ld_stream_i32(p.rowptr + i, pol);
+        re = ld_stream_i32(p.rowptr + i + 1, pol);
+        bi = ld_stream_f64(p.b + i, pol);
+    }
+    if (tid == 0) {
+        if (p.trace) {
+            atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
+            atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
+        }
+        cta_ticket(p, s_blk, s_epoch);
+    }
+    __syncthreads();
+    const uint32_t epoch = s_epoch;
+    if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
+        i = (int)s_blk * kLeanCta + tid;
+        if (UPPER) i = p.n - 1 - i;
+        rs = 0, re = 1, bi = 0.0;
+        if (i >= 0 && i < p.n) {
+            rs = ld_stream_i32(p.rowptr + i, pol);
+            re = ld_stream_i32(p.rowptr + i + 1, pol);
+            bi = ld_stream_f64(p.b + i, pol);
+        }
+    }
+    const bool act = i >= 0 && i < p.n;
+    lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);
     if (p.trace && lane == 0) atomicMax(&p.trace[3 * (size_t)p.n + 1], globaltimer_ns());  // last warp exit
 }
 

@@ -18,6 +18,7 @@
 #include "solve_k.cuh"
 #include "solve_dyn.cuh"
 #include "solve_lean.cuh"
+#include "solve_tri.cuh"
 #include "solve_multi.cuh"
 #include "solve_paper.cuh"
 #include "sptrsv.h"
@@ -238,7 +239,8 @@ int build_plan(sptrsv_handle_s *h) {
             rc = SPTRSV_ERR_ALLOC;
             break;
         }
-        k_plan_count<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_bt, d_bg);
+        const bool rev = h->tri & SPTRSV_TRI_UPPER;  // f4 upper: plan over logical (reversed) rows
+        k_plan_count<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_bt, d_bg, rev);
         if (cudaGetLastError() != cudaSuccess ||
             cudaMemcpy(bt.data(), d_bt, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess ||
             cudaMemcpy(bg.data(), d_bg, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess) {
@@ -274,7 +276,7 @@ int build_plan(sptrsv_handle_s *h) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
             }
-            k_plan_write<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_off, h->ws.tasks);
+            k_plan_write<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_off, h->ws.tasks, rev);
             if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
@@ -349,7 +351,6 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
     h->colidx = colidx;
     h->val = val;
     h->tri = tri_flags;
-    if (tri_flags) h->mode = 1;  // f4 forms run on the thread-level LEAN engine only
     unsigned long long *d_status = nullptr, *d_near = nullptr;
     int32_t *d_maxrow = nullptr;
     do {
@@ -459,13 +460,15 @@ int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem,
 // ENGINE_AUTO: all-thread-level plans go to the LEAN engine unless a quarter or
 // more of the dependencies are "near" (within 256 rows: chains, grid wavefronts),
 // where the staged one-shot engine's shared-memory local resolution wins; plans
-// with warp-level rows use the staged one-shot engine.  (Round-1 B200 sweeps,
-// DESIGN.md section 8.)
+// with warp-level rows use the HYBRID engine (2-13% faster than the staged
+// one-shot engine on every warp-plan shape measured, tools/hybrid_probe.py).
+// (Round-1 B200 sweeps.)
 int resolve_engine(const sptrsv_handle_s *h) {
-    if (h->tri) return 3;  // upper / unit-diagonal handles: LEAN only
+    if (h->tri) return h->plan == PLAN_THREAD ? 3 : 6;  // f4 handles: LEAN or tri hybrid
     if (h->engine != 5) return h->engine;
     const long long offdiag = h->nnz - h->n;
     if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_deps < offdiag)) return 3;
+    if (h->plan != PLAN_THREAD) return 6;
     return 0;
 }
 
@@ -475,6 +478,11 @@ int resolve_engine(const sptrsv_handle_s *h) {
 // chains): 2 rows per lane in 128-thread CTAs; on plans with warp-level rows:
 // 64-thread CTAs; everything else 256 threads, 1 row per lane.
 void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) {
+    if (engine == 3 || engine == 6) {  // fixed geometry: LEAN 256 threads, HYBRID 64
+        *cta = (engine == 6 && h->plan != PLAN_THREAD) ? kTriWarpCta : kLeanCta;
+        *K = 1;
+        return;
+    }
     int c = 256, k = 1;
     if (engine == 0) {
         if (h->plan == PLAN_THREAD && h->nnz > h->n && 4 * h->near_deps >= h->nnz - h->n) {
@@ -499,14 +507,31 @@ lean_fn lean_tri_kernel(int proto, int tri) {
     return tab[tri & 3][proto ? 1 : 0];
 }
 
+lean_fn tri_warp_kernel(int proto, int tri, int plan) {
+#define TRI_ROW(U, N)                                                                              \
+    {k_solve_tri_warp<PROTO_FLAGS, U, N, PLAN_WARP>, k_solve_tri_warp<PROTO_FUSED, U, N, PLAN_WARP>, \
+     k_solve_tri_warp<PROTO_FLAGS, U, N, PLAN_LIST>, k_solve_tri_warp<PROTO_FUSED, U, N, PLAN_LIST>}
+    static const lean_fn tab[4][4] = {TRI_ROW(false, false), TRI_ROW(true, false), TRI_ROW(false, true),
+                                      TRI_ROW(true, true)};
+#undef TRI_ROW
+    return tab[tri & 3][(plan == PLAN_LIST ? 2 : 0) + (proto ? 1 : 0)];
+}
+
 int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
-    if (h->tri) {  // f4: upper / unit-diagonal forms on the LEAN engine (solve_lean.cuh)
-        L->fn = (const void *)lean_tri_kernel(h->proto, h->tri);
+    if (h->tri || (!h->variant && resolve_engine(h) == 6)) {  // f4 forms, or ENGINE_HYBRID (solve_lean.cuh / solve_tri.cuh)
         L->kind = 0;
-        L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
-        L->block = dim3((unsigned)kLeanCta);
         L->smem = 0;
-        L->key = 7000000 + h->proto * 100000 + h->tri * 10000;
+        if (h->plan != PLAN_THREAD) {  // warp-level rows present: one task per warp
+            L->fn = (const void *)tri_warp_kernel(h->proto, h->tri, h->plan);
+            L->grid = dim3((unsigned)((h->n_tasks + kTriWarpCta / 32 - 1) / (kTriWarpCta / 32)));
+            L->block = dim3((unsigned)kTriWarpCta);
+            L->key = 7500000 + h->proto * 100000 + h->tri * 10000 + h->plan * 1000;
+        } else {  // all thread level: LEAN
+            L->fn = (const void *)lean_tri_kernel(h->proto, h->tri);
+            L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
+            L->block = dim3((unsigned)kLeanCta);
+            L->key = 7000000 + h->proto * 100000 + h->tri * 10000;
+        }
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
@@ -817,11 +842,8 @@ int sptrsv_destroy(sptrsv_handle_t h) {
 
 int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
-    if (h->tri) {  // f4 handles: thread-level LEAN only; the paper's variants are lower-only
-        if ((key == SPTRSV_OPT_MODE && value == 2) || (key == SPTRSV_OPT_VARIANT && value != 0))
-            return SPTRSV_ERR_INVALID_ARG;
-        if (key == SPTRSV_OPT_MODE) return (value < 0 || value > 2) ? SPTRSV_ERR_INVALID_ARG : SPTRSV_OK;
-    }
+    if (h->tri && key == SPTRSV_OPT_VARIANT && value != 0)
+        return SPTRSV_ERR_INVALID_ARG;  // the paper's kernels are lower-only
     switch (key) {
         case SPTRSV_OPT_MODE:
             if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
@@ -883,7 +905,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->local = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
-            if (value < 0 || value > 5) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 6) return SPTRSV_ERR_INVALID_ARG;
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_STAGES:

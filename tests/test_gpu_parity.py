@@ -344,15 +344,39 @@ def test_lean_engine(cap, proto):
 
 
 def test_engine_auto_choice(cap):
-    """ENGINE_AUTO: far dependencies -> LEAN (3); chains / grid wavefronts -> staged one-shot (0)."""
+    """ENGINE_AUTO: far dependencies -> LEAN (3); chains / grid wavefronts -> staged one-shot (0);
+    plans with warp-level rows -> HYBRID (6)."""
     for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 0, 128, 2),
                               (lambda: synth.gen_chain(3000), 0, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
-                              (lambda: synth.gen_c4(n=5000, nlevels=50), 0, 64, 1)):
+                              (lambda: synth.gen_c4(n=5000, nlevels=50), 6, 64, 1)):
         s = gen()
         x, info = gpu_solve(cap, s)
         assert (info["engine"], info["cta_threads"], info["rows_per_lane"]) == (want, cta, K), (s.name, info)
         ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
         assert relerr(x, ref) <= TOL
+
+
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("mode", MODES)
+def test_hybrid_engine(cap, proto, mode):
+    """ENGINE_HYBRID (6): warp tasks + 32-row thread groups in 64-thread CTAs, lower handles."""
+    for n in (1, 31, 33, 257, 4099):
+        s = synth.gen_random_lower(n, 24, seed=n + 17)
+        x, info = gpu_solve(cap, s, mode, protocol=proto, engine=6)
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        assert info["engine"] == 6
+        if mode == 1:
+            assert np.array_equal(x, ref), n
+        else:
+            assert relerr(x, ref) <= TOL, n
+    for gen in (lambda: synth.gen_c4(n=60_000, nlevels=120), lambda: synth.gen_grid(150),
+                lambda: synth.gen_dense_lower(300), lambda: synth.gen_leveled(100_000, 10, 1, 40, 3, "l")):
+        s = gen()
+        x, _ = gpu_solve(cap, s, mode, protocol=proto, engine=6)
+        assert relerr(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)) <= TOL, s.name
+    si = synth.integerize(synth.gen_leveled(50_000, 20, 1, 30, 4, "l"))
+    x, _ = gpu_solve(cap, si, mode, protocol=proto, engine=6)
+    assert np.array_equal(x, si.x_true)
 
 
 @pytest.mark.parametrize("nrhs", [1, 2, 3, 4, 7, 8, 16, 32])

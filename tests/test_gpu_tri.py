@@ -15,6 +15,11 @@ pytestmark = pytest.mark.gpu
 
 U, UNIT = oracle.UPPER, oracle.UNIT_DIAG
 FORMS = [U, UNIT, U | UNIT]
+TOL = 1e-12  # warp-level rows (lane-strided sums), as tests/test_gpu_parity.py
+
+
+def relerr(a, ref):
+    return float(np.max(np.abs(a - ref) / np.maximum(np.abs(ref), 1e-300)))
 
 
 @pytest.fixture(scope="module")
@@ -75,8 +80,10 @@ def test_tri_structured_bit_exact(cap, which, flags):
             "dense": lambda: synth.gen_dense_lower(400), "chain": lambda: synth.gen_chain(30_000)}[which]()
     s = form(base, flags)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
-    x, _ = gpu_solve(cap, s, flags)
+    x, _ = gpu_solve(cap, s, flags, mode=1)  # thread level everywhere: bit-exact
     assert np.array_equal(x, ref)
+    x, _ = gpu_solve(cap, s, flags)  # AUTO (warp rows where long): warp-mode bound
+    assert relerr(x, ref) <= TOL
 
 
 @pytest.mark.parametrize("flags", [0, U, UNIT, U | UNIT])
@@ -130,6 +137,47 @@ def test_unit_lower_chain_closed_form(cap):
     s = synth.CSRSystem("uc", n, rp, ci, -np.ones(n - 1), np.ones(n), None, {})
     x, _ = gpu_solve(cap, s, UNIT)
     assert np.array_equal(x, np.arange(1, n + 1, dtype=float))
+
+
+@pytest.mark.parametrize("n", [1, 2, 33, 1000, 4099])
+@pytest.mark.parametrize("flags", FORMS)
+@pytest.mark.parametrize("proto", [0, 1])
+def test_tri_warp_mode(cap, n, flags, proto):
+    """MODE = 2: one warp per row (k_solve_tri_warp); lane-strided sums -> warp-mode bound."""
+    s = form(synth.gen_random_lower(n, 40, seed=n + 3), flags)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
+    x, info = gpu_solve(cap, s, flags, mode=2, protocol=proto)
+    assert info["engine"] == 6 and info["n_warp_rows"] == n
+    assert relerr(x, ref) <= TOL
+
+
+@pytest.mark.parametrize("flags", FORMS)
+def test_tri_c4_auto_picks_warp(cap, flags):
+    """c4-like rows (~64 entries) in each form: AUTO plans every row warp-level."""
+    s = form(synth.gen_c4(n=100_000, nlevels=100), flags)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
+    x, info = gpu_solve(cap, s, flags)
+    assert info["engine"] == 6
+    assert relerr(x, ref) <= TOL
+    assert relerr(x, s.x_true) <= TOL
+
+
+@pytest.mark.parametrize("flags", FORMS)
+def test_tri_integer_warp_mode_bit_exact(cap, flags):
+    """Exact-integer values: any summation order is exact, so warp rows are bit-exact too."""
+    s = synth.integerize(synth.gen_random_lower(20_000, 30, 31))
+    if flags & U:
+        s = synth.to_upper(s)
+    if flags & UNIT:
+        rows = np.repeat(np.arange(s.n), np.diff(s.rowptr))
+        keep = s.colidx != rows
+        rp = np.zeros(s.n + 1, np.int64)
+        np.cumsum(np.bincount(rows[keep], minlength=s.n), out=rp[1:])
+        ci, v = s.colidx[keep], s.val[keep]
+        b = s.x_true + np.bincount(rows[keep], weights=v * s.x_true[ci], minlength=s.n)
+        s = synth.CSRSystem("u", s.n, rp.astype(np.int32), ci, v, b, s.x_true, {})
+    x, _ = gpu_solve(cap, s, flags, mode=2)
+    assert np.array_equal(x, s.x_true)
 
 
 @pytest.mark.parametrize("flags", FORMS)
@@ -230,8 +278,6 @@ def test_tri_unsupported_calls_fail_loudly(cap):
             h.solve_multi(torch.zeros((s.n, 2), dtype=torch.float64, device="cuda:0"))
         with pytest.raises(cap.SptrsvError):
             h.levels()
-        with pytest.raises(cap.SptrsvError):
-            h.set_option(cap.OPT_MODE, cap.MODE_WARP)
         with pytest.raises(cap.SptrsvError):
             h.set_option(cap._lib.OPT_VARIANT, 5)
         # still solves correctly after the refused calls
