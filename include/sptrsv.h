@@ -103,6 +103,14 @@ typedef enum sptrsv_option {
                                       ONE-SHOT engine with CTAs of <= 256 threads          */
     SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5 (default), 6 or 8
                                       resident 256-thread CTAs per SM                       */
+    SPTRSV_OPT_PREFETCH = 18,      /* L2 bulk prefetch (cp.async.bulk.prefetch.L2) of the
+                                      CSR range of the CTA this many logical blocks ahead:
+                                      -1 (default) = the engine's measured choice, 0 = off.
+                                      A cache hint only; never changes a result            */
+    SPTRSV_OPT_POLL_GAP_NS = 19,   /* LEAN: __nanosleep after a pass that progressed but left
+                                      lanes waiting (0 = default, none)                    */
+    SPTRSV_OPT_POLL_ONE = 20,      /* LEAN: 1 = poll one dependency per lane per pass
+                                      (default 0: the next two, DESIGN G21)                 */
     SPTRSV_OPT_VARIANT = 16        /* ablation: 0 (default) product path; 3, 4, 5
                                       = the paper's Alg.3 SyncFree (warp per row), Alg.4
                                       Two-Phase, Alg.5 Writing-First with their printed

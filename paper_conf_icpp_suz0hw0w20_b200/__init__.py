@@ -142,9 +142,10 @@ class Handle:
     def trace(self, b, x=None, stream=None):
         """Diagnostic solve: (x, trace) with trace[:n] = publish time (ns, %globaltimer) of each
         x_i, trace[n:2n] = when (thread-level) row i consumed its last dependency (0 = none) and
-        trace[2n:] = when its solve loop started (0 = not recorded)."""
+        trace[2n:3n] = when its solve loop started (0 = not recorded), trace[3n:3n+3] = kernel
+        first entry / last exit / CTAs started, trace[3n+3:4n+3] = when row i's CTA entered (LEAN)."""
         import torch
-        tr = torch.zeros(3 * self.n + 3, dtype=torch.int64, device=self.device)
+        tr = torch.zeros(4 * self.n + 3, dtype=torch.int64, device=self.device)
         tr[3 * self.n] = (1 << 63) - 1
         check(lib.sptrsv_set_trace(self._h, tr.data_ptr()), "sptrsv_set_trace")
         try:
@@ -194,7 +195,9 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
             "pipe_stages": _lib.OPT_PIPE_STAGES, "pipe_batch": _lib.OPT_PIPE_BATCH,
             "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
-            "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY}
+            "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY,
+            "prefetch": _lib.OPT_PREFETCH, "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
+            "poll_one": _lib.OPT_POLL_ONE}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

@@ -54,6 +54,9 @@ OPT_PIPE_ENTRIES = 14
 OPT_ROWS_PER_LANE = 15
 OPT_VARIANT = 16
 OPT_LEAN_OCCUPANCY = 17
+OPT_PREFETCH = 18
+OPT_POLL_GAP_NS = 19
+OPT_POLL_ONE = 20
 ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2

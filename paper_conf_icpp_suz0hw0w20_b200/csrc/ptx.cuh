@@ -98,6 +98,19 @@ __device__ __forceinline__ double ld_stream_f64(const double *p, uint64_t pol) {
     return v;
 }
 
+// Bulk L2 prefetch (TMA unit, no shared memory, no completion to wait for) of the
+// byte range [lo, hi), shrunk inward to 16-byte boundaries so it never touches a
+// byte outside the caller's arrays.  A hint only: it changes no result.
+__device__ __forceinline__ void bulk_prefetch_l2(const void *lo, const void *hi) {
+    uintptr_t a = ((uintptr_t)lo + 15) & ~(uintptr_t)15;
+    const uintptr_t e = (uintptr_t)hi & ~(uintptr_t)15;
+    while (a < e) {
+        const uintptr_t c = (e - a) > 65536 ? 65536 : (e - a);
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((unsigned)c) : "memory");
+        a += c;
+    }
+}
+
 __device__ __forceinline__ void nanosleep_ns(uint32_t ns) {
     asm volatile("nanosleep.u32 %0;" ::"r"(ns));
 }

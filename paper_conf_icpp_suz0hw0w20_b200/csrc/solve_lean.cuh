@@ -23,6 +23,16 @@
 namespace sptrsv_dev {
 
 constexpr int kLeanCta = 256;
+constexpr int kLeanPrefetchDefault = 0;  // SPTRSV_OPT_PREFETCH = -1 resolves to this (CTAs ahead)
+
+// L2 bulk prefetch of the physical rows [A, B): rowptr[A..B], b[A..B) and the
+// entries [pa, pb) = [rowptr[A], rowptr[B]) of colidx and val.
+__device__ __forceinline__ void prefetch_rows_l2(const SolveParams &p, int A, int B, int pa, int pb) {
+    bulk_prefetch_l2(p.rowptr + A, p.rowptr + B + 1);
+    bulk_prefetch_l2(p.b + A, p.b + B);
+    bulk_prefetch_l2(p.colidx + pa, p.colidx + pb);
+    bulk_prefetch_l2(p.val + pa, p.val + pb);
+}
 
 // One warp, one row per lane (Alg.5 l.3-18): lane's row i (act: i is a real row), its
 // bounds [rs, re) and b_i already loaded.  Returns when every lane of the warp has
@@ -45,6 +55,7 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
     int nc2 = (act && inr(j + dir)) ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
     Diag dg;
     dg.init(dv);
+    if (p.trace && act && nc != -2) p.trace[2 * (size_t)p.n + i] = globaltimer_ns();  // loads landed
     double ls = 0.0;
     bool done = !act;
     Cta nocta;
@@ -71,7 +82,7 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
                 // poll the next two dependencies together, consume the ready prefix in row order
                 unsigned long long a0, a1, c0 = 0, c1 = 0;
                 poll1<PROTO>(p, nc, a0, a1);
-                const int cc2 = nc2;
+                const int cc2 = p.poll_one ? -1 : nc2;
                 if (cc2 >= 0) poll1<PROTO>(p, cc2, c0, c1);
                 if (ready1<PROTO>(a0, a1, epoch)) {
                     if (p.trace) p.trace[p.n + i] = globaltimer_ns();
@@ -93,6 +104,7 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
         if (__ballot_sync(FULL, prog)) {
             backoff = p.backoff_min;
             idle = 0;
+            if (p.poll_gap) nanosleep_ns(p.poll_gap);
             continue;
         }
         if (backoff) nanosleep_ns(backoff);
@@ -127,9 +139,23 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
     int rs = 0, re = 1;
     double bi = 0.0;
     if (i >= 0 && i < p.n) {
+        if (p.trace) p.trace[3 * (size_t)p.n + 3 + i] = globaltimer_ns();  // CTA entry
         rs = ld_stream_i32(p.rowptr + i, pol);
         re = ld_stream_i32(p.rowptr + i + 1, pol);
         bi = ld_stream_f64(p.b + i, pol);
+    }
+    // ---- L2 bulk prefetch of the block pf_dist logical blocks ahead (speculatively
+    // blockIdx.x + pf_dist): its bounds load overlaps the ticket, the copy is issued after it
+    int pfA = 0, pfB = 0, pfa = 0, pfb = 0;
+    if (p.pf_dist > 0 && tid == 32) {
+        const long long r0 = ((long long)blockIdx.x + p.pf_dist) * kLeanCta;
+        if (r0 < p.n) {
+            const int r1 = (int)min((long long)p.n, r0 + kLeanCta);
+            pfA = UPPER ? p.n - r1 : (int)r0;
+            pfB = UPPER ? p.n - (int)r0 : r1;
+            pfa = ld_stream_i32(p.rowptr + pfA, pol);
+            pfb = ld_stream_i32(p.rowptr + pfB, pol);
+        }
     }
     if (tid == 0) {
         if (p.trace) {
@@ -140,6 +166,7 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
     }
     __syncthreads();
     const uint32_t epoch = s_epoch;
+    if (pfB > pfA) prefetch_rows_l2(p, pfA, pfB, pfa, pfb);
     if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
         i = (int)s_blk * kLeanCta + tid;
         if (UPPER) i = p.n - 1 - i;

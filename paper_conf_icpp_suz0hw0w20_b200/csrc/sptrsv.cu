@@ -80,6 +80,9 @@ struct sptrsv_handle_s {
     int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
     int lean_minb = 5;      // LEAN: minimum resident CTAs per SM the register budget targets
+    int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
+    uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
+    int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
     int grid_cache = 0;
@@ -440,6 +443,7 @@ struct Launch {
     size_t smem = 0;
     PipeGeom geom;
     int key = 0;  // configuration identity (the epoch arithmetic needs a fixed grid per key)
+    int pf_dist = 0;  // SolveParams::pf_dist (engines that implement the L2 prefetch)
 };
 
 int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem, int key, int *out) {
@@ -616,6 +620,7 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
         L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
         L->block = dim3((unsigned)kLeanCta);
         L->smem = 0;
+        L->pf_dist = h->pf_dist < 0 ? kLeanPrefetchDefault : h->pf_dist;
         L->key = 5000000 + h->proto * 100000 + h->lean_minb * 1000;
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;
@@ -665,7 +670,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
         if (rc) return rc;
         h->launch_key = L.key;
     }
-    SolveParams p;
+    SolveParams p{};
     p.rowptr = h->rowptr;
     p.colidx = h->colidx;
     p.val = h->val;
@@ -685,6 +690,9 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.spin_limit = h->spin_limit;
     p.stage = h->stage;
     p.local = h->local;
+    p.pf_dist = L.pf_dist;
+    p.poll_gap = h->poll_gap;
+    p.poll_one = h->poll_one;
     p.trace = h->trace;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = L.grid;
@@ -932,6 +940,18 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 5 && value != 6 && value != 8) return SPTRSV_ERR_INVALID_ARG;
             h->lean_minb = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_PREFETCH:
+            if (value < -1 || value > (1 << 24)) return SPTRSV_ERR_INVALID_ARG;
+            h->pf_dist = (int)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_POLL_GAP_NS:
+            if (value < 0 || value > 1000000) return SPTRSV_ERR_INVALID_ARG;
+            h->poll_gap = (uint32_t)value;
+            return SPTRSV_OK;
+        case SPTRSV_OPT_POLL_ONE:
+            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            h->poll_one = (int)value;
+            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -957,6 +977,9 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_ROWS_PER_LANE: *value = h->rows_per_lane; return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT: *value = h->variant; return SPTRSV_OK;
         case SPTRSV_OPT_LEAN_OCCUPANCY: *value = h->lean_minb; return SPTRSV_OK;
+        case SPTRSV_OPT_PREFETCH: *value = h->pf_dist; return SPTRSV_OK;
+        case SPTRSV_OPT_POLL_GAP_NS: *value = h->poll_gap; return SPTRSV_OK;
+        case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }

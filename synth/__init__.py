@@ -367,4 +367,9 @@ CONFIGS = {
 def make(name: str, **kw) -> CSRSystem:
     if name.startswith("c5_"):
         return gen_c5(int(name[3:]), **kw)
+    if name.startswith("diag:"):  # scratch shapes for the perf tools: diag:N, lev:N:L
+        return gen_diag(int(name.split(":")[1]))
+    if name.startswith("lev:"):
+        _, n, nl = name.split(":")
+        return gen_leveled(int(n), int(nl), 1, 1, 2, name)
     return CONFIGS[name](**kw)

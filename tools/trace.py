@@ -40,6 +40,20 @@ out["per_level_us_p10_50_90"] = [round(float(a), 3) for a in q]
 if nl <= 40:
     out["level_done_us"] = [round(float(a) / 1e3, 2) for a in lvl_done]
     out["level_first_us"] = [round(float(a) / 1e3, 2) for a in lvl_first]
+    stv = tt[2 * s.n:3 * s.n]
+    if (stv > 0).all():
+        st0 = stv - t0
+        out["level_start_p0_50_100_us"] = [[round(float(np.percentile(st0[lv == l], q)) / 1e3, 2) for q in (0, 50, 100)]
+                                           for l in range(nl)]
+        out["level_publish_p50_us"] = [round(float(np.percentile(t[lv == l], 50)) / 1e3, 2) for l in range(nl)]
+    ent = tt[3 * s.n + 3:4 * s.n + 3] if tt.size >= 4 * s.n + 3 else np.zeros(0)
+    if ent.size and (ent > 0).all():
+        e0 = ent - t0
+        out["level_entry_p0_50_100_us"] = [[round(float(np.percentile(e0[lv == l], q)) / 1e3, 2) for q in (0, 50, 100)]
+                                           for l in range(nl)]
+        if (stv > 0).all():
+            ld = (stv - ent)
+            out["load_latency_ns_p10_50_90"] = [int(np.percentile(ld, q)) for q in (10, 50, 90)]
 if name == "chain":
     dt = np.diff(t)
     idx = np.arange(1, s.n)
