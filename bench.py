@@ -473,7 +473,8 @@ def main():
                        "mode": {0: "auto", 1: "thread", 2: "warp"}[args.mode],
                        "plan": {"thread_groups": info["n_thread_groups"], "warp_rows": info["n_warp_rows"]},
                        "engine": {0: "one-shot (staged, in-CTA x copy)", 1: "pipe (TMA ring)", 2: "dyn",
-                                  3: "lean", 4: "dyn-static", 6: "hybrid (warp tasks + 32-row thread groups)"}.get(info["engine"], str(info["engine"])),
+                                  3: "lean", 4: "dyn-static", 6: "hybrid (warp tasks + 32-row thread groups)",
+                                  7: "chain (in-warp shuffle chain)"}.get(info["engine"], str(info["engine"])),
                        "cta_threads": info["cta_threads"], "rows_per_lane": info["rows_per_lane"],
                        "analyse_ms": round(info["analyse_ms"], 3),
                        "l2": "flushed between timed steps (256 MiB write, outside the per-step events)",

@@ -111,6 +111,9 @@ typedef enum sptrsv_option {
                                       lanes waiting (0 = default, none)                    */
     SPTRSV_OPT_POLL_ONE = 20,      /* LEAN: 1 = poll one dependency per lane per pass
                                       (default 0: the next two, DESIGN G21)                 */
+    SPTRSV_OPT_CHAIN_PUBLISH = 21, /* CHAIN engine (FUSED): finalized rows are published in
+                                      warp-wide batches every this many chain steps, 1..64
+                                      (default 32)                                         */
     SPTRSV_OPT_VARIANT = 16        /* ablation: 0 (default) product path; 3, 4, 5
                                       = the paper's Alg.3 SyncFree (warp per row), Alg.4
                                       Two-Phase, Alg.5 Writing-First with their printed
@@ -128,6 +131,7 @@ typedef struct sptrsv_info {
     float analyse_ms;         /* wall time of sptrsv_analyse_csr (Table 1 analogue)        */
     uint32_t solves;          /* solves enqueued through this handle                      */
     int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
+    int64_t warp_deps;        /* dependencies inside the row's own 32-row group            */
     int32_t engine;           /* engine the next solve uses (AUTO resolved)                */
     int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */

@@ -57,7 +57,9 @@ OPT_LEAN_OCCUPANCY = 17
 OPT_PREFETCH = 18
 OPT_POLL_GAP_NS = 19
 OPT_POLL_ONE = 20
+OPT_CHAIN_PUBLISH = 21
 ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
+ENGINE_HYBRID, ENGINE_CHAIN = 6, 7
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
 
@@ -74,6 +76,7 @@ class sptrsv_info(ctypes.Structure):
         ("analyse_ms", ctypes.c_float),
         ("solves", ctypes.c_uint32),
         ("near_deps", ctypes.c_int64),
+        ("warp_deps", ctypes.c_int64),
         ("engine", ctypes.c_int32),
         ("cta_threads", ctypes.c_int32),
         ("rows_per_lane", ctypes.c_int32),

@@ -19,8 +19,8 @@ enum : int {  // same numbering as sptrsv_status (negated)
 // status: 64-bit min over (row << 8 | code) -> the lowest offending row wins,
 // which is the row-ordered error the oracle reports too.
 // Also counts "near" dependencies (|i - col| < 256: produced within about one CTA
-// of rows) -- the statistic ENGINE_AUTO uses to choose between the shared-memory
-// local resolution of the staged engine and the lean engine.
+// of rows) and in-warp ones (i and col in the same 32-row group) -- the statistics
+// ENGINE_AUTO uses to choose between the LEAN, ONE-SHOT and CHAIN engines.
 // tri: bit 0 UPPER (entries j >= i, diagonal FIRST), bit 1 UNIT
 // (diagonal implicit 1, not stored: entries strictly inside the triangle).
 __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ rowptr,
@@ -32,7 +32,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
     const bool upper = tri & 1, unit = tri & 2;
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     int len = 0;
-    unsigned near = 0;
+    unsigned near = 0, wdep = 0;
     if (i < n) {
         const int64_t s = rowptr[i], e = rowptr[i + 1];
         int code = 0;
@@ -50,6 +50,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
                 if (c >= n) { code = E_BAD_COL; break; }  // upper only (lower has c <= i < n)
                 if (j > s && c <= prev) { code = E_UNSORTED; break; }
                 if (c != i && (c > i ? c - i : i - c) < 256) ++near;
+                if (c != i && (c >> 5) == (i >> 5)) ++wdep;
                 prev = c;
             }
             if (!code && !unit) {
@@ -65,9 +66,12 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
     for (int off = 16; off > 0; off >>= 1) {
         len = max(len, __shfl_xor_sync(0xffffffffu, len, off));
         near += __shfl_xor_sync(0xffffffffu, near, off);
+        wdep += __shfl_xor_sync(0xffffffffu, wdep, off);
     }
     if ((threadIdx.x & 31) == 0 && len > 0) atomicMax(max_row, len);
-    if ((threadIdx.x & 31) == 0 && near) atomicAdd(near_deps, (unsigned long long)near);
+    // both totals are < nnz < 2^31: near in the low word, wdep in the high word
+    if ((threadIdx.x & 31) == 0 && (near | wdep))
+        atomicAdd(near_deps, (unsigned long long)near | ((unsigned long long)wdep << 32));
 }
 
 // mode: 0 auto, 1 all thread-level, 2 all warp-level.

@@ -1,0 +1,268 @@
+// solve_chain.cuh -- ENGINE_CHAIN: warp-sequential resolution of in-warp dependency chains.
+//
+// The same per-row method as every engine -- Alg.5 Writing-First for
+// thread-level rows: stream the row, consume ready
+// dependencies in row order, divide at the diagonal, publish -- but with the
+// dependencies that fall INSIDE a warp's own rows resolved in registers instead
+// of through a flag / record round trip.  That is the shape of the paper's
+// "pure chain" and grid-wavefront regimes (bidiagonal and 5-point lower
+// factors: row i depends on i-1), where the one-shot engine paid ~0.3 us per
+// in-warp hop (shared-memory local rounds) and the record protocol ~0.5 us.
+//
+// A warp owns R = 32K consecutive rows r0 .. r0+R-1 (lane l owns r0 + l + 32k).
+// A row's off-diagonals split, by the sorted CSR order, into EXTERNAL ones
+// (col < r0, other warps: global FUSED / FLAGS protocol) followed by INTERNAL
+// ones (col in [r0, i), rows of this warp).  Each pass:
+//   A. external: every unfinished row whose next entry is external issues a poll
+//      (K polls per lane in flight while B and C run; consumed in D);
+//   B. catch-up: rows whose next entries are internal and already finalized
+//      read them from the warp's shared-memory copy s_x;
+//   C. chain: from the first unfinalized row s, while row s has no external
+//      entry left, its owner divides and publishes, the value is broadcast
+//      with one __shfl_sync, and every row whose next entry is column r0+s
+//      consumes it -- one step per row, no memory round trip on the chain;
+//   D. the polls of A are consumed (ready ones advance their row).
+// Accumulation stays in row order with separately rounded mul and add (external
+// entries precede internal ones in a sorted row), so x is bit-identical to
+// Alg.1, like every thread-level path.  Forward progress: a
+// row only waits on external rows (earlier warps / CTAs, which started first by
+// the CTA ticket) or on earlier rows of its own warp, finalized in order.
+#pragma once
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "solve.cuh"
+
+namespace sptrsv_dev {
+
+constexpr int kChainCta = 128;  // 4 warps
+constexpr int kChainEPR = 4;    // staged CSR entries per row (a longer slice reads global memory)
+
+__host__ __device__ constexpr int chain_warp_smem_bytes(int K) {
+    // s_val [32K*EPR] f64 | s_x [32K] f64 | s_col [32K*EPR] i32 | s_rp [32K+1] i32   (16-B multiple)
+    return ((8 * 32 * K * kChainEPR + 8 * 32 * K + 4 * 32 * K * kChainEPR + 4 * (32 * K + 1)) + 15) / 16 * 16;
+}
+
+template <int PROTO, int K>
+__global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams p) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ uint32_t s_blk, s_epoch;
+    constexpr int RT = 32 * K;
+    constexpr int ECAP = RT * kChainEPR;
+    const int warps = blockDim.x >> 5;
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) cta_ticket(p, s_blk, s_epoch);
+    __syncthreads();
+    const uint32_t epoch = s_epoch;
+    const int r0 = ((int)s_blk * warps + warp) * RT;
+    if (r0 >= p.n) return;
+    const int rows = min(RT, p.n - r0);
+    const uint64_t pol = policy_evict_first();
+    p.local = 0;  // no CTA-wide x copy in this engine (publish() skips it)
+    Cta nocta;
+    nocta.R0 = nocta.R1 = 0;
+    nocta.xc = nullptr;
+    nocta.xc_s = 0;
+    unsigned char *wsm = smem + (size_t)warp * chain_warp_smem_bytes(K);
+    double *s_val = reinterpret_cast<double *>(wsm);
+    double *s_x = s_val + ECAP;
+    int32_t *s_col = reinterpret_cast<int32_t *>(s_x + RT);
+    int32_t *s_rp = s_col + ECAP;
+    // ---- stage rowptr, b, then the warp's contiguous CSR slice (coalesced)
+    double bk[K];
+#pragma unroll
+    for (int k = 0; k <= K; ++k) {
+        const int idx = lane + 32 * k;
+        if (idx <= rows) s_rp[idx] = ld_stream_i32(p.rowptr + r0 + idx, pol);
+    }
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+        const int idx = lane + 32 * k;
+        bk[k] = idx < rows ? ld_stream_f64(p.b + r0 + idx, pol) : 0.0;
+    }
+    __syncwarp();
+    const int base = s_rp[0];
+    const int len = s_rp[rows] - base;
+    const bool staged = len <= ECAP;  // warp-uniform
+    if (staged) {
+#pragma unroll 4
+        for (int e = lane; e < len; e += 32) {
+            s_col[e] = ld_stream_i32(p.colidx + base + e, pol);
+            s_val[e] = ld_stream_f64(p.val + base + e, pol);
+        }
+    }
+    __syncwarp();
+    auto col_at = [&](int jj) -> int { return staged ? s_col[jj - base] : ld_stream_i32(p.colidx + jj, pol); };
+    auto val_at = [&](int jj) -> double { return staged ? s_val[jj - base] : ld_stream_f64(p.val + jj, pol); };
+    // ---- per-row state: cursor j, diagonal index je, next column / value, partial sum
+    int j[K], je[K], nc[K];
+    double nv[K], ls[K], xm[K];
+    Diag dg[K];
+    unsigned done = 0;  // bit k: row k of this lane finalized (or not a row)
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+        const int idx = lane + 32 * k;
+        const bool a = idx < rows;
+        j[k] = a ? s_rp[idx] : 0;
+        je[k] = a ? s_rp[idx + 1] - 1 : 0;
+        nc[k] = (a && j[k] < je[k]) ? col_at(j[k]) : -1;
+        nv[k] = (a && j[k] < je[k]) ? val_at(j[k]) : 0.0;
+        ls[k] = 0.0;
+        xm[k] = 0.0;
+        dg[k].init(a ? val_at(je[k]) : 1.0);
+        if (!a) done |= 1u << k;
+    }
+    auto advance = [&](int k) {
+        ++j[k];
+        const bool more = j[k] < je[k];
+        nc[k] = more ? col_at(j[k]) : -1;
+        nv[k] = more ? val_at(j[k]) : 0.0;
+    };
+    int s = 0;  // next row (warp-relative) to finalize; rows < s are published
+    uint32_t backoff = p.backoff_min, idle = 0;
+    while (true) {
+        bool prog = false;
+        // ---- A. external dependencies: one poll per unfinished row, K in flight
+        unsigned long long w0[K], w1[K];
+        unsigned gm = 0;
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            w0[k] = 0;
+            w1[k] = 0;
+            if (!(done >> k & 1u) && nc[k] >= 0 && nc[k] < r0) {
+                gm |= 1u << k;
+                poll1<PROTO>(p, nc[k], w0[k], w1[k]);
+            }
+        }
+        // ---- consume the ready polls
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            if ((gm >> k & 1u) && ready1<PROTO>(w0[k], w1[k], epoch)) {
+                if (p.trace) p.trace[p.n + r0 + lane + 32 * k] = globaltimer_ns();
+                ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], value1<PROTO>(p, nc[k], w0[k], w1[k])));
+                advance(k);
+                prog = true;
+            }
+        }
+        // ---- B. internal entries finalized in an earlier run: read the warp's smem copy
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            while (!(done >> k & 1u) && nc[k] >= r0 && nc[k] < r0 + s) {
+                ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], s_x[nc[k] - r0]));
+                advance(k);
+                prog = true;
+            }
+        }
+        // ---- C. the chain: rows with no external entry left, finalized in row order
+        unsigned long long ok = 0;  // bit t: warp row t is done or has only internal entries / the diagonal left
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const bool rdy = (done >> k & 1u) || nc[k] < 0 || nc[k] >= r0;
+            ok |= (unsigned long long)__ballot_sync(FULL, rdy) << (32 * k);
+        }
+        const int s0 = s;
+        const unsigned long long nok = ~ok >> s;
+        const int run_end = min(rows, nok ? s + __ffsll((long long)nok) - 1 : 64);
+        // One step per row: the owner divides (Diag: the Markstein step, RN(a/d) inside the
+        // guard) and its value is broadcast by one __shfl_sync to the rows that consume it.
+        // FUSED publishes each value at once (one 16-byte record store, the only per-step
+        // store); x, the smem copy and FLAGS publication are written per run, coalesced.
+#pragma unroll
+        for (int k = 0; k < K; ++k) {  // rows r0 + 32k .. r0 + 32k + 31: owner lane = s - 32k
+            const int hi = min(run_end, 32 * (k + 1));
+            for (; s < hi; ++s) {
+                const int owner = s - 32 * k;
+                const double a = __dsub_rn(bk[k], ls[k]);
+                double q = dg[k].cand(a);
+                if (lane == owner && !dg[k].ok(a)) q = __ddiv_rn(a, dg[k].d);  // rare: outside the guard
+                const double xv = __shfl_sync(FULL, q, owner);
+                if (lane == owner) {
+                    xm[k] = q;
+                    done |= 1u << k;
+                    if (PROTO == PROTO_FUSED) {
+                        unsigned long long bits = (unsigned long long)__double_as_longlong(q);
+                        if (bits == kSentinel) bits = kCanonNaN;  // same canonicalisation as publish()
+                        const unsigned long long e = (unsigned long long)epoch << 32;
+                        st_relaxed_v2_u64(p.rec + 2 * (size_t)(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
+                        if (p.trace) p.trace[r0 + s] = globaltimer_ns();
+                    }
+                }
+                const int cs = r0 + s;
+#pragma unroll
+                for (int m = 0; m < K; ++m) {
+                    if (nc[m] == cs) {  // done rows hold nc = -1
+                        ls[m] = __dadd_rn(ls[m], __dmul_rn(nv[m], xv));
+                        advance(m);
+                    }
+                }
+            }
+        }
+        if (s > s0) {
+            // the run's x (output), the smem copy for later in-warp consumers and, for FLAGS, the
+            // release pattern (PTX model, G6): x stores, one gpu-scope fence, relaxed flags
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+                const int t = lane + 32 * k;
+                if (t >= s0 && t < s) {
+                    p.x[r0 + t] = xm[k];
+                    s_x[t] = xm[k];
+                    if (PROTO == PROTO_FLAGS && p.trace) p.trace[r0 + t] = globaltimer_ns();
+                }
+            }
+            if (PROTO == PROTO_FLAGS) {
+                fence_acq_rel_gpu();
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    const int t = lane + 32 * k;
+                    if (t >= s0 && t < s) st_relaxed_u32(p.flags + r0 + t, epoch);
+                }
+            }
+        }
+        if (s >= rows) break;
+        if (s > s0) prog = true;
+        if (__ballot_sync(FULL, prog)) {
+            backoff = p.backoff_min;
+            idle = 0;
+            continue;
+        }
+        // ---- lean wait: nothing moved, so every unfinished row is blocked on an external entry;
+        // re-poll only those (a few instructions per round instead of a full pass) until one is
+        // ready, then consume it and run a full pass
+        bool woke = false;
+        while (!woke) {
+            if (backoff) nanosleep_ns(backoff);
+            backoff = min(max(backoff * 2u, 32u), p.backoff_max);
+            if ((++idle & 63u) == 0) {
+                uint32_t ab = 0;
+                if (lane == 0) {
+                    if (p.spin_limit && idle >= p.spin_limit) {
+                        atomicCAS(&p.st->error.v, 0u, 1u);
+                        st_relaxed_u32(&p.st->abort.v, 1u);
+                    }
+                    ab = ld_relaxed_u32(&p.st->abort.v);
+                }
+                if (__shfl_sync(FULL, ab, 0)) return;
+            }
+            bool got = false;
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+                if (!(done >> k & 1u) && nc[k] >= 0 && nc[k] < r0) {
+                    unsigned long long a0, a1;
+                    poll1<PROTO>(p, nc[k], a0, a1);
+                    if (ready1<PROTO>(a0, a1, epoch)) {
+                        if (p.trace) p.trace[p.n + r0 + lane + 32 * k] = globaltimer_ns();
+                        ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], value1<PROTO>(p, nc[k], a0, a1)));
+                        advance(k);
+                        got = true;
+                    }
+                }
+            }
+            woke = __ballot_sync(FULL, got) != 0;
+        }
+        backoff = p.backoff_min;
+    }
+}
+
+}  // namespace sptrsv_dev

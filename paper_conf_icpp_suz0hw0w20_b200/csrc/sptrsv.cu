@@ -21,6 +21,7 @@
 #include "solve_tri.cuh"
 #include "solve_multi.cuh"
 #include "solve_paper.cuh"
+#include "solve_chain.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -62,6 +63,7 @@ struct sptrsv_handle_s {
     int32_t n_warp_rows = 0;
     int32_t max_row = 0;
     int64_t near_deps = 0;  // dependencies within 256 rows (analyse statistic for ENGINE_AUTO)
+    int64_t warp_deps = 0;  // dependencies inside the row's own 32-row group (ditto)
     // options
     int mode = 0;
     int threshold = 16;
@@ -83,6 +85,7 @@ struct sptrsv_handle_s {
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
+    int chain_pub = 32;     // CHAIN: publication batch in chain steps (SPTRSV_OPT_CHAIN_PUBLISH)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
     int grid_cache = 0;
@@ -404,6 +407,8 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
             rc = SPTRSV_ERR_CUDA;
             break;
         }
+        h->warp_deps = (int64_t)((uint64_t)h->near_deps >> 32);
+        h->near_deps &= 0xFFFFFFFFll;
         if (status != ~0ull) {
             rc = -(int)(status & 0xff);
             break;
@@ -462,8 +467,11 @@ int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem,
 }
 
 // ENGINE_AUTO: all-thread-level plans go to the LEAN engine unless a quarter or
-// more of the dependencies are "near" (within 256 rows: chains, grid wavefronts),
-// where the staged one-shot engine's shared-memory local resolution wins; plans
+// more of the dependencies are "near" (within 256 rows: chains, grid wavefronts).
+// Of those, plans with a quarter or more of their dependencies inside the row's own
+// 32-row group (bidiagonal chains, grid west neighbours) use the CHAIN engine
+// (in-warp shuffle chain); the rest the staged one-shot engine's shared-memory
+// local resolution; plans
 // with warp-level rows use the HYBRID engine (2-13% faster than the staged
 // one-shot engine on every warp-plan shape measured, tools/hybrid_probe.py).
 // (Round-1 B200 sweeps.)
@@ -473,6 +481,7 @@ int resolve_engine(const sptrsv_handle_s *h) {
     const long long offdiag = h->nnz - h->n;
     if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_deps < offdiag)) return 3;
     if (h->plan != PLAN_THREAD) return 6;
+    if (4 * h->warp_deps >= offdiag) return 7;  // in-warp chains: CHAIN
     return 0;
 }
 
@@ -488,7 +497,10 @@ void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) 
         return;
     }
     int c = 256, k = 1;
-    if (engine == 0) {
+    if (engine == 7) {
+        c = kChainCta;
+        k = 2;
+    } else if (engine == 0) {
         if (h->plan == PLAN_THREAD && h->nnz > h->n && 4 * h->near_deps >= h->nnz - h->n) {
             c = 128;
             k = 2;
@@ -605,6 +617,21 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
             return SPTRSV_OK;
         }
     }
+    // ---- ENGINE_CHAIN: warp-sequential in-warp chains (solve_chain.cuh), all-thread-level plans
+    if (engine == 7 && h->plan == PLAN_THREAD && cta <= 256) {
+        const int K = Kq >= 2 ? 2 : 1;
+        const int warps = cta / 32;
+        L->fn = K == 2 ? (h->proto ? (const void *)k_solve_chain<PROTO_FUSED, 2> : (const void *)k_solve_chain<PROTO_FLAGS, 2>)
+                       : (h->proto ? (const void *)k_solve_chain<PROTO_FUSED, 1> : (const void *)k_solve_chain<PROTO_FLAGS, 1>);
+        L->kind = 0;
+        const long long rows_per_cta = (long long)warps * 32 * K;
+        L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
+        L->block = dim3((unsigned)cta);
+        L->smem = (size_t)warps * chain_warp_smem_bytes(K);
+        L->key = 8000000 + h->proto * 100000 + K * 10000 + cta;
+        L->key ^= (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
     // ---- ENGINE_LEAN: minimal one-shot kernel for all-thread-level plans
     if (engine == 3 && h->plan == PLAN_THREAD) {
         // LEAN occupancy: minimum resident CTAs per SM = 5 (default), 6 or 8 (option rows_per_lane
@@ -693,6 +720,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.pf_dist = L.pf_dist;
     p.poll_gap = h->poll_gap;
     p.poll_one = h->poll_one;
+    p.chain_pub = h->chain_pub;
     p.trace = h->trace;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = L.grid;
@@ -913,7 +941,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->local = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
-            if (value < 0 || value > 6) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 7) return SPTRSV_ERR_INVALID_ARG;
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_STAGES:
@@ -952,6 +980,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->poll_one = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_CHAIN_PUBLISH:
+            if (value < 1 || value > 64) return SPTRSV_ERR_INVALID_ARG;
+            h->chain_pub = (int)value;
+            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -980,6 +1012,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_PREFETCH: *value = h->pf_dist; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_GAP_NS: *value = h->poll_gap; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
+        case SPTRSV_OPT_CHAIN_PUBLISH: *value = h->chain_pub; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }
@@ -996,6 +1029,7 @@ int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
     out->analyse_ms = h->analyse_ms;
     out->solves = h->solves;
     out->near_deps = h->near_deps;
+    out->warp_deps = h->warp_deps;
     out->engine = resolve_engine(h);
     effective_geometry(h, out->engine, &out->cta_threads, &out->rows_per_lane);
     return SPTRSV_OK;

@@ -369,6 +369,8 @@ def make(name: str, **kw) -> CSRSystem:
         return gen_c5(int(name[3:]), **kw)
     if name.startswith("diag:"):  # scratch shapes for the perf tools: diag:N, lev:N:L
         return gen_diag(int(name.split(":")[1]))
+    if name.startswith("chain:"):
+        return gen_chain(int(name.split(":")[1]))
     if name.startswith("lev:"):
         _, n, nl = name.split(":")
         return gen_leveled(int(n), int(nl), 1, 1, 2, name)

@@ -343,11 +343,40 @@ def test_lean_engine(cap, proto):
     assert np.array_equal(x, si.x_true)
 
 
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("K", [1, 2])
+@pytest.mark.parametrize("cta", [64, 128, 256])
+def test_chain_engine(cap, proto, K, cta):
+    """ENGINE_CHAIN (in-warp dependencies resolved by a warp-sequential shuffle chain): bit-exact
+    like every thread-level path -- ragged tails, slices longer than the staging cap (dense rows),
+    chains, grids, far and interleaved dependencies, diagonal-only."""
+    for n in (1, 31, 33, 63, 65, 255, 257, 4099):
+        s = synth.gen_random_lower(n, 4, seed=n + 17)
+        x, info = gpu_solve(cap, s, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+        assert info["engine"] == 7
+        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
+    for gen in (lambda: synth.gen_c2i(n=100_000), lambda: synth.gen_c2(n=200_000), lambda: synth.gen_grid(200),
+                lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100), lambda: synth.gen_diag(70_001),
+                lambda: synth.gen_c1()):
+        s = gen()
+        x, _ = gpu_solve(cap, s, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        assert np.array_equal(x, ref), s.name
+    si = synth.integerize(synth.gen_c2i(n=50_000))
+    x, _ = gpu_solve(cap, si, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+    assert np.array_equal(x, si.x_true)
+    sc = synth.gen_chain(10_000)  # closed form x_i = 1 - 2^-(i+1) (i <= 52), 1 after
+    x, _ = gpu_solve(cap, sc, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+    i = np.arange(sc.n)
+    assert np.array_equal(x, np.where(i <= 52, 1.0 - np.ldexp(1.0, -(np.minimum(i, 52) + 1)), 1.0))
+
+
 def test_engine_auto_choice(cap):
-    """ENGINE_AUTO: far dependencies -> LEAN (3); chains / grid wavefronts -> staged one-shot (0);
-    plans with warp-level rows -> HYBRID (6)."""
-    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 0, 128, 2),
-                              (lambda: synth.gen_chain(3000), 0, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
+    """ENGINE_AUTO: far dependencies -> LEAN (3); in-warp chains / grid wavefronts -> CHAIN (7);
+    other near-dependency plans -> staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""
+    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 7, 128, 2),
+                              (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
+                              (lambda: synth.gen_c1(), 0, 128, 2),
                               (lambda: synth.gen_c4(n=5000, nlevels=50), 6, 64, 1)):
         s = gen()
         x, info = gpu_solve(cap, s)

@@ -54,7 +54,7 @@ if nl <= 40:
         if (stv > 0).all():
             ld = (stv - ent)
             out["load_latency_ns_p10_50_90"] = [int(np.percentile(ld, q)) for q in (10, 50, 90)]
-if name == "chain":
+if name.startswith("chain"):
     dt = np.diff(t)
     idx = np.arange(1, s.n)
     inwarp = (idx % 32) != 0
