@@ -54,6 +54,20 @@ __device__ __forceinline__ void st_relaxed_v2_u64(unsigned long long *p, unsigne
     asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
 
+// Predicated forms: one store instruction guarded by a predicate register, so a
+// single-lane store inside warp-uniform code does not open a divergent branch.
+__device__ __forceinline__ void st_relaxed_v2_u64_if(bool pr, unsigned long long *p, unsigned long long a,
+                                                     unsigned long long b) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};\n\t}" ::"l"(p),
+                 "l"(a), "l"(b), "r"((unsigned)pr)
+                 : "memory");
+}
+__device__ __forceinline__ void st_u64_if(bool pr, unsigned long long *p, unsigned long long v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.u64 [%0], %1;\n\t}" ::"l"(p), "l"(v),
+                 "r"((unsigned)pr)
+                 : "memory");
+}
+
 __device__ __forceinline__ void st_release_u32(uint32_t *p, uint32_t v) {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }

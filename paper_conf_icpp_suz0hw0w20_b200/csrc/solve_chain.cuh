@@ -39,12 +39,14 @@ constexpr int kChainCta = 128;  // 4 warps
 constexpr int kChainEPR = 4;    // staged CSR entries per row (a longer slice reads global memory)
 
 __host__ __device__ constexpr int chain_warp_smem_bytes(int K) {
-    // s_val [32K*EPR] f64 | s_x [32K] f64 | s_col [32K*EPR] i32 | s_rp [32K+1] i32   (16-B multiple)
-    return ((8 * 32 * K * kChainEPR + 8 * 32 * K + 4 * 32 * K * kChainEPR + 4 * (32 * K + 1)) + 15) / 16 * 16;
+    // s_val [32K*EPR] f64 | s_x [32K] f64 | f_b, f_d, f_r, f_ls, f_v [32K] f64 |
+    // s_col [32K*EPR] i32 | f_has [32K] i32 | s_rp [32K+1] i32   (16-B multiple)
+    return ((8 * 32 * K * kChainEPR + 8 * 32 * K + 5 * 8 * 32 * K + 4 * 32 * K * kChainEPR + 4 * 32 * K +
+             4 * (32 * K + 1)) + 15) / 16 * 16;
 }
 
 template <int PROTO, int K>
-__global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams p) {
+__global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams p) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t s_blk, s_epoch;
     constexpr int RT = 32 * K;
@@ -67,8 +69,10 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
     unsigned char *wsm = smem + (size_t)warp * chain_warp_smem_bytes(K);
     double *s_val = reinterpret_cast<double *>(wsm);
     double *s_x = s_val + ECAP;
-    int32_t *s_col = reinterpret_cast<int32_t *>(s_x + RT);
-    int32_t *s_rp = s_col + ECAP;
+    double *f_b = s_x + RT, *f_d = f_b + RT, *f_r = f_d + RT, *f_ls = f_r + RT, *f_v = f_ls + RT;
+    int32_t *s_col = reinterpret_cast<int32_t *>(f_v + RT);
+    int32_t *f_has = s_col + ECAP;
+    int32_t *s_rp = f_has + RT;
     // ---- stage rowptr, b, then the warp's contiguous CSR slice (coalesced)
     double bk[K];
 #pragma unroll
@@ -112,6 +116,9 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
         xm[k] = 0.0;
         dg[k].init(a ? val_at(je[k]) : 1.0);
         if (!a) done |= 1u << k;
+        f_b[idx] = bk[k];  // the rows' constants, for the warp-redundant fast path (section C)
+        f_d[idx] = dg[k].d;
+        f_r[idx] = dg[k].r;
     }
     auto advance = [&](int k) {
         ++j[k];
@@ -119,6 +126,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
         nc[k] = more ? col_at(j[k]) : -1;
         nv[k] = more ? val_at(j[k]) : 0.0;
     };
+    const bool tracing = p.trace != nullptr;
     int s = 0;  // next row (warp-relative) to finalize; rows < s are published
     uint32_t backoff = p.backoff_min, idle = 0;
     while (true) {
@@ -169,6 +177,64 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
         // guard) and its value is broadcast by one __shfl_sync to the rows that consume it.
         // FUSED publishes each value at once (one 16-byte record store, the only per-step
         // store); x, the smem copy and FLAGS publication are written per run, coalesced.
+        // Fast path (bidiagonal chains, grid west neighbours): when every row of the run has
+        // at most ONE internal entry left and it is the previous row, the run is the scalar
+        // recurrence x_t = (b_t - (ls_t + v_t x_{t-1})) / d_t.  All 32 lanes then evaluate it
+        // REDUNDANTLY from the run's operands in shared memory (broadcast loads): no shuffle and
+        // no lane-to-lane hop on the chain, only its dependent fp64 operations.  Same
+        // operations in the same order as Alg.1 (mul, add, sub, division), so bit-exact.
+        bool el = true;
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const int t = lane + 32 * k;
+            if (!(done >> k & 1u) && t >= s && t < run_end) {
+                const bool none = nc[k] < 0;
+                const bool prev = nc[k] == r0 + t - 1 && j[k] + 1 == je[k];
+                el = el && (none || (prev && t > s));
+                f_ls[t] = ls[k];
+                f_v[t] = prev ? nv[k] : 0.0;
+                f_has[t] = prev ? 1 : 0;
+            }
+        }
+        if (run_end > s && __all_sync(FULL, el)) {
+            __syncwarp();
+            double xp = 0.0;  // x of row t - 1 (read only when row t has that entry)
+            // operands of row t are loaded one iteration ahead, off the dependency chain
+            double lsv = f_ls[s], bv = f_b[s], vv = f_v[s], dv = f_d[s], rv = f_r[s];
+            int hv = f_has[s];
+            for (int t = s; t < run_end; ++t) {
+                const int tn = min(t + 1, run_end - 1);
+                const double lsn = f_ls[tn], bn = f_b[tn], vn = f_v[tn], dn = f_d[tn], rn = f_r[tn];
+                const int hn = f_has[tn];
+                const double u = hv ? __dadd_rn(lsv, __dmul_rn(vv, xp)) : lsv;
+                const double a = __dsub_rn(bv, u);
+                Diag g;
+                g.d = dv;
+                g.r = rv;
+                double q = g.cand(a);
+                // guard (Diag::ok) in integer ops; warp-uniform here: every lane holds the same a
+                if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0), 0)) q = __ddiv_rn(a, dv);
+                const int owner = t & 31, kk = t >> 5;
+                const bool mine = lane == owner;
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    const bool mk = mine && kk == k;
+                    xm[k] = mk ? q : xm[k];
+                    done |= mk ? (1u << k) : 0u;
+                    nc[k] = mk ? -1 : nc[k];
+                }
+                if (PROTO == PROTO_FUSED) {  // the owner's record: one predicated store, no branch
+                    unsigned long long bits = (unsigned long long)__double_as_longlong(q);
+                    bits = bits == kSentinel ? kCanonNaN : bits;
+                    const unsigned long long e = (unsigned long long)epoch << 32;
+                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)(r0 + t), e | (bits & 0xffffffffull), e | (bits >> 32));
+                    if (tracing) st_u64_if(mine, p.trace + r0 + t, globaltimer_ns());
+                }
+                xp = q;
+                lsv = lsn, bv = bn, vv = vn, dv = dn, rv = rn, hv = hn;
+            }
+            s = run_end;
+        }
 #pragma unroll
         for (int k = 0; k < K; ++k) {  // rows r0 + 32k .. r0 + 32k + 31: owner lane = s - 32k
             const int hi = min(run_end, 32 * (k + 1));
@@ -176,26 +242,29 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 const int owner = s - 32 * k;
                 const double a = __dsub_rn(bk[k], ls[k]);
                 double q = dg[k].cand(a);
-                if (lane == owner && !dg[k].ok(a)) q = __ddiv_rn(a, dg[k].d);  // rare: outside the guard
-                const double xv = __shfl_sync(FULL, q, owner);
-                if (lane == owner) {
-                    xm[k] = q;
-                    done |= 1u << k;
-                    if (PROTO == PROTO_FUSED) {
-                        unsigned long long bits = (unsigned long long)__double_as_longlong(q);
-                        if (bits == kSentinel) bits = kCanonNaN;  // same canonicalisation as publish()
-                        const unsigned long long e = (unsigned long long)epoch << 32;
-                        st_relaxed_v2_u64(p.rec + 2 * (size_t)(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
-                        if (p.trace) p.trace[r0 + s] = globaltimer_ns();
-                    }
+                const int bad = !dg[k].ok(a);
+                double xv = __shfl_sync(FULL, q, owner);
+                if (__shfl_sync(FULL, bad, owner)) {  // warp-uniform, rare: outside the guard
+                    q = __ddiv_rn(a, dg[k].d);
+                    xv = __shfl_sync(FULL, q, owner);
+                }
+                const bool mine = lane == owner;
+                xm[k] = mine ? q : xm[k];
+                done |= mine ? (1u << k) : 0u;
+                if (PROTO == PROTO_FUSED) {
+                    unsigned long long bits = (unsigned long long)__double_as_longlong(q);
+                    if (bits == kSentinel) bits = kCanonNaN;  // same canonicalisation as publish()
+                    const unsigned long long e = (unsigned long long)epoch << 32;
+                    if (mine) st_relaxed_v2_u64(p.rec + 2 * (size_t)(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
+                    if (tracing && mine) p.trace[r0 + s] = globaltimer_ns();
                 }
                 const int cs = r0 + s;
 #pragma unroll
-                for (int m = 0; m < K; ++m) {
-                    if (nc[m] == cs) {  // done rows hold nc = -1
-                        ls[m] = __dadd_rn(ls[m], __dmul_rn(nv[m], xv));
-                        advance(m);
-                    }
+                for (int m = 0; m < K; ++m) {  // done rows hold nc = -1
+                    const bool c = nc[m] == cs;
+                    const double t = __dadd_rn(ls[m], __dmul_rn(nv[m], xv));
+                    ls[m] = c ? t : ls[m];
+                    if (c) advance(m);
                 }
             }
         }

@@ -628,6 +628,11 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
         L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
         L->block = dim3((unsigned)cta);
         L->smem = (size_t)warps * chain_warp_smem_bytes(K);
+        if (L->smem > 48 * 1024 &&
+            cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_CUDA;
+        }
         L->key = 8000000 + h->proto * 100000 + K * 10000 + cta;
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;

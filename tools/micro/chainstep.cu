@@ -152,6 +152,59 @@ __global__ void k_step(long long *cyc, int steps, double d0, unsigned long long 
     if (lane == 0) cyc[W] = (t1 - t0) / steps + (long long)(xm * 0) + done * 0;
 }
 
+// The CHAIN engine's warp-redundant fast path (solve_chain.cuh) in isolation: operands in
+// smem, all lanes evaluate x_t = (b_t - (ls_t + v_t x_{t-1})) / d_t; W selects the per-step
+// publication: 0 none, 1 owner's 16-B relaxed.gpu record store, 2 weak 16-B store, 3 strong
+// store + globaltimer trace.
+template <int W>
+__global__ void k_fast(long long *cyc, int steps, unsigned long long *rec, unsigned long long *tr) {
+    __shared__ double f_ls[64], f_b[64], f_v[64], f_d[64], f_r[64];
+    __shared__ int f_has[64];
+    const int lane = threadIdx.x;
+    for (int t = lane; t < 64; t += 32) {
+        f_ls[t] = 0.0; f_b[t] = 1.0; f_v[t] = -1.0; f_d[t] = 2.0 + t * 1e-3; f_r[t] = __drcp_rn(f_d[t]); f_has[t] = t > 0;
+    }
+    __syncwarp();
+    double xp = 0.0, xm = 0.0;
+    long long t0 = clock64();
+    for (int it = 0; it < steps / 32; ++it) {
+        double lsv = f_ls[0], bv = f_b[0], vv = f_v[0], dv = f_d[0], rv = f_r[0];
+        int hv = f_has[0];
+        for (int t = 0; t < 32; ++t) {
+            const int tn = min(t + 1, 31);
+            const double lsn = f_ls[tn], bn = f_b[tn], vn = f_v[tn], dn = f_d[tn], rn = f_r[tn];
+            const int hn = f_has[tn];
+            const double u = hv ? __dadd_rn(lsv, __dmul_rn(vv, xp)) : lsv;
+            const double a = __dsub_rn(bv, u);
+            Diag g;
+            g.d = dv;
+            g.r = rv;
+            double q = g.div_fast(a);
+            const unsigned ex = ((unsigned)__double2hiint(a) >> 20) & 0x7FFu;
+            if (!(rv != 0.0 && ex - (1023u - 400u) <= 800u)) q = __ddiv_rn(a, dv);
+            const bool mine = lane == t;
+            xm = mine ? q : xm;
+            unsigned long long bits = (unsigned long long)__double_as_longlong(q), e = 1ull << 32;
+            const size_t ix = 2 * (size_t)((it * 32 + t) & 4095);
+            if (W == 1 || W == 3) {
+                if (mine) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(rec + ix), "l"(e | (bits & 0xffffffffull)), "l"(e | (bits >> 32)) : "memory");
+            }
+            if (W == 2) {
+                if (mine) asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(rec + ix), "l"(e | (bits & 0xffffffffull)), "l"(e | (bits >> 32)) : "memory");
+            }
+            if (W == 3 && mine) {
+                unsigned long long tt;
+                asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tt));
+                tr[(it * 32 + t) & 4095] = tt;
+            }
+            xp = q;
+            lsv = lsn, bv = bn, vv = vn, dv = dn, rv = rn, hv = hn;
+        }
+    }
+    long long t1 = clock64();
+    if (lane == 0) cyc[W] = (t1 - t0) / steps + (long long)(xm * 0);
+}
+
 __global__ void k_lat(long long *cyc, double a0, int iters) {
     double a = a0, b = 1.0000001;
     long long t0 = clock64();
@@ -179,7 +232,7 @@ int main() {
     double *out;
     long long *cyc, h[8];
     cudaMalloc(&out, 64);
-    cudaMalloc(&cyc, 64);
+    cudaMalloc(&cyc, 128);
     k_lat<<<1, 32>>>(cyc, 1.5, 10000);
     cudaMemcpy(h, cyc, 40, cudaMemcpyDeviceToHost);
     printf("dependent latency (cycles): DFMA %lld  DMUL %lld  SHFL.64 %lld  __ddiv_rn %lld\n", h[0], h[1], h[2], h[3]);
@@ -213,6 +266,14 @@ int main() {
     k_step<4><<<1, 32>>>(cyc, 32000, 4.0, rec, cols);
     k_step<7><<<1, 32>>>(cyc, 32000, 4.0, rec, cols);
     cudaMemcpy(h, cyc, 64, cudaMemcpyDeviceToHost);
+    k_fast<0><<<1, 32>>>(cyc + 8, 32000, rec, (unsigned long long *)xg);
+    k_fast<1><<<1, 32>>>(cyc + 8, 32000, rec, (unsigned long long *)xg);
+    k_fast<2><<<1, 32>>>(cyc + 8, 32000, rec, (unsigned long long *)xg);
+    k_fast<3><<<1, 32>>>(cyc + 8, 32000, rec, (unsigned long long *)xg);
+    long long hf[4];
+    cudaMemcpy(hf, cyc + 8, 32, cudaMemcpyDeviceToHost);
+    printf("fast path step: no store %lld | strong rec store %lld | weak store %lld | strong + trace %lld cycles\n",
+           hf[0], hf[1], hf[2], hf[3]);
     printf("kernel step: bare %lld | +check/vote %lld | +store %lld | +check+store %lld | +consume %lld | all %lld cycles\n",
            h[0], h[1], h[2], h[3], h[4], h[7]);
     return 0;
