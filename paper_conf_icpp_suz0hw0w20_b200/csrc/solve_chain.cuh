@@ -46,7 +46,7 @@ __host__ __device__ constexpr int chain_warp_smem_bytes(int K) {
 }
 
 template <int PROTO, int K>
-__global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams p) {
+__global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams p) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t s_blk, s_epoch;
     constexpr int RT = 32 * K;
@@ -74,7 +74,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams
     int32_t *f_has = s_col + ECAP;
     int32_t *s_rp = f_has + RT;
     // ---- stage rowptr, b, then the warp's contiguous CSR slice (coalesced)
-    double bk[K];
+    double bk[K];  // staging only: the rows' constants live in smem (f_b, f_d, f_r) afterwards
 #pragma unroll
     for (int k = 0; k <= K; ++k) {
         const int idx = lane + 32 * k;
@@ -102,7 +102,6 @@ __global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams
     // ---- per-row state: cursor j, diagonal index je, next column / value, partial sum
     int j[K], je[K], nc[K];
     double nv[K], ls[K], xm[K];
-    Diag dg[K];
     unsigned done = 0;  // bit k: row k of this lane finalized (or not a row)
 #pragma unroll
     for (int k = 0; k < K; ++k) {
@@ -114,11 +113,12 @@ __global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams
         nv[k] = (a && j[k] < je[k]) ? val_at(j[k]) : 0.0;
         ls[k] = 0.0;
         xm[k] = 0.0;
-        dg[k].init(a ? val_at(je[k]) : 1.0);
+        Diag dg;
+        dg.init(a ? val_at(je[k]) : 1.0);
         if (!a) done |= 1u << k;
-        f_b[idx] = bk[k];  // the rows' constants, for the warp-redundant fast path (section C)
-        f_d[idx] = dg[k].d;
-        f_r[idx] = dg[k].r;
+        f_b[idx] = bk[k];  // the rows' constants (both chain paths read them from smem)
+        f_d[idx] = dg.d;
+        f_r[idx] = dg.r;
     }
     auto advance = [&](int k) {
         ++j[k];
@@ -240,12 +240,15 @@ __global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams
             const int hi = min(run_end, 32 * (k + 1));
             for (; s < hi; ++s) {
                 const int owner = s - 32 * k;
-                const double a = __dsub_rn(bk[k], ls[k]);
-                double q = dg[k].cand(a);
-                const int bad = !dg[k].ok(a);
+                Diag g;
+                g.d = f_d[s];
+                g.r = f_r[s];
+                const double a = __dsub_rn(f_b[s], ls[k]);
+                double q = g.cand(a);
+                const int bad = !g.ok(a);
                 double xv = __shfl_sync(FULL, q, owner);
                 if (__shfl_sync(FULL, bad, owner)) {  // warp-uniform, rare: outside the guard
-                    q = __ddiv_rn(a, dg[k].d);
+                    q = __ddiv_rn(a, g.d);
                     xv = __shfl_sync(FULL, q, owner);
                 }
                 const bool mine = lane == owner;
@@ -253,10 +256,10 @@ __global__ void __launch_bounds__(256, K == 1 ? 3 : 2) k_solve_chain(SolveParams
                 done |= mine ? (1u << k) : 0u;
                 if (PROTO == PROTO_FUSED) {
                     unsigned long long bits = (unsigned long long)__double_as_longlong(q);
-                    if (bits == kSentinel) bits = kCanonNaN;  // same canonicalisation as publish()
+                    bits = bits == kSentinel ? kCanonNaN : bits;  // same canonicalisation as publish()
                     const unsigned long long e = (unsigned long long)epoch << 32;
-                    if (mine) st_relaxed_v2_u64(p.rec + 2 * (size_t)(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
-                    if (tracing && mine) p.trace[r0 + s] = globaltimer_ns();
+                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
+                    if (tracing) st_u64_if(mine, p.trace + r0 + s, globaltimer_ns());
                 }
                 const int cs = r0 + s;
 #pragma unroll
