@@ -404,7 +404,9 @@ def main():
     peak, peak_src = peaks()
     alg_bytes = systems[0].alg_bytes()
     achieved = alg_bytes / kernel_s / 1e9
-    roof = {"bound": "hbm", "kernel": "k_solve", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
+    kname = {0: "k_solve", 1: "k_solve_pipe", 2: "k_solve_dyn", 3: "k_solve_lean", 4: "k_solve_dyn",
+             6: "k_solve_tri_warp", 7: "k_solve_chain"}.get(handles[0].info()["engine"], "k_solve")
+    roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 5), "traffic": ncu_traffic(args.config),
             "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src,
             "alg_bytes_formula": "4(n+1) + 12*nnz + 8n (b) + 8n (x) + 4n (flags)"}

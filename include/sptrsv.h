@@ -101,7 +101,7 @@ typedef enum sptrsv_option {
                                       r0+lane+32k), or 0 (default) = the engine's measured
                                       best; applies to all-thread-level plans on the
                                       ONE-SHOT engine with CTAs of <= 256 threads          */
-    SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5 (default), 6 or 8
+    SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 6)
                                       resident 256-thread CTAs per SM                       */
     SPTRSV_OPT_PREFETCH = 18,      /* L2 bulk prefetch (cp.async.bulk.prefetch.L2) of the
                                       CSR range of the CTA this many logical blocks ahead:

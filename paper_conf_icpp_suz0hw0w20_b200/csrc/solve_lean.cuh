@@ -127,14 +127,14 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
 // j > i) are taken in REVERSE order -- logical row r is row n-1-r, so the ticket
 // order is again a topological order; UNIT: the diagonal is implicitly 1 and
 // not stored.
-template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false>
-__global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
+template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false, int CT = kLeanCta>
+__global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint64_t pol = policy_evict_first();
     // ---- speculative first-level loads for logical block == blockIdx.x
-    int i = (int)blockIdx.x * kLeanCta + tid;
+    int i = (int)blockIdx.x * CT + tid;
     if (UPPER) i = p.n - 1 - i;
     int rs = 0, re = 1;
     double bi = 0.0;
@@ -148,9 +148,9 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
     // blockIdx.x + pf_dist): its bounds load overlaps the ticket, the copy is issued after it
     int pfA = 0, pfB = 0, pfa = 0, pfb = 0;
     if (p.pf_dist > 0 && tid == 32) {
-        const long long r0 = ((long long)blockIdx.x + p.pf_dist) * kLeanCta;
+        const long long r0 = ((long long)blockIdx.x + p.pf_dist) * CT;
         if (r0 < p.n) {
-            const int r1 = (int)min((long long)p.n, r0 + kLeanCta);
+            const int r1 = (int)min((long long)p.n, r0 + CT);
             pfA = UPPER ? p.n - r1 : (int)r0;
             pfB = UPPER ? p.n - (int)r0 : r1;
             pfa = ld_stream_i32(p.rowptr + pfA, pol);
@@ -168,7 +168,7 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_lean(SolveParams p) {
     const uint32_t epoch = s_epoch;
     if (pfB > pfA) prefetch_rows_l2(p, pfA, pfB, pfa, pfb);
     if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
-        i = (int)s_blk * kLeanCta + tid;
+        i = (int)s_blk * CT + tid;
         if (UPPER) i = p.n - 1 - i;
         rs = 0, re = 1, bi = 0.0;
         if (i >= 0 && i < p.n) {

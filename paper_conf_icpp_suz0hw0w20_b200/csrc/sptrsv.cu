@@ -81,7 +81,7 @@ struct sptrsv_handle_s {
     int pipe_entries = 0;   // 0 = 4 per row of a round
     int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
-    int lean_minb = 5;      // LEAN: minimum resident CTAs per SM the register budget targets
+    int lean_minb = 6;      // LEAN: resident 256-thread CTAs per SM the register budget targets (5..8)
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
@@ -487,12 +487,17 @@ int resolve_engine(const sptrsv_handle_s *h) {
 
 // CTA size and rows per lane actually used: the user's values, else the
 // per-engine defaults measured best on B200 in round 1:
-// staged one-shot on near-dependency thread-level plans (grid wavefronts,
-// chains): 2 rows per lane in 128-thread CTAs; on plans with warp-level rows:
-// 64-thread CTAs; everything else 256 threads, 1 row per lane.
+// CHAIN 2 rows per lane in 128-thread CTAs; staged one-shot on plans with
+// warp-level rows: 64-thread CTAs; everything else 256 threads, 1 row per lane
+// (the one-shot's former 2-rows/128-thread geometry for near-dependency plans
+// predates CHAIN, which now takes grids and chains; on c1 it measured 69.7 us
+// vs 30.7 us for 256/1).
 void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) {
-    if (engine == 3 || engine == 6) {  // fixed geometry: LEAN 256 threads, HYBRID 64
-        *cta = (engine == 6 && h->plan != PLAN_THREAD) ? kTriWarpCta : kLeanCta;
+    if (engine == 3 || engine == 6) {  // LEAN 256 threads (lower: option CTA_THREADS 128/512), HYBRID 64
+        *cta = (engine == 6 && h->plan != PLAN_THREAD) ? kTriWarpCta
+               : (engine == 3 && !h->tri && h->plan == PLAN_THREAD &&
+                  (h->cta_threads == 128 || h->cta_threads == 512)) ? h->cta_threads
+                                                                                       : kLeanCta;
         *K = 1;
         return;
     }
@@ -500,25 +505,39 @@ void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) 
     if (engine == 7) {
         c = kChainCta;
         k = 2;
-    } else if (engine == 0) {
-        if (h->plan == PLAN_THREAD && h->nnz > h->n && 4 * h->near_deps >= h->nnz - h->n) {
-            c = 128;
-            k = 2;
-        } else if (h->plan != PLAN_THREAD) {
-            c = 64;
-        }
+    } else if (engine == 0 && h->plan != PLAN_THREAD) {
+        c = 64;
     }
     *cta = h->cta_threads ? h->cta_threads : c;
     *K = h->rows_per_lane ? h->rows_per_lane : k;
 }
 
 typedef void (*lean_fn)(SolveParams);
+
+// LEAN for lower thread-level plans: CTA size ct in {128, 256, 512} (0 = 256) and the
+// register budget occ = resident 256-thread CTAs per SM targeted (5..8), i.e.
+// __launch_bounds__(ct, occ * 256 / ct).  Returns nullptr for an unsupported pair.
+#define LEAN_OCC(CT_, M5, M6, M7, M8)                                                               \
+    {{k_solve_lean<PROTO_FLAGS, M5, false, false, CT_>, k_solve_lean<PROTO_FUSED, M5, false, false, CT_>}, \
+     {k_solve_lean<PROTO_FLAGS, M6, false, false, CT_>, k_solve_lean<PROTO_FUSED, M6, false, false, CT_>}, \
+     {k_solve_lean<PROTO_FLAGS, M7, false, false, CT_>, k_solve_lean<PROTO_FUSED, M7, false, false, CT_>}, \
+     {k_solve_lean<PROTO_FLAGS, M8, false, false, CT_>, k_solve_lean<PROTO_FUSED, M8, false, false, CT_>}}
+lean_fn lean_lower_kernel(int proto, int occ, int cta, int *ct_out) {
+    static const lean_fn tab[3][4][2] = {LEAN_OCC(128, 10, 12, 14, 16), LEAN_OCC(256, 5, 6, 7, 8),
+                                         LEAN_OCC(512, 2, 3, 3, 4)};
+    const int ct = (cta == 128 || cta == 512) ? cta : kLeanCta;  // other sizes: the default 256
+    const int c = ct == 128 ? 0 : ct == 256 ? 1 : 2;
+    if (occ < 5 || occ > 8) return nullptr;
+    *ct_out = ct;
+    return tab[c][occ - 5][proto ? 1 : 0];
+}
+#undef LEAN_OCC
 lean_fn lean_tri_kernel(int proto, int tri) {
     static const lean_fn tab[4][2] = {
-        {k_solve_lean<PROTO_FLAGS, 5>, k_solve_lean<PROTO_FUSED, 5>},
-        {k_solve_lean<PROTO_FLAGS, 5, true, false>, k_solve_lean<PROTO_FUSED, 5, true, false>},
-        {k_solve_lean<PROTO_FLAGS, 5, false, true>, k_solve_lean<PROTO_FUSED, 5, false, true>},
-        {k_solve_lean<PROTO_FLAGS, 5, true, true>, k_solve_lean<PROTO_FUSED, 5, true, true>},
+        {k_solve_lean<PROTO_FLAGS, 6>, k_solve_lean<PROTO_FUSED, 6>},
+        {k_solve_lean<PROTO_FLAGS, 6, true, false>, k_solve_lean<PROTO_FUSED, 6, true, false>},
+        {k_solve_lean<PROTO_FLAGS, 6, false, true>, k_solve_lean<PROTO_FUSED, 6, false, true>},
+        {k_solve_lean<PROTO_FLAGS, 6, true, true>, k_solve_lean<PROTO_FUSED, 6, true, true>},
     };
     return tab[tri & 3][proto ? 1 : 0];
 }
@@ -639,21 +658,17 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
     }
     // ---- ENGINE_LEAN: minimal one-shot kernel for all-thread-level plans
     if (engine == 3 && h->plan == PLAN_THREAD) {
-        // LEAN occupancy: minimum resident CTAs per SM = 5 (default), 6 or 8 (option rows_per_lane
-        // is not used by LEAN; lean_minb selects the register budget)
-        const int mb = h->lean_minb;
-        if (mb == 8)
-            L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED, 8> : (const void *)k_solve_lean<PROTO_FLAGS, 8>;
-        else if (mb == 6)
-            L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED, 6> : (const void *)k_solve_lean<PROTO_FLAGS, 6>;
-        else
-            L->fn = h->proto ? (const void *)k_solve_lean<PROTO_FUSED, 5> : (const void *)k_solve_lean<PROTO_FLAGS, 5>;
+        // LEAN geometry: CTA size 128 / 256 (default) / 512 (option CTA_THREADS) and the register
+        // budget (option LEAN_OCCUPANCY = resident 256-thread CTAs per SM it targets: 5..8)
+        int ct = 0;
+        L->fn = (const void *)lean_lower_kernel(h->proto, h->lean_minb, h->cta_threads, &ct);
+        if (!L->fn) return SPTRSV_ERR_INVALID_ARG;
         L->kind = 0;
-        L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
-        L->block = dim3((unsigned)kLeanCta);
+        L->grid = dim3((unsigned)((h->n + ct - 1) / ct));
+        L->block = dim3((unsigned)ct);
         L->smem = 0;
         L->pf_dist = h->pf_dist < 0 ? kLeanPrefetchDefault : h->pf_dist;
-        L->key = 5000000 + h->proto * 100000 + h->lean_minb * 1000;
+        L->key = 5000000 + h->proto * 100000 + h->lean_minb * 1000 + ct;
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
@@ -970,7 +985,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->variant = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_LEAN_OCCUPANCY:
-            if (value != 5 && value != 6 && value != 8) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 5 || value > 8) return SPTRSV_ERR_INVALID_ARG;
             h->lean_minb = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_PREFETCH:
