@@ -93,7 +93,11 @@ typedef enum sptrsv_option {
                                       6 HYBRID: 64-thread CTAs, one task per warp -- a
                                       warp-level row (Alg.3) or a 32-row thread group
                                       (LEAN's per-lane loop), no staging / in-CTA copy;
-                                      all-thread-level plans run LEAN                        */
+                                      all-thread-level plans run LEAN.
+                                      8 LEAN_K: LEAN with K = ROWS_PER_LANE (2 default, 3, 4)
+                                      rows per lane, row constants in shared memory; a larger
+                                      resident-row window for wide levels (CTA_THREADS 128
+                                      or 256; LEAN_OCCUPANCY 2..5 picks the register budget) */
     SPTRSV_OPT_PIPE_STAGES = 12,   /* PIPE ring depth, 2..8 (default 3)                     */
     SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
     SPTRSV_OPT_PIPE_ENTRIES = 14,  /* PIPE colidx/val entries per stage (0 = 4 per row)     */
@@ -102,7 +106,8 @@ typedef enum sptrsv_option {
                                       best; applies to all-thread-level plans on the
                                       ONE-SHOT engine with CTAs of <= 256 threads          */
     SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 6)
-                                      resident 256-thread CTAs per SM                       */
+                                      resident 256-thread CTAs per SM; LEAN_K: 2..5 (per-K
+                                      default)                                              */
     SPTRSV_OPT_PREFETCH = 18,      /* L2 bulk prefetch (cp.async.bulk.prefetch.L2) of the
                                       CSR range of the CTA this many logical blocks ahead:
                                       -1 (default) = the engine's measured choice, 0 = off.

@@ -18,6 +18,7 @@
 #include "solve_k.cuh"
 #include "solve_dyn.cuh"
 #include "solve_lean.cuh"
+#include "solve_lk.cuh"
 #include "solve_tri.cuh"
 #include "solve_multi.cuh"
 #include "solve_paper.cuh"
@@ -81,6 +82,7 @@ struct sptrsv_handle_s {
     int pipe_entries = 0;   // 0 = 4 per row of a round
     int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
+    int lk_occ = 0;         // LEAN_K register budget (0 = per-K default; SPTRSV_OPT_LEAN_OCCUPANCY)
     int lean_minb = 6;      // LEAN: resident 256-thread CTAs per SM the register budget targets (5..8)
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
@@ -502,6 +504,11 @@ void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) 
         return;
     }
     int c = 256, k = 1;
+    if (engine == 8) {  // LEAN_K: 256-thread CTAs, K = 2 (1 is LEAN itself)
+        *cta = (h->cta_threads == 128) ? 128 : 256;
+        *K = (h->rows_per_lane >= 2 && h->rows_per_lane <= 4) ? h->rows_per_lane : 2;
+        return;
+    }
     if (engine == 7) {
         c = kChainCta;
         k = 2;
@@ -532,6 +539,34 @@ lean_fn lean_lower_kernel(int proto, int occ, int cta, int *ct_out) {
     return tab[c][occ - 5][proto ? 1 : 0];
 }
 #undef LEAN_OCC
+
+// LEAN_K (solve_lk.cuh): K in {2, 3, 4} rows per lane, CTA 128 or 256 threads, and the
+// register budget occ = resident 256-thread CTAs per SM targeted.  Supported occ per K:
+// K=2: 3, 4 (default), 5;  K=3: 2, 3 (default);  K=4: 2 (default), 3.
+#define LK_PAIR(K_, CT_, MB_) {k_solve_lk<PROTO_FLAGS, K_, CT_, MB_>, k_solve_lk<PROTO_FUSED, K_, CT_, MB_>}
+lean_fn lean_k_kernel(int proto, int K, int cta, int occ, int *occ_out) {
+    static const lean_fn t2[2][3][2] = {{LK_PAIR(2, 128, 6), LK_PAIR(2, 128, 8), LK_PAIR(2, 128, 10)},
+                                        {LK_PAIR(2, 256, 3), LK_PAIR(2, 256, 4), LK_PAIR(2, 256, 5)}};
+    static const lean_fn t3[2][2][2] = {{LK_PAIR(3, 128, 4), LK_PAIR(3, 128, 6)},
+                                        {LK_PAIR(3, 256, 2), LK_PAIR(3, 256, 3)}};
+    static const lean_fn t4[2][2][2] = {{LK_PAIR(4, 128, 4), LK_PAIR(4, 128, 6)},
+                                        {LK_PAIR(4, 256, 2), LK_PAIR(4, 256, 3)}};
+    const int c = cta == 128 ? 0 : 1, pr = proto ? 1 : 0;
+    if (K == 2) {
+        const int o = (occ >= 3 && occ <= 5) ? occ : 4;
+        *occ_out = o;
+        return t2[c][o - 3][pr];
+    }
+    if (K == 3) {
+        const int o = (occ == 2 || occ == 3) ? occ : 3;
+        *occ_out = o;
+        return t3[c][o - 2][pr];
+    }
+    const int o = (occ == 2 || occ == 3) ? occ : 2;
+    *occ_out = o;
+    return t4[c][o - 2][pr];
+}
+#undef LK_PAIR
 lean_fn lean_tri_kernel(int proto, int tri) {
     static const lean_fn tab[4][2] = {
         {k_solve_lean<PROTO_FLAGS, 6>, k_solve_lean<PROTO_FUSED, 6>},
@@ -653,6 +688,19 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
             return SPTRSV_ERR_CUDA;
         }
         L->key = 8000000 + h->proto * 100000 + K * 10000 + cta;
+        L->key ^= (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
+    // ---- ENGINE_LEAN_K: LEAN with K rows per lane (all-thread-level lower plans)
+    if (engine == 8 && h->plan == PLAN_THREAD) {
+        int occ = 0;
+        L->fn = (const void *)lean_k_kernel(h->proto, Kq, cta, h->lk_occ, &occ);
+        L->kind = 0;
+        const long long rows_per_cta = (long long)cta * Kq;
+        L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
+        L->block = dim3((unsigned)cta);
+        L->smem = 0;
+        L->key = 9000000 + h->proto * 100000 + Kq * 10000 + occ * 1000 + cta;
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
@@ -961,7 +1009,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->local = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
-            if (value < 0 || value > 7) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 8) return SPTRSV_ERR_INVALID_ARG;
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_PIPE_STAGES:
@@ -985,8 +1033,9 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->variant = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_LEAN_OCCUPANCY:
-            if (value < 5 || value > 8) return SPTRSV_ERR_INVALID_ARG;
-            h->lean_minb = (int)value;
+            if (value < 2 || value > 8) return SPTRSV_ERR_INVALID_ARG;
+            if (value >= 5) h->lean_minb = (int)value;  // LEAN: 5..8
+            h->lk_occ = (int)value;                     // LEAN_K: per K, see lean_k_kernel
             return SPTRSV_OK;
         case SPTRSV_OPT_PREFETCH:
             if (value < -1 || value > (1 << 24)) return SPTRSV_ERR_INVALID_ARG;

@@ -344,6 +344,34 @@ def test_lean_engine(cap, proto):
 
 
 @pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("K,cta,occ", [(2, 256, 0), (2, 128, 0), (2, 256, 3), (2, 256, 5), (3, 256, 0), (3, 128, 2),
+                                       (4, 256, 0), (4, 256, 3), (4, 128, 0)])
+def test_lean_k_engine(cap, proto, K, cta, occ):
+    """ENGINE_LEAN_K (8): K rows per lane, two preloaded dependencies per row, row constants in smem:
+    bit-exact like every thread-level path -- ragged tails (n not a multiple of 32K or of the CTA's
+    rows), rows longer than the two preloaded entries (dense), in-warp chains (same lane, k-strided
+    rows), grids, interleaved levels, diagonal-only; exact-integer systems give x_true."""
+    opts = dict(protocol=proto, engine=8, rows_per_lane=K, cta_threads=cta)
+    if occ:
+        opts["lean_occupancy"] = occ
+    for n in (1, 31, 33, 63, 65, 255, 257, 1023, 1025, 4099):
+        s = synth.gen_random_lower(n, 4, seed=n + 19)
+        x, info = gpu_solve(cap, s, 1, **opts)
+        assert info["engine"] == 8 and info["rows_per_lane"] == K and info["cta_threads"] == cta, info
+        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
+    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=300_000), lambda: synth.gen_grid(200),
+                lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100), lambda: synth.gen_diag(70_001),
+                lambda: synth.gen_c1()):
+        s = gen()
+        x, _ = gpu_solve(cap, s, 1, **opts)
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        assert np.array_equal(x, ref), s.name
+    si = synth.integerize(synth.gen_c2i(n=50_000))
+    x, _ = gpu_solve(cap, si, 1, **opts)
+    assert np.array_equal(x, si.x_true)
+
+
+@pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("K", [1, 2])
 @pytest.mark.parametrize("cta", [64, 128, 256])
 def test_chain_engine(cap, proto, K, cta):

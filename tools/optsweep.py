@@ -11,6 +11,16 @@ name = sys.argv[1]
 sets = json.loads(sys.argv[2]) if len(sys.argv) > 2 else [{}]
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 30
 flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+FLUSH = os.environ.get("FLUSH", "dirty")  # dirty (bench.py's 256 MiB write), clean (write + read), none
+sink = torch.empty(1, dtype=torch.float32, device="cuda")
+
+
+def do_flush():
+    if FLUSH == "none":
+        return
+    flush.zero_()
+    if FLUSH == "clean":
+        sink.add_(flush.sum())
 s = synth.make(name)
 d = torch.device("cuda")
 rp, ci, v, b = (torch.from_numpy(a).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
@@ -23,7 +33,7 @@ for rnd in range(2):  # two passes: the spread between them is the noise floor
         h.check()
         ts = []
         for _ in range(reps):
-            flush.zero_()
+            do_flush()
             e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
             e0.record(); h.solve(b, x); e1.record(); torch.cuda.synchronize()
             ts.append(e0.elapsed_time(e1) * 1e-3)
@@ -31,7 +41,7 @@ for rnd in range(2):  # two passes: the spread between them is the noise floor
         t = float(np.median(ts))
         err = float(np.max(np.abs(x.cpu().numpy() - s.x_true) / np.abs(s.x_true))) if s.x_true is not None else -1
         inf = h.info()
-        print(json.dumps({"cfg": name, "pass": rnd, "opts": opts, "t_us": round(t * 1e6, 2),
+        print(json.dumps({"cfg": name, "pass": rnd, "flush": FLUSH, "opts": opts, "t_us": round(t * 1e6, 2),
                           "p10": round(float(np.percentile(ts, 10)) * 1e6, 2),
                           "p90": round(float(np.percentile(ts, 90)) * 1e6, 2),
                           "gflops": round(2 * s.nnz / t / 1e9, 2), "roof": round(s.alg_bytes() / t / PEAK, 4),
