@@ -1,0 +1,39 @@
+"""Publish-time trace of the 2D grid (c3-shaped) solve: north / west hop costs and the wavefront.
+usage: python tools/trace_grid.py G [key=value ...]   (G x G 5-point lower factor)"""
+import os, sys, json
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import synth
+import paper_conf_icpp_suz0hw0w20_b200 as cap
+
+g = int(sys.argv[1])
+opts = {k: int(v) for k, v in (a.split("=") for a in sys.argv[2:])}
+s = synth.gen_grid(g)
+d = torch.device("cuda")
+rp, ci, v, b = (torch.from_numpy(a).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+h = cap.analyse(rp, ci, v, **opts)
+x = torch.empty_like(b)
+for _ in range(3):
+    h.solve(b, x)
+h.check()
+x, tr = h.trace(b, x)
+t = tr.cpu().numpy().astype(np.int64)[: s.n]
+t = (t - t.min()).reshape(g, g) / 1e3  # us
+inf = h.info()
+K = inf["rows_per_lane"]
+R = 32 * K
+north = t[1:, :] - t[:-1, :]          # T(r,c) - T(r-1,c)
+west = t[:, 1:] - t[:, :-1]           # T(r,c) - T(r,c-1)
+wb = (np.arange(1, g) % R) == 0       # west step crossing a warp boundary
+q = lambda a: [round(float(np.percentile(a, p)), 3) for p in (10, 50, 90)]
+rows_done = t.max(axis=1)
+rows_first = t.min(axis=1)
+out = {"g": g, "opts": opts, "engine": inf["engine"], "K": K, "total_us": round(float(t.max()), 1),
+       "north_us_p10_50_90": q(north), "west_inwarp_us_p10_50_90": q(west[:, ~wb]),
+       "west_warp_boundary_us_p10_50_90": q(west[:, wb]),
+       "row_span_us_p10_50_90": q(rows_done - rows_first),
+       "row_first_gap_us_p10_50_90": q(np.diff(rows_first)),
+       "row_done_gap_us_p10_50_90": q(np.diff(rows_done)),
+       "col0_per_row_us": round(float(t[-1, 0] / (g - 1)), 3),
+       "lastcol_per_row_us": round(float((t[-1, -1] - t[0, -1]) / (g - 1)), 3)}
+print(json.dumps(out))
