@@ -1,5 +1,5 @@
-mkdir -p gpurun_out
-timeout 600 python -m pytest tests/test_gpu_parity.py -x -q -k "chain or auto_choice" > gpurun_out/t_chain.log 2>&1
-python tools/optsweep.py c3 '[{}, {"rows_per_lane":1}, {"backoff_max_ns":512}]' 5 > gpurun_out/sweep10_c3.txt 2>&1
-python tools/optsweep.py chain '[{}]' 5 > gpurun_out/sweep10_chain.txt 2>&1
-python tools/trace_grid.py 2048 > gpurun_out/trace_grid10.txt 2>&1
+mkdir -p gpurun_out/final
+for c in c2 c1 c3 c4 c5; do timeout 400 python bench.py --config $c > gpurun_out/final/bench_$c.json 2> gpurun_out/final/bench_$c.err; done
+ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/final/launches_c2.csv python bench.py --profile --steps 5 --warmup 3 > gpurun_out/final/launches_c2.log 2>&1
+ncu --set full --clock-control none --import-source on -k regex:k_solve_lean --launch-skip 3 -c 1 -o gpurun_out/final/r01_lean6_c2 python bench.py --profile --config c2 --steps 1 --warmup 3 > gpurun_out/final/ncu_c2.log 2>&1
+timeout 300 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/final/ref.json 2> gpurun_out/final/ref.err
