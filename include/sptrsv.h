@@ -189,14 +189,17 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
  * missing / misplaced diagonal -> MISSING_DIAG; as sptrsv_analyse_csr
  * otherwise (lowest offending row wins).  Same ownership and synchronisation
  * as sptrsv_analyse_csr.
- * A handle with tri_flags != 0 runs the thread-level LEAN engine, or -- when
- * the plan is all warp-level (SPTRSV_OPT_MODE = 2, or AUTO with every 32-row
- * group above the warp threshold) -- one warp per row (k_solve_tri_warp).
+ * A handle with tri_flags != 0 runs, for an all-thread-level plan, the LEAN
+ * engine or -- when >= 1/4 of its dependencies fall inside their own 32-row
+ * group of logical rows (grids, chains) -- the CHAIN engine; a plan with
+ * warp-level rows runs k_solve_tri_warp (one warp per long row, 32-row thread
+ * groups for the rest).
  * Upper rows are taken in reverse order behind the same start ticket, so the
  * ticket order is a topological order.  Each row's off-diagonals are summed
  * earliest-solved first: ascending column (lower), descending column (upper).
  * sptrsv_solve, sptrsv_solve_host, sptrsv_get_indegree, sptrsv_check and the
- * options work as for lower handles (ENGINE is ignored);
+ * options work as for lower handles (ENGINE: only 3 LEAN and 7 CHAIN are
+ * honoured, for all-thread-level plans);
  * sptrsv_solve_multi, sptrsv_levels and VARIANT != 0 return
  * SPTRSV_ERR_INVALID_ARG.  Thread-level rows are bit-exact with that fp64
  * substitution (one rounded multiply and add each); warp rows are within the

@@ -50,7 +50,8 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
                 if (c >= n) { code = E_BAD_COL; break; }  // upper only (lower has c <= i < n)
                 if (j > s && c <= prev) { code = E_UNSORTED; break; }
                 if (c != i && (c > i ? c - i : i - c) < 256) ++near;
-                if (c != i && (c >> 5) == (i >> 5)) ++wdep;
+                // same 32-row group of LOGICAL rows (upper handles run row n-1-r as logical r)
+                if (c != i && (upper ? ((n - 1 - c) >> 5) == ((n - 1 - i) >> 5) : (c >> 5) == (i >> 5))) ++wdep;
                 prev = c;
             }
             if (!code && !unit) {

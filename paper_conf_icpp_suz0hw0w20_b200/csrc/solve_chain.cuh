@@ -45,7 +45,13 @@ __host__ __device__ constexpr int chain_warp_smem_bytes(int K) {
              4 * (32 * K + 1)) + 15) / 16 * 16;
 }
 
-template <int PROTO, int K>
+// UPPER / UNIT (G25): the warp owns LOGICAL rows r0 .. r0+R-1, logical row
+// r = physical row n-1-r for upper handles, so the ticket order stays a topological order.  All
+// the chain logic runs on logical indices (dependencies: logical column < logical row); a row's
+// off-diagonals are walked earliest-solved first (descending physical column for upper), its
+// diagonal is the first entry (upper), the last (lower) or implicit 1 (unit).  Loads of CSR
+// entries, polls and publication use physical indices.
+template <int PROTO, int K, bool UPPER = false, bool UNIT = false>
 __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams p) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t s_blk, s_epoch;
@@ -73,17 +79,22 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
     int32_t *s_col = reinterpret_cast<int32_t *>(f_v + RT);
     int32_t *f_has = s_col + ECAP;
     int32_t *s_rp = f_has + RT;
+    // logical <-> physical (upper: reversed); s_rp holds the slice's rowptr in PHYSICAL order
+    const int p0 = UPPER ? p.n - r0 - rows : r0;                  // first physical row of the slice
+    auto phys = [&](int lr) { return UPPER ? p.n - 1 - lr : lr; };  // logical row / column -> physical
+    auto slot = [&](int t) { return UPPER ? rows - 1 - t : t; };    // warp row t -> s_rp index
+    constexpr int dir = UPPER ? -1 : 1;                             // entry walk, earliest-solved first
     // ---- stage rowptr, b, then the warp's contiguous CSR slice (coalesced)
     double bk[K];  // staging only: the rows' constants live in smem (f_b, f_d, f_r) afterwards
 #pragma unroll
     for (int k = 0; k <= K; ++k) {
         const int idx = lane + 32 * k;
-        if (idx <= rows) s_rp[idx] = ld_stream_i32(p.rowptr + r0 + idx, pol);
+        if (idx <= rows) s_rp[idx] = ld_stream_i32(p.rowptr + p0 + idx, pol);
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
         const int idx = lane + 32 * k;
-        bk[k] = idx < rows ? ld_stream_f64(p.b + r0 + idx, pol) : 0.0;
+        bk[k] = idx < rows ? ld_stream_f64(p.b + phys(r0 + idx), pol) : 0.0;
     }
     __syncwarp();
     const int base = s_rp[0];
@@ -99,31 +110,37 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
     __syncwarp();
     auto col_at = [&](int jj) -> int { return staged ? s_col[jj - base] : ld_stream_i32(p.colidx + jj, pol); };
     auto val_at = [&](int jj) -> double { return staged ? s_val[jj - base] : ld_stream_f64(p.val + jj, pol); };
-    // ---- per-row state: cursor j, diagonal index je, next column / value, partial sum
+    // ---- per-row state: cursor j, end je (one step past the last off-diagonal: the diagonal,
+    // or the row's edge for unit forms), next LOGICAL column / value, partial sum
     int j[K], je[K], nc[K];
     double nv[K], ls[K], xm[K];
     unsigned done = 0;  // bit k: row k of this lane finalized (or not a row)
+    auto lcol = [&](int jj) { return UPPER ? p.n - 1 - col_at(jj) : col_at(jj); };
 #pragma unroll
     for (int k = 0; k < K; ++k) {
         const int idx = lane + 32 * k;
         const bool a = idx < rows;
-        j[k] = a ? s_rp[idx] : 0;
-        je[k] = a ? s_rp[idx + 1] - 1 : 0;
-        nc[k] = (a && j[k] < je[k]) ? col_at(j[k]) : -1;
-        nv[k] = (a && j[k] < je[k]) ? val_at(j[k]) : 0.0;
+        const int rs = a ? s_rp[slot(idx)] : 0, re = a ? s_rp[slot(idx) + 1] : 0;
+        // lower: [rs, re-1) ascending, diagonal re-1; upper: (rs, re) descending, diagonal rs;
+        // unit: every stored entry is an off-diagonal
+        j[k] = UPPER ? re - 1 : rs;
+        je[k] = UPPER ? (UNIT ? rs - 1 : rs) : (UNIT ? re : re - 1);
+        if (!a) j[k] = je[k] = 0;
+        nc[k] = (a && j[k] != je[k]) ? lcol(j[k]) : -1;
+        nv[k] = (a && j[k] != je[k]) ? val_at(j[k]) : 0.0;
         ls[k] = 0.0;
         xm[k] = 0.0;
         Diag dg;
-        dg.init(a ? val_at(je[k]) : 1.0);
+        dg.init((a && !UNIT) ? val_at(UPPER ? rs : re - 1) : 1.0);
         if (!a) done |= 1u << k;
         f_b[idx] = bk[k];  // the rows' constants (both chain paths read them from smem)
         f_d[idx] = dg.d;
         f_r[idx] = dg.r;
     }
     auto advance = [&](int k) {
-        ++j[k];
-        const bool more = j[k] < je[k];
-        nc[k] = more ? col_at(j[k]) : -1;
+        j[k] += dir;
+        const bool more = j[k] != je[k];
+        nc[k] = more ? lcol(j[k]) : -1;
         nv[k] = more ? val_at(j[k]) : 0.0;
     };
     const bool tracing = p.trace != nullptr;
@@ -140,15 +157,15 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
             w1[k] = 0;
             if (!(done >> k & 1u) && nc[k] >= 0 && nc[k] < r0) {
                 gm |= 1u << k;
-                poll1<PROTO>(p, nc[k], w0[k], w1[k]);
+                poll1<PROTO>(p, phys(nc[k]), w0[k], w1[k]);
             }
         }
         // ---- consume the ready polls
 #pragma unroll
         for (int k = 0; k < K; ++k) {
             if ((gm >> k & 1u) && ready1<PROTO>(w0[k], w1[k], epoch)) {
-                if (p.trace) p.trace[p.n + r0 + lane + 32 * k] = globaltimer_ns();
-                ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], value1<PROTO>(p, nc[k], w0[k], w1[k])));
+                if (p.trace) p.trace[p.n + phys(r0 + lane + 32 * k)] = globaltimer_ns();
+                ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], value1<PROTO>(p, phys(nc[k]), w0[k], w1[k])));
                 advance(k);
                 prog = true;
             }
@@ -189,7 +206,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
             const int t = lane + 32 * k;
             if (!(done >> k & 1u) && t >= s && t < run_end) {
                 const bool none = nc[k] < 0;
-                const bool prev = nc[k] == r0 + t - 1 && j[k] + 1 == je[k];
+                const bool prev = nc[k] == r0 + t - 1 && j[k] + dir == je[k];
                 el = el && (none || (prev && t > s));
                 f_ls[t] = ls[k];
                 f_v[t] = prev ? nv[k] : 0.0;
@@ -227,8 +244,8 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                     unsigned long long bits = (unsigned long long)__double_as_longlong(q);
                     bits = bits == kSentinel ? kCanonNaN : bits;
                     const unsigned long long e = (unsigned long long)epoch << 32;
-                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)(r0 + t), e | (bits & 0xffffffffull), e | (bits >> 32));
-                    if (tracing) st_u64_if(mine, p.trace + r0 + t, globaltimer_ns());
+                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)phys(r0 + t), e | (bits & 0xffffffffull), e | (bits >> 32));
+                    if (tracing) st_u64_if(mine, p.trace + phys(r0 + t), globaltimer_ns());
                 }
                 xp = q;
                 lsv = lsn, bv = bn, vv = vn, dv = dn, rv = rn, hv = hn;
@@ -258,8 +275,8 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                     unsigned long long bits = (unsigned long long)__double_as_longlong(q);
                     bits = bits == kSentinel ? kCanonNaN : bits;  // same canonicalisation as publish()
                     const unsigned long long e = (unsigned long long)epoch << 32;
-                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
-                    if (tracing) st_u64_if(mine, p.trace + r0 + s, globaltimer_ns());
+                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)phys(r0 + s), e | (bits & 0xffffffffull), e | (bits >> 32));
+                    if (tracing) st_u64_if(mine, p.trace + phys(r0 + s), globaltimer_ns());
                 }
                 const int cs = r0 + s;
 #pragma unroll
@@ -278,9 +295,9 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
             for (int k = 0; k < K; ++k) {
                 const int t = lane + 32 * k;
                 if (t >= s0 && t < s) {
-                    p.x[r0 + t] = xm[k];
+                    p.x[phys(r0 + t)] = xm[k];
                     s_x[t] = xm[k];
-                    if (PROTO == PROTO_FLAGS && p.trace) p.trace[r0 + t] = globaltimer_ns();
+                    if (PROTO == PROTO_FLAGS && p.trace) p.trace[phys(r0 + t)] = globaltimer_ns();
                 }
             }
             if (PROTO == PROTO_FLAGS) {
@@ -288,7 +305,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
 #pragma unroll
                 for (int k = 0; k < K; ++k) {
                     const int t = lane + 32 * k;
-                    if (t >= s0 && t < s) st_relaxed_u32(p.flags + r0 + t, epoch);
+                    if (t >= s0 && t < s) st_relaxed_u32(p.flags + phys(r0 + t), epoch);
                 }
             }
         }
@@ -322,10 +339,10 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
             for (int k = 0; k < K; ++k) {
                 if (!(done >> k & 1u) && nc[k] >= 0 && nc[k] < r0) {
                     unsigned long long a0, a1;
-                    poll1<PROTO>(p, nc[k], a0, a1);
+                    poll1<PROTO>(p, phys(nc[k]), a0, a1);
                     if (ready1<PROTO>(a0, a1, epoch)) {
-                        if (p.trace) p.trace[p.n + r0 + lane + 32 * k] = globaltimer_ns();
-                        ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], value1<PROTO>(p, nc[k], a0, a1)));
+                        if (p.trace) p.trace[p.n + phys(r0 + lane + 32 * k)] = globaltimer_ns();
+                        ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], value1<PROTO>(p, phys(nc[k]), a0, a1)));
                         advance(k);
                         got = true;
                     }

@@ -478,9 +478,14 @@ int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem,
 // one-shot engine on every warp-plan shape measured, tools/hybrid_probe.py).
 // (Round-1 B200 sweeps.)
 int resolve_engine(const sptrsv_handle_s *h) {
-    if (h->tri) return h->plan == PLAN_THREAD ? 3 : 6;  // f4 handles: LEAN or tri hybrid
+    // stored off-diagonals (unit handles store no diagonal)
+    const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;
+    if (h->tri) {  // f4 handles: tri hybrid for warp rows, else CHAIN or LEAN (ENGINE 3 / 7 honoured)
+        if (h->plan != PLAN_THREAD) return 6;
+        if (h->engine == 3 || h->engine == 7) return h->engine;
+        return (offdiag > 0 && 4 * h->warp_deps >= offdiag) ? 7 : 3;
+    }
     if (h->engine != 5) return h->engine;
-    const long long offdiag = h->nnz - h->n;
     if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_deps < offdiag)) return 3;
     if (h->plan != PLAN_THREAD) return 6;
     if (4 * h->warp_deps >= offdiag) return 7;  // in-warp chains: CHAIN
@@ -588,7 +593,8 @@ lean_fn tri_warp_kernel(int proto, int tri, int plan) {
 }
 
 int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
-    if (h->tri || (!h->variant && resolve_engine(h) == 6)) {  // f4 forms, or ENGINE_HYBRID (solve_lean.cuh / solve_tri.cuh)
+    if ((h->tri && resolve_engine(h) != 7) || (!h->tri && !h->variant && resolve_engine(h) == 6)) {
+        // f4 forms (LEAN / tri hybrid), or ENGINE_HYBRID (solve_lean.cuh / solve_tri.cuh)
         L->kind = 0;
         L->smem = 0;
         if (h->plan != PLAN_THREAD) {  // warp-level rows present: one task per warp
@@ -675,8 +681,13 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
     if (engine == 7 && h->plan == PLAN_THREAD && cta <= 256) {
         const int K = Kq >= 2 ? 2 : 1;
         const int warps = cta / 32;
-        L->fn = K == 2 ? (h->proto ? (const void *)k_solve_chain<PROTO_FUSED, 2> : (const void *)k_solve_chain<PROTO_FLAGS, 2>)
-                       : (h->proto ? (const void *)k_solve_chain<PROTO_FUSED, 1> : (const void *)k_solve_chain<PROTO_FLAGS, 1>);
+#define CHAIN_ROW(U_, N_)                                                                              \
+    {{k_solve_chain<PROTO_FLAGS, 1, U_, N_>, k_solve_chain<PROTO_FUSED, 1, U_, N_>},                   \
+     {k_solve_chain<PROTO_FLAGS, 2, U_, N_>, k_solve_chain<PROTO_FUSED, 2, U_, N_>}}
+        static const lean_fn ctab[4][2][2] = {CHAIN_ROW(false, false), CHAIN_ROW(true, false),
+                                              CHAIN_ROW(false, true), CHAIN_ROW(true, true)};
+#undef CHAIN_ROW
+        L->fn = (const void *)ctab[h->tri & 3][K - 1][h->proto ? 1 : 0];
         L->kind = 0;
         const long long rows_per_cta = (long long)warps * 32 * K;
         L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
@@ -687,7 +698,7 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
             (void)cudaGetLastError();
             return SPTRSV_ERR_CUDA;
         }
-        L->key = 8000000 + h->proto * 100000 + K * 10000 + cta;
+        L->key = 8000000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta;
         L->key ^= (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }

@@ -68,8 +68,12 @@ def test_tri_random_sizes_bit_exact(cap, n, gen, flags, proto):
     s = form(GENS[gen](n), flags)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     x, info = gpu_solve(cap, s, flags, protocol=proto)
-    assert info["engine"] == 3
+    assert info["engine"] in (3, 7)  # LEAN, or CHAIN when >= 1/4 of the dependencies are in-warp
     assert np.array_equal(x, ref)
+    for engine in (3, 7):  # both thread-level engines, forced
+        x, info = gpu_solve(cap, s, flags, protocol=proto, engine=engine)
+        assert info["engine"] == engine
+        assert np.array_equal(x, ref)
 
 
 @pytest.mark.parametrize("which", ["c2", "c2i", "grid", "c4", "dense", "chain"])
@@ -285,3 +289,42 @@ def test_tri_unsupported_calls_fail_loudly(cap):
         x = h.solve(b)
         h.check()
         assert np.array_equal(x.cpu().numpy(), oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, U))
+
+
+@pytest.mark.parametrize("which", ["grid", "chain", "c2i", "rand4"])
+@pytest.mark.parametrize("flags", FORMS)
+@pytest.mark.parametrize("proto", [0, 1])
+@pytest.mark.parametrize("K,cta", [(1, 128), (2, 128), (2, 64), (2, 256)])
+def test_tri_chain_engine_bit_exact(cap, which, flags, proto, K, cta):
+    """CHAIN (in-warp chains in registers) on f4 handles: logical rows reversed for upper, the
+    diagonal first / implicit, entries walked earliest-solved first -- bit-exact vs solve_tri."""
+    base = {"grid": lambda: synth.gen_grid(150), "chain": lambda: synth.gen_chain(20_000),
+            "c2i": lambda: synth.gen_c2i(n=60_000), "rand4": lambda: synth.gen_random_lower(4099, 4, seed=5)}[which]()
+    s = form(base, flags)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
+    x, info = gpu_solve(cap, s, flags, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+    assert (info["engine"], info["rows_per_lane"], info["cta_threads"]) == (7, K, cta), info
+    assert np.array_equal(x, ref)
+
+
+@pytest.mark.parametrize("flags", FORMS)
+def test_tri_chain_auto_choice_and_closed_forms(cap, flags):
+    """AUTO sends f4 grids and chains to CHAIN; the f4 bidiagonal closed forms stay exact."""
+    s = form(synth.gen_grid(200), flags)
+    x, info = gpu_solve(cap, s, flags)
+    assert info["engine"] == 7, info
+    assert np.array_equal(x, oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags))
+    s = form(synth.gen_c2(n=100_000), flags)
+    _, info = gpu_solve(cap, s, flags)
+    assert info["engine"] == 3, info  # far dependencies stay on LEAN
+    n = 100_000  # upper bidiagonal U_ii = 2, U_{i,i+1} = -1, b = 1 (as test_upper_bidiagonal_closed_form)
+    rp = np.r_[np.arange(0, 2 * n, 2), 2 * n - 1].astype(np.int32)
+    ci = np.empty(2 * n - 1, np.int32)
+    v = np.empty(2 * n - 1)
+    ci[0::2], v[0::2] = np.arange(n), 2.0
+    ci[1::2], v[1::2] = np.arange(1, n), -1.0
+    sb = synth.CSRSystem("ub", n, rp, ci, v, np.ones(n), None, {})
+    x, info = gpu_solve(cap, sb, U)
+    assert info["engine"] == 7
+    k = np.arange(n - 53, n)
+    assert np.array_equal(x[k], 1.0 - 2.0 ** -(n - k).astype(float))
