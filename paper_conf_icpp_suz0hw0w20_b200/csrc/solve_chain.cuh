@@ -219,7 +219,8 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
             // operands of row t are loaded one iteration ahead, off the dependency chain
             double lsv = f_ls[s], bv = f_b[s], vv = f_v[s], dv = f_d[s], rv = f_r[s];
             int hv = f_has[s];
-            for (int t = s; t < run_end; ++t) {
+            int t = s;
+            for (; t < run_end; ++t) {
                 const int tn = min(t + 1, run_end - 1);
                 const double lsn = f_ls[tn], bn = f_b[tn], vn = f_v[tn], dn = f_d[tn], rn = f_r[tn];
                 const int hn = f_has[tn];
@@ -228,9 +229,12 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 Diag g;
                 g.d = dv;
                 g.r = rv;
-                double q = g.cand(a);
-                // guard (Diag::ok) in integer ops; warp-uniform here: every lane holds the same a
-                if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0), 0)) q = __ddiv_rn(a, dv);
+                const double q = g.cand(a);
+                // guard (Diag::ok) in integer ops, warp-uniform here (every lane holds the same a).  A
+                // failure LEAVES the fast loop instead of branching around an in-loop __ddiv_rn: the
+                // loop body then has no reconvergence point, and the guard resolves from a while the
+                // Markstein step is still in flight (chain step ~140 -> ~90 cycles, chainstep.cu)
+                if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0), 0)) break;
                 const int owner = t & 31, kk = t >> 5;
                 const bool mine = lane == owner;
 #pragma unroll
@@ -250,7 +254,20 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 xp = q;
                 lsv = lsn, bv = bn, vv = vn, dv = dn, rv = rn, hv = hn;
             }
-            s = run_end;
+            if (t < run_end && hv) {
+                // the guard failed at row t: the exact loop below finishes the run from t.  Row t's
+                // previous-row entry is consumed first, by its owner, with the same mul and add as the
+                // fast step (so the sum stays bit-identical to Alg.1)
+                const int owner = t & 31, kk = t >> 5;
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    if (lane == owner && kk == k) {
+                        ls[k] = __dadd_rn(ls[k], __dmul_rn(nv[k], xp));
+                        advance(k);
+                    }
+                }
+            }
+            s = t;
         }
 #pragma unroll
         for (int k = 0; k < K; ++k) {  // rows r0 + 32k .. r0 + 32k + 31: owner lane = s - 32k

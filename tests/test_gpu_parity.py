@@ -399,6 +399,34 @@ def test_chain_engine(cap, proto, K, cta):
     assert np.array_equal(x, np.where(i <= 52, 1.0 - np.ldexp(1.0, -(np.minimum(i, 52) + 1)), 1.0))
 
 
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("K", [1, 2])
+def test_chain_engine_division_guard_exits(cap, proto, K):
+    """CHAIN's fast (bidiagonal / grid-west) loop leaves to the exact loop when the Markstein
+    range guard fails (|a| or |L_ii| outside [2^-400, 2^401)): chains whose diagonals and
+    right-hand sides span 2^+-600 -- guard failures at arbitrary steps, overflow, underflow --
+    must still match Alg.1 bit for bit (NaN positions included)."""
+    rng = np.random.default_rng(31 + K)
+    for n, frac in ((3000, 0.02), (3000, 0.5), (700, 1.0)):
+        rp = np.r_[0, np.arange(1, 2 * n, 2)].astype(np.int32)
+        ci = np.empty(2 * n - 1, np.int32)
+        v = np.empty(2 * n - 1)
+        ci[0], ci[1::2], ci[2::2] = 0, np.arange(0, n - 1), np.arange(1, n)
+        d = rng.uniform(1, 2, n) * rng.choice([-1.0, 1.0], n)
+        wild = rng.random(n) < frac
+        d[wild] = np.ldexp(d[wild], rng.integers(-600, 600, wild.sum()))
+        v[0], v[2::2] = d[0], d[1:]
+        v[1::2] = -np.ldexp(1.0, rng.integers(-20, 20, n - 1))
+        b = rng.uniform(-1, 1, n)
+        bw = rng.random(n) < frac
+        b[bw] = np.ldexp(b[bw], rng.integers(-600, 600, bw.sum()))
+        s = synth.CSRSystem("wild", n, rp, ci, v, b, None, {})
+        x, info = gpu_solve(cap, s, 1, protocol=proto, engine=7, rows_per_lane=K)
+        assert info["engine"] == 7
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        assert np.array_equal(x, ref, equal_nan=True), (n, frac)
+
+
 def test_engine_auto_choice(cap):
     """ENGINE_AUTO: far dependencies -> LEAN (3); in-warp chains / grid wavefronts -> CHAIN (7);
     other near-dependency plans -> staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""

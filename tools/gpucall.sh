@@ -1,4 +1,5 @@
 mkdir -p gpurun_out
-timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/t_all13.log 2>&1
-timeout 400 python bench.py --config c3 --no-cpu-baseline > gpurun_out/bench13_c3.json 2> gpurun_out/bench13_c3.err
-python tools/optsweep.py chain '[{}]' 5 > gpurun_out/sweep13_chain.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_tri.py -x -q -k "chain or auto_choice or division or closed" > gpurun_out/t_chain16.log 2>&1
+python tools/optsweep.py c3 '[{}]' 5 > gpurun_out/sweep16_c3.txt 2>&1
+python tools/optsweep.py chain '[{}]' 5 > gpurun_out/sweep16_chain.txt 2>&1
+python tools/trace_grid.py 2048 > gpurun_out/trace_grid16.txt 2>&1

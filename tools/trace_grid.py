@@ -36,4 +36,15 @@ out = {"g": g, "opts": opts, "engine": inf["engine"], "K": K, "total_us": round(
        "row_done_gap_us_p10_50_90": q(np.diff(rows_done)),
        "col0_per_row_us": round(float(t[-1, 0] / (g - 1)), 3),
        "lastcol_per_row_us": round(float((t[-1, -1] - t[0, -1]) / (g - 1)), 3)}
+pos = np.arange(g) % R
+for name, m in (("pos0", pos == 0), ("pos1", pos == 1), ("pos2_7", (pos >= 2) & (pos < 8)),
+                ("pos8_31", (pos >= 8) & (pos < 32)), ("pos32_63", pos >= 32)):
+    if m.any():
+        out["north_us_p50_" + name] = round(float(np.percentile(north[:, m], 50)), 3)
+out["north_us_p50_col0"] = round(float(np.percentile(north[:, 0], 50)), 3)
+# how far the row below trails inside one warp: publish time of the warp's first cell relative to
+# the north warp's last cell
+first = t[1:, ::R]
+north_last = t[:-1, R - 1::R][:, : first.shape[1]]
+out["warp_first_minus_north_warp_last_us_p10_50_90"] = q(first[:, : north_last.shape[1]] - north_last)
 print(json.dumps(out))
