@@ -53,6 +53,9 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
     int nc = (act && inr(j)) ? ld_stream_i32(p.colidx + j, pol) : -1;
     double nv = (act && inr(j)) ? ld_stream_f64(p.val + j, pol) : 0.0;
     int nc2 = (act && inr(j + dir)) ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
+    // the second dependency's VALUE is preloaded too: consuming both dependencies in one pass
+    // (the common case when the earlier one is long solved) then never waits on a reload
+    double nv2 = (act && inr(j + dir)) ? ld_stream_f64(p.val + j + dir, pol) : 0.0;
     Diag dg;
     dg.init(dv);
     if (p.trace && act && nc != -2) p.trace[2 * (size_t)p.n + i] = globaltimer_ns();  // loads landed
@@ -68,8 +71,10 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
     auto advance = [&]() {
         j += dir;
         nc = nc2;
-        nv = (nc >= 0) ? ld_stream_f64(p.val + j, pol) : 0.0;
-        nc2 = inr(j + dir) ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
+        nv = nv2;
+        const bool more = inr(j + dir);
+        nc2 = more ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
+        nv2 = more ? ld_stream_f64(p.val + j + dir, pol) : 0.0;
     };
     while (true) {
         bool prog = false;
