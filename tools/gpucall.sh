@@ -1,6 +1,3 @@
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_tri.py -x -q -k "lean or tri or hybrid" > gpurun_out/t_lean17.log 2>&1
-python tools/optsweep.py c2 '[{}, {"lean_occupancy":5}]' 30 > gpurun_out/sweep17_c2.txt 2>&1
-python tools/optsweep.py c5_0 '[{}]' 20 > gpurun_out/sweep17_c5.txt 2>&1
-python tools/optsweep.py c4 '[{}]' 10 > gpurun_out/sweep17_c4.txt 2>&1
-python tools/optsweep.py diag:1000000 '[{}]' 20 > gpurun_out/sweep17_diag.txt 2>&1
+timeout 900 compute-sanitizer --tool memcheck --print-limit 20 python tools/memcheck_small.py > gpurun_out/memcheck18.txt 2>&1; echo "rc=$?" >> gpurun_out/memcheck18.txt
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/t_all18.log 2>&1
