@@ -72,3 +72,52 @@ def test_chain_full_closed_form(proto):
     x1, _, _ = _run(s, protocol=proto)
     want = np.array([1.0 - 2.0 ** -(i + 1) if i <= 52 else 1.0 for i in range(s.n)])
     assert np.array_equal(x1, want)
+
+
+@pytest.mark.parametrize("proto", [0, 1])
+def test_c2_full_default_launch(proto):
+    """c2 in exactly the bench.py configuration: default options, AUTO -> LEAN."""
+    s = synth.gen_c2()
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    x1, x2, info = _run(s, protocol=proto)
+    assert info["engine"] == 3
+    assert np.array_equal(x1, ref) and np.array_equal(x2, ref)
+
+
+def test_c3_full_default_launch():
+    """c3 in the bench.py configuration: AUTO -> CHAIN with 2 rows per lane, 128-thread CTAs."""
+    s = synth.gen_c3(ones=True)
+    x1, x2, info = _run(s)
+    assert (info["engine"], info["rows_per_lane"], info["cta_threads"]) == (7, 2, 128), info
+    assert np.array_equal(x1, np.ones(s.n)) and np.array_equal(x2, np.ones(s.n))
+    s = synth.gen_c3()
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    x1, x2, _ = _run(s)
+    assert np.array_equal(x1, ref) and np.array_equal(x2, ref)
+
+
+@pytest.mark.parametrize("cfg,flags", [("c2", 1), ("c2", 2), ("c2", 3), ("c3", 1), ("c3", 2), ("c3", 3),
+                                       ("c4", 1), ("c4", 3)])
+def test_f4_forms_full(cfg, flags):
+    """SURVEY f4 at full BASELINE sizes, the bench's triangular_forms_leg configuration (AUTO):
+    upper (flags 1), unit lower (2), unit upper (3) -- LEAN (c2), CHAIN (c3), HYBRID (c4)."""
+    import paper_conf_icpp_suz0hw0w20_b200 as cap
+    s = {"c2": synth.gen_c2, "c3": synth.gen_c3, "c4": synth.gen_c4}[cfg]()
+    if flags & 1:
+        s = synth.to_upper(s)
+    if flags & 2:
+        s = synth.to_unit(s)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
+    d = torch.device("cuda:0")
+    rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+    with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2)) as h:
+        x = torch.full_like(b, float("nan"))
+        h.solve(b, x)
+        h.check()
+        info = h.info()
+        got = x.cpu().numpy()
+    assert info["engine"] == {"c2": 3, "c3": 7, "c4": 6}[cfg], info
+    if cfg == "c4":
+        assert np.max(np.abs(got - ref) / np.abs(ref)) <= TOL
+    else:
+        assert np.array_equal(got, ref)
