@@ -234,9 +234,15 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
                        sptrsv_stream_t stream);
 
 /*
- * sptrsv_solve_host -- end-to-end convenience: copies b (host) to handle-owned
- * device staging, solves, copies x back to host, and synchronises `stream`.
- * b_host/x_host: host double[n] (pinned memory gives full PCIe bandwidth).
+ * sptrsv_solve_host -- end-to-end convenience from host buffers; synchronises
+ * `stream` before returning.  b_host/x_host: host double[n].
+ *   - Both pinned (page-locked, UVA-mapped; e.g. cudaHostAlloc or torch
+ *     pin_memory) and the handle runs LEAN: no separate copies.  The kernel
+ *     reads b straight from host memory over PCIe and every CTA writes its
+ *     finished rows of x to x_host as one contiguous block, so both transfers
+ *     overlap the solve (x also lands in handle-owned device staging).
+ *   - Otherwise: b is copied to handle-owned device staging, solved, and x is
+ *     copied back (cudaMemcpyAsync; pageable buffers are staged by the driver).
  */
 int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host,
                       sptrsv_stream_t stream);

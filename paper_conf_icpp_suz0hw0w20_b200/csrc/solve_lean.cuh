@@ -185,6 +185,17 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     const bool act = i >= 0 && i < p.n;
     lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);
     if (p.trace && lane == 0) atomicMax(&p.trace[3 * (size_t)p.n + 1], globaltimer_ns());  // last warp exit
+    if (p.x_host) {
+        // sptrsv_solve_host: the CTA's finished rows go to pinned host memory over PCIe as one
+        // contiguous, coalesced block per CTA (8-byte per-row publishes would each be a TLP),
+        // overlapping the device->host transfer with the rest of the solve
+        __syncthreads();
+        const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
+        if (lr0 < lr1) {
+            const int a = UPPER ? p.n - lr1 : lr0, e = UPPER ? p.n - lr0 : lr1;
+            for (int r = a + tid; r < e; r += CT) p.x_host[r] = __ldcg(p.x + r);
+        }
+    }
 }
 
 }  // namespace sptrsv_dev

@@ -758,7 +758,14 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
 
 }  // namespace
 
+static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream);
+
 int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream) {
+    return solve_impl(h, b, x, nullptr, stream);
+}
+
+// x_host (LEAN only, from sptrsv_solve_host): device-mapped pinned host copy target of x
+static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!b || !x || b == x) return SPTRSV_ERR_INVALID_ARG;
@@ -800,6 +807,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
     p.poll_gap = h->poll_gap;
     p.poll_one = h->poll_one;
     p.chain_pub = h->chain_pub;
+    p.x_host = x_host;
     p.trace = h->trace;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = L.grid;
@@ -935,6 +943,22 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         }
     }
     cudaStream_t s = (cudaStream_t)stream;
+    // Pinned host buffers and the LEAN engine: no separate copies.  The kernel reads b straight
+    // from host memory (UVA mapping, each warp one coalesced 256-byte PCIe read) and every CTA
+    // writes its finished rows of x to host memory as one contiguous block, so both transfers
+    // overlap the solve instead of bracketing it.  x still lands in device memory first (the
+    // FLAGS protocol reads it back; FUSED consumers read the records).
+    cudaPointerAttributes ab, ax;
+    const bool pinned = cudaPointerGetAttributes(&ab, b_host) == cudaSuccess &&
+                        cudaPointerGetAttributes(&ax, x_host) == cudaSuccess && ab.type == cudaMemoryTypeHost &&
+                        ax.type == cudaMemoryTypeHost && ab.devicePointer && ax.devicePointer;
+    (void)cudaGetLastError();
+    if (pinned && !h->variant && resolve_engine(h) == 3 && h->plan == PLAN_THREAD) {
+        int rc = solve_impl(h, (const double *)ab.devicePointer, h->ws.x_stage, (double *)ax.devicePointer, stream);
+        if (rc) return rc;
+        CK(cudaStreamSynchronize(s));
+        return SPTRSV_OK;
+    }
     CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
     int rc = sptrsv_solve(h, h->ws.b_stage, h->ws.x_stage, stream);
     if (rc) return rc;

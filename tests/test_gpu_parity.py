@@ -200,13 +200,44 @@ def test_many_solves_on_side_stream_and_graph_capture(cap, proto, engine):
             assert np.array_equal(x2.cpu().numpy(), ref)
 
 
-def test_solve_host_e2e(cap):
-    s = synth.gen_c2(n=100_000)
-    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("engine", [5, 0, 7])
+@pytest.mark.parametrize("pinned", [True, False])
+def test_solve_host_e2e(cap, proto, engine, pinned):
+    """sptrsv_solve_host from pinned host buffers (LEAN: b read over PCIe inside the kernel, x
+    written per CTA to host memory -- no staging copies) and from pageable numpy buffers
+    (staged copies), every engine family, ragged sizes, repeated solves on one handle."""
+    for s in (synth.gen_c2(n=100_000), synth.gen_random_lower(1000, 3, seed=4), synth.gen_random_lower(33, 2, seed=5)):
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        rp, ci, v, _ = dev_csr(s)
+        with cap.analyse(rp, ci, v, protocol=proto, engine=engine) as h:
+            if pinned:
+                bh = torch.from_numpy(s.b).pin_memory()
+                xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
+            else:
+                bh = s.b.copy()
+                xh = np.full(s.n, np.nan)
+            for _ in range(3):
+                (xh.fill_ if pinned else xh.fill)(float("nan"))
+                h.solve_host(bh, xh)
+                got = xh.numpy() if pinned else xh
+                assert np.array_equal(got, ref), (s.name, proto, engine, pinned)
+
+
+@pytest.mark.parametrize("flags", [1, 2, 3])
+def test_solve_host_e2e_f4_lean(cap, flags):
+    """The pinned path for upper / unit handles on LEAN (physical row ranges of reversed CTAs)."""
+    s = synth.gen_c2(n=70_000)  # 70000 % 256 = 112: a ragged last CTA
+    if flags & 1:
+        s = synth.to_upper(s)
+    if flags & 2:
+        s = synth.to_unit(s)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     rp, ci, v, _ = dev_csr(s)
-    with cap.analyse(rp, ci, v) as h:
+    with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2)) as h:
+        assert h.info()["engine"] == 3
         bh = torch.from_numpy(s.b).pin_memory()
-        xh = torch.empty(s.n, dtype=torch.float64).pin_memory()
+        xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
         h.solve_host(bh, xh)
         assert np.array_equal(xh.numpy(), ref)
 

@@ -1,3 +1,3 @@
 mkdir -p gpurun_out
-timeout 900 compute-sanitizer --tool memcheck --print-limit 20 python tools/memcheck_small.py > gpurun_out/memcheck18.txt 2>&1; echo "rc=$?" >> gpurun_out/memcheck18.txt
-timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/t_all18.log 2>&1
+timeout 600 python -m pytest tests/test_gpu_parity.py -x -q -k "solve_host or lean" > gpurun_out/t_host24.log 2>&1
+timeout 400 python bench.py --config c4 --no-cpu-baseline --no-flags-leg --no-tri-leg --nrhs 0 > gpurun_out/bench24_c4.json 2> gpurun_out/bench24_c4.err
