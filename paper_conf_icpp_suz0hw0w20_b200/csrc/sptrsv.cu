@@ -88,6 +88,7 @@ struct sptrsv_handle_s {
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
     int chain_pub = 32;     // CHAIN: publication batch in chain steps (SPTRSV_OPT_CHAIN_PUBLISH)
+    int split_last = 1;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
     int grid_cache = 0;
@@ -807,6 +808,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.poll_gap = h->poll_gap;
     p.poll_one = h->poll_one;
     p.chain_pub = h->chain_pub;
+    p.split_last = h->split_last;
     p.x_host = x_host;
     p.trace = h->trace;
     cudaLaunchConfig_t cfg = {};
@@ -1084,6 +1086,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->poll_one = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_WARP_SPLIT_LAST:
+            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            h->split_last = (int)value;
+            return SPTRSV_OK;
         case SPTRSV_OPT_CHAIN_PUBLISH:
             if (value < 1 || value > 64) return SPTRSV_ERR_INVALID_ARG;
             h->chain_pub = (int)value;
@@ -1117,6 +1123,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_POLL_GAP_NS: *value = h->poll_gap; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
         case SPTRSV_OPT_CHAIN_PUBLISH: *value = h->chain_pub; return SPTRSV_OK;
+        case SPTRSV_OPT_WARP_SPLIT_LAST: *value = h->split_last; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }

@@ -1,3 +1,3 @@
 mkdir -p gpurun_out
-timeout 600 python -m pytest tests/test_gpu_parity.py -x -q -k "solve_host or lean" > gpurun_out/t_host24.log 2>&1
-timeout 400 python bench.py --config c4 --no-cpu-baseline --no-flags-leg --no-tri-leg --nrhs 0 > gpurun_out/bench24_c4.json 2> gpurun_out/bench24_c4.err
+python tools/optsweep.py c4 '[{"warp_split_last":0}, {"warp_split_last":1}, {"warp_split_last":0,"backoff_max_ns":0}, {"warp_split_last":1,"backoff_max_ns":0}]' 10 > gpurun_out/sweep27_c4.txt 2>&1
+python tools/optsweep.py lev:200000:400 '[{"warp_split_last":0,"mode":2}, {"warp_split_last":1,"mode":2}]' 10 > gpurun_out/sweep27_lev.txt 2>&1
