@@ -116,10 +116,12 @@ typedef enum sptrsv_option {
                                       lanes waiting (0 = default, none)                    */
     SPTRSV_OPT_POLL_ONE = 20,      /* LEAN: 1 = poll one dependency per lane per pass
                                       (default 0: the next two, DESIGN G21)                 */
-    SPTRSV_OPT_WARP_SPLIT_LAST = 22,/* warp-level rows: 1 (default) = the row's last
+    SPTRSV_OPT_WARP_SPLIT_LAST = 22,/* warp-level rows: 2 (default) = the row's last
                                       off-diagonal (its nearest dependency) is added after
-                                      the lane-strided tree, by lane 0 alone; 0 = it is part
-                                      of the tree.  Both orders are fixed (deterministic) */
+                                      the lane-strided tree by lane 0 alone, which polls it
+                                      with at most 32 ns sleeps; 1 = the same with the
+                                      handle's backoff; 0 = it is part of the tree.  Every
+                                      order is fixed (deterministic)                       */
     SPTRSV_OPT_CHAIN_PUBLISH = 21, /* CHAIN engine (FUSED): finalized rows are published in
                                       warp-wide batches every this many chain steps, 1..64
                                       (default 32)                                         */

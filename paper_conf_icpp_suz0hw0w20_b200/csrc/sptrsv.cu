@@ -88,7 +88,7 @@ struct sptrsv_handle_s {
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
     int chain_pub = 32;     // CHAIN: publication batch in chain steps (SPTRSV_OPT_CHAIN_PUBLISH)
-    int split_last = 1;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
+    int split_last = 2;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
     int grid_cache = 0;
@@ -1087,7 +1087,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->poll_one = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST:
-            if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
             h->split_last = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_CHAIN_PUBLISH:
