@@ -122,9 +122,7 @@ typedef enum sptrsv_option {
                                       with at most 32 ns sleeps; 1 = the same with the
                                       handle's backoff; 0 = it is part of the tree.  Every
                                       order is fixed (deterministic)                       */
-    SPTRSV_OPT_CHAIN_PUBLISH = 21, /* CHAIN engine (FUSED): finalized rows are published in
-                                      warp-wide batches every this many chain steps, 1..64
-                                      (default 32)                                         */
+    /* 21: retired (CHAIN publishes every finalized row at once)                        */
     SPTRSV_OPT_VARIANT = 16        /* ablation: 0 (default) product path; 3, 4, 5
                                       = the paper's Alg.3 SyncFree (warp per row), Alg.4
                                       Two-Phase, Alg.5 Writing-First with their printed

@@ -197,7 +197,7 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
             "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY,
             "prefetch": _lib.OPT_PREFETCH, "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
-            "poll_one": _lib.OPT_POLL_ONE, "chain_publish": _lib.OPT_CHAIN_PUBLISH,
+            "poll_one": _lib.OPT_POLL_ONE,
             "warp_split_last": _lib.OPT_WARP_SPLIT_LAST}
     for k, v in options.items():
         h.set_option(keys[k], v)

@@ -87,7 +87,6 @@ struct sptrsv_handle_s {
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
-    int chain_pub = 32;     // CHAIN: publication batch in chain steps (SPTRSV_OPT_CHAIN_PUBLISH)
     int split_last = 2;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
@@ -807,7 +806,6 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.pf_dist = L.pf_dist;
     p.poll_gap = h->poll_gap;
     p.poll_one = h->poll_one;
-    p.chain_pub = h->chain_pub;
     p.split_last = h->split_last;
     p.x_host = x_host;
     p.trace = h->trace;
@@ -1090,10 +1088,6 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
             h->split_last = (int)value;
             return SPTRSV_OK;
-        case SPTRSV_OPT_CHAIN_PUBLISH:
-            if (value < 1 || value > 64) return SPTRSV_ERR_INVALID_ARG;
-            h->chain_pub = (int)value;
-            return SPTRSV_OK;
         default:
             return SPTRSV_ERR_INVALID_ARG;
     }
@@ -1122,7 +1116,6 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_PREFETCH: *value = h->pf_dist; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_GAP_NS: *value = h->poll_gap; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
-        case SPTRSV_OPT_CHAIN_PUBLISH: *value = h->chain_pub; return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST: *value = h->split_last; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
