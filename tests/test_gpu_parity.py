@@ -463,7 +463,7 @@ def test_engine_auto_choice(cap):
     other near-dependency plans -> staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""
     for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 7, 128, 2),
                               (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
-                              (lambda: synth.gen_c1(), 0, 256, 1),
+                              (lambda: synth.gen_c1(), 0, 1024, 1),
                               (lambda: synth.gen_c4(n=5000, nlevels=50), 6, 64, 1)):
         s = gen()
         x, info = gpu_solve(cap, s)
