@@ -116,6 +116,11 @@ typedef enum sptrsv_option {
                                       lanes waiting (0 = default, none)                    */
     SPTRSV_OPT_POLL_ONE = 20,      /* LEAN: 1 = poll one dependency per lane per pass
                                       (default 0: the next two, DESIGN G21)                 */
+    SPTRSV_OPT_HOST_IO = 23,       /* sptrsv_solve_host with pinned buffers on LEAN: bit 0 =
+                                      the kernel reads b over PCIe, bit 1 = each CTA writes
+                                      its rows of x to host memory; a cleared bit uses a
+                                      cudaMemcpyAsync before / after the solve instead.
+                                      Default 2 (b by DMA, x written per CTA)              */
     SPTRSV_OPT_WARP_SPLIT_LAST = 22,/* warp-level rows: 2 (default) = the row's last
                                       off-diagonal (its nearest dependency) is added after
                                       the lane-strided tree by lane 0 alone, which polls it
@@ -241,10 +246,10 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
  * sptrsv_solve_host -- end-to-end convenience from host buffers; synchronises
  * `stream` before returning.  b_host/x_host: host double[n].
  *   - Both pinned (page-locked, UVA-mapped; e.g. cudaHostAlloc or torch
- *     pin_memory) and the handle runs LEAN: no separate copies.  The kernel
- *     reads b straight from host memory over PCIe and every CTA writes its
- *     finished rows of x to x_host as one contiguous block, so both transfers
- *     overlap the solve (x also lands in handle-owned device staging).
+ *     pin_memory) and the handle runs LEAN: b is copied to device staging,
+ *     and every CTA writes its finished rows of x to x_host as one contiguous
+ *     block, so the device->host transfer overlaps the solve (x also lands in
+ *     handle-owned device staging).  SPTRSV_OPT_HOST_IO selects the variants.
  *   - Otherwise: b is copied to handle-owned device staging, solved, and x is
  *     copied back (cudaMemcpyAsync; pageable buffers are staged by the driver).
  */

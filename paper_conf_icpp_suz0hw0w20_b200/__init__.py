@@ -198,7 +198,8 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY,
             "prefetch": _lib.OPT_PREFETCH, "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
             "poll_one": _lib.OPT_POLL_ONE,
-            "warp_split_last": _lib.OPT_WARP_SPLIT_LAST}
+            "warp_split_last": _lib.OPT_WARP_SPLIT_LAST,
+            "host_io": _lib.OPT_HOST_IO}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

@@ -58,6 +58,7 @@ OPT_PREFETCH = 18
 OPT_POLL_GAP_NS = 19
 OPT_POLL_ONE = 20
 OPT_WARP_SPLIT_LAST = 22
+OPT_HOST_IO = 23
 ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
 ENGINE_HYBRID, ENGINE_CHAIN = 6, 7
 PROTO_FLAGS, PROTO_FUSED = 0, 1

@@ -87,6 +87,7 @@ struct sptrsv_handle_s {
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
+    int host_io = 2;        // sptrsv_solve_host on LEAN with pinned buffers (SPTRSV_OPT_HOST_IO)
     int split_last = 2;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
@@ -948,19 +949,24 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         }
     }
     cudaStream_t s = (cudaStream_t)stream;
-    // Pinned host buffers and the LEAN engine: no separate copies.  The kernel reads b straight
-    // from host memory (UVA mapping, each warp one coalesced 256-byte PCIe read) and every CTA
-    // writes its finished rows of x to host memory as one contiguous block, so both transfers
-    // overlap the solve instead of bracketing it.  x still lands in device memory first (the
-    // FLAGS protocol reads it back; FUSED consumers read the records).
+    // Pinned host buffers and the LEAN engine: every CTA writes its finished rows of x to host
+    // memory as one contiguous block (UVA mapping), so the device->host transfer overlaps the
+    // solve instead of following it; x still lands in device memory first (the FLAGS protocol
+    // reads it back; FUSED consumers read the records).  b is copied in by DMA first: reading
+    // it in-kernel over PCIe (HOST_IO bit 0) measured slower (c2: 469 us vs 330 us per step,
+    // tools/e2e_probe.py; staged copies both ways 357 us).
     cudaPointerAttributes ab, ax;
     const bool pinned = cudaPointerGetAttributes(&ab, b_host) == cudaSuccess &&
                         cudaPointerGetAttributes(&ax, x_host) == cudaSuccess && ab.type == cudaMemoryTypeHost &&
                         ax.type == cudaMemoryTypeHost && ab.devicePointer && ax.devicePointer;
     (void)cudaGetLastError();
-    if (pinned && !h->variant && resolve_engine(h) == 3 && h->plan == PLAN_THREAD) {
-        int rc = solve_impl(h, (const double *)ab.devicePointer, h->ws.x_stage, (double *)ax.devicePointer, stream);
+    const int io = h->host_io;  // bit 0: b read in-kernel over PCIe, bit 1: x written per CTA
+    if (pinned && io && !h->variant && resolve_engine(h) == 3 && h->plan == PLAN_THREAD) {
+        if (!(io & 1)) CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
+        int rc = solve_impl(h, (io & 1) ? (const double *)ab.devicePointer : h->ws.b_stage, h->ws.x_stage,
+                            (io & 2) ? (double *)ax.devicePointer : nullptr, stream);
         if (rc) return rc;
+        if (!(io & 2)) CK(cudaMemcpyAsync(x_host, h->ws.x_stage, bytes, cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         return SPTRSV_OK;
     }
@@ -1089,6 +1095,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->poll_one = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_HOST_IO:
+            if (value < 0 || value > 3) return SPTRSV_ERR_INVALID_ARG;
+            h->host_io = (int)value;
+            return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST:
             if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
             h->split_last = (int)value;
@@ -1122,6 +1132,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_POLL_GAP_NS: *value = h->poll_gap; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST: *value = h->split_last; return SPTRSV_OK;
+        case SPTRSV_OPT_HOST_IO: *value = h->host_io; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }

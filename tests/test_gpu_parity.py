@@ -201,16 +201,16 @@ def test_many_solves_on_side_stream_and_graph_capture(cap, proto, engine):
 
 
 @pytest.mark.parametrize("proto", PROTOS)
-@pytest.mark.parametrize("engine", [5, 0, 7])
+@pytest.mark.parametrize("engine,host_io", [(5, 0), (5, 1), (5, 2), (5, 3), (0, 2), (7, 2)])
 @pytest.mark.parametrize("pinned", [True, False])
-def test_solve_host_e2e(cap, proto, engine, pinned):
+def test_solve_host_e2e(cap, proto, engine, host_io, pinned):
     """sptrsv_solve_host from pinned host buffers (LEAN: b read over PCIe inside the kernel, x
     written per CTA to host memory -- no staging copies) and from pageable numpy buffers
     (staged copies), every engine family, ragged sizes, repeated solves on one handle."""
     for s in (synth.gen_c2(n=100_000), synth.gen_random_lower(1000, 3, seed=4), synth.gen_random_lower(33, 2, seed=5)):
         ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
         rp, ci, v, _ = dev_csr(s)
-        with cap.analyse(rp, ci, v, protocol=proto, engine=engine) as h:
+        with cap.analyse(rp, ci, v, protocol=proto, engine=engine, host_io=host_io) as h:
             if pinned:
                 bh = torch.from_numpy(s.b).pin_memory()
                 xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
@@ -221,7 +221,7 @@ def test_solve_host_e2e(cap, proto, engine, pinned):
                 (xh.fill_ if pinned else xh.fill)(float("nan"))
                 h.solve_host(bh, xh)
                 got = xh.numpy() if pinned else xh
-                assert np.array_equal(got, ref), (s.name, proto, engine, pinned)
+                assert np.array_equal(got, ref), (s.name, proto, engine, host_io, pinned)
 
 
 @pytest.mark.parametrize("flags", [1, 2, 3])
