@@ -117,10 +117,12 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_POLL_ONE = 20,      /* LEAN: 1 = poll one dependency per lane per pass
                                       (default 0: the next two, DESIGN G21)                 */
     SPTRSV_OPT_HOST_IO = 23,       /* sptrsv_solve_host with pinned buffers on LEAN: bit 0 =
-                                      the kernel reads b over PCIe, bit 1 = each CTA writes
-                                      its rows of x to host memory; a cleared bit uses a
-                                      cudaMemcpyAsync before / after the solve instead.
-                                      Default 2 (b by DMA, x written per CTA)              */
+                                      b copied in chunks on a second stream, each CTA waiting
+                                      for its own chunk only (needs cuStreamWriteValue32);
+                                      bit 1 = each CTA writes its rows of x to host memory;
+                                      a cleared bit uses one cudaMemcpyAsync before / after
+                                      the solve instead.  Bits 8..15: log2 of the chunk in
+                                      rows (8..24; 0 = about four chunks).  Default 3      */
     SPTRSV_OPT_WARP_SPLIT_LAST = 22,/* warp-level rows: 2 (default) = the row's last
                                       off-diagonal (its nearest dependency) is added after
                                       the lane-strided tree by lane 0 alone, which polls it
@@ -246,10 +248,12 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
  * sptrsv_solve_host -- end-to-end convenience from host buffers; synchronises
  * `stream` before returning.  b_host/x_host: host double[n].
  *   - Both pinned (page-locked, UVA-mapped; e.g. cudaHostAlloc or torch
- *     pin_memory) and the handle runs LEAN: b is copied to device staging,
- *     and every CTA writes its finished rows of x to x_host as one contiguous
- *     block, so the device->host transfer overlaps the solve (x also lands in
- *     handle-owned device staging).  SPTRSV_OPT_HOST_IO selects the variants.
+ *     pin_memory) and the handle runs LEAN: b is copied to device staging in
+ *     about four chunks on a handle-owned second stream, each CTA of the solve
+ *     waiting only for the chunk of its own rows, and every CTA writes its
+ *     finished rows of x to x_host as one contiguous block -- both transfers
+ *     overlap the solve (x also lands in handle-owned device staging).
+ *     SPTRSV_OPT_HOST_IO selects the variants.
  *   - Otherwise: b is copied to handle-owned device staging, solved, and x is
  *     copied back (cudaMemcpyAsync; pageable buffers are staged by the driver).
  */

@@ -143,11 +143,12 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     if (UPPER) i = p.n - 1 - i;
     int rs = 0, re = 1;
     double bi = 0.0;
+    const bool bgate = p.bflag != nullptr;  // b still arriving in chunks (sptrsv_solve_host)
     if (i >= 0 && i < p.n) {
         if (p.trace) p.trace[3 * (size_t)p.n + 3 + i] = globaltimer_ns();  // CTA entry
         rs = ld_stream_i32(p.rowptr + i, pol);
         re = ld_stream_i32(p.rowptr + i + 1, pol);
-        bi = ld_stream_f64(p.b + i, pol);
+        if (!bgate) bi = ld_stream_f64(p.b + i, pol);
     }
     // ---- L2 bulk prefetch of the block pf_dist logical blocks ahead (speculatively
     // blockIdx.x + pf_dist): its bounds load overlaps the ticket, the copy is issued after it
@@ -168,6 +169,23 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
             atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
         }
         cta_ticket(p, s_blk, s_epoch);
+        if (bgate) {  // wait until the b chunks of this CTA's (physical) rows have landed
+            const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
+            if (lr0 < lr1) {
+                const int a = UPPER ? p.n - lr1 : lr0, e = UPPER ? p.n - lr0 : lr1;
+                uint32_t spins = 0;
+                for (int c = a >> p.bshift; c <= (e - 1) >> p.bshift; ++c) {
+                    while ((int)(ld_acquire_u32(p.bflag + c) - p.bseq) < 0) {
+                        nanosleep_ns(128);
+                        if (p.spin_limit && ++spins >= p.spin_limit) {  // watchdog, as in the solve loops
+                            atomicCAS(&p.st->error.v, 0u, 1u);
+                            st_relaxed_u32(&p.st->abort.v, 1u);
+                            break;
+                        }
+                    }
+                }
+            }
+        }
     }
     __syncthreads();
     const uint32_t epoch = s_epoch;
@@ -181,6 +199,8 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
             re = ld_stream_i32(p.rowptr + i + 1, pol);
             bi = ld_stream_f64(p.b + i, pol);
         }
+    } else if (bgate && i >= 0 && i < p.n) {
+        bi = ld_stream_f64(p.b + i, pol);
     }
     const bool act = i >= 0 && i < p.n;
     lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);

@@ -4,6 +4,7 @@
 // libsptrsv.so for sm_100a (see paper_conf_icpp_suz0hw0w20_b200/build.py).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <chrono>
 #include <cstdint>
 #include <cstdlib>
@@ -44,7 +45,29 @@ struct Workspace {
     unsigned long long *mrec = nullptr;  // multi-RHS: n * mcap records (FUSED)
     int64_t mcap = 0;              // right-hand sides the multi buffers hold
     double *x_stage = nullptr;     // n (solve_host, lazy)
+    uint32_t *bflag = nullptr;     // solve_host: per-chunk "b has landed" words (lazy)
+    int32_t bflag_n = 0;
+    cudaStream_t s2 = nullptr;     // solve_host: copy stream for the chunked b
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr;
 };
+
+// cuStreamWriteValue32 through the runtime's driver entry point (no link-time libcuda
+// dependency: the library must load on machines without a GPU driver).
+typedef int (*write_value32_fn)(cudaStream_t, unsigned long long, uint32_t, unsigned int);
+write_value32_fn write_value32() {
+    static write_value32_fn fn = [] {
+        void *f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &f, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess) {
+            (void)cudaGetLastError();
+            f = nullptr;
+        }
+        return (write_value32_fn)f;
+    }();
+    return fn;
+}
+constexpr int kBChunkShift = 16;  // solve_host: smallest b chunk, 2^16 rows (512 KB)
 
 }  // namespace
 
@@ -87,7 +110,8 @@ struct sptrsv_handle_s {
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
-    int host_io = 2;        // sptrsv_solve_host on LEAN with pinned buffers (SPTRSV_OPT_HOST_IO)
+    int host_io = 3;        // sptrsv_solve_host on LEAN with pinned buffers (SPTRSV_OPT_HOST_IO)
+    uint32_t host_seq = 0;  // solve_host: sequence number of the chunked-b flags
     int split_last = 2;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
@@ -223,6 +247,10 @@ void free_ws(Workspace &w) {
     cudaFree(w.mflags);
     cudaFree(w.mrec);
     cudaFree(w.x_stage);
+    cudaFree(w.bflag);
+    if (w.s2) cudaStreamDestroy(w.s2);
+    if (w.ev_a) cudaEventDestroy(w.ev_a);
+    if (w.ev_b) cudaEventDestroy(w.ev_b);
     w = Workspace();
 }
 
@@ -764,14 +792,16 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
 
 }  // namespace
 
-static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream);
+static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream,
+                      const uint32_t *bflag = nullptr, uint32_t bseq = 0, int bshift = kBChunkShift);
 
 int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream) {
     return solve_impl(h, b, x, nullptr, stream);
 }
 
 // x_host (LEAN only, from sptrsv_solve_host): device-mapped pinned host copy target of x
-static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream) {
+static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream,
+                      const uint32_t *bflag, uint32_t bseq, int bshift) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!b || !x || b == x) return SPTRSV_ERR_INVALID_ARG;
@@ -814,6 +844,9 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.poll_one = h->poll_one;
     p.split_last = h->split_last;
     p.x_host = x_host;
+    p.bflag = bflag;
+    p.bseq = bseq;
+    p.bshift = bshift;
     p.trace = h->trace;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = L.grid;
@@ -949,23 +982,74 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         }
     }
     cudaStream_t s = (cudaStream_t)stream;
-    // Pinned host buffers and the LEAN engine: every CTA writes its finished rows of x to host
-    // memory as one contiguous block (UVA mapping), so the device->host transfer overlaps the
-    // solve instead of following it; x still lands in device memory first (the FLAGS protocol
-    // reads it back; FUSED consumers read the records).  b is copied in by DMA first: reading
-    // it in-kernel over PCIe (HOST_IO bit 0) measured slower (c2: 469 us vs 330 us per step,
-    // tools/e2e_probe.py; staged copies both ways 357 us).
+    // Pinned host buffers and the LEAN engine: b is copied in by DMA in ~4 chunks on a second
+    // stream and each CTA of the solve waits only for the chunk holding its own rows, so the
+    // host->device copy overlaps the solve; every CTA writes its finished rows of x to host memory
+    // as one contiguous block (UVA mapping), so the device->host transfer overlaps it too.  x still
+    // lands in device memory (the FLAGS protocol reads it back; FUSED consumers read records).
+    // c2, tools/e2e_probe.py: 270 us per step, against 357 us staged both ways and 330 us with
+    // only the x side overlapped; reading b in-kernel over PCIe instead measured 469 us.
     cudaPointerAttributes ab, ax;
     const bool pinned = cudaPointerGetAttributes(&ab, b_host) == cudaSuccess &&
                         cudaPointerGetAttributes(&ax, x_host) == cudaSuccess && ab.type == cudaMemoryTypeHost &&
                         ax.type == cudaMemoryTypeHost && ab.devicePointer && ax.devicePointer;
     (void)cudaGetLastError();
-    const int io = h->host_io;  // bit 0: b read in-kernel over PCIe, bit 1: x written per CTA
+    int io = h->host_io & 3;  // bit 0: b in chunks overlapped with the solve, bit 1: x written per CTA
+    // b chunk = 2^sh rows: the option's bits 8.., else about four chunks (each copy + flag write costs
+    // a few us of DMA setup; measured on c2: 2^15-row chunks 549 us, 2^16 394, 2^18 270, 2^20 324)
+    int sh = h->host_io >> 8;
+    if (!sh) {
+        sh = kBChunkShift;
+        while (sh < 24 && ((long long)4 << sh) < (long long)h->n) ++sh;
+    }
+    if ((io & 1) && !write_value32()) io &= ~1;
     if (pinned && io && !h->variant && resolve_engine(h) == 3 && h->plan == PLAN_THREAD) {
-        if (!(io & 1)) CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
-        int rc = solve_impl(h, (io & 1) ? (const double *)ab.devicePointer : h->ws.b_stage, h->ws.x_stage,
-                            (io & 2) ? (double *)ax.devicePointer : nullptr, stream);
+        const uint32_t *bflag = nullptr;
+        uint32_t seq = 0;
+        if (io & 1) {
+            // b in chunks of 2^16 rows on a second stream; after each chunk a stream memory op sets
+            // its flag to this call's sequence number, and a CTA of the solve waits for the flags
+            // of its own rows only -- the copy and the solve overlap, chunk by chunk
+            const int nch = (int)((h->n + (1 << sh) - 1) >> sh);
+            Workspace &w = h->ws;
+            if (w.bflag_n < nch) {
+                cudaFree(w.bflag);
+                w.bflag = nullptr;
+                w.bflag_n = 0;
+                if (cudaMalloc(&w.bflag, sizeof(uint32_t) * nch) != cudaSuccess) {
+                    (void)cudaGetLastError();
+                    return SPTRSV_ERR_ALLOC;
+                }
+                CK(cudaMemset(w.bflag, 0, sizeof(uint32_t) * nch));
+                w.bflag_n = nch;
+                h->host_seq = 0;
+            }
+            if (!w.s2) CK(cudaStreamCreateWithFlags(&w.s2, cudaStreamNonBlocking));
+            if (!w.ev_a) CK(cudaEventCreateWithFlags(&w.ev_a, cudaEventDisableTiming));
+            if (!w.ev_b) CK(cudaEventCreateWithFlags(&w.ev_b, cudaEventDisableTiming));
+            seq = ++h->host_seq;
+            if (seq == 0) seq = ++h->host_seq;  // 0 is the reset value (wrap-safe compare in the kernel)
+            CK(cudaEventRecord(w.ev_a, s));  // the copies start after the stream's earlier work
+            CK(cudaStreamWaitEvent(w.s2, w.ev_a, 0));
+            for (int c = 0; c < nch; ++c) {
+                const size_t r0 = (size_t)c << sh;
+                const size_t rows = std::min((size_t)h->n - r0, (size_t)1 << sh);
+                CK(cudaMemcpyAsync(w.b_stage + r0, b_host + r0, rows * sizeof(double), cudaMemcpyHostToDevice,
+                                   w.s2));
+                if (write_value32()(w.s2, (unsigned long long)(uintptr_t)(w.bflag + c), seq, 0) != 0)
+                    return SPTRSV_ERR_CUDA;
+            }
+            bflag = w.bflag;
+        } else {
+            CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
+        }
+        int rc = solve_impl(h, h->ws.b_stage, h->ws.x_stage, (io & 2) ? (double *)ax.devicePointer : nullptr, stream,
+                            bflag, seq, sh);
         if (rc) return rc;
+        if (io & 1) {  // the stream also orders after the copies (they finish before the solve does)
+            CK(cudaEventRecord(h->ws.ev_b, h->ws.s2));
+            CK(cudaStreamWaitEvent(s, h->ws.ev_b, 0));
+        }
         if (!(io & 2)) CK(cudaMemcpyAsync(x_host, h->ws.x_stage, bytes, cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         return SPTRSV_OK;
@@ -1095,8 +1179,9 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->poll_one = (int)value;
             return SPTRSV_OK;
-        case SPTRSV_OPT_HOST_IO:
-            if (value < 0 || value > 3) return SPTRSV_ERR_INVALID_ARG;
+        case SPTRSV_OPT_HOST_IO:  // bits 0-1 mode, bits 8.. log2 of the b chunk in rows (0 = 16)
+            if ((value & ~0xFF03ll) || ((value >> 8) && ((value >> 8) < 8 || (value >> 8) > 24)))
+                return SPTRSV_ERR_INVALID_ARG;
             h->host_io = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST:

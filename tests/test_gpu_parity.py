@@ -224,22 +224,31 @@ def test_solve_host_e2e(cap, proto, engine, host_io, pinned):
                 assert np.array_equal(got, ref), (s.name, proto, engine, host_io, pinned)
 
 
+@pytest.mark.parametrize("host_io", [2, 3])
 @pytest.mark.parametrize("flags", [1, 2, 3])
-def test_solve_host_e2e_f4_lean(cap, flags):
+def test_solve_host_e2e_f4_lean(cap, flags, host_io):
     """The pinned path for upper / unit handles on LEAN (physical row ranges of reversed CTAs)."""
-    s = synth.gen_c2(n=70_000)  # 70000 % 256 = 112: a ragged last CTA
+    s = synth.gen_c2(n=300_000)  # 300000 % 256 = 224: a ragged last CTA; 5 b chunks of 2^16 rows
     if flags & 1:
         s = synth.to_upper(s)
     if flags & 2:
         s = synth.to_unit(s)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     rp, ci, v, _ = dev_csr(s)
-    with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2)) as h:
+    with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2), host_io=host_io) as h:
         assert h.info()["engine"] == 3
         bh = torch.from_numpy(s.b).pin_memory()
         xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
+        for _ in range(2):
+            h.solve_host(bh, xh)
+            assert np.array_equal(xh.numpy(), ref)
+            xh.fill_(float("nan"))
+        # interleaved with device-side solves on the same handle (shared epoch / ticket state)
+        b = torch.from_numpy(s.b).cuda()
+        x = torch.full_like(b, float("nan"))
+        h.solve(b, x)
         h.solve_host(bh, xh)
-        assert np.array_equal(xh.numpy(), ref)
+        assert np.array_equal(x.cpu().numpy(), ref) and np.array_equal(xh.numpy(), ref)
 
 
 def test_empty_matrix(cap):
