@@ -1,5 +1,5 @@
 """Small solves through every engine / form for compute-sanitizer (memcheck / racecheck-free kernels):
-usage: compute-sanitizer --tool memcheck python tools/memcheck_small.py"""
+usage: compute-sanitizer --tool memcheck python tests/memcheck_driver.py (a test harness: it runs the oracle)"""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch

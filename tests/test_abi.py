@@ -70,3 +70,14 @@ def test_product_package_never_imports_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 txt = open(os.path.join(dp, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt and "oracle.c" not in txt, f
+
+
+def test_only_tests_smoke_and_bench_touch_the_oracle():
+    """The oracle is test infrastructure: outside tests/, only __graft_entry__.smoke() and
+    bench.py's cpu_baseline / reference legs may import it (tools/, synth/ and include/ never do)."""
+    for sub in ("tools", "synth", "include"):
+        for dp, _, fs in os.walk(os.path.join(ROOT, sub)):
+            for f in fs:
+                if f.endswith((".py", ".cu", ".cuh", ".h", ".c")):
+                    txt = open(os.path.join(dp, f)).read()
+                    assert "import oracle" not in txt and "from oracle" not in txt, os.path.join(dp, f)

@@ -3,7 +3,7 @@ usage: python tools/trace.py CONFIG [key=value ...]"""
 import os, sys, json
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
-import synth, oracle
+import synth
 import paper_conf_icpp_suz0hw0w20_b200 as cap
 
 name = sys.argv[1]
@@ -26,7 +26,7 @@ if tt.size >= 3 * s.n + 3 and tt[3 * s.n + 1] > 0:
 t = tt[: s.n] - t0
 seen = np.where(tt[s.n:2 * s.n] > 0, tt[s.n:2 * s.n] - t0, -1)
 start = np.where(tt[2 * s.n:3 * s.n] > 0, tt[2 * s.n:3 * s.n] - t0, -1)
-lv = oracle.levels_dp(s.rowptr, s.colidx)
+lv = h.levels()[0].cpu().numpy()  # the GPU level diagnostic (tools/ never run the oracle)
 nl = int(lv.max()) + 1
 # completion time of each level = max publish time of its rows
 lvl_done = np.full(nl, 0, np.int64)
