@@ -60,7 +60,14 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
     const int warps = blockDim.x >> 5;
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
-    if (threadIdx.x == 0) cta_ticket(p, s_blk, s_epoch);
+    if (threadIdx.x == 0) {
+        cta_ticket(p, s_blk, s_epoch);
+        if (p.bflag) {  // sptrsv_solve_host: this CTA's b chunks (physical rows)
+            const int lr0 = (int)s_blk * (int)(blockDim.x >> 5) * 32 * K;
+            const int lr1 = min(p.n, lr0 + (int)(blockDim.x >> 5) * 32 * K);
+            wait_b_chunks(p, UPPER ? p.n - lr1 : lr0, UPPER ? p.n - lr0 : lr1);
+        }
+    }
     __syncthreads();
     const uint32_t epoch = s_epoch;
     const int r0 = ((int)s_blk * warps + warp) * RT;
@@ -326,7 +333,16 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 }
             }
         }
-        if (s >= rows) break;
+        if (s >= rows) {
+            if (p.x_host) {  // sptrsv_solve_host: the warp's rows to pinned host memory, coalesced
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    const int t = lane + 32 * k;
+                    if (t < rows) p.x_host[phys(r0 + t)] = xm[k];
+                }
+            }
+            break;
+        }
         if (s > s0) prog = true;
         if (__ballot_sync(FULL, prog)) {
             backoff = p.backoff_min;

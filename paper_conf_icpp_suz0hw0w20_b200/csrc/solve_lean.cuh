@@ -171,20 +171,7 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         cta_ticket(p, s_blk, s_epoch);
         if (bgate) {  // wait until the b chunks of this CTA's (physical) rows have landed
             const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
-            if (lr0 < lr1) {
-                const int a = UPPER ? p.n - lr1 : lr0, e = UPPER ? p.n - lr0 : lr1;
-                uint32_t spins = 0;
-                for (int c = a >> p.bshift; c <= (e - 1) >> p.bshift; ++c) {
-                    while ((int)(ld_acquire_u32(p.bflag + c) - p.bseq) < 0) {
-                        nanosleep_ns(128);
-                        if (p.spin_limit && ++spins >= p.spin_limit) {  // watchdog, as in the solve loops
-                            atomicCAS(&p.st->error.v, 0u, 1u);
-                            st_relaxed_u32(&p.st->abort.v, 1u);
-                            break;
-                        }
-                    }
-                }
-            }
+            wait_b_chunks(p, UPPER ? p.n - lr1 : lr0, UPPER ? p.n - lr0 : lr1);
         }
     }
     __syncthreads();

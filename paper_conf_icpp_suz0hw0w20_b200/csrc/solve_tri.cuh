@@ -52,7 +52,23 @@ template <int PROTO, bool UPPER, bool UNIT, int PLAN>
 __global__ void __launch_bounds__(kTriWarpCta) k_solve_tri_warp(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (threadIdx.x == 0) cta_ticket(p, s_blk, s_epoch);
+    if (threadIdx.x == 0) {
+        cta_ticket(p, s_blk, s_epoch);
+        if (p.bflag) {  // sptrsv_solve_host: the b chunks of this CTA's tasks' (physical) rows
+            int lo = p.n, hi = 0;  // logical row range of the CTA's tasks
+            for (int t = (int)s_blk * (kTriWarpCta / 32); t < min(p.n_tasks, ((int)s_blk + 1) * (kTriWarpCta / 32)); ++t) {
+                int r0 = t, r1 = t + 1;
+                if (PLAN == PLAN_LIST) {
+                    const int v = p.tasks[t];
+                    r0 = v >= 0 ? v : ~v;
+                    r1 = v >= 0 ? min(p.n, v + 32) : r0 + 1;
+                }
+                lo = min(lo, r0);
+                hi = max(hi, r1);
+            }
+            if (lo < hi) wait_b_chunks(p, UPPER ? p.n - hi : lo, UPPER ? p.n - lo : hi);
+        }
+    }
     __syncthreads();
     const uint32_t epoch = s_epoch;
     const int task = (int)s_blk * (kTriWarpCta / 32) + warp;

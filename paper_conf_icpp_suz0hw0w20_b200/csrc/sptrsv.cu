@@ -982,11 +982,12 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         }
     }
     cudaStream_t s = (cudaStream_t)stream;
-    // Pinned host buffers and the LEAN engine: b is copied in by DMA in ~4 chunks on a second
+    // Pinned host buffers and the LEAN / CHAIN / HYBRID engines: b is copied in by DMA in ~4 chunks on a second
     // stream and each CTA of the solve waits only for the chunk holding its own rows, so the
-    // host->device copy overlaps the solve; every CTA writes its finished rows of x to host memory
-    // as one contiguous block (UVA mapping), so the device->host transfer overlaps it too.  x still
-    // lands in device memory (the FLAGS protocol reads it back; FUSED consumers read records).
+    // host->device copy overlaps the solve; every LEAN CTA / CHAIN warp writes its finished rows of
+    // x to host memory as one contiguous block (UVA mapping), so the device->host transfer overlaps
+    // it too (HYBRID copies x back after the solve).  x still lands in device memory (the FLAGS
+    // protocol reads it back; FUSED consumers read records).
     // c2, tools/e2e_probe.py: 270 us per step, against 357 us staged both ways and 330 us with
     // only the x side overlapped; reading b in-kernel over PCIe instead measured 469 us.
     cudaPointerAttributes ab, ax;
@@ -1003,7 +1004,11 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         while (sh < 24 && ((long long)4 << sh) < (long long)h->n) ++sh;
     }
     if ((io & 1) && !write_value32()) io &= ~1;
-    if (pinned && io && !h->variant && resolve_engine(h) == 3 && h->plan == PLAN_THREAD) {
+    // engines that take the chunked b (wait_b_chunks) and, for LEAN / CHAIN, write x per CTA / warp
+    const int eng = h->variant ? -1 : resolve_engine(h);
+    const bool gated = (eng == 3 || eng == 7) ? h->plan == PLAN_THREAD : eng == 6;
+    if (!(eng == 3 || eng == 7)) io &= ~2;
+    if (pinned && io && gated) {
         const uint32_t *bflag = nullptr;
         uint32_t seq = 0;
         if (io & 1) {

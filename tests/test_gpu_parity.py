@@ -201,7 +201,7 @@ def test_many_solves_on_side_stream_and_graph_capture(cap, proto, engine):
 
 
 @pytest.mark.parametrize("proto", PROTOS)
-@pytest.mark.parametrize("engine,host_io", [(5, 0), (5, 1), (5, 2), (5, 3), (0, 2), (7, 2)])
+@pytest.mark.parametrize("engine,host_io", [(5, 0), (5, 1), (5, 2), (5, 3), (0, 2), (7, 2), (7, 1), (7, 3)])
 @pytest.mark.parametrize("pinned", [True, False])
 def test_solve_host_e2e(cap, proto, engine, host_io, pinned):
     """sptrsv_solve_host from pinned host buffers (LEAN: b read over PCIe inside the kernel, x
@@ -222,6 +222,37 @@ def test_solve_host_e2e(cap, proto, engine, host_io, pinned):
                 h.solve_host(bh, xh)
                 got = xh.numpy() if pinned else xh
                 assert np.array_equal(got, ref), (s.name, proto, engine, host_io, pinned)
+
+
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("host_io", [0, 1, 3])
+@pytest.mark.parametrize("case", ["grid", "grid_upper", "c4", "c4_unit_upper", "mixed"])
+def test_solve_host_e2e_chain_hybrid(cap, proto, host_io, case):
+    """sptrsv_solve_host on CHAIN (grids, upper grids) and HYBRID (warp rows, f4 warp rows, mixed
+    plans): chunked b gated per CTA, x written per CHAIN warp -- element by element vs the oracle."""
+    flags = {"grid_upper": 1, "c4_unit_upper": 3}.get(case, 0)
+    s = {"grid": lambda: synth.gen_grid(600), "grid_upper": lambda: synth.gen_grid(600),
+         "c4": lambda: synth.gen_c4(n=150_000, nlevels=300), "c4_unit_upper": lambda: synth.gen_c4(n=150_000, nlevels=300),
+         "mixed": lambda: synth.gen_random_lower(150_001, 20, seed=9)}[case]()
+    if flags & 1:
+        s = synth.to_upper(s)
+    if flags & 2:
+        s = synth.to_unit(s)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags) if flags else oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, _ = dev_csr(s)
+    with cap.analyse(rp, ci, v, protocol=proto, host_io=host_io, upper=bool(flags & 1), unit_diag=bool(flags & 2)) as h:
+        eng = h.info()["engine"]
+        assert eng == (7 if "grid" in case else 6), (case, eng)
+        bh = torch.from_numpy(s.b).pin_memory()
+        xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
+        for _ in range(2):
+            h.solve_host(bh, xh)
+            got = xh.numpy()
+            if eng == 7:
+                assert np.array_equal(got, ref), case
+            else:
+                assert np.max(np.abs(got - ref) / np.abs(ref)) <= TOL, case
+            xh.fill_(float("nan"))
 
 
 @pytest.mark.parametrize("host_io", [2, 3])
