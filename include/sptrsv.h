@@ -208,11 +208,11 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
  * Upper rows are taken in reverse order behind the same start ticket, so the
  * ticket order is a topological order.  Each row's off-diagonals are summed
  * earliest-solved first: ascending column (lower), descending column (upper).
- * sptrsv_solve, sptrsv_solve_host, sptrsv_get_indegree, sptrsv_check and the
+ * sptrsv_solve, sptrsv_solve_multi (column by column), sptrsv_solve_host,
+ * sptrsv_get_indegree, sptrsv_check and the
  * options work as for lower handles (ENGINE: only 3 LEAN and 7 CHAIN are
  * honoured, for all-thread-level plans);
- * sptrsv_solve_multi, sptrsv_levels and VARIANT != 0 return
- * SPTRSV_ERR_INVALID_ARG.  Thread-level rows are bit-exact with that fp64
+ * sptrsv_levels and VARIANT != 0 return SPTRSV_ERR_INVALID_ARG.  Thread-level rows are bit-exact with that fp64
  * substitution (one rounded multiply and add each); warp rows are within the
  * warp-mode bound, as for lower handles.  sptrsv_info.engine: 3 LEAN, 6 warp.
  */
@@ -239,7 +239,10 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
  * 1 <= nrhs <= 32, ldb, ldx >= nrhs; B and X device, must not alias.  Same
  * protocol option and options as sptrsv_solve; asynchronous, one launch.
  * Each component (i, r) has its own ready word, so the handle keeps
- * n * nrhs of them (allocated on first use).
+ * n * nrhs of them (allocated on first use).  Handles whose solve runs the
+ * CHAIN engine, and upper / unit-diagonal handles, solve column by column
+ * instead (gather, sptrsv_solve, scatter per column, on `stream`): their
+ * in-register chains beat one shared hop per row.
  */
 int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nrhs, int64_t ldb, int64_t ldx,
                        sptrsv_stream_t stream);

@@ -562,6 +562,21 @@ def test_multi_rhs(cap, nrhs, proto):
             assert torch.isnan(Xp[:, nrhs:]).all()
 
 
+@pytest.mark.parametrize("nrhs", [1, 5, 8])
+def test_multi_rhs_chain_plans_by_column(cap, nrhs):
+    """Plans that run CHAIN (grids, chains) solve multi-RHS column by column: bit-exact per column."""
+    rng = np.random.default_rng(100 + nrhs)
+    for s in (synth.gen_grid(300), synth.gen_chain(20_000, closed_form=False)):
+        B = rng.uniform(-1, 1, (s.n, nrhs))
+        ref = oracle.solve_multi(s.rowptr, s.colidx, s.val, B)
+        rp, ci, v, _ = dev_csr(s)
+        with cap.analyse(rp, ci, v) as h:
+            assert h.info()["engine"] == 7
+            X = h.solve_multi(torch.from_numpy(B).cuda())
+            h.check()
+            assert np.array_equal(X.cpu().numpy(), ref), s.name
+
+
 @pytest.mark.parametrize("variant", [3, 4, 5])
 def test_paper_variants(cap, variant):
     """The paper's Alg.3 / Alg.4 / Alg.5 kernels (ablation): same result -- thread-level ones
