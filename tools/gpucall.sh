@@ -1,3 +1,4 @@
 mkdir -p gpurun_out
-timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29511 bench.py --gpus 1 --steps 10 --warmup 3 > gpurun_out/torchrun44.json 2> gpurun_out/torchrun44.err
-timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29512 bench.py --gpus 1 --steps 3 --warmup 3 --impl reference > gpurun_out/torchrun44_ref.json 2> gpurun_out/torchrun44_ref.err
+python tools/optsweep.py c4 '[{"warp_split_last":2}, {"warp_split_last":3}]' 10 > gpurun_out/sweep45_c4.txt 2>&1
+python tools/optsweep.py lev:200000:400 '[{"warp_split_last":2,"mode":2}, {"warp_split_last":3,"mode":2}]' 10 > gpurun_out/sweep45_lev.txt 2>&1
+python tools/optsweep.py lev:1000000:1000 '[{"warp_split_last":2,"mode":2}, {"warp_split_last":3,"mode":2}]' 10 > gpurun_out/sweep45_lev2.txt 2>&1
