@@ -311,6 +311,37 @@ def main():
                      "value": round(2.0 * nnz_all * args.steps / ft / 1e9, 3), "unit": UNIT,
                      "ms_per_step": round(ft / args.steps * 1e3, 5)}
 
+    # ---- comparison leg: the same solve without the persisting L2 window over the ready words
+    # (the window keeps the solver's records L2-resident across the flush; CSR, b and x stream cold)
+    nowin_leg = None
+    if not args.no_flags_leg and not args.profile and opts.get("l2_window", 1) != 0:
+        for h in handles:
+            h.set_option(cap.OPT_L2_WINDOW, 0)
+        for i in range(args.warmup):
+            flush.zero_()
+            step(i)
+        ev3 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            flush.zero_()
+            ev3[i][0].record(stream)
+            step(i)
+            ev3[i][1].record(stream)
+        torch.cuda.synchronize()
+        for h in handles:
+            h.check(stream)
+            h.set_option(cap.OPT_L2_WINDOW, opts.get("l2_window", 1))
+        wt = float(np.sum([a.elapsed_time(b) for a, b in ev3])) * 1e-3
+        if dist:
+            t = torch.tensor([wt], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            wt = float(t.item())
+        nowin_leg = {"what": "same solve, no persisting L2 window over the ready words (SPTRSV_OPT_L2_WINDOW=0)",
+                     "value": round(2.0 * nnz_all * args.steps / wt / 1e9, 3), "unit": UNIT,
+                     "ms_per_step": round(wt / args.steps * 1e3, 5)}
+
     # ---- multi-RHS leg: sptrsv_solve_multi with nrhs right-hand sides, same timing rules
     multi_leg = None
     if args.nrhs > 0 and not args.profile:
@@ -479,12 +510,16 @@ def main():
                                   7: "chain (in-warp shuffle chain)"}.get(info["engine"], str(info["engine"])),
                        "cta_threads": info["cta_threads"], "rows_per_lane": info["rows_per_lane"],
                        "analyse_ms": round(info["analyse_ms"], 3),
-                       "l2": "flushed between timed steps (256 MiB write, outside the per-step events)",
+                       "l2": "flushed between timed steps (256 MiB write, outside the per-step events): CSR, b and "
+                             "x are read / written cold; the solver's ready words (16-B records per row) sit in a "
+                             "persisting L2 access-policy window (north_star) and survive the flush -- see "
+                             "no_l2_window_leg",
                        "parallelism": f"replicas x{world}" if args.config != "c5" else f"systems sharded over {world}",
                        "options": opts},
             "protocol": {1: "fused (epoch-tagged 16-byte value records, no fences)",
                          0: "flags (st.release.gpu / ld.acquire.gpu)"}[opts.get("protocol", 1)],
             "flags_protocol_leg": flags_leg,
+            "no_l2_window_leg": nowin_leg,
             "multi_rhs_leg": multi_leg,
             "triangular_forms_leg": tri_leg,
             "roofline": roof,

@@ -65,7 +65,11 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_BACKOFF_MIN_NS = 4, /* __nanosleep after a pass where no lane progressed     */
     SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
     SPTRSV_OPT_SPIN_LIMIT = 6,     /* watchdog: idle passes per warp before TIMEOUT (0=off) */
-    SPTRSV_OPT_L2_WINDOW = 7,      /* 1: cudaAccessPolicyWindow persisting over the flags   */
+    SPTRSV_OPT_L2_WINDOW = 7,      /* 1 (default): a persisting cudaAccessPolicyWindow over
+                                      the ready words (FLAGS: flags, FUSED: records); the
+                                      device's persisting L2 set-aside is grown to the window
+                                      (up to persistingL2CacheMaxSize) at the first solve.
+                                      0: no window                                         */
     SPTRSV_OPT_STAGE_SMEM = 8,     /* 1 (default): thread-level warps stage their CSR slice
                                       in shared memory with coalesced loads                 */
     SPTRSV_OPT_PROTOCOL = 9,       /* cross-CTA ready protocol: 0 FLAGS = uint32 epoch flags,
