@@ -68,7 +68,8 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_L2_WINDOW = 7,      /* 1 (default): a persisting cudaAccessPolicyWindow over
                                       the ready words (FLAGS: flags, FUSED: records); the
                                       device's persisting L2 set-aside is grown to the window
-                                      (up to persistingL2CacheMaxSize) at the first solve.
+                                      (up to persistingL2CacheMaxSize) at the first solve;
+                                      ready words larger than that run without a window.
                                       0: no window                                         */
     SPTRSV_OPT_STAGE_SMEM = 8,     /* 1 (default): thread-level warps stage their CSR slice
                                       in shared memory with coalesced loads                 */
