@@ -1,10 +1,5 @@
-mkdir -p gpurun_out
-python -c "
-import ctypes, torch
-torch.cuda.init()
-lib = ctypes.CDLL('libcudart.so.12') if False else None
-print(torch.cuda.get_device_properties(0))
-" > gpurun_out/props56.txt 2>&1
-python tools/optsweep.py c3 '[{}, {"l2_window":0}]' 5 > gpurun_out/sweep56_c3.txt 2>&1
-python tools/optsweep.py c2 '[{}, {"l2_window":0}]' 20 > gpurun_out/sweep56_c2.txt 2>&1
-python tools/optsweep.py c4 '[{}]' 10 > gpurun_out/sweep56_c4.txt 2>&1
+mkdir -p gpurun_out/final5
+timeout 1800 python -m pytest tests -m gpu -q > gpurun_out/final5/tests.log 2>&1
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/final5/smoke.log 2>&1
+for c in c2 c1 c3 c4 c5; do timeout 400 python bench.py --config $c > gpurun_out/final5/bench_$c.json 2> gpurun_out/final5/bench_$c.err; done
+timeout 300 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/final5/ref.json 2> gpurun_out/final5/ref.err
