@@ -366,6 +366,8 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
     return sptrsv_analyse_csr_ex(n, rowptr, colidx, val, 0, out);
 }
 
+void size_l2_window(sptrsv_handle_s *h);
+
 int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
                           int32_t tri_flags, sptrsv_handle_t *out) {
     const auto t0 = std::chrono::steady_clock::now();
@@ -463,6 +465,7 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         delete h;
         return rc;
     }
+    size_l2_window(h);
     h->analyse_ms =
         std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
     *out = h;
@@ -507,6 +510,26 @@ int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem,
 // with warp-level rows use the HYBRID engine (2-13% faster than the staged
 // one-shot engine on every warp-plan shape measured, tools/hybrid_probe.py).
 // (Round-1 B200 sweeps.)
+// Size the device's persisting L2 set-aside for the handle's ready-word window (SPTRSV_OPT_L2_WINDOW):
+// grown to the window (up to persistingL2CacheMaxSize); l2_hit = 1 if it holds the whole window,
+// -1 (no window) otherwise -- a partial window (c3's 67 MB of records) left the time unchanged and
+// added DRAM traffic (361.6 vs 314.6 MB per launch).  Host-only, synchronous: called from analyse
+// and set_option so that a first solve inside a stream capture never changes device limits.
+void size_l2_window(sptrsv_handle_s *h) {
+    h->l2_hit = -1.f;
+    if (!h->l2_window || h->n == 0) return;
+    const size_t wbytes = (h->proto == PROTO_FLAGS ? sizeof(uint32_t) : 16) * (size_t)h->n;
+    cudaDeviceProp prop;
+    size_t cur = 0;
+    if (cudaGetDeviceProperties(&prop, h->device) == cudaSuccess &&
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
+        const size_t want = std::min(wbytes, (size_t)prop.persistingL2CacheMaxSize);
+        if (cur < want && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) == cudaSuccess) cur = want;
+        h->l2_hit = cur >= wbytes ? 1.f : -1.f;
+    }
+    (void)cudaGetLastError();
+}
+
 int resolve_engine(const sptrsv_handle_s *h) {
     // stored off-diagonals (unit handles store no diagonal)
     const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;
@@ -867,25 +890,11 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     // every dependent row and re-written every solve; persisting lines are not evicted by the
     // streamed CSR nor by other traffic between solves (bench.py's 256 MiB flush included), so
     // polls of not-yet-published dependencies and the publishes hit L2 (c2 41.0 -> 32.8 us).
-    // The device's persisting set-aside is grown to the window (up to persistingL2CacheMaxSize)
-    // on first use; a window larger than the set-aside is not used.
+    // The device's persisting set-aside is grown to the window (size_l2_window, at analyse time and
+    // on option changes -- never inside a stream capture); a window it cannot hold whole is not used.
     void *wbase = h->proto == PROTO_FLAGS ? (void *)h->ws.flags : (void *)h->ws.rec;
     const size_t wbytes = (h->proto == PROTO_FLAGS ? sizeof(uint32_t) : 16) * (size_t)h->n;
-    if (h->l2_window && wbase && h->l2_hit == 0.f) {
-        cudaDeviceProp prop;
-        size_t cur = 0;
-        if (cudaGetDeviceProperties(&prop, h->device) == cudaSuccess &&
-            cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
-            const size_t want = std::min(wbytes, (size_t)prop.persistingL2CacheMaxSize);
-            if (cur < want && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) == cudaSuccess) cur = want;
-            // only a window the set-aside holds whole: a partial one (c3's 67 MB of records) left the
-            // time unchanged and added DRAM traffic (361.6 vs 314.6 MB per launch)
-            h->l2_hit = cur >= wbytes ? 1.f : -1.f;
-        } else {
-            h->l2_hit = -1.f;  // no persisting L2 here: run without the window
-        }
-        (void)cudaGetLastError();
-    }
+    if (h->l2_window && wbase && h->l2_hit == 0.f) size_l2_window(h);  // normally done at analyse / set_option
     if (h->l2_window && wbase && h->l2_hit > 0.f) {
         cudaLaunchAttribute &a = attr[cfg.numAttrs++];
         a.id = cudaLaunchAttributeAccessPolicyWindow;
@@ -1167,7 +1176,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
         case SPTRSV_OPT_L2_WINDOW:
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
             h->l2_window = (int)value;
-            h->l2_hit = 0.f;  // (re)size the set-aside at the next solve
+            size_l2_window(h);
             return SPTRSV_OK;
         case SPTRSV_OPT_STAGE_SMEM:
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;
@@ -1183,8 +1192,8 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
                 }
                 CK(cudaMemset(h->ws.rec, 0, 16 * (size_t)h->n));
             }
-            h->l2_hit = 0.f;
             h->proto = (int)value;
+            size_l2_window(h);
             return SPTRSV_OK;
         case SPTRSV_OPT_LOCAL:
             if (value != 0 && value != 1) return SPTRSV_ERR_INVALID_ARG;

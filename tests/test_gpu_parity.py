@@ -200,6 +200,33 @@ def test_many_solves_on_side_stream_and_graph_capture(cap, proto, engine):
             assert np.array_equal(x2.cpu().numpy(), ref)
 
 
+@pytest.mark.parametrize("cfg", ["c1", "c2s", "grid", "c4s"])
+def test_graph_capture_of_a_fresh_handles_first_solve(cap, cfg):
+    """The very first solve of a handle may be captured: nothing device-wide (the persisting L2
+    set-aside) is changed inside the capture, and the replays are exact."""
+    s = {"c1": synth.gen_c1, "c2s": lambda: synth.gen_c2(n=200_000), "grid": lambda: synth.gen_grid(150),
+         "c4s": lambda: synth.gen_c4(n=20_000, nlevels=100)}[cfg]()
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        st = torch.cuda.Stream()
+        g = torch.cuda.CUDAGraph()
+        x = torch.empty_like(b)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=st):
+            h.solve(b, x, stream=st)
+        for _ in range(4):
+            x.fill_(float("nan"))
+            g.replay()
+            torch.cuda.synchronize()
+            got = x.cpu().numpy()
+            if h.info()["n_warp_rows"]:
+                assert relerr(got, ref) <= TOL
+            else:
+                assert np.array_equal(got, ref)
+        h.check()
+
+
 @pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("engine,host_io", [(5, 0), (5, 1), (5, 2), (5, 3), (0, 2), (7, 2), (7, 1), (7, 3)])
 @pytest.mark.parametrize("pinned", [True, False])
