@@ -156,6 +156,10 @@ typedef struct sptrsv_info {
     int32_t engine;           /* engine the next solve uses (AUTO resolved)                */
     int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
+    int64_t prev_deps;        /* dependencies on the previous row in solve order (i - 1;
+                                 i + 1 for upper handles): AUTO's CHAIN criterion           */
+    int64_t near_rows;        /* rows whose nearest dependency is < 256 rows away: AUTO's
+                                 LEAN criterion (LEAN when < n/4)                          */
 } sptrsv_info;
 
 /*

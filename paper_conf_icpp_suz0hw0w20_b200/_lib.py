@@ -81,6 +81,8 @@ class sptrsv_info(ctypes.Structure):
         ("engine", ctypes.c_int32),
         ("cta_threads", ctypes.c_int32),
         ("rows_per_lane", ctypes.c_int32),
+        ("prev_deps", ctypes.c_int64),
+        ("near_rows", ctypes.c_int64),
     ]
 
 

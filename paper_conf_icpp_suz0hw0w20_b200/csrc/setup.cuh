@@ -32,7 +32,8 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
     const bool upper = tri & 1, unit = tri & 2;
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     int len = 0;
-    unsigned near = 0, wdep = 0;
+    unsigned near = 0, wdep = 0, pdep = 0, nrow = 0;
+    int dmin = 0x7fffffff;  // the row's nearest dependency (distance in rows)
     if (i < n) {
         const int64_t s = rowptr[i], e = rowptr[i + 1];
         int code = 0;
@@ -52,6 +53,8 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
                 if (c != i && (c > i ? c - i : i - c) < 256) ++near;
                 // same 32-row group of LOGICAL rows (upper handles run row n-1-r as logical r)
                 if (c != i && (upper ? ((n - 1 - c) >> 5) == ((n - 1 - i) >> 5) : (c >> 5) == (i >> 5))) ++wdep;
+                if (c == (upper ? i + 1 : i - 1)) ++pdep;  // the previous row in solve order (chains)
+                if (c != i) dmin = min(dmin, c > i ? c - i : i - c);
                 prev = c;
             }
             if (!code && !unit) {
@@ -60,6 +63,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
                 else if (val[jd] == 0.0) code = E_ZERO_DIAG;
             }
         }
+        if (!code && dmin < 256) nrow = 1;  // the row's latest-solved dependency is near
         if (code) atomicMin(status, ((unsigned long long)i << 8) | (unsigned long long)code);
         len = code ? 0 : (int)(e - s);
         indeg[i] = code ? 0 : (int)(e - s - (unit ? 0 : 1));
@@ -68,11 +72,16 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
         len = max(len, __shfl_xor_sync(0xffffffffu, len, off));
         near += __shfl_xor_sync(0xffffffffu, near, off);
         wdep += __shfl_xor_sync(0xffffffffu, wdep, off);
+        pdep += __shfl_xor_sync(0xffffffffu, pdep, off);
+        nrow += __shfl_xor_sync(0xffffffffu, nrow, off);
     }
     if ((threadIdx.x & 31) == 0 && len > 0) atomicMax(max_row, len);
     // both totals are < nnz < 2^31: near in the low word, wdep in the high word
     if ((threadIdx.x & 31) == 0 && (near | wdep))
         atomicAdd(near_deps, (unsigned long long)near | ((unsigned long long)wdep << 32));
+    // previous-row dependencies in the low word, rows with a near (< 256) nearest dependency in the high word
+    if ((threadIdx.x & 31) == 0 && (pdep | nrow))
+        atomicAdd(near_deps + 1, (unsigned long long)pdep | ((unsigned long long)nrow << 32));
 }
 
 // mode: 0 auto, 1 all thread-level, 2 all warp-level.

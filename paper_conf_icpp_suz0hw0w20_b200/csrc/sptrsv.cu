@@ -88,6 +88,8 @@ struct sptrsv_handle_s {
     int32_t max_row = 0;
     int64_t near_deps = 0;  // dependencies within 256 rows (analyse statistic for ENGINE_AUTO)
     int64_t warp_deps = 0;  // dependencies inside the row's own 32-row group (ditto)
+    int64_t prev_deps = 0;  // dependencies on the previous row in solve order (ditto: chains)
+    int64_t near_rows = 0;  // rows whose nearest dependency is < 256 rows away (ditto)
     // options
     int mode = 0;
     int threshold = 16;
@@ -416,13 +418,13 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
             cudaMalloc(&h->ws.st, sizeof(SolveState)) != cudaSuccess ||
             cudaMalloc(&d_status, sizeof(unsigned long long)) != cudaSuccess ||
             cudaMalloc(&d_maxrow, sizeof(int32_t)) != cudaSuccess ||
-            cudaMalloc(&d_near, sizeof(unsigned long long)) != cudaSuccess) {
+            cudaMalloc(&d_near, 2 * sizeof(unsigned long long)) != cudaSuccess) {
             rc = SPTRSV_ERR_ALLOC;
             break;
         }
         if (cudaMemset(d_status, 0xff, sizeof(unsigned long long)) != cudaSuccess ||
             cudaMemset(d_maxrow, 0, sizeof(int32_t)) != cudaSuccess ||
-            cudaMemset(d_near, 0, sizeof(unsigned long long)) != cudaSuccess) {
+            cudaMemset(d_near, 0, 2 * sizeof(unsigned long long)) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
@@ -437,12 +439,15 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         unsigned long long status = 0;
         if (cudaMemcpy(&status, d_status, sizeof(status), cudaMemcpyDeviceToHost) != cudaSuccess ||
             cudaMemcpy(&h->max_row, d_maxrow, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(&h->near_deps, d_near, sizeof(int64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+            cudaMemcpy(&h->near_deps, d_near, sizeof(int64_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(&h->prev_deps, d_near + 1, sizeof(int64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
         h->warp_deps = (int64_t)((uint64_t)h->near_deps >> 32);
         h->near_deps &= 0xFFFFFFFFll;
+        h->near_rows = (int64_t)((uint64_t)h->prev_deps >> 32);
+        h->prev_deps &= 0xFFFFFFFFll;
         if (status != ~0ull) {
             rc = -(int)(status & 0xff);
             break;
@@ -536,12 +541,14 @@ int resolve_engine(const sptrsv_handle_s *h) {
     if (h->tri) {  // f4 handles: tri hybrid for warp rows, else CHAIN or LEAN (ENGINE 3 / 7 honoured)
         if (h->plan != PLAN_THREAD) return 6;
         if (h->engine == 3 || h->engine == 7) return h->engine;
-        return (offdiag > 0 && 4 * h->warp_deps >= offdiag) ? 7 : 3;
+        return (offdiag > 0 && 4 * h->prev_deps >= offdiag) ? 7 : 3;
     }
     if (h->engine != 5) return h->engine;
-    if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_deps < offdiag)) return 3;
+    // LEAN unless >= 1/4 of the rows wait on a near row (small levels, grids, chains): those resolve
+    // in-CTA (one-shot's shared-memory copy) or in-warp (CHAIN)
+    if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n)) return 3;
     if (h->plan != PLAN_THREAD) return 6;
-    if (4 * h->warp_deps >= offdiag) return 7;  // in-warp chains: CHAIN
+    if (4 * h->prev_deps >= offdiag) return 7;  // chains (>= 1/4 of the dependencies on row i-1): CHAIN
     return 0;
 }
 
@@ -1296,6 +1303,8 @@ int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
     out->solves = h->solves;
     out->near_deps = h->near_deps;
     out->warp_deps = h->warp_deps;
+    out->prev_deps = h->prev_deps;
+    out->near_rows = h->near_rows;
     out->engine = resolve_engine(h);
     effective_geometry(h, out->engine, &out->cta_threads, &out->rows_per_lane);
     return SPTRSV_OK;
