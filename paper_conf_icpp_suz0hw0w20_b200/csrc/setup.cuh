@@ -64,6 +64,12 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
             }
         }
         if (!code && dmin < 256) nrow = 1;  // the row's latest-solved dependency is near
+        if (!code && dmin != 0x7fffffff) {  // histogram of floor(log2(nearest-dependency distance))
+            const int bk = 31 - __clz(dmin);
+            const unsigned same = __match_any_sync(__activemask(), bk);
+            if ((threadIdx.x & 31) == __ffs(same) - 1)
+                atomicAdd(near_deps + 2 + bk, (unsigned long long)__popc(same));
+        }
         if (code) atomicMin(status, ((unsigned long long)i << 8) | (unsigned long long)code);
         len = code ? 0 : (int)(e - s);
         indeg[i] = code ? 0 : (int)(e - s - (unit ? 0 : 1));

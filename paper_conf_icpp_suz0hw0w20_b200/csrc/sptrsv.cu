@@ -93,6 +93,8 @@ struct sptrsv_handle_s {
     // options
     int mode = 0;
     int threshold = 16;
+    bool threshold_user = false;  // SPTRSV_OPT_WARP_THRESHOLD set explicitly
+    int dmin_log2 = -1;           // floor(log2(median nearest-dependency distance)), -1 = no dependencies
     int cta_threads = 0;    // 0 = per-engine default (see effective_geometry)
     uint32_t backoff_min = 0;
     uint32_t backoff_max = 256;
@@ -369,6 +371,19 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
 }
 
 void size_l2_window(sptrsv_handle_s *h);
+// AUTO's per-32-row-group warp threshold (mean nnz/row above which a group runs warp-level), from
+// floor(log2) of the median distance to a row's nearest dependency -- on leveled matrices about the
+// level width, which moves the thread/warp crossover (profiles/r01_ablation_final.md,
+// tools/dispatch_probe.py): < 64 rows: in-CTA / in-warp resolution wins, thread level only;
+// 64..1023: warp from 2 nnz/row; 1024..8191: from 6; wider: from 20.
+int auto_warp_threshold(int med_log2) {
+    if (med_log2 < 0) return 16;  // no dependencies at all
+    if (med_log2 <= 5) return 1 << 30;
+    if (med_log2 <= 9) return 2;
+    if (med_log2 <= 12) return 6;
+    return 20;
+}
+
 
 int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
                           int32_t tri_flags, sptrsv_handle_t *out) {
@@ -418,13 +433,13 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
             cudaMalloc(&h->ws.st, sizeof(SolveState)) != cudaSuccess ||
             cudaMalloc(&d_status, sizeof(unsigned long long)) != cudaSuccess ||
             cudaMalloc(&d_maxrow, sizeof(int32_t)) != cudaSuccess ||
-            cudaMalloc(&d_near, 2 * sizeof(unsigned long long)) != cudaSuccess) {
+            cudaMalloc(&d_near, 34 * sizeof(unsigned long long)) != cudaSuccess) {
             rc = SPTRSV_ERR_ALLOC;
             break;
         }
         if (cudaMemset(d_status, 0xff, sizeof(unsigned long long)) != cudaSuccess ||
             cudaMemset(d_maxrow, 0, sizeof(int32_t)) != cudaSuccess ||
-            cudaMemset(d_near, 0, 2 * sizeof(unsigned long long)) != cudaSuccess) {
+            cudaMemset(d_near, 0, 34 * sizeof(unsigned long long)) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
@@ -448,6 +463,27 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         h->near_deps &= 0xFFFFFFFFll;
         h->near_rows = (int64_t)((uint64_t)h->prev_deps >> 32);
         h->prev_deps &= 0xFFFFFFFFll;
+        {   // the AUTO warp threshold from the median nearest-dependency distance (f2)
+            unsigned long long hist[32];
+            if (cudaMemcpy(hist, d_near + 2, sizeof(hist), cudaMemcpyDeviceToHost) != cudaSuccess) {
+                rc = SPTRSV_ERR_CUDA;
+                break;
+            }
+            unsigned long long tot = 0, acc = 0;
+            for (int k = 0; k < 32; ++k) tot += hist[k];
+            int med = -1;
+            for (int k = 0; k < 32 && tot; ++k) {
+                acc += hist[k];
+                if (2 * acc >= tot) {
+                    med = k;
+                    break;
+                }
+            }
+            h->dmin_log2 = med;
+            // a system that fits one 1024-thread one-shot CTA resolves everything in shared memory:
+            // thread level only (c1: 28.2 us vs 32.9 us with warp rows)
+            if (!h->threshold_user) h->threshold = h->n <= 1024 ? (1 << 30) : auto_warp_threshold(med);
+        }
         if (status != ~0ull) {
             rc = -(int)(status & 0xff);
             break;
@@ -1162,6 +1198,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
         case SPTRSV_OPT_WARP_THRESHOLD:
             if (value < 0 || value > (1 << 30)) return SPTRSV_ERR_INVALID_ARG;
             h->threshold = (int)value;
+            h->threshold_user = true;
             return build_plan(h);
         case SPTRSV_OPT_CTA_THREADS:
             if (value != 0 && value != 64 && value != 128 && value != 256 && value != 512 && value != 1024)

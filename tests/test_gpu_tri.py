@@ -67,11 +67,11 @@ GENS = {
 def test_tri_random_sizes_bit_exact(cap, n, gen, flags, proto):
     s = form(GENS[gen](n), flags)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
-    x, info = gpu_solve(cap, s, flags, protocol=proto)
-    assert info["engine"] in (3, 7)  # LEAN, or CHAIN when >= 1/4 of the dependencies are in-warp
+    x, info = gpu_solve(cap, s, flags, protocol=proto, mode=1)  # thread level: bit-exact
+    assert info["engine"] in (3, 7)  # LEAN, or CHAIN when >= 1/4 of the dependencies are on the previous row
     assert np.array_equal(x, ref)
     for engine in (3, 7):  # both thread-level engines, forced
-        x, info = gpu_solve(cap, s, flags, protocol=proto, engine=engine)
+        x, info = gpu_solve(cap, s, flags, protocol=proto, engine=engine, mode=1)
         assert info["engine"] == engine
         assert np.array_equal(x, ref)
 
@@ -300,7 +300,7 @@ def test_tri_chain_engine_bit_exact(cap, which, flags, proto, K, cta):
             "c2i": lambda: synth.gen_c2i(n=60_000), "rand4": lambda: synth.gen_random_lower(4099, 4, seed=5)}[which]()
     s = form(base, flags)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
-    x, info = gpu_solve(cap, s, flags, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+    x, info = gpu_solve(cap, s, flags, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta, mode=1)
     assert (info["engine"], info["rows_per_lane"], info["cta_threads"]) == (7, K, cta), info
     assert np.array_equal(x, ref)
 
