@@ -57,8 +57,11 @@ typedef enum sptrsv_option {
                                       Alg.5), 2 WARP (every row warp-level, Alg.3).
                                       Setting it re-plans (synchronous).                    */
     SPTRSV_OPT_WARP_THRESHOLD = 2, /* AUTO: a 32-row group goes warp-level when its mean
-                                      nnz/row exceeds this (default 16; sec.4.4, DESIGN G10).
-                                      Setting it re-plans (synchronous).                    */
+                                      nnz/row exceeds this.  Default: derived at analyse from
+                                      the median distance to each row's nearest dependency
+                                      (< 64 rows: never; 64-1023: 2; 1024-8191: 6; wider: 20;
+                                      n <= 1024: never; sec.4.4, DESIGN G10).  Setting it
+                                      overrides that and re-plans (synchronous).            */
     SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 64, 128, 256, 512, 1024, or 0 (default)
                                       = the engine's measured best; the PIPE engine uses one
                                       of the warps as its loader                            */
