@@ -8,6 +8,8 @@ near-diagonal and far dependencies, empty-ish rows, ragged sizes.
 Bar: bit-exact where every row is thread level, else max componentwise
 relative error <= 1e-12 (the solutions are x_true ~ U[1, 2], |x| >= 1).
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -63,7 +65,7 @@ ENGINES = [(5, {}), (0, {}), (3, {}), (6, {}), (7, {}), (8, {"rows_per_lane": 2}
            (7, {"rows_per_lane": 1, "cta_threads": 64}), (3, {"cta_threads": 128})]
 
 
-@pytest.mark.parametrize("seed", range(100))
+@pytest.mark.parametrize("seed", range(int(os.environ.get("SPTRSV_FUZZ_SEEDS", "100"))))
 def test_fuzz_engines_vs_oracle(seed):
     import paper_conf_icpp_suz0hw0w20_b200 as cap
     rng = np.random.default_rng(1000 + seed)

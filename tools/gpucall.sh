@@ -1,4 +1,2 @@
 mkdir -p gpurun_out
-python tools/optsweep.py c3 '[{}]' 5 > gpurun_out/sweep72_c3.txt 2>&1
-python tools/optsweep.py chain '[{}]' 5 > gpurun_out/sweep72_chain.txt 2>&1
-python tools/optsweep.py c3 '[{"rows_per_lane":1}]' 5 > gpurun_out/sweep72_c3k1.txt 2>&1
+SPTRSV_FUZZ_SEEDS=600 timeout 1800 python -m pytest tests/test_gpu_fuzz.py -q > gpurun_out/fuzz600.log 2>&1
