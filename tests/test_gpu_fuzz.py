@@ -89,3 +89,33 @@ def test_fuzz_engines_vs_oracle(seed):
                 else:
                     err = float(np.max(np.abs(got - ref) / np.abs(ref))) if s.n else 0.0
                     assert err <= TOL, (s.name, s.n, engine, proto, extra, info, err)
+
+
+@pytest.mark.parametrize("seed", range(int(os.environ.get("SPTRSV_FUZZ_SEEDS", "100")) // 2))
+def test_fuzz_triangular_forms_vs_oracle(seed):
+    """The same random structures as upper / unit-lower / unit-upper systems through
+    AUTO and the forced thread-level engines (LEAN, CHAIN), two solves each, vs oracle.solve_tri."""
+    import paper_conf_icpp_suz0hw0w20_b200 as cap
+    rng = np.random.default_rng(5000 + seed)
+    s = random_structure(rng)
+    flags = int(rng.integers(1, 4))  # 1 upper, 2 unit lower, 3 unit upper
+    if flags & 1:
+        s = synth.to_upper(s)
+    if flags & 2:
+        s = synth.to_unit(s)
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
+    d = torch.device("cuda:0")
+    rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+    for opts in ({}, {"engine": 3, "mode": 1}, {"engine": 7, "mode": 1}):
+        proto = int(rng.integers(0, 2))
+        with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2), protocol=proto, **opts) as h:
+            for _ in range(2):
+                x = torch.full_like(b, float("nan"))
+                h.solve(b, x)
+                h.check()
+                got = x.cpu().numpy()
+                if h.info()["n_warp_rows"] == 0:
+                    assert np.array_equal(got, ref), (s.name, s.n, flags, opts, proto)
+                else:
+                    err = float(np.max(np.abs(got - ref) / np.abs(ref))) if s.n else 0.0
+                    assert err <= TOL, (s.name, s.n, flags, opts, proto, err)
