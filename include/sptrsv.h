@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SPTRSV_ABI_VERSION 2
+#define SPTRSV_ABI_VERSION 3
 
 typedef struct sptrsv_handle_s *sptrsv_handle_t;
 typedef void *sptrsv_stream_t; /* cudaStream_t */
@@ -47,7 +47,12 @@ typedef enum sptrsv_status {
     SPTRSV_ERR_TOO_LARGE = -8,    /* n > 2^31 - 2 (int32 CSR)                  */
     SPTRSV_ERR_CUDA = -9,         /* a CUDA runtime call failed (launch, copy, ...)         */
     SPTRSV_ERR_ALLOC = -10,       /* device / pinned allocation failed                      */
-    SPTRSV_ERR_TIMEOUT = -11      /* watchdog: a solve spun past SPTRSV_OPT_SPIN_LIMIT      */
+    SPTRSV_ERR_TIMEOUT = -11,     /* watchdog: a solve spun past SPTRSV_OPT_SPIN_LIMIT      */
+    SPTRSV_ERR_STALE_LAUNCH = -12 /* a solve captured in a CUDA graph was replayed after the
+                                     handle's launch configuration changed (an option
+                                     change or a watchdog reset re-zeroes the ready words
+                                     under a new generation): the stale launch did not
+                                     solve; re-capture the graph                           */
 } sptrsv_status;
 
 /* Options (sptrsv_set_option / sptrsv_get_option).  None changes the result
@@ -62,9 +67,9 @@ typedef enum sptrsv_option {
                                       (< 64 rows: never; 64-1023: 2; 1024-8191: 6; wider: 20;
                                       n <= 1024: never; sec.4.4, DESIGN G10).  Setting it
                                       overrides that and re-plans (synchronous).            */
-    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA: 64, 128, 256, 512, 1024, or 0 (default)
-                                      = the engine's measured best; the PIPE engine uses one
-                                      of the warps as its loader                            */
+    SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA, or 0 (default) = the engine's measured
+                                      best.  ONE-SHOT: 64..1024; LEAN (lower): 128, 256, 512;
+                                      CHAIN: 64, 128, 256; other values / engines: default  */
     SPTRSV_OPT_BACKOFF_MIN_NS = 4, /* __nanosleep after a pass where no lane progressed     */
     SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
     SPTRSV_OPT_SPIN_LIMIT = 6,     /* watchdog: idle passes per warp before TIMEOUT (0=off) */
@@ -83,39 +88,28 @@ typedef enum sptrsv_option {
                                                                      */
     SPTRSV_OPT_LOCAL = 10,         /* 1 (default): dependencies produced inside the same CTA
                                       are read from a shared-memory copy of x               */
-    SPTRSV_OPT_ENGINE = 11,        /* 5 (default) AUTO: LEAN for all-thread-level plans whose
-                                      dependencies are mostly far (< 1/4 within 256 rows),
-                                      HYBRID for plans with warp-level rows, else ONE-SHOT.  0 ONE-SHOT: one CTA per row range,
-                                      ticketed, smem-staged, in-CTA x copy;
-                                      1 PIPE: persistent CTAs, a loader warp streams rounds
-                                      of rows into a shared-memory ring by TMA bulk copy.
-                                      PIPE needs 16-byte aligned rowptr/colidx/val/b and a
-                                      ring that fits; it falls back to ONE-SHOT otherwise.
-                                      2 DYN: persistent warps, every lane slot takes the next
-                                      row as soon as its row is published (all-thread-level
-                                      plans; ROWS_PER_LANE = slots per lane, 1/2/4).
-                                      3 LEAN: minimal-latency one-shot kernel for
-                                      all-thread-level plans (no staging, speculative rows).
-                                      4 DYN-STATIC: DYN with static round-robin 32-row units
-                                      (no ticket), launched cooperatively.
-                                      6 HYBRID: 64-thread CTAs, one task per warp -- a
-                                      warp-level row (Alg.3) or a 32-row thread group
-                                      (LEAN's per-lane loop), no staging / in-CTA copy;
-                                      all-thread-level plans run LEAN.
-                                      8 LEAN_K: LEAN with K = ROWS_PER_LANE (2 default, 3, 4)
-                                      rows per lane, row constants in shared memory; a larger
-                                      resident-row window for wide levels (CTA_THREADS 128
-                                      or 256; LEAN_OCCUPANCY 2..5 picks the register budget) */
-    SPTRSV_OPT_PIPE_STAGES = 12,   /* PIPE ring depth, 2..8 (default 3)                     */
-    SPTRSV_OPT_PIPE_BATCH = 13,    /* accepted for compatibility; PIPE takes 1 round/ticket */
-    SPTRSV_OPT_PIPE_ENTRIES = 14,  /* PIPE colidx/val entries per stage (0 = 4 per row)     */
-    SPTRSV_OPT_ROWS_PER_LANE = 15, /* K = 1..4 thread-level rows per lane (lane owns rows
-                                      r0+lane+32k), or 0 (default) = the engine's measured
-                                      best; applies to all-thread-level plans on the
-                                      ONE-SHOT engine with CTAs of <= 256 threads          */
+    SPTRSV_OPT_ENGINE = 11,        /* 5 (default) AUTO, from analyse's statistics (DESIGN.md
+                                      section 6): HYBRID for plans with warp-level rows; for
+                                      all-thread-level plans LEAN when < 1/4 of the rows wait
+                                      on a row < 256 away, CHAIN when >= 1/4 of the
+                                      dependencies are on the previous row, else ONE-SHOT.
+                                      Forced engines:
+                                      0 ONE-SHOT (lower): one CTA per row range, ticketed,
+                                      smem-staged CSR slices, in-CTA x copy in smem;
+                                      3 LEAN: minimal-latency kernel, one row per lane, no
+                                      staging, speculative rows;
+                                      6 HYBRID: one task per warp -- a warp-level row (Alg.3)
+                                      or a 32-row thread group (LEAN's per-lane loop);
+                                      7 CHAIN: in-warp dependency chains resolved in
+                                      registers / shared memory, external ones by polling.
+                                      LEAN and CHAIN need an all-thread-level plan; a plan
+                                      with warp-level rows runs HYBRID (ONE-SHOT if forced on
+                                      a lower handle).  sptrsv_info.engine reports the engine
+                                      that runs.  Other values: INVALID_ARG                 */
+    /* 12, 13, 14: retired (the PIPE ablation engine left the library in round 2)       */
+    SPTRSV_OPT_ROWS_PER_LANE = 15, /* CHAIN: K = 1 or 2 (0 = default 2) rows per lane       */
     SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 6)
-                                      resident 256-thread CTAs per SM; LEAN_K: 2..5 (per-K
-                                      default)                                              */
+                                      resident 256-thread CTAs per SM                       */
     SPTRSV_OPT_PREFETCH = 18,      /* L2 bulk prefetch (cp.async.bulk.prefetch.L2) of the
                                       CSR range of the CTA this many logical blocks ahead:
                                       -1 (default) = the engine's measured choice, 0 = off.
@@ -156,7 +150,8 @@ typedef struct sptrsv_info {
     uint32_t solves;          /* solves enqueued through this handle                      */
     int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
     int64_t warp_deps;        /* dependencies inside the row's own 32-row group            */
-    int32_t engine;           /* engine the next solve uses (AUTO resolved)                */
+    int32_t engine;           /* engine the next solve launches (0 ONE-SHOT, 3 LEAN,
+                                 6 HYBRID, 7 CHAIN; 33/34/35 the paper's Alg.3/4/5)        */
     int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
     int64_t prev_deps;        /* dependencies on the previous row in solve order (i - 1;
@@ -313,7 +308,9 @@ int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev,
 int sptrsv_set_trace(sptrsv_handle_t h, uint64_t *trace_dev);
 
 /* sptrsv_check -- synchronises `stream`, returns SPTRSV_ERR_TIMEOUT if the
- * watchdog fired in any solve since the last check (and clears it), else OK. */
+ * watchdog fired in any solve since the last check, SPTRSV_ERR_STALE_LAUNCH if
+ * a stale graph launch was refused, else OK.  Clears the condition: the next
+ * solve re-zeroes the ready words first, so it is correct again. */
 int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream);
 
 /*
@@ -330,6 +327,19 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream);
  * Synchronous.
  */
 int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop, double *sm_mhz);
+
+/*
+ * sptrsv_hop_scan -- diagnostic, placement-controlled t_hop (the critical-path latency bound's
+ * hop): one CTA per SM on the current device; the CTAs on SM sm_a (the
+ * lowest SM id present) and on each other SM b ping-pong `iters` rounds through the solve's
+ * publish / poll pair (protocol 0 FLAGS: st.release flag, ld.acquire poll + x load; 1 FUSED:
+ * 16-byte epoch record, relaxed store / poll) and the mean one-way hop in ns is reported per b.
+ *   capacity    entries sm_b_out / ns_out can hold (host arrays).
+ *   sm_a_out    host int32, receives sm_a.   count  host int32, receives the pairs measured.
+ * Synchronous.  The two dies of a B200 show as two latency modes over b.
+ */
+int sptrsv_hop_scan(int32_t iters, int32_t protocol, int32_t capacity, int32_t *sm_a_out, int32_t *sm_b_out,
+                    double *ns_out, int32_t *count);
 
 const char *sptrsv_strerror(int status);
 int sptrsv_abi_version(void);

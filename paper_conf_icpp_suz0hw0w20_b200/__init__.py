@@ -17,25 +17,27 @@ from ._lib import (MODE_AUTO, MODE_THREAD, MODE_WARP, OPT_BACKOFF_MAX_NS, OPT_BA
                    OPT_CTA_THREADS, OPT_L2_WINDOW, OPT_LOCAL, OPT_MODE, OPT_PROTOCOL, OPT_SPIN_LIMIT,
                    OPT_STAGE_SMEM, OPT_WARP_THRESHOLD, PROTO_FLAGS, PROTO_FUSED, SptrsvError, check)
 
-__all__ = ["analyse", "Handle", "SptrsvError", "flag_latency", "MODE_AUTO", "MODE_THREAD",
+__all__ = ["analyse", "Handle", "SptrsvError", "flag_latency", "hop_scan", "MODE_AUTO", "MODE_THREAD",
            "MODE_WARP", "PROTO_FLAGS", "PROTO_FUSED", "lib"]
 
 lib = _lib.lib
 
 
-def _stream_ptr(stream) -> int | None:
+def _stream_ptr(stream, device=None) -> int | None:
     import torch
     if stream is None:
-        stream = torch.cuda.current_stream()
+        stream = torch.cuda.current_stream(device)
     if isinstance(stream, int):
         return stream
     return stream.cuda_stream
 
 
-def _need(t, dtype, n, name):
+def _need(t, dtype, n, name, device=None):
     import torch
     if not isinstance(t, torch.Tensor) or not t.is_cuda:
         raise TypeError(f"{name} must be a CUDA tensor")
+    if device is not None and t.device != device:
+        raise ValueError(f"{name} is on {t.device}, the handle on {device}")
     if t.dtype != dtype:
         raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
     if not t.is_contiguous():
@@ -74,12 +76,13 @@ class Handle:
     def solve(self, b, x=None, stream=None):
         """x <- L^{-1} b (fp64, device tensors), enqueued on ``stream`` (default: current)."""
         import torch
-        _need(b, torch.float64, self.n, "b")
+        _need(b, torch.float64, self.n, "b", self.device)
         if x is None:
             x = torch.empty_like(b)
-        _need(x, torch.float64, self.n, "x")
+        _need(x, torch.float64, self.n, "x", self.device)
         if self.n:
-            check(lib.sptrsv_solve(self._h, b.data_ptr(), x.data_ptr(), _stream_ptr(stream)), "sptrsv_solve")
+            with torch.cuda.device(self.device):
+                check(lib.sptrsv_solve(self._h, b.data_ptr(), x.data_ptr(), _stream_ptr(stream, self.device)), "sptrsv_solve")
         return x
 
     def solve_multi(self, B, X=None, stream=None):
@@ -89,14 +92,17 @@ class Handle:
             raise TypeError("B must be a 2-D float64 CUDA tensor")
         if B.shape[0] != self.n or B.stride(1) != 1:
             raise ValueError("B must be (n, nrhs) with unit column stride")
+        if B.device != self.device:
+            raise ValueError(f"B is on {B.device}, the handle on {self.device}")
         nrhs = B.shape[1]
         if X is None:
             X = torch.empty_like(B)
-        if X.shape != B.shape or X.stride(1) != 1 or X.dtype != torch.float64 or not X.is_cuda:
+        if X.shape != B.shape or X.stride(1) != 1 or X.dtype != torch.float64 or X.device != B.device:
             raise ValueError("X must match B")
         if self.n and nrhs:
-            check(lib.sptrsv_solve_multi(self._h, B.data_ptr(), X.data_ptr(), nrhs, B.stride(0), X.stride(0),
-                                         _stream_ptr(stream)), "sptrsv_solve_multi")
+            with torch.cuda.device(self.device):
+                check(lib.sptrsv_solve_multi(self._h, B.data_ptr(), X.data_ptr(), nrhs, B.stride(0), X.stride(0),
+                                             _stream_ptr(stream, self.device)), "sptrsv_solve_multi")
         return X
 
     def solve_host(self, b_host, x_host, stream=None):
@@ -112,19 +118,19 @@ class Handle:
             assert a.is_contiguous() and a.numel() == self.n
             return a.data_ptr()
         with torch.cuda.device(self.device):
-            check(lib.sptrsv_solve_host(self._h, ptr(b_host), ptr(x_host), _stream_ptr(stream)),
+            check(lib.sptrsv_solve_host(self._h, ptr(b_host), ptr(x_host), _stream_ptr(stream, self.device)),
                   "sptrsv_solve_host")
         return x_host
 
     def check(self, stream=None):
         """Synchronise and raise SptrsvError(ERR_TIMEOUT) if the watchdog fired."""
-        check(lib.sptrsv_check(self._h, _stream_ptr(stream)), "sptrsv_check")
+        check(lib.sptrsv_check(self._h, _stream_ptr(stream, self.device)), "sptrsv_check")
 
     # -- diagnostics ---------------------------------------------------------------------
     def indegree(self, stream=None):
         import torch
         out = torch.empty(self.n, dtype=torch.int32, device=self.device)
-        check(lib.sptrsv_get_indegree(self._h, out.data_ptr() if self.n else None, _stream_ptr(stream)),
+        check(lib.sptrsv_get_indegree(self._h, out.data_ptr() if self.n else None, _stream_ptr(stream, self.device)),
               "sptrsv_get_indegree")
         return out
 
@@ -136,7 +142,7 @@ class Handle:
         nl = ctypes.c_int32(0)
         if self.n:
             check(lib.sptrsv_levels(self._h, lv.data_ptr(), counts.data_ptr(), ctypes.byref(nl),
-                                    _stream_ptr(stream)), "sptrsv_levels")
+                                    _stream_ptr(stream, self.device)), "sptrsv_levels")
         return lv, int(nl.value), counts[: nl.value]
 
     def trace(self, b, x=None, stream=None):
@@ -193,8 +199,7 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "backoff_min_ns": OPT_BACKOFF_MIN_NS, "backoff_max_ns": OPT_BACKOFF_MAX_NS,
             "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
-            "pipe_stages": _lib.OPT_PIPE_STAGES, "pipe_batch": _lib.OPT_PIPE_BATCH,
-            "pipe_entries": _lib.OPT_PIPE_ENTRIES, "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
+            "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
             "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY,
             "prefetch": _lib.OPT_PREFETCH, "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
             "poll_one": _lib.OPT_POLL_ONE,
@@ -203,6 +208,18 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h
+
+
+def hop_scan(iters: int = 4000, protocol: int = 1, capacity: int = 512):
+    """Placement-controlled one-way hop (ns) from the lowest-id SM to every other SM of the current
+    device (``sptrsv_hop_scan``): returns (partner SM ids, ns per hop) as numpy arrays."""
+    import numpy as np
+    sm_b = np.zeros(capacity, dtype=np.int32)
+    ns = np.zeros(capacity, dtype=np.float64)
+    a, cnt = ctypes.c_int32(0), ctypes.c_int32(0)
+    check(lib.sptrsv_hop_scan(iters, protocol, capacity, ctypes.byref(a), sm_b.ctypes.data, ns.ctypes.data,
+                              ctypes.byref(cnt)), "sptrsv_hop_scan")
+    return sm_b[: cnt.value], ns[: cnt.value]
 
 
 def flag_latency(iters: int = 20000, protocol: int = 0, with_clock: bool = False):

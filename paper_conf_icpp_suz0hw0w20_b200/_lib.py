@@ -35,6 +35,7 @@ TRI_UNIT_DIAG = 2
 ERR_CUDA = -9
 ERR_ALLOC = -10
 ERR_TIMEOUT = -11
+ERR_STALE_LAUNCH = -12
 
 # options
 OPT_MODE = 1
@@ -48,9 +49,6 @@ OPT_STAGE_SMEM = 8
 OPT_PROTOCOL = 9
 OPT_LOCAL = 10
 OPT_ENGINE = 11
-OPT_PIPE_STAGES = 12
-OPT_PIPE_BATCH = 13
-OPT_PIPE_ENTRIES = 14
 OPT_ROWS_PER_LANE = 15
 OPT_VARIANT = 16
 OPT_LEAN_OCCUPANCY = 17
@@ -59,8 +57,7 @@ OPT_POLL_GAP_NS = 19
 OPT_POLL_ONE = 20
 OPT_WARP_SPLIT_LAST = 22
 OPT_HOST_IO = 23
-ENGINE_ONESHOT, ENGINE_PIPE, ENGINE_DYN, ENGINE_LEAN, ENGINE_DYN_STATIC, ENGINE_AUTO = 0, 1, 2, 3, 4, 5
-ENGINE_HYBRID, ENGINE_CHAIN = 6, 7
+ENGINE_ONESHOT, ENGINE_LEAN, ENGINE_AUTO, ENGINE_HYBRID, ENGINE_CHAIN = 0, 3, 5, 6, 7
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
 
@@ -106,6 +103,7 @@ EXPORTS = {
     "sptrsv_set_trace": (ctypes.c_int, [_h, _p]),
     "sptrsv_flag_latency": (ctypes.c_int, [_i32, _i32, ctypes.POINTER(ctypes.c_double),
                                            ctypes.POINTER(ctypes.c_double)]),
+    "sptrsv_hop_scan": (ctypes.c_int, [_i32, _i32, _i32, ctypes.POINTER(_i32), _p, _p, ctypes.POINTER(_i32)]),
     "sptrsv_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "sptrsv_abi_version": (ctypes.c_int, []),
 }

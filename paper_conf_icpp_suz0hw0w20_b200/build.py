@@ -5,6 +5,7 @@
 """
 from __future__ import annotations
 
+import glob
 import os
 import subprocess
 import sys
@@ -14,8 +15,9 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libsptrsv.so")
 SOURCES = [os.path.join(CSRC, f) for f in ("sptrsv.cu",)]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("solve.cuh", "solve_pipe.cuh", "solve_k.cuh", "solve_dyn.cuh", "solve_lean.cuh", "solve_tri.cuh", "solve_multi.cuh", "solve_paper.cuh", "setup.cuh", "ptx.cuh", "diag.cuh")] + [
-    os.path.join(ROOT, "include", "sptrsv.h")]
+DEPS = SOURCES + sorted(glob.glob(os.path.join(CSRC, "*.cuh"))) + [os.path.join(ROOT, "include", "sptrsv.h")]
+# ptxas register / spill report of the last build (untracked: build() must not dirty the tree)
+PTXAS_INFO = os.path.join(ROOT, "build", "ptxas_info.txt")
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
@@ -49,7 +51,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed building libsptrsv.so")
     if verbose:
         sys.stderr.write(res.stderr)
-    with open(os.path.join(CSRC, "ptxas_info.txt"), "w") as f:
+    os.makedirs(os.path.dirname(PTXAS_INFO), exist_ok=True)
+    with open(PTXAS_INFO, "w") as f:
         f.write(res.stderr)
     os.replace(tmp, LIB)
     return LIB

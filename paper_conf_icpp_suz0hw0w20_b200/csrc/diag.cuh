@@ -168,4 +168,69 @@ __global__ void k_pingpong(uint32_t *flags, double *xs, int iters, int protocol,
     sink[me] = acc;
 }
 
+// ---------------------------------------------------------------- placement-controlled hop (t_hop per die pair)
+// One CTA per SM: the launch requests more than half of an SM's shared memory, so the grid of
+// #SMs CTAs lands one per SM, all co-resident.  k_smids records which SM each CTA landed on;
+// in k_pingpong_sm the CTAs on SMs sm_a and sm_b ping-pong `iters` rounds through the solve's
+// protocol (0: st.release flag / ld.acquire poll + relaxed x load; 1: FUSED 16-byte epoch
+// record, relaxed store / relaxed poll) and the others exit at once.  The one-way hop between
+// a given pair of SMs is then independent of where the scheduler puts CTAs.
+__device__ __forceinline__ unsigned smid_u32() {
+    unsigned s;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+    return s;
+}
+
+__global__ void k_smids(int32_t *out) {
+    extern __shared__ unsigned char pad_[];
+    if (threadIdx.x == 0) {
+        pad_[0] = 0;
+        out[blockIdx.x] = (int32_t)smid_u32();
+    }
+}
+
+__global__ void k_pingpong_sm(unsigned long long *rec, uint32_t *flags, double *xs, int iters, int protocol,
+                              int sm_a, int sm_b, unsigned long long *out, double *sink) {
+    extern __shared__ unsigned char pad_[];
+    if (threadIdx.x != 0) return;
+    pad_[0] = 0;
+    const int s = (int)smid_u32();
+    const int me = s == sm_a ? 0 : s == sm_b ? 1 : -1;
+    if (me < 0) return;
+    unsigned long long *myr = rec + 16 * me, *orr = rec + 16 * (1 - me);  // 128 B apart
+    uint32_t *myf = flags + 32 * me, *of = flags + 32 * (1 - me);
+    double *myx = xs + 16 * me, *ox = xs + 16 * (1 - me);
+    double acc = 0.0;
+    const uint64_t t0 = globaltimer_ns();
+    for (int k = 1; k <= iters; ++k) {
+        for (int phase = 0; phase < 2; ++phase) {
+            const bool send = (phase == 0) == (me == 0);
+            if (send) {
+                if (protocol == 0) {
+                    myx[0] = (double)k;
+                    st_release_u32(myf, (uint32_t)k);
+                } else {
+                    const unsigned long long bits = (unsigned long long)__double_as_longlong((double)k);
+                    const unsigned long long e = (unsigned long long)k << 32;
+                    st_relaxed_v2_u64(myr, e | (bits & 0xffffffffull), e | (bits >> 32));
+                }
+            } else {
+                if (protocol == 0) {
+                    while (ld_acquire_u32(of) != (uint32_t)k) {}
+                    acc += ld_relaxed_f64(ox);
+                } else {
+                    unsigned long long a, b;
+                    do {
+                        ld_relaxed_v2_u64(orr, a, b);
+                    } while ((uint32_t)(a >> 32) != (uint32_t)k || (uint32_t)(b >> 32) != (uint32_t)k);
+                    acc += __longlong_as_double((long long)((a & 0xffffffffull) | (b << 32)));
+                }
+            }
+        }
+    }
+    const uint64_t t1 = globaltimer_ns();
+    if (me == 0) out[0] = t1 - t0;
+    sink[me] = acc;
+}
+
 }  // namespace sptrsv_dev

@@ -69,6 +69,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
         }
     }
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     const int r0 = ((int)s_blk * warps + warp) * RT;
     if (r0 >= p.n) return;
@@ -101,7 +102,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
 #pragma unroll
     for (int k = 0; k < K; ++k) {
         const int idx = lane + 32 * k;
-        bk[k] = idx < rows ? ld_stream_f64(p.b + phys(r0 + idx), pol) : 0.0;
+        bk[k] = idx < rows ? ld_b(p, phys(r0 + idx), pol) : 0.0;
     }
     __syncwarp();
     const int base = s_rp[0];
@@ -360,7 +361,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 uint32_t ab = 0;
                 if (lane == 0) {
                     if (p.spin_limit && idle >= p.spin_limit) {
-                        atomicCAS(&p.st->error.v, 0u, 1u);
+                        atomicCAS(&p.st->error.v, 0u, kErrTimeout);
                         st_relaxed_u32(&p.st->abort.v, 1u);
                     }
                     ab = ld_relaxed_u32(&p.st->abort.v);

@@ -118,7 +118,7 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int r
             uint32_t ab = 0;
             if (lane == 0) {
                 if (p.spin_limit && idle >= p.spin_limit) {
-                    atomicCAS(&p.st->error.v, 0u, 1u);
+                    atomicCAS(&p.st->error.v, 0u, kErrTimeout);
                     st_relaxed_u32(&p.st->abort.v, 1u);
                 }
                 ab = ld_relaxed_u32(&p.st->abort.v);
@@ -148,7 +148,7 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         if (p.trace) p.trace[3 * (size_t)p.n + 3 + i] = globaltimer_ns();  // CTA entry
         rs = ld_stream_i32(p.rowptr + i, pol);
         re = ld_stream_i32(p.rowptr + i + 1, pol);
-        if (!bgate) bi = ld_stream_f64(p.b + i, pol);
+        if (!bgate) bi = ld_b(p, i, pol);
     }
     // ---- L2 bulk prefetch of the block pf_dist logical blocks ahead (speculatively
     // blockIdx.x + pf_dist): its bounds load overlaps the ticket, the copy is issued after it
@@ -175,6 +175,7 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         }
     }
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     if (pfB > pfA) prefetch_rows_l2(p, pfA, pfB, pfa, pfb);
     if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
@@ -184,10 +185,10 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         if (i >= 0 && i < p.n) {
             rs = ld_stream_i32(p.rowptr + i, pol);
             re = ld_stream_i32(p.rowptr + i + 1, pol);
-            bi = ld_stream_f64(p.b + i, pol);
+            bi = ld_b(p, i, pol);
         }
     } else if (bgate && i >= 0 && i < p.n) {
-        bi = ld_stream_f64(p.b + i, pol);
+        bi = ld_b(p, i, pol);
     }
     const bool act = i >= 0 && i < p.n;
     lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);

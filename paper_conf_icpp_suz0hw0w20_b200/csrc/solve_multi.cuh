@@ -37,6 +37,7 @@ __global__ void __launch_bounds__(256) k_solve_multi(SolveParams p, MultiParams 
     const uint64_t pol = policy_evict_first();
     if (tid == 0) cta_ticket(p, s_blk, s_epoch);
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     const int rows_per_cta = blockDim.x / m.g;
     const int i = (int)s_blk * rows_per_cta + tid / m.g;  // row
@@ -116,7 +117,7 @@ __global__ void __launch_bounds__(256) k_solve_multi(SolveParams p, MultiParams 
             uint32_t ab = 0;
             if (lane == 0) {
                 if (p.spin_limit && idle >= p.spin_limit) {
-                    atomicCAS(&p.st->error.v, 0u, 1u);
+                    atomicCAS(&p.st->error.v, 0u, kErrTimeout);
                     st_relaxed_u32(&p.st->abort.v, 1u);
                 }
                 ab = ld_relaxed_u32(&p.st->abort.v);

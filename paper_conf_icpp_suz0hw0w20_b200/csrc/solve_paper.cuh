@@ -41,6 +41,7 @@ __global__ void __launch_bounds__(kPaperCta) k_paper_alg5(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
     if (threadIdx.x == 0) cta_ticket(p, s_blk, s_epoch);
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     const int i = (int)s_blk * kPaperCta + threadIdx.x;  // l.3: one thread for one component
     if (i >= p.n) return;
@@ -67,6 +68,7 @@ __global__ void __launch_bounds__(kPaperCta) k_paper_alg4(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
     if (threadIdx.x == 0) cta_ticket(p, s_blk, s_epoch);
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     const int i = (int)s_blk * kPaperCta + threadIdx.x;  // l.3
     const bool act = i < p.n;
@@ -114,6 +116,7 @@ __global__ void __launch_bounds__(kPaperCta) k_paper_alg3(SolveParams p) {
     __shared__ double left_sum_s[kPaperCta];          // l.4: left_sum[WARP_SIZE] per warp
     if (threadIdx.x == 0) cta_ticket(p, s_blk, s_epoch);
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     const int warp = threadIdx.x >> 5, tid = threadIdx.x & 31;
     const int i = (int)s_blk * (kPaperCta / 32) + warp;  // l.3: one warp for one component

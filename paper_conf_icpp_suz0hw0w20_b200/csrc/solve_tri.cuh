@@ -31,7 +31,7 @@ __device__ __forceinline__ void tri_warp_row(SolveParams &p, int r, uint32_t epo
     const int hi = (UPPER || UNIT) ? re : re - 1;
     double bi = 0.0, dv = 1.0;
     if (lane == 0) {
-        bi = ld_stream_f64(p.b + i, pol);
+        bi = ld_b(p, i, pol);
         if (!UNIT) dv = ld_stream_f64(p.val + (UPPER ? rs : re - 1), pol);
     }
     Cta nocta;
@@ -70,6 +70,7 @@ __global__ void __launch_bounds__(kTriWarpCta) k_solve_tri_warp(SolveParams p) {
         }
     }
     __syncthreads();
+    if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
     const int task = (int)s_blk * (kTriWarpCta / 32) + warp;
     if (task >= p.n_tasks) return;
@@ -92,7 +93,7 @@ __global__ void __launch_bounds__(kTriWarpCta) k_solve_tri_warp(SolveParams p) {
     if (act) {
         rs = ld_stream_i32(p.rowptr + i, pol);
         re = ld_stream_i32(p.rowptr + i + 1, pol);
-        bi = ld_stream_f64(p.b + i, pol);
+        bi = ld_b(p, i, pol);
     }
     lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);
 }

@@ -9,21 +9,19 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <vector>
 
 #include "diag.cuh"
 #include "setup.cuh"
 #include "solve.cuh"
-#include "solve_pipe.cuh"
-#include "solve_k.cuh"
-#include "solve_dyn.cuh"
 #include "solve_lean.cuh"
-#include "solve_lk.cuh"
 #include "solve_tri.cuh"
 #include "solve_multi.cuh"
 #include "solve_paper.cuh"
 #include "solve_chain.cuh"
+#include "solve_chainp.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -31,6 +29,9 @@ using namespace sptrsv_dev;
 namespace {
 
 constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
+
+// engines (SPTRSV_OPT_ENGINE values, include/sptrsv.h)
+enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_CHAINP = 8 };
 
 struct Workspace {
     uint32_t *flags = nullptr;     // n      (PROTO_FLAGS)
@@ -95,22 +96,19 @@ struct sptrsv_handle_s {
     int threshold = 16;
     bool threshold_user = false;  // SPTRSV_OPT_WARP_THRESHOLD set explicitly
     int dmin_log2 = -1;           // floor(log2(median nearest-dependency distance)), -1 = no dependencies
-    int cta_threads = 0;    // 0 = per-engine default (see effective_geometry)
+    int cta_threads = 0;    // 0 = per-engine default (see plan_launch)
     uint32_t backoff_min = 0;
     uint32_t backoff_max = 256;
     uint32_t spin_limit = 1u << 24;
     int l2_window = 1;      // persisting L2 window over the ready words (SPTRSV_OPT_L2_WINDOW)
     float l2_hit = 0.f;     // its hitRatio once the set-aside is sized (0 = not yet)
+    bool l2_user = false;   // counted among the device's persisting-L2 users (l2_limit_*)
     int stage = 1;
     int proto = PROTO_FUSED;
     int local = 1;
-    int engine = 5;         // 5 AUTO; 0 one-shot, 1 pipe, 2 dyn, 3 lean, 4 dyn-static
-    int pipe_stages = 3;
-    int pipe_batch = 1;  // (kept for the ABI; the loader takes one round per ticket)
-    int pipe_entries = 0;   // 0 = 4 per row of a round
-    int rows_per_lane = 0;  // K: thread-level rows per lane; 0 = per-engine default
+    int engine = ENG_AUTO;  // SPTRSV_OPT_ENGINE: ENG_AUTO or a forced engine (resolve_engine)
+    int rows_per_lane = 0;  // CHAIN: K rows per lane (0 = 2)
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
-    int lk_occ = 0;         // LEAN_K register budget (0 = per-K default; SPTRSV_OPT_LEAN_OCCUPANCY)
     int lean_minb = 6;      // LEAN: resident 256-thread CTAs per SM the register budget targets (5..8)
     int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
@@ -124,11 +122,42 @@ struct sptrsv_handle_s {
     int launch_key = -1;  // configuration of the last launch (see sptrsv_solve)
     long long mlaunch_key = -1;  // same for sptrsv_solve_multi
     uint32_t msince_reset = 0;
+    uint32_t gen = 0, mgen = 0;  // configuration generations of the solve / multi-RHS state (cta_ticket)
     unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
     uint32_t since_reset = 0;
     float analyse_ms = 0.f;
+};
+
+namespace {
+// The persisting-L2 set-aside is a device-wide limit.  The library grows it for handles whose
+// ready-word window it can hold, remembers the value it found, and restores that value when the
+// last handle using a window on the device is destroyed (or turns its window off), so a host
+// application's L2 is only shared while a windowed handle exists.
+struct L2Limit {
+    size_t orig = 0;
+    int users = 0;
+};
+std::mutex g_l2_mu;
+L2Limit g_l2[256];
+
+void l2_limit_release(sptrsv_handle_s *h);
+}  // namespace
+
+// Makes a handle's device current for a host entry point and restores the caller's on exit.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) cudaSetDevice(dev);
+        (void)cudaGetLastError();
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+        (void)cudaGetLastError();
+    }
 };
 
 #define CK(call)                                        \
@@ -140,6 +169,18 @@ struct sptrsv_handle_s {
     } while (0)
 
 namespace {
+
+void l2_limit_release(sptrsv_handle_s *h) {
+    std::lock_guard<std::mutex> lk(g_l2_mu);
+    if (!h->l2_user) return;
+    h->l2_user = false;
+    L2Limit &e = g_l2[h->device & 255];
+    if (--e.users == 0) {
+        (void)cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, e.orig);
+        (void)cudaGetLastError();
+        e.orig = 0;
+    }
+}
 
 // dynamic smem: x copy [warps*32] doubles, then (if staging) [warps][kStageCap] doubles + ints
 size_t solve_smem_bytes(int cta_threads, int stage) {
@@ -157,82 +198,15 @@ solve_fn solve_kernel(int plan, int proto) {
     return tab[plan][proto];
 }
 
-solve_fn solve_k_kernel(int proto, int K) {
-    if (K == 2) return proto ? k_solve_k<PROTO_FUSED, 2> : k_solve_k<PROTO_FLAGS, 2>;
-    if (K == 3) return proto ? k_solve_k<PROTO_FUSED, 3> : k_solve_k<PROTO_FLAGS, 3>;
-    return proto ? k_solve_k<PROTO_FUSED, 4> : k_solve_k<PROTO_FLAGS, 4>;
-}
-
-solve_fn solve_dyn_kernel(int proto, int K, bool stat) {
-    if (stat) {
-        if (K == 2) return proto ? k_solve_dyn<PROTO_FUSED, 2, true> : k_solve_dyn<PROTO_FLAGS, 2, true>;
-        if (K == 4) return proto ? k_solve_dyn<PROTO_FUSED, 4, true> : k_solve_dyn<PROTO_FLAGS, 4, true>;
-        return proto ? k_solve_dyn<PROTO_FUSED, 1, true> : k_solve_dyn<PROTO_FLAGS, 1, true>;
-    }
-    if (K == 2) return proto ? k_solve_dyn<PROTO_FUSED, 2, false> : k_solve_dyn<PROTO_FLAGS, 2, false>;
-    if (K == 4) return proto ? k_solve_dyn<PROTO_FUSED, 4, false> : k_solve_dyn<PROTO_FLAGS, 4, false>;
-    return proto ? k_solve_dyn<PROTO_FUSED, 1, false> : k_solve_dyn<PROTO_FLAGS, 1, false>;
-}
-
-size_t solve_k_smem_bytes(int cta_threads, int K) {
-    const size_t w = (size_t)(cta_threads / 32);
-    return w * 32 * K * sizeof(double) + w * (size_t)k_warp_smem_bytes(K);
-}
-
-typedef void (*pipe_fn)(SolveParams, PipeGeom);
-pipe_fn pipe_kernel(int plan, int proto) {
-    static const pipe_fn tab[3][2] = {
-        {k_solve_pipe<PLAN_THREAD, PROTO_FLAGS>, k_solve_pipe<PLAN_THREAD, PROTO_FUSED>},
-        {k_solve_pipe<PLAN_WARP, PROTO_FLAGS>, k_solve_pipe<PLAN_WARP, PROTO_FUSED>},
-        {k_solve_pipe<PLAN_LIST, PROTO_FLAGS>, k_solve_pipe<PLAN_LIST, PROTO_FUSED>},
-    };
-    return tab[plan][proto];
-}
-
-int round16(int b) { return (b + 15) & ~15; }
-constexpr int kPipeMaxSmem = 200 * 1024;  // ring bytes per CTA, at most (227 KB minus static smem and slack)
-
-PipeGeom pipe_geom(const sptrsv_handle_s *h, int cta) {
-    PipeGeom g;
-    g.W = cta / 32 - 1;
-    g.S = h->pipe_stages;
-    g.B = h->pipe_batch;
-    g.RB = 32 * g.W;
-    g.E = h->pipe_entries > 0 ? h->pipe_entries : 4 * g.RB;
-    int off = 64;  // StageHdr
-    g.off_rp = off;
-    off += round16(4 * (g.RB + 1) + 32);
-    g.off_b = off;
-    off += round16(8 * g.RB + 32);
-    g.off_col = off;
-    off += round16(4 * g.E + 32);
-    g.off_val = off;
-    off += round16(8 * g.E + 32);
-    g.off_xc = off;
-    off += round16(8 * g.RB);
-    g.stage_bytes = round16(off);
-    return g;
-}
-
 int set_kernel_attrs() {
     static int done = 0;
     static int rc = SPTRSV_OK;
     if (done) return rc;
     const int maxb = (int)solve_smem_bytes(1024, 1);
     for (int pl = 0; pl < 3; ++pl)
-        for (int pr = 0; pr < 2; ++pr) {
+        for (int pr = 0; pr < 2; ++pr)
             if (cudaFuncSetAttribute(solve_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize, maxb) !=
-                    cudaSuccess ||
-                cudaFuncSetAttribute(pipe_kernel(pl, pr), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     kPipeMaxSmem) != cudaSuccess) {
-                (void)cudaGetLastError();
-                rc = SPTRSV_ERR_CUDA;
-            }
-        }
-    for (int pr = 0; pr < 2; ++pr)
-        for (int K = 2; K <= 4; ++K)
-            if (cudaFuncSetAttribute(solve_k_kernel(pr, K), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)solve_k_smem_bytes(256, K)) != cudaSuccess) {
+                cudaSuccess) {
                 (void)cudaGetLastError();
                 rc = SPTRSV_ERR_CUDA;
             }
@@ -332,13 +306,41 @@ int build_plan(sptrsv_handle_s *h) {
     return rc;
 }
 
+// discard.global.L2 over [p, p + bytes) (whole 128-B lines inside the range): drops a dead window's
+// lines from L2 without write-back, which also ends their persisting status.
+__global__ void k_l2_discard(char *p, size_t bytes) {
+    const size_t lines = bytes / 128;
+    for (size_t l = blockIdx.x * (size_t)blockDim.x + threadIdx.x; l < lines; l += (size_t)gridDim.x * blockDim.x)
+        asm volatile("discard.global.L2 [%0], 128;" ::"l"(p + l * 128) : "memory");
+}
+
+// SolveState := 0 with the start ticket at gen << kGenShift (solve.cuh cta_ticket).  A kernel, not
+// a host copy, so that a reset inside a stream capture is capturable.
+__global__ void k_state_init(SolveState *st, uint32_t gen) {
+    st->tk.v = (unsigned long long)gen << kGenShift;
+}
+
+int init_state(SolveState *st, uint32_t gen, cudaStream_t s) {
+    CK(cudaMemsetAsync(st, 0, sizeof(SolveState), s));
+    k_state_init<<<1, 1, 0, s>>>(st, gen);
+    CK(cudaGetLastError());
+    return SPTRSV_OK;
+}
+
 int reset_state(sptrsv_handle_s *h, cudaStream_t s) {
-    // flags / records := 0 (no epoch matches), counters := 0; the next solve has epoch 1
+    // flags / records := 0 (no epoch matches), counters := 0 under a new generation; the next
+    // solve has epoch 1
     CK(cudaMemsetAsync(h->ws.flags, 0, sizeof(uint32_t) * (size_t)(h->n > 0 ? h->n : 1), s));
     if (h->ws.rec) CK(cudaMemsetAsync(h->ws.rec, 0, 16 * (size_t)(h->n > 0 ? h->n : 1), s));
-    CK(cudaMemsetAsync(h->ws.st, 0, sizeof(SolveState), s));
+    h->gen = (h->gen + 1) & 0xFFFFFFu;
     h->since_reset = 0;
-    return SPTRSV_OK;
+    return init_state(h->ws.st, h->gen, s);
+}
+
+// a reset is due before the next launch: new configuration, epoch about to wrap, or the 40-bit
+// ticket count of this generation about to overflow
+bool reset_due(uint32_t since, unsigned grid) {
+    return since >= kEpochResetAt || (unsigned long long)(since + 1) * grid >= (1ull << (kGenShift - 1));
 }
 
 }  // namespace
@@ -361,6 +363,8 @@ const char *sptrsv_strerror(int status) {
         case SPTRSV_ERR_CUDA: return "CUDA runtime error";
         case SPTRSV_ERR_ALLOC: return "allocation failed";
         case SPTRSV_ERR_TIMEOUT: return "watchdog timeout in solve";
+        case SPTRSV_ERR_STALE_LAUNCH:
+            return "a captured solve was replayed after the handle's launch configuration changed (re-capture)";
         default: return "unknown status";
     }
 }
@@ -515,114 +519,69 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
 
 namespace {
 
-// One solve launch: which kernel, its geometry, and how it is parameterised.
+// One solve launch: which kernel, its geometry, and how it is parameterised.  plan_launch is the
+// single source of truth: sptrsv_get_info, sptrsv_solve_host's transfer overlap and the epoch
+// arithmetic all read the engine / geometry it actually picked.
 struct Launch {
     const void *fn = nullptr;
-    int kind = 0;  // 0 SolveParams only, 1 SolveParams + PipeGeom
-    bool coop = false;  // cooperative launch (co-residency guaranteed)
     dim3 grid, block;
     size_t smem = 0;
-    PipeGeom geom;
-    int key = 0;  // configuration identity (the epoch arithmetic needs a fixed grid per key)
-    int pf_dist = 0;  // SolveParams::pf_dist (engines that implement the L2 prefetch)
+    int key = 0;      // configuration identity (the epoch arithmetic needs a fixed grid per key)
+    int pf_dist = 0;  // SolveParams::pf_dist (LEAN's optional L2 prefetch)
+    int engine = 0;   // engine launched (ENG_*; 30 + v for the paper's Alg. v)
+    int cta = 0;      // threads per CTA
+    int K = 1;        // thread-level rows per lane
 };
 
-int occupancy_grid(sptrsv_handle_s *h, const void *fn, int threads, size_t smem, int key, int *out) {
-    if (key != h->grid_cache_key) {
-        int per_sm = 0, sms = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem) != cudaSuccess ||
-            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device) != cudaSuccess) {
-            (void)cudaGetLastError();
-            return SPTRSV_ERR_CUDA;
-        }
-        h->grid_cache = per_sm * sms;
-        h->grid_cache_key = key;
-    }
-    *out = h->grid_cache;
-    return SPTRSV_OK;
-}
-
-// ENGINE_AUTO: all-thread-level plans go to the LEAN engine unless a quarter or
-// more of the dependencies are "near" (within 256 rows: chains, grid wavefronts).
-// Of those, plans with a quarter or more of their dependencies inside the row's own
-// 32-row group (bidiagonal chains, grid west neighbours) use the CHAIN engine
-// (in-warp shuffle chain); the rest the staged one-shot engine's shared-memory
-// local resolution; plans
-// with warp-level rows use the HYBRID engine (2-13% faster than the staged
-// one-shot engine on every warp-plan shape measured, tools/hybrid_probe.py).
-// (Round-1 B200 sweeps.)
 // Size the device's persisting L2 set-aside for the handle's ready-word window (SPTRSV_OPT_L2_WINDOW):
 // grown to the window (up to persistingL2CacheMaxSize); l2_hit = 1 if it holds the whole window,
 // -1 (no window) otherwise -- a partial window (c3's 67 MB of records) left the time unchanged and
 // added DRAM traffic (361.6 vs 314.6 MB per launch).  Host-only, synchronous: called from analyse
-// and set_option so that a first solve inside a stream capture never changes device limits.
+// and set_option so that a first solve inside a stream capture never changes device limits.  The
+// limit the library found is remembered per device and restored by the last handle's destroy.
 void size_l2_window(sptrsv_handle_s *h) {
     h->l2_hit = -1.f;
-    if (!h->l2_window || h->n == 0) return;
+    if (!h->l2_window || h->n == 0) {
+        l2_limit_release(h);
+        return;
+    }
     const size_t wbytes = (h->proto == PROTO_FLAGS ? sizeof(uint32_t) : 16) * (size_t)h->n;
-    cudaDeviceProp prop;
+    int maxp = 0;
     size_t cur = 0;
-    if (cudaGetDeviceProperties(&prop, h->device) == cudaSuccess &&
-        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
-        const size_t want = std::min(wbytes, (size_t)prop.persistingL2CacheMaxSize);
-        if (cur < want && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) == cudaSuccess) cur = want;
-        h->l2_hit = cur >= wbytes ? 1.f : -1.f;
+    {
+        std::lock_guard<std::mutex> lk(g_l2_mu);
+        L2Limit &e = g_l2[h->device & 255];
+        if (cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, h->device) == cudaSuccess &&
+            cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
+            if (e.users == 0) e.orig = cur;  // the value found before any windowed handle
+            const size_t want = std::min(wbytes, (size_t)maxp);
+            if (cur < want && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) == cudaSuccess) cur = want;
+            h->l2_hit = cur >= wbytes ? 1.f : -1.f;
+            if (h->l2_hit > 0.f && !h->l2_user) {
+                h->l2_user = true;
+                e.users++;
+            }
+            if (e.users == 0 && cur != e.orig) (void)cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, e.orig);
+        }
+        (void)cudaGetLastError();
     }
-    (void)cudaGetLastError();
+    if (h->l2_hit <= 0.f) l2_limit_release(h);
 }
 
+// ENGINE_AUTO, from analyse's O(nnz) statistics:
+//   plans with warp-level rows                                   -> HYBRID
+//   all-thread plans, < 1/4 of the rows waiting on a row < 256 away -> LEAN
+//   all-thread plans, >= 1/4 of the dependencies on row i-1 (chains, grids) -> CHAIN
+//   other near-dependency plans (small levels, c1)               -> ONE-SHOT (in-CTA smem copy of x)
+// f4 (upper / unit) handles: HYBRID for warp rows, else CHAIN (chains) or LEAN.
 int resolve_engine(const sptrsv_handle_s *h) {
-    // stored off-diagonals (unit handles store no diagonal)
-    const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;
-    if (h->tri) {  // f4 handles: tri hybrid for warp rows, else CHAIN or LEAN (ENGINE 3 / 7 honoured)
-        if (h->plan != PLAN_THREAD) return 6;
-        if (h->engine == 3 || h->engine == 7) return h->engine;
-        return (offdiag > 0 && 4 * h->prev_deps >= offdiag) ? 7 : 3;
-    }
-    if (h->engine != 5) return h->engine;
-    // LEAN unless >= 1/4 of the rows wait on a near row (small levels, grids, chains): those resolve
-    // in-CTA (one-shot's shared-memory copy) or in-warp (CHAIN)
-    if (h->plan == PLAN_THREAD && (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n)) return 3;
-    if (h->plan != PLAN_THREAD) return 6;
-    if (4 * h->prev_deps >= offdiag) return 7;  // chains (>= 1/4 of the dependencies on row i-1): CHAIN
-    return 0;
-}
-
-// CTA size and rows per lane actually used: the user's values, else the
-// per-engine defaults measured best on B200 in round 1:
-// CHAIN 2 rows per lane in 128-thread CTAs; staged one-shot on plans with
-// warp-level rows: 64-thread CTAs; everything else 256 threads, 1 row per lane
-// (the one-shot's former 2-rows/128-thread geometry for near-dependency plans
-// predates CHAIN, which now takes grids and chains; on c1 it measured 69.7 us
-// vs 30.7 us for 256/1), 1024 threads for small (n <= 32768) thread-level systems.
-void effective_geometry(const sptrsv_handle_s *h, int engine, int *cta, int *K) {
-    if (engine == 3 || engine == 6) {  // LEAN 256 threads (lower: option CTA_THREADS 128/512), HYBRID 64
-        *cta = (engine == 6 && h->plan != PLAN_THREAD) ? kTriWarpCta
-               : (engine == 3 && !h->tri && h->plan == PLAN_THREAD &&
-                  (h->cta_threads == 128 || h->cta_threads == 512)) ? h->cta_threads
-                                                                                       : kLeanCta;
-        *K = 1;
-        return;
-    }
-    int c = 256, k = 1;
-    if (engine == 8) {  // LEAN_K: 256-thread CTAs, K = 2 (1 is LEAN itself)
-        *cta = (h->cta_threads == 128) ? 128 : 256;
-        *K = (h->rows_per_lane >= 2 && h->rows_per_lane <= 4) ? h->rows_per_lane : 2;
-        return;
-    }
-    if (engine == 7) {
-        c = kChainCta;
-        k = 2;
-    } else if (engine == 0 && h->plan != PLAN_THREAD) {
-        c = 64;
-    } else if (engine == 0 && h->n <= 32768) {
-        // small thread-level systems: 1024-thread CTAs keep more dependencies inside one CTA
-        // (resolved through the shared-memory copy of x): c1 29.7 -> 26.7 us, a 4000-row
-        // 40-level system 47.1 -> 34.9 us
-        c = 1024;
-    }
-    *cta = h->cta_threads ? h->cta_threads : c;
-    *K = h->rows_per_lane ? h->rows_per_lane : k;
+    const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;  // unit handles store no diagonal
+    const bool chains = offdiag > 0 && 4 * h->prev_deps >= offdiag;
+    if (h->plan != PLAN_THREAD) return (h->engine == ENG_ONESHOT && !h->tri) ? ENG_ONESHOT : ENG_HYBRID;
+    if (h->engine != ENG_AUTO) return (h->tri && h->engine == ENG_ONESHOT) ? ENG_LEAN : h->engine;
+    if (h->tri) return chains ? ENG_CHAIN : ENG_LEAN;
+    if (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n) return ENG_LEAN;
+    return chains ? ENG_CHAIN : ENG_ONESHOT;
 }
 
 typedef void (*lean_fn)(SolveParams);
@@ -635,44 +594,15 @@ typedef void (*lean_fn)(SolveParams);
      {k_solve_lean<PROTO_FLAGS, M6, false, false, CT_>, k_solve_lean<PROTO_FUSED, M6, false, false, CT_>}, \
      {k_solve_lean<PROTO_FLAGS, M7, false, false, CT_>, k_solve_lean<PROTO_FUSED, M7, false, false, CT_>}, \
      {k_solve_lean<PROTO_FLAGS, M8, false, false, CT_>, k_solve_lean<PROTO_FUSED, M8, false, false, CT_>}}
-lean_fn lean_lower_kernel(int proto, int occ, int cta, int *ct_out) {
+lean_fn lean_lower_kernel(int proto, int occ, int ct) {
     static const lean_fn tab[3][4][2] = {LEAN_OCC(128, 10, 12, 14, 16), LEAN_OCC(256, 5, 6, 7, 8),
                                          LEAN_OCC(512, 2, 3, 3, 4)};
-    const int ct = (cta == 128 || cta == 512) ? cta : kLeanCta;  // other sizes: the default 256
     const int c = ct == 128 ? 0 : ct == 256 ? 1 : 2;
     if (occ < 5 || occ > 8) return nullptr;
-    *ct_out = ct;
     return tab[c][occ - 5][proto ? 1 : 0];
 }
 #undef LEAN_OCC
 
-// LEAN_K (solve_lk.cuh): K in {2, 3, 4} rows per lane, CTA 128 or 256 threads, and the
-// register budget occ = resident 256-thread CTAs per SM targeted.  Supported occ per K:
-// K=2: 3, 4 (default), 5;  K=3: 2, 3 (default);  K=4: 2 (default), 3.
-#define LK_PAIR(K_, CT_, MB_) {k_solve_lk<PROTO_FLAGS, K_, CT_, MB_>, k_solve_lk<PROTO_FUSED, K_, CT_, MB_>}
-lean_fn lean_k_kernel(int proto, int K, int cta, int occ, int *occ_out) {
-    static const lean_fn t2[2][3][2] = {{LK_PAIR(2, 128, 6), LK_PAIR(2, 128, 8), LK_PAIR(2, 128, 10)},
-                                        {LK_PAIR(2, 256, 3), LK_PAIR(2, 256, 4), LK_PAIR(2, 256, 5)}};
-    static const lean_fn t3[2][2][2] = {{LK_PAIR(3, 128, 4), LK_PAIR(3, 128, 6)},
-                                        {LK_PAIR(3, 256, 2), LK_PAIR(3, 256, 3)}};
-    static const lean_fn t4[2][2][2] = {{LK_PAIR(4, 128, 4), LK_PAIR(4, 128, 6)},
-                                        {LK_PAIR(4, 256, 2), LK_PAIR(4, 256, 3)}};
-    const int c = cta == 128 ? 0 : 1, pr = proto ? 1 : 0;
-    if (K == 2) {
-        const int o = (occ >= 3 && occ <= 5) ? occ : 4;
-        *occ_out = o;
-        return t2[c][o - 3][pr];
-    }
-    if (K == 3) {
-        const int o = (occ == 2 || occ == 3) ? occ : 3;
-        *occ_out = o;
-        return t3[c][o - 2][pr];
-    }
-    const int o = (occ == 2 || occ == 3) ? occ : 2;
-    *occ_out = o;
-    return t4[c][o - 2][pr];
-}
-#undef LK_PAIR
 lean_fn lean_tri_kernel(int proto, int tri) {
     static const lean_fn tab[4][2] = {
         {k_solve_lean<PROTO_FLAGS, 6>, k_solve_lean<PROTO_FUSED, 6>},
@@ -693,29 +623,29 @@ lean_fn tri_warp_kernel(int proto, int tri, int plan) {
     return tab[tri & 3][(plan == PLAN_LIST ? 2 : 0) + (proto ? 1 : 0)];
 }
 
-int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
-    if ((h->tri && resolve_engine(h) != 7) || (!h->tri && !h->variant && resolve_engine(h) == 6)) {
-        // f4 forms (LEAN / tri hybrid), or ENGINE_HYBRID (solve_lean.cuh / solve_tri.cuh)
-        L->kind = 0;
-        L->smem = 0;
-        if (h->plan != PLAN_THREAD) {  // warp-level rows present: one task per warp
-            L->fn = (const void *)tri_warp_kernel(h->proto, h->tri, h->plan);
-            L->grid = dim3((unsigned)((h->n_tasks + kTriWarpCta / 32 - 1) / (kTriWarpCta / 32)));
-            L->block = dim3((unsigned)kTriWarpCta);
-            L->key = 7500000 + h->proto * 100000 + h->tri * 10000 + h->plan * 1000;
-        } else {  // all thread level: LEAN
-            L->fn = (const void *)lean_tri_kernel(h->proto, h->tri);
-            L->grid = dim3((unsigned)((h->n + kLeanCta - 1) / kLeanCta));
-            L->block = dim3((unsigned)kLeanCta);
-            L->key = 7000000 + h->proto * 100000 + h->tri * 10000;
-        }
-        L->key ^= (int)L->grid.x * 7919;
-        return SPTRSV_OK;
-    }
+lean_fn chain_kernel(int proto, int tri, int K) {
+#define CHAIN_ROW(U_, N_)                                                                              \
+    {{k_solve_chain<PROTO_FLAGS, 1, U_, N_>, k_solve_chain<PROTO_FUSED, 1, U_, N_>},                   \
+     {k_solve_chain<PROTO_FLAGS, 2, U_, N_>, k_solve_chain<PROTO_FUSED, 2, U_, N_>}}
+    static const lean_fn tab[4][2][2] = {CHAIN_ROW(false, false), CHAIN_ROW(true, false),
+                                         CHAIN_ROW(false, true), CHAIN_ROW(true, true)};
+#undef CHAIN_ROW
+    return tab[tri & 3][K - 1][proto ? 1 : 0];
+}
+
+lean_fn chainp_kernel(int proto, int tri, int K) {
+#define CHAINP_ROW(U_, N_)                                                                             \
+    {{k_solve_chainp<PROTO_FLAGS, 1, U_, N_>, k_solve_chainp<PROTO_FUSED, 1, U_, N_>},                 \
+     {k_solve_chainp<PROTO_FLAGS, 2, U_, N_>, k_solve_chainp<PROTO_FUSED, 2, U_, N_>}}
+    static const lean_fn tab[4][2][2] = {CHAINP_ROW(false, false), CHAINP_ROW(true, false),
+                                         CHAINP_ROW(false, true), CHAINP_ROW(true, true)};
+#undef CHAINP_ROW
+    return tab[tri & 3][K - 1][proto ? 1 : 0];
+}
+
+int plan_launch(sptrsv_handle_s *h, Launch *L) {
     if (h->variant) {  // the paper's kernels, control flow as printed (solve_paper.cuh; ablation only)
-        L->kind = 0;
         L->block = dim3(kPaperCta);
-        L->smem = 0;
         if (h->variant == 3) {
             L->fn = (const void *)k_paper_alg3;
             L->grid = dim3((unsigned)((h->n + kPaperCta / 32 - 1) / (kPaperCta / 32)));
@@ -723,74 +653,34 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
             L->fn = h->variant == 4 ? (const void *)k_paper_alg4 : (const void *)k_paper_alg5;
             L->grid = dim3((unsigned)((h->n + kPaperCta - 1) / kPaperCta));
         }
-        L->key = 6000000 + h->variant * 100000;
-        L->key ^= (int)L->grid.x * 7919;
+        L->engine = 30 + h->variant;
+        L->cta = kPaperCta;
+        L->key = (6000000 + h->variant * 100000) ^ (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
     const int engine = resolve_engine(h);
-    int cta = 256, Kq = 1;
-    effective_geometry(h, engine, &cta, &Kq);
-    // ---- ENGINE_PIPE: persistent, loader warp + TMA ring
-    if (engine == 1 && aligned && cta >= 64) {
-        const PipeGeom g = pipe_geom(h, cta);
-        const size_t smem = (size_t)g.S * g.stage_bytes;
-        if (smem <= (size_t)kPipeMaxSmem) {
-            const void *fn = (const void *)pipe_kernel(h->plan, h->proto);
-            const int key = 1000000 + (h->plan * 2 + h->proto) * 100000 + cta * 16 + g.S;
-            int cap = 0;
-            int rc = occupancy_grid(h, fn, cta, smem, key, &cap);
-            if (rc) return rc;
-            if (cap >= 1) {
-                const int rounds = (h->n_tasks + g.W - 1) / g.W;
-                L->fn = fn;
-                L->kind = 1;
-                L->grid = dim3((unsigned)(rounds < cap ? (rounds > 0 ? rounds : 1) : cap));
-                L->block = dim3((unsigned)cta);
-                L->smem = smem;
-                L->geom = g;
-                L->key = key ^ (int)L->grid.x * 7919;
-                return SPTRSV_OK;
-            }
-        }
-    }
-    // ---- ENGINE_DYN: persistent, lane slots refilled row by row
-    if ((engine == 2 || engine == 4) && h->plan == PLAN_THREAD && cta <= 256) {
-        const int K = Kq == 3 ? 2 : Kq;
-        const bool stat = engine == 4;
-        const void *fn = (const void *)solve_dyn_kernel(h->proto, K, stat);
-        const size_t smem = (size_t)(cta / 32) * kDynWarpSmem;
-        const int key = 2000000 + h->proto * 100000 + K * 10000 + cta + (stat ? 500 : 0);
-        int cap = 0;
-        int rc = occupancy_grid(h, fn, cta, smem, key, &cap);
-        if (rc) return rc;
-        if (cap >= 1) {
-            long long grid = cap;
-            const long long need = stat ? ((long long)h->n + kDynSub * (cta / 32) - 1) / (kDynSub * (cta / 32))
-                                        : ((long long)h->n + kDynCtaChunk - 1) / kDynCtaChunk;
-            if (grid > need) grid = need;
-            L->fn = fn;
-            L->kind = 0;
-            L->coop = stat;
-            L->grid = dim3((unsigned)(grid > 0 ? grid : 1));
-            L->block = dim3((unsigned)cta);
-            L->smem = smem;
-            L->key = key ^ (int)L->grid.x * 7919;
+    const int user = h->cta_threads;
+    L->engine = engine;
+    if (engine == ENG_HYBRID) {  // warp-level rows: one task per warp (solve_tri.cuh), any triangular form
+        L->fn = (const void *)tri_warp_kernel(h->proto, h->tri, h->plan == PLAN_THREAD ? PLAN_LIST : h->plan);
+        if (h->plan == PLAN_THREAD) {  // HYBRID forced on an all-thread plan: run it as LEAN
+            L->engine = ENG_LEAN;
+        } else {
+            L->cta = kTriWarpCta;
+            L->grid = dim3((unsigned)((h->n_tasks + kTriWarpCta / 32 - 1) / (kTriWarpCta / 32)));
+            L->block = dim3((unsigned)kTriWarpCta);
+            L->key = (7500000 + h->proto * 100000 + h->tri * 10000 + h->plan * 1000) ^ (int)L->grid.x * 7919;
             return SPTRSV_OK;
         }
     }
-    // ---- ENGINE_CHAIN: warp-sequential in-warp chains (solve_chain.cuh), all-thread-level plans
-    if (engine == 7 && h->plan == PLAN_THREAD && cta <= 256) {
-        const int K = Kq >= 2 ? 2 : 1;
+    if (L->engine == ENG_CHAIN) {  // warp-sequential in-warp chains (solve_chain.cuh): 64..256 threads
+        const int K = h->rows_per_lane == 1 ? 1 : 2;
+        const int cta = (user == 64 || user == 128 || user == 256) ? user : kChainCta;
         const int warps = cta / 32;
-#define CHAIN_ROW(U_, N_)                                                                              \
-    {{k_solve_chain<PROTO_FLAGS, 1, U_, N_>, k_solve_chain<PROTO_FUSED, 1, U_, N_>},                   \
-     {k_solve_chain<PROTO_FLAGS, 2, U_, N_>, k_solve_chain<PROTO_FUSED, 2, U_, N_>}}
-        static const lean_fn ctab[4][2][2] = {CHAIN_ROW(false, false), CHAIN_ROW(true, false),
-                                              CHAIN_ROW(false, true), CHAIN_ROW(true, true)};
-#undef CHAIN_ROW
-        L->fn = (const void *)ctab[h->tri & 3][K - 1][h->proto ? 1 : 0];
-        L->kind = 0;
         const long long rows_per_cta = (long long)warps * 32 * K;
+        L->fn = (const void *)chain_kernel(h->proto, h->tri, K);
+        L->cta = cta;
+        L->K = K;
         L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
         L->block = dim3((unsigned)cta);
         L->smem = (size_t)warps * chain_warp_smem_bytes(K);
@@ -799,61 +689,54 @@ int plan_launch(sptrsv_handle_s *h, bool aligned, Launch *L) {
             (void)cudaGetLastError();
             return SPTRSV_ERR_CUDA;
         }
-        L->key = 8000000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta;
-        L->key ^= (int)L->grid.x * 7919;
+        L->key = (8000000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta) ^ (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
-    // ---- ENGINE_LEAN_K: LEAN with K rows per lane (all-thread-level lower plans)
-    if (engine == 8 && h->plan == PLAN_THREAD) {
-        int occ = 0;
-        L->fn = (const void *)lean_k_kernel(h->proto, Kq, cta, h->lk_occ, &occ);
-        L->kind = 0;
-        const long long rows_per_cta = (long long)cta * Kq;
+    if (L->engine == ENG_CHAINP) {  // chain warps with poller warps (solve_chainp.cuh): 1..4 pairs per CTA
+        const int K = h->rows_per_lane == 1 ? 1 : 2;
+        const int cta = (user == 64 || user == 128 || user == 256) ? user : 64 * kChainPPairs;
+        const int pairs = cta / 64;
+        const long long rows_per_cta = (long long)pairs * 32 * K;
+        L->fn = (const void *)chainp_kernel(h->proto, h->tri, K);
+        L->cta = cta;
+        L->K = K;
         L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
         L->block = dim3((unsigned)cta);
-        L->smem = 0;
-        L->key = 9000000 + h->proto * 100000 + Kq * 10000 + occ * 1000 + cta;
-        L->key ^= (int)L->grid.x * 7919;
+        L->smem = (size_t)pairs * chainp_pair_smem_bytes(K);
+        L->key = (8500000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta) ^ (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
-    // ---- ENGINE_LEAN: minimal one-shot kernel for all-thread-level plans
-    if (engine == 3 && h->plan == PLAN_THREAD) {
-        // LEAN geometry: CTA size 128 / 256 (default) / 512 (option CTA_THREADS) and the register
-        // budget (option LEAN_OCCUPANCY = resident 256-thread CTAs per SM it targets: 5..8)
-        int ct = 0;
-        L->fn = (const void *)lean_lower_kernel(h->proto, h->lean_minb, h->cta_threads, &ct);
-        if (!L->fn) return SPTRSV_ERR_INVALID_ARG;
-        L->kind = 0;
+    if (L->engine == ENG_LEAN) {  // minimal one-shot kernel for all-thread-level plans (solve_lean.cuh)
+        int ct = kLeanCta;
+        if (h->tri) {
+            L->fn = (const void *)lean_tri_kernel(h->proto, h->tri);
+        } else {
+            // CTA size 128 / 256 (default) / 512 (option CTA_THREADS) and the register budget
+            // (option LEAN_OCCUPANCY = resident 256-thread CTAs per SM it targets: 5..8)
+            if (user == 128 || user == 512) ct = user;
+            L->fn = (const void *)lean_lower_kernel(h->proto, h->lean_minb, ct);
+            if (!L->fn) return SPTRSV_ERR_INVALID_ARG;
+            L->pf_dist = h->pf_dist < 0 ? kLeanPrefetchDefault : h->pf_dist;
+        }
+        L->cta = ct;
         L->grid = dim3((unsigned)((h->n + ct - 1) / ct));
         L->block = dim3((unsigned)ct);
-        L->smem = 0;
-        L->pf_dist = h->pf_dist < 0 ? kLeanPrefetchDefault : h->pf_dist;
-        L->key = 5000000 + h->proto * 100000 + h->lean_minb * 1000 + ct;
-        L->key ^= (int)L->grid.x * 7919;
+        L->key = (5000000 + h->proto * 100000 + h->lean_minb * 1000 + h->tri * 10 + ct / 128) ^ (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
-    // ---- ONE-SHOT, K rows per lane
-    if (engine == 0 && h->plan == PLAN_THREAD && Kq > 1 && cta <= 256) {
-        const int K = Kq;
-        const long long rows_per_cta = (long long)(cta / 32) * 32 * K;
-        L->fn = (const void *)solve_k_kernel(h->proto, K);
-        L->kind = 0;
-        L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
-        L->block = dim3((unsigned)cta);
-        L->smem = solve_k_smem_bytes(cta, K);
-        L->key = 3000000 + h->proto * 100000 + K * 10000 + cta;
-        L->key ^= (int)L->grid.x * 7919;
-        return SPTRSV_OK;
-    }
-    // ---- ONE-SHOT (default)
+    // ONE-SHOT (solve.cuh k_solve), lower handles only: staged CSR slices and an in-CTA shared-memory copy of
+    // x.  64-thread CTAs on plans with warp-level rows; 1024 for small (n <= 32768) thread-level systems
+    // (more dependencies resolved in-CTA: c1 29.7 -> 26.7 us); else 256.
+    int cta = h->plan != PLAN_THREAD ? 64 : h->n <= 32768 ? 1024 : 256;
+    if (user) cta = user;
     const int warps = cta / 32;
+    L->engine = ENG_ONESHOT;
     L->fn = (const void *)solve_kernel(h->plan, h->proto);
-    L->kind = 0;
+    L->cta = cta;
     L->grid = dim3((unsigned)((h->n_tasks + warps - 1) / warps));
     L->block = dim3((unsigned)cta);
     L->smem = solve_smem_bytes(cta, h->stage && h->plan != PLAN_WARP);
-    L->key = 4000000 + (h->plan * 2 + h->proto) * 100000 + cta;
-    L->key ^= (int)L->grid.x * 7919;
+    L->key = (4000000 + (h->plan * 2 + h->proto) * 100000 + cta) ^ (int)L->grid.x * 7919;
     return SPTRSV_OK;
 }
 
@@ -873,15 +756,18 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     if (h->n == 0) return SPTRSV_OK;
     if (!b || !x || b == x) return SPTRSV_ERR_INVALID_ARG;
     cudaStream_t s = (cudaStream_t)stream;
-    const bool aligned =
-        ((((uintptr_t)h->rowptr) | ((uintptr_t)h->colidx) | ((uintptr_t)h->val) | ((uintptr_t)b)) & 15) == 0;
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != h->device) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_INVALID_ARG;  // the handle's device must be current (its stream, its workspace)
+    }
     Launch L;
-    int rc = plan_launch(h, aligned, &L);
+    int rc = plan_launch(h, &L);
     if (rc) return rc;
     // The epoch of a solve is derived on the device from the start ticket and the
     // grid size (solve.cuh SolveState); a new launch configuration, or an epoch
     // about to wrap, re-zeroes the flags / records and the counters first.
-    if (L.key != h->launch_key || h->since_reset >= kEpochResetAt) {
+    if (L.key != h->launch_key || reset_due(h->since_reset, L.grid.x)) {
         rc = reset_state(h, s);
         if (rc) return rc;
         h->launch_key = L.key;
@@ -900,6 +786,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.n = h->n;
     p.n_tasks = h->n_tasks;
     p.epoch0 = 1;
+    p.gen = h->gen;
     p.grid = L.grid.x;
     p.backoff_min = h->backoff_min;
     p.backoff_max = h->backoff_max;
@@ -920,14 +807,9 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     cfg.blockDim = L.block;
     cfg.dynamicSmemBytes = L.smem;
     cfg.stream = s;
-    cudaLaunchAttribute attr[2];
+    cudaLaunchAttribute attr[1];
     cfg.numAttrs = 0;
     cfg.attrs = attr;
-    if (L.coop) {
-        attr[cfg.numAttrs].id = cudaLaunchAttributeCooperative;
-        attr[cfg.numAttrs].val.cooperative = 1;
-        cfg.numAttrs++;
-    }
     // The ready words (FLAGS: flags, FUSED: records) in a persisting L2 window -- north_star's
     // "L2 access-policy window pinning the flags".  They are the handle's workspace, re-read by
     // every dependent row and re-written every solve; persisting lines are not evicted by the
@@ -947,11 +829,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
         a.val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
         a.val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
     }
-    cudaError_t e;
-    if (L.kind == 1)
-        e = cudaLaunchKernelEx(&cfg, (void (*)(SolveParams, PipeGeom))L.fn, p, L.geom);
-    else
-        e = cudaLaunchKernelEx(&cfg, (void (*)(SolveParams))L.fn, p);
+    const cudaError_t e = cudaLaunchKernelEx(&cfg, (void (*)(SolveParams))L.fn, p);
     if (e != cudaSuccess) {
         (void)cudaGetLastError();
         return SPTRSV_ERR_CUDA;
@@ -978,8 +856,16 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
     if (nrhs < 1 || nrhs > 32 || ldb < nrhs || ldx < nrhs) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!B || !X || (const double *)X == B) return SPTRSV_ERR_INVALID_ARG;
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != h->device) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_INVALID_ARG;
+    }
     cudaStream_t s = (cudaStream_t)stream;
-    if (h->tri || (!h->variant && resolve_engine(h) == 7)) {
+    Launch L0;
+    int rc0 = plan_launch(h, &L0);
+    if (rc0) return rc0;
+    if (h->tri || L0.engine == ENG_CHAIN) {
         // Column by column through the handle's own engine: f4 (upper / unit) handles, and plans
         // that run CHAIN, whose in-register chains are worth more than k_solve_multi's one hop per
         // row for all columns (c3, 8 columns: 77 ms in k_solve_multi, 8 x 5 ms here).  Each column
@@ -1024,10 +910,12 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
     const int rows_per_cta = 256 / g;
     const unsigned grid = (unsigned)((h->n + rows_per_cta - 1) / rows_per_cta);
     const long long key = ((long long)grid << 8) | ((long long)nrhs << 1) | h->proto;
-    if (key != h->mlaunch_key || h->msince_reset >= kEpochResetAt) {
+    if (key != h->mlaunch_key || reset_due(h->msince_reset, grid)) {
         CK(cudaMemsetAsync(h->ws.mflags, 0, 4 * words, s));
         CK(cudaMemsetAsync(h->ws.mrec, 0, 16 * words, s));
-        CK(cudaMemsetAsync(h->ws.mst, 0, sizeof(SolveState), s));
+        h->mgen = (h->mgen + 1) & 0xFFFFFFu;
+        const int rc = init_state(h->ws.mst, h->mgen, s);
+        if (rc) return rc;
         h->mlaunch_key = key;
         h->msince_reset = 0;
     }
@@ -1042,6 +930,7 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
     p.n = h->n;
     p.n_tasks = h->n_tasks;
     p.epoch0 = 1;
+    p.gen = h->mgen;
     p.grid = grid;
     p.backoff_min = h->backoff_min;
     p.backoff_max = h->backoff_max;
@@ -1073,6 +962,14 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!b_host || !x_host) return SPTRSV_ERR_INVALID_ARG;
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != h->device) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_INVALID_ARG;
+    }
+    Launch L0;
+    const int rc0 = plan_launch(h, &L0);
+    if (rc0) return rc0;
     const size_t bytes = sizeof(double) * (size_t)h->n;
     if (!h->ws.b_stage) {
         if (cudaMalloc(&h->ws.b_stage, bytes) != cudaSuccess) {
@@ -1110,9 +1007,9 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
     }
     if ((io & 1) && !write_value32()) io &= ~1;
     // engines that take the chunked b (wait_b_chunks) and, for LEAN / CHAIN, write x per CTA / warp
-    const int eng = h->variant ? -1 : resolve_engine(h);
-    const bool gated = (eng == 3 || eng == 7) ? h->plan == PLAN_THREAD : eng == 6;
-    if (!(eng == 3 || eng == 7)) io &= ~2;
+    const int eng = L0.engine;
+    const bool gated = eng == ENG_LEAN || eng == ENG_CHAIN || eng == ENG_HYBRID;
+    if (!(eng == ENG_LEAN || eng == ENG_CHAIN)) io &= ~2;
     if (pinned && io && gated) {
         const uint32_t *bflag = nullptr;
         uint32_t seq = 0;
@@ -1174,14 +1071,22 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
 
 int sptrsv_destroy(sptrsv_handle_t h) {
     if (!h) return SPTRSV_OK;
-    int prev = 0;
-    cudaGetDevice(&prev);
-    cudaSetDevice(h->device);
+    DeviceGuard g(h->device);
     cudaDeviceSynchronize();
-    if (h->l2_window && h->l2_hit > 0.f) cudaCtxResetPersistingL2Cache();  // demote this handle's lines
+    if (h->l2_user) {
+        // demote this handle's persisting lines only (a context-wide reset would demote every
+        // other handle's window too): discard the window's L2 lines -- the records are dead
+        void *wbase = h->proto == PROTO_FLAGS ? (void *)h->ws.flags : (void *)h->ws.rec;
+        const size_t wbytes = (h->proto == PROTO_FLAGS ? sizeof(uint32_t) : 16) * (size_t)h->n;
+        if (wbase) {
+            k_l2_discard<<<(unsigned)std::min<size_t>((wbytes / 128 + 255) / 256, 4096), 256>>>(
+                (char *)wbase, wbytes);
+            cudaDeviceSynchronize();
+        }
+        l2_limit_release(h);
+    }
     (void)cudaGetLastError();
     free_ws(h->ws);
-    cudaSetDevice(prev);
     delete h;
     return SPTRSV_OK;
 }
@@ -1190,6 +1095,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->tri && key == SPTRSV_OPT_VARIANT && value != 0)
         return SPTRSV_ERR_INVALID_ARG;  // the paper's kernels are lower-only
+    DeviceGuard g(h->device);
     switch (key) {
         case SPTRSV_OPT_MODE:
             if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
@@ -1244,23 +1150,13 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->local = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
-            if (value < 0 || value > 8) return SPTRSV_ERR_INVALID_ARG;
+            if (value != ENG_ONESHOT && value != ENG_LEAN && value != ENG_AUTO && value != ENG_HYBRID &&
+                value != ENG_CHAIN && value != ENG_CHAINP)
+                return SPTRSV_ERR_INVALID_ARG;
             h->engine = (int)value;
             return SPTRSV_OK;
-        case SPTRSV_OPT_PIPE_STAGES:
-            if (value < 2 || value > 8) return SPTRSV_ERR_INVALID_ARG;
-            h->pipe_stages = (int)value;
-            return SPTRSV_OK;
-        case SPTRSV_OPT_PIPE_BATCH:
-            if (value < 1 || value > 32) return SPTRSV_ERR_INVALID_ARG;
-            h->pipe_batch = (int)value;
-            return SPTRSV_OK;
-        case SPTRSV_OPT_PIPE_ENTRIES:
-            if (value < 0 || value > (1 << 16)) return SPTRSV_ERR_INVALID_ARG;
-            h->pipe_entries = (int)value;
-            return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE:
-            if (value < 0 || value > 4) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
             h->rows_per_lane = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT:
@@ -1268,9 +1164,8 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->variant = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_LEAN_OCCUPANCY:
-            if (value < 2 || value > 8) return SPTRSV_ERR_INVALID_ARG;
-            if (value >= 5) h->lean_minb = (int)value;  // LEAN: 5..8
-            h->lk_occ = (int)value;                     // LEAN_K: per K, see lean_k_kernel
+            if (value < 5 || value > 8) return SPTRSV_ERR_INVALID_ARG;
+            h->lean_minb = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_PREFETCH:
             if (value < -1 || value > (1 << 24)) return SPTRSV_ERR_INVALID_ARG;
@@ -1312,9 +1207,6 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_PROTOCOL: *value = h->proto; return SPTRSV_OK;
         case SPTRSV_OPT_LOCAL: *value = h->local; return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE: *value = h->engine; return SPTRSV_OK;
-        case SPTRSV_OPT_PIPE_STAGES: *value = h->pipe_stages; return SPTRSV_OK;
-        case SPTRSV_OPT_PIPE_BATCH: *value = h->pipe_batch; return SPTRSV_OK;
-        case SPTRSV_OPT_PIPE_ENTRIES: *value = h->pipe_entries; return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE: *value = h->rows_per_lane; return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT: *value = h->variant; return SPTRSV_OK;
         case SPTRSV_OPT_LEAN_OCCUPANCY: *value = h->lean_minb; return SPTRSV_OK;
@@ -1342,14 +1234,19 @@ int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
     out->warp_deps = h->warp_deps;
     out->prev_deps = h->prev_deps;
     out->near_rows = h->near_rows;
-    out->engine = resolve_engine(h);
-    effective_geometry(h, out->engine, &out->cta_threads, &out->rows_per_lane);
+    Launch L;
+    const int rc = plan_launch(h, &L);
+    if (rc) return rc;
+    out->engine = L.engine;
+    out->cta_threads = L.cta;
+    out->rows_per_lane = L.K;
     return SPTRSV_OK;
 }
 
 int sptrsv_get_indegree(sptrsv_handle_t h, int32_t *out_dev, sptrsv_stream_t stream) {
     if (!h || (!out_dev && h->n > 0)) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
+    DeviceGuard g(h->device);
     CK(cudaMemcpyAsync(out_dev, h->ws.indeg, sizeof(int32_t) * (size_t)h->n, cudaMemcpyDeviceToDevice,
                        (cudaStream_t)stream));
     return SPTRSV_OK;
@@ -1360,6 +1257,7 @@ int sptrsv_levels(sptrsv_handle_t h, int32_t *level_dev, int32_t *counts_dev, in
     if (!h || !nlevels_host || h->tri) return SPTRSV_ERR_INVALID_ARG;
     *nlevels_host = 0;
     if (h->n == 0) return SPTRSV_OK;
+    DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
     const size_t n = (size_t)h->n;
     if (!h->ws.lvl) {
@@ -1390,6 +1288,7 @@ int sptrsv_set_trace(sptrsv_handle_t h, uint64_t *trace_dev) {
 
 int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
+    DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
     CK(cudaStreamSynchronize(s));
     uint32_t err = 0, merr = 0;
@@ -1399,16 +1298,84 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
         if (merr) {
             CK(cudaMemset(h->ws.mst, 0, sizeof(SolveState)));
             h->mlaunch_key = -1;
-            return SPTRSV_ERR_TIMEOUT;
         }
     }
     if (err) {
         CK(cudaMemset(&h->ws.st->error.v, 0, sizeof(uint32_t)));
         CK(cudaMemset(&h->ws.st->abort.v, 0, sizeof(uint32_t)));
         h->launch_key = -1;  // flags of the aborted solve are partial: re-zero before the next one
-        return SPTRSV_ERR_TIMEOUT;
     }
-    return SPTRSV_OK;
+    const uint32_t e = err ? err : merr;
+    if (e == kErrStale) return SPTRSV_ERR_STALE_LAUNCH;
+    return e ? SPTRSV_ERR_TIMEOUT : SPTRSV_OK;
+}
+
+int sptrsv_hop_scan(int32_t iters, int32_t protocol, int32_t capacity, int32_t *sm_a_out, int32_t *sm_b_out,
+                    double *ns_out, int32_t *count) {
+    if (iters <= 0 || (protocol != 0 && protocol != 1) || capacity < 0 || !count || !sm_a_out ||
+        (capacity > 0 && (!sm_b_out || !ns_out)))
+        return SPTRSV_ERR_INVALID_ARG;
+    *count = 0;
+    int dev = 0, nsm = 0, smem_sm = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) ||
+        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev)) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_CUDA;
+    }
+    const int smem = smem_sm / 2 + 1024;  // > half an SM: one CTA per SM
+    if (cudaFuncSetAttribute(k_smids, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
+        cudaFuncSetAttribute(k_pingpong_sm, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return SPTRSV_ERR_CUDA;
+    }
+    unsigned long long *rec = nullptr, *ns = nullptr;
+    uint32_t *flags = nullptr;
+    double *xs = nullptr, *sink = nullptr;
+    int32_t *ids = nullptr;
+    int rc = SPTRSV_OK;
+    do {
+        if (cudaMalloc(&rec, 512) != cudaSuccess || cudaMalloc(&flags, 512) != cudaSuccess ||
+            cudaMalloc(&xs, 512) != cudaSuccess || cudaMalloc(&sink, 16) != cudaSuccess ||
+            cudaMalloc(&ns, 16) != cudaSuccess || cudaMalloc(&ids, sizeof(int32_t) * nsm) != cudaSuccess) {
+            rc = SPTRSV_ERR_ALLOC;
+            break;
+        }
+        std::vector<int32_t> h_ids(nsm);
+        k_smids<<<nsm, 32, smem>>>(ids);
+        if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess ||
+            cudaMemcpy(h_ids.data(), ids, sizeof(int32_t) * nsm, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            rc = SPTRSV_ERR_CUDA;
+            break;
+        }
+        std::sort(h_ids.begin(), h_ids.end());
+        h_ids.erase(std::unique(h_ids.begin(), h_ids.end()), h_ids.end());
+        const int a = h_ids[0];
+        *sm_a_out = a;
+        for (size_t k = 1; k < h_ids.size() && *count < capacity; ++k) {
+            if (cudaMemset(rec, 0, 512) != cudaSuccess || cudaMemset(flags, 0, 512) != cudaSuccess) {
+                rc = SPTRSV_ERR_CUDA;
+                break;
+            }
+            k_pingpong_sm<<<nsm, 32, smem>>>(rec, flags, xs, iters, protocol, a, h_ids[k], ns, sink);
+            unsigned long long t = 0;
+            if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess ||
+                cudaMemcpy(&t, ns, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+                rc = SPTRSV_ERR_CUDA;
+                break;
+            }
+            sm_b_out[*count] = h_ids[k];
+            ns_out[*count] = (double)t / (2.0 * iters);
+            ++*count;
+        }
+    } while (0);
+    (void)cudaGetLastError();
+    cudaFree(rec);
+    cudaFree(flags);
+    cudaFree(xs);
+    cudaFree(sink);
+    cudaFree(ns);
+    cudaFree(ids);
+    return rc;
 }
 
 int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop, double *sm_mhz) {

@@ -39,7 +39,7 @@ def test_library_exports_every_declared_symbol(libpath):
 def test_binding_covers_header_and_loads(libpath):
     import paper_conf_icpp_suz0hw0w20_b200._lib as L
     assert sorted(L.EXPORTS) == _declared()
-    assert L.lib.sptrsv_abi_version() == 2
+    assert L.lib.sptrsv_abi_version() == 3
     assert L.lib.sptrsv_strerror(-3).decode().startswith("row without a diagonal")
     # argument validation happens before any CUDA call
     assert L.lib.sptrsv_analyse_csr(-1, None, None, None, None) == L.ERR_INVALID_ARG
@@ -81,3 +81,28 @@ def test_only_tests_smoke_and_bench_touch_the_oracle():
                 if f.endswith((".py", ".cu", ".cuh", ".h", ".c")):
                     txt = open(os.path.join(dp, f)).read()
                     assert "import oracle" not in txt and "from oracle" not in txt, os.path.join(dp, f)
+
+
+def test_reference_arm_loads_no_product_library():
+    """bench.py --impl reference runs the oracle only: the product package (and libsptrsv.so)
+    must not be imported, so the driver's native-library census of that arm lists oracle/ alone."""
+    code = ("import sys, bench; a = bench.parse(['--impl', 'reference', '--config', 'c1', '--steps', '2', "
+            "'--warmup', '1']); bench.run_reference(a, 0, 1); "
+            "assert not any(m.startswith('paper_conf_icpp_suz0hw0w20_b200') for m in sys.modules), 'product imported'; "
+            "import os; maps = open('/proc/self/maps').read(); assert 'libsptrsv' not in maps")
+    r = subprocess.run(["python", "-c", code], cwd=ROOT, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    line = [l for l in r.stdout.splitlines() if l.startswith("{")][-1]
+    import json
+    d = json.loads(line)
+    assert d["impl"] == "reference" and d["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_bench_defaults():
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    assert bench.parse([]).config == "c2" and bench.parse([]).gpus == 1
+    assert bench.parse(["--gpus", "4"]).config == "c5"
+    a = bench.parse(["--gpus", "2", "--config", "c2"])
+    assert a.config == "c2"

@@ -48,7 +48,7 @@ def relerr(a, ref):
 
 MODES = [0, 1, 2]
 PROTOS = [0, 1]  # 0 FLAGS (release/acquire), 1 FUSED (epoch-tagged value records)
-ENGINES = [0, 1]  # 0 one-shot k_solve, 1 pipelined k_solve_pipe (TMA ring + loader warp)
+ENGINES = [0, 3]  # 0 one-shot k_solve (staged, in-CTA x copy), 3 LEAN
 
 
 # ------------------------------------------------------------------ small, many tiles + ragged tails
@@ -370,59 +370,6 @@ def test_indegree_and_levels_bit_exact(cap, gen):
         assert np.array_equal(counts.cpu().numpy(), ocounts)
 
 
-@pytest.mark.parametrize("stages,batch,entries,cta", [(2, 1, 0, 64), (3, 2, 0, 256), (4, 4, 64, 256),
-                                                      (8, 32, 0, 1024), (2, 3, 100, 512)])
-def test_pipe_geometry_variants(cap, stages, batch, entries, cta):
-    """Ring depth, ticket batch, stage capacity (tiny -> direct global reads) and CTA size."""
-    for gen in (lambda: synth.gen_c2i(n=60_000), lambda: synth.gen_c4(n=8_000, nlevels=40),
-                lambda: synth.gen_random_lower(5000, 6, seed=9)):
-        s = gen()
-        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-        for proto in PROTOS:
-            x, _ = gpu_solve(cap, s, 0, engine=1, pipe_stages=stages, pipe_batch=batch, pipe_entries=entries,
-                             cta_threads=cta, protocol=proto)
-            assert relerr(x, ref) <= TOL
-
-
-@pytest.mark.parametrize("K", [2, 3, 4])
-@pytest.mark.parametrize("proto", PROTOS)
-def test_rows_per_lane(cap, K, proto):
-    """K thread-level rows per lane (coarsened Writing-First): bit-exact like K = 1."""
-    for n in (1, 31, 33, 200, 4099):
-        s = synth.gen_random_lower(n, 4, seed=n + 7)
-        x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K)
-        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
-    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=100_000), lambda: synth.gen_grid(300),
-                lambda: synth.gen_chain(20_000), lambda: synth.gen_dense_lower(120)):
-        s = gen()
-        for local, cta in ((1, 256), (0, 256), (1, 128), (1, 64)):
-            x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K, local=local, cta_threads=cta)
-            assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), (s.name, local, cta)
-    si = synth.integerize(synth.gen_c2i(n=50_000))
-    x, _ = gpu_solve(cap, si, 1, protocol=proto, rows_per_lane=K)
-    assert np.array_equal(x, si.x_true)
-
-
-@pytest.mark.parametrize("K", [1, 2, 4])
-@pytest.mark.parametrize("proto", PROTOS)
-@pytest.mark.parametrize("engine", [2, 4])
-def test_dyn_engine(cap, K, proto, engine):
-    """ENGINE_DYN (rows re-assigned to lane slots as they finish): bit-exact like the others."""
-    for n in (1, 31, 33, 129, 200, 4099):
-        s = synth.gen_random_lower(n, 4, seed=n + 11)
-        x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K, engine=engine)
-        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
-    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=300_000), lambda: synth.gen_grid(200),
-                lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100)):
-        s = gen()
-        for cta in (256, 64):
-            x, _ = gpu_solve(cap, s, 1, protocol=proto, rows_per_lane=K, engine=engine, cta_threads=cta)
-            assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), (s.name, cta)
-    si = synth.integerize(synth.gen_c2i(n=50_000))
-    x, _ = gpu_solve(cap, si, 1, protocol=proto, rows_per_lane=K, engine=engine)
-    assert np.array_equal(x, si.x_true)
-
-
 @pytest.mark.parametrize("proto", PROTOS)
 def test_lean_engine(cap, proto):
     """ENGINE_LEAN (no staging, speculative rows): bit-exact like the others."""
@@ -441,65 +388,42 @@ def test_lean_engine(cap, proto):
     assert np.array_equal(x, si.x_true)
 
 
-@pytest.mark.parametrize("proto", PROTOS)
-@pytest.mark.parametrize("K,cta,occ", [(2, 256, 0), (2, 128, 0), (2, 256, 3), (2, 256, 5), (3, 256, 0), (3, 128, 2),
-                                       (4, 256, 0), (4, 256, 3), (4, 128, 0)])
-def test_lean_k_engine(cap, proto, K, cta, occ):
-    """ENGINE_LEAN_K (8): K rows per lane, two preloaded dependencies per row, row constants in smem:
-    bit-exact like every thread-level path -- ragged tails (n not a multiple of 32K or of the CTA's
-    rows), rows longer than the two preloaded entries (dense), in-warp chains (same lane, k-strided
-    rows), grids, interleaved levels, diagonal-only; exact-integer systems give x_true."""
-    opts = dict(protocol=proto, engine=8, rows_per_lane=K, cta_threads=cta)
-    if occ:
-        opts["lean_occupancy"] = occ
-    for n in (1, 31, 33, 63, 65, 255, 257, 1023, 1025, 4099):
-        s = synth.gen_random_lower(n, 4, seed=n + 19)
-        x, info = gpu_solve(cap, s, 1, **opts)
-        assert info["engine"] == 8 and info["rows_per_lane"] == K and info["cta_threads"] == cta, info
-        assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
-    for gen in (lambda: synth.gen_c2i(n=200_000), lambda: synth.gen_c2(n=300_000), lambda: synth.gen_grid(200),
-                lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100), lambda: synth.gen_diag(70_001),
-                lambda: synth.gen_c1()):
-        s = gen()
-        x, _ = gpu_solve(cap, s, 1, **opts)
-        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-        assert np.array_equal(x, ref), s.name
-    si = synth.integerize(synth.gen_c2i(n=50_000))
-    x, _ = gpu_solve(cap, si, 1, **opts)
-    assert np.array_equal(x, si.x_true)
+CHAIN_ENGINES = [7, 8]
 
 
 @pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("K", [1, 2])
 @pytest.mark.parametrize("cta", [64, 128, 256])
-def test_chain_engine(cap, proto, K, cta):
+@pytest.mark.parametrize("eng", CHAIN_ENGINES)
+def test_chain_engine(cap, proto, K, cta, eng):
     """ENGINE_CHAIN (in-warp dependencies resolved by a warp-sequential shuffle chain): bit-exact
     like every thread-level path -- ragged tails, slices longer than the staging cap (dense rows),
     chains, grids, far and interleaved dependencies, diagonal-only."""
     for n in (1, 31, 33, 63, 65, 255, 257, 4099):
         s = synth.gen_random_lower(n, 4, seed=n + 17)
-        x, info = gpu_solve(cap, s, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
-        assert info["engine"] == 7
+        x, info = gpu_solve(cap, s, 1, protocol=proto, engine=eng, rows_per_lane=K, cta_threads=cta)
+        assert info["engine"] == eng
         assert np.array_equal(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)), n
     for gen in (lambda: synth.gen_c2i(n=100_000), lambda: synth.gen_c2(n=200_000), lambda: synth.gen_grid(200),
                 lambda: synth.gen_chain(5_000), lambda: synth.gen_dense_lower(100), lambda: synth.gen_diag(70_001),
                 lambda: synth.gen_c1()):
         s = gen()
-        x, _ = gpu_solve(cap, s, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+        x, _ = gpu_solve(cap, s, 1, protocol=proto, engine=eng, rows_per_lane=K, cta_threads=cta)
         ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
         assert np.array_equal(x, ref), s.name
     si = synth.integerize(synth.gen_c2i(n=50_000))
-    x, _ = gpu_solve(cap, si, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+    x, _ = gpu_solve(cap, si, 1, protocol=proto, engine=eng, rows_per_lane=K, cta_threads=cta)
     assert np.array_equal(x, si.x_true)
     sc = synth.gen_chain(10_000)  # closed form x_i = 1 - 2^-(i+1) (i <= 52), 1 after
-    x, _ = gpu_solve(cap, sc, 1, protocol=proto, engine=7, rows_per_lane=K, cta_threads=cta)
+    x, _ = gpu_solve(cap, sc, 1, protocol=proto, engine=eng, rows_per_lane=K, cta_threads=cta)
     i = np.arange(sc.n)
     assert np.array_equal(x, np.where(i <= 52, 1.0 - np.ldexp(1.0, -(np.minimum(i, 52) + 1)), 1.0))
 
 
 @pytest.mark.parametrize("proto", PROTOS)
 @pytest.mark.parametrize("K", [1, 2])
-def test_chain_engine_division_guard_exits(cap, proto, K):
+@pytest.mark.parametrize("eng", CHAIN_ENGINES)
+def test_chain_engine_division_guard_exits(cap, proto, K, eng):
     """CHAIN's fast (bidiagonal / grid-west) loop leaves to the exact loop when the Markstein
     range guard fails (|a| or |L_ii| outside [2^-400, 2^401)): chains whose diagonals and
     right-hand sides span 2^+-600 -- guard failures at arbitrary steps, overflow, underflow --
@@ -519,8 +443,8 @@ def test_chain_engine_division_guard_exits(cap, proto, K):
         bw = rng.random(n) < frac
         b[bw] = np.ldexp(b[bw], rng.integers(-600, 600, bw.sum()))
         s = synth.CSRSystem("wild", n, rp, ci, v, b, None, {})
-        x, info = gpu_solve(cap, s, 1, protocol=proto, engine=7, rows_per_lane=K)
-        assert info["engine"] == 7
+        x, info = gpu_solve(cap, s, 1, protocol=proto, engine=eng, rows_per_lane=K)
+        assert info["engine"] == eng
         ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
         assert np.array_equal(x, ref, equal_nan=True), (n, frac)
 
@@ -619,21 +543,6 @@ def test_paper_variants(cap, variant):
             assert relerr(x, ref) <= TOL, s.name
         else:
             assert np.array_equal(x, ref), s.name
-
-
-def test_pipe_unaligned_b_falls_back(cap):
-    """b at an 8-byte (not 16-byte) offset: the TMA ring needs 16-byte alignment -> one-shot engine."""
-    s = synth.gen_c2(n=20_000)
-    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-    rp, ci, v, _ = dev_csr(s)
-    store = torch.zeros(s.n + 1, dtype=torch.float64, device="cuda:0")
-    store[1:] = torch.from_numpy(s.b).cuda()
-    b_off = store[1:]
-    with cap.analyse(rp, ci, v, engine=1) as h:
-        x = torch.full_like(b_off, float("nan"))
-        h.solve(b_off, x)
-        h.check()
-        assert np.array_equal(x.cpu().numpy(), ref)
 
 
 def test_protocol_switch_on_one_handle(cap):

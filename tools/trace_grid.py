@@ -47,4 +47,14 @@ out["north_us_p50_col0"] = round(float(np.percentile(north[:, 0], 50)), 3)
 first = t[1:, ::R]
 north_last = t[:-1, R - 1::R][:, : first.shape[1]]
 out["warp_first_minus_north_warp_last_us_p10_50_90"] = q(first[:, : north_last.shape[1]] - north_last)
+# north split: [n+i] = when cell (r,c) consumed its north (external) dependency (CHAIN / LEAN)
+tc = tr.cpu().numpy().astype(np.int64)[s.n: 2 * s.n]
+if (tc[g:] > 0).mean() > 0.5:
+    t0 = tr.cpu().numpy().astype(np.int64)[: s.n].min()
+    tcu = ((tc - t0) / 1e3).reshape(g, g)
+    seen = tcu[1:, :] - t[:-1, :]      # north published -> consumed by the cell below
+    pub = t[1:, :] - tcu[1:, :]        # north consumed -> the cell's own publish
+    ok = tc.reshape(g, g)[1:, :] > 0
+    out["north_seen_us_p10_50_90"] = q(seen[ok])
+    out["north_consumed_to_publish_us_p10_50_90"] = q(pub[ok])
 print(json.dumps(out))
