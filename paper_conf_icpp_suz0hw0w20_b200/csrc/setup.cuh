@@ -13,7 +13,24 @@
 namespace sptrsv_dev {
 
 enum : int {  // same numbering as sptrsv_status (negated)
-    E_NOT_LOWER = 2, E_MISSING_DIAG = 3, E_ZERO_DIAG = 4, E_UNSORTED = 5, E_BAD_ROWPTR = 6, E_BAD_COL = 7
+    E_INVALID_ARG = 1, E_NOT_LOWER = 2, E_MISSING_DIAG = 3, E_ZERO_DIAG = 4, E_UNSORTED = 5, E_BAD_ROWPTR = 6,
+    E_BAD_COL = 7
+};
+
+// Everything analyse learns on the device, read back by the host in ONE copy at the end
+// (sptrsv.cu sptrsv_analyse_csr_ex): the whole setup is a handful of kernels on one stream.
+struct AnalyseOut {
+    unsigned long long status;   // min over ((row + 1) << 8 | code); key 0 << 8 | code: a global
+                                 // rowptr error; ~0 = valid (the lowest offending row wins)
+    long long nnz;               // rowptr[n]
+    int32_t max_row;             // longest row (entries)
+    int32_t threshold;           // AUTO warp threshold the plan used (sec.4.4)
+    int32_t med_log2;            // floor(log2(median nearest-dependency distance)), -1 = none
+    int32_t n_tasks, n_tgroups;  // plan: warp tasks, 32-row thread groups
+    int32_t pad;
+    unsigned long long near;     // near_deps | warp_deps << 32
+    unsigned long long prev;     // prev_deps | near_rows << 32
+    unsigned long long hist[32]; // rows by floor(log2(nearest-dependency distance))
 };
 
 // status: 64-bit min over (row << 8 | code) -> the lowest offending row wins,
@@ -26,11 +43,20 @@ enum : int {  // same numbering as sptrsv_status (negated)
 __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ rowptr,
                                                   const int32_t *__restrict__ colidx,
                                                   const double *__restrict__ val, int32_t n,
-                                                  int64_t nnz, int32_t *indeg,
-                                                  unsigned long long *status, int32_t *max_row,
-                                                  unsigned long long *near_deps, int tri) {
+                                                  int32_t *indeg, AnalyseOut *out, int tri) {
     const bool upper = tri & 1, unit = tri & 2;
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned long long *status = &out->status;
+    int32_t *max_row = &out->max_row;
+    unsigned long long *near_deps = &out->near;  // near, prev, hist[32] are consecutive
+    const int64_t nnz = rowptr[n];  // the nnz the caller's rowptr declares
+    if (i == 0) {
+        out->nnz = nnz;
+        if (rowptr[0] != 0 || nnz < 0) atomicMin(status, (unsigned long long)E_BAD_ROWPTR);  // key row 0: global
+        // a row with entries needs colidx / val (unit handles may pass NULL for an empty matrix)
+        if (nnz > 0 && (!colidx || (!val && !unit))) atomicMin(status, (unsigned long long)E_INVALID_ARG);
+    }
+    if (nnz > 0 && (!colidx || (!val && !unit))) return;
     int len = 0;
     unsigned near = 0, wdep = 0, pdep = 0, nrow = 0;
     int dmin = 0x7fffffff;  // the row's nearest dependency (distance in rows)
@@ -70,7 +96,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
             if ((threadIdx.x & 31) == __ffs(same) - 1)
                 atomicAdd(near_deps + 2 + bk, (unsigned long long)__popc(same));
         }
-        if (code) atomicMin(status, ((unsigned long long)i << 8) | (unsigned long long)code);
+        if (code) atomicMin(status, ((unsigned long long)(i + 1) << 8) | (unsigned long long)code);
         len = code ? 0 : (int)(e - s);
         indeg[i] = code ? 0 : (int)(e - s - (unit ? 0 : 1));
     }
@@ -133,9 +159,10 @@ __device__ __forceinline__ int block_exclusive_scan(int v, int *s_warp, int *tot
 }
 
 __global__ void __launch_bounds__(1024) k_plan_count(const int32_t *__restrict__ rowptr, int32_t n,
-                                                     int32_t ngroups, int mode, int threshold,
+                                                     int32_t ngroups, int mode, const AnalyseOut *out,
                                                      int32_t *blk_tasks, int32_t *blk_tgroups, bool rev) {
     __shared__ int s_warp[33];
+    const int threshold = out->threshold;
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
     int t = 0, tg = 0;
     if (g < ngroups) {
@@ -153,10 +180,11 @@ __global__ void __launch_bounds__(1024) k_plan_count(const int32_t *__restrict__
 }
 
 __global__ void __launch_bounds__(1024) k_plan_write(const int32_t *__restrict__ rowptr, int32_t n,
-                                                     int32_t ngroups, int mode, int threshold,
+                                                     int32_t ngroups, int mode, const AnalyseOut *out,
                                                      const int32_t *__restrict__ blk_offset,
                                                      int32_t *tasks, bool rev) {
     __shared__ int s_warp[33];
+    const int threshold = out->threshold;
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
     int t = 0;
     bool w = false;
@@ -169,6 +197,59 @@ __global__ void __launch_bounds__(1024) k_plan_write(const int32_t *__restrict__
         } else {
             tasks[off] = g * 32;  // thread task: first row of the group
         }
+    }
+}
+
+// AUTO's per-32-row-group warp threshold (mean nnz/row above which a group runs warp-level), from
+// floor(log2) of the median distance to a row's nearest dependency -- on leveled matrices about the
+// level width, which moves the thread/warp crossover (f2 sweep): < 64 rows:
+// thread level only; 64..1023: warp from 2 nnz/row; 1024..8191: from 6; wider: from 20.  A system
+// that fits one 1024-thread one-shot CTA resolves in shared memory: thread level only.
+// user >= 0: SPTRSV_OPT_WARP_THRESHOLD was set, use it.  One thread.
+__global__ void k_auto_threshold(AnalyseOut *out, int32_t n, int32_t user) {
+    unsigned long long tot = 0, acc = 0;
+    for (int k = 0; k < 32; ++k) tot += out->hist[k];
+    int med = -1;
+    for (int k = 0; k < 32 && tot; ++k) {
+        acc += out->hist[k];
+        if (2 * acc >= tot) {
+            med = k;
+            break;
+        }
+    }
+    out->med_log2 = med;
+    int t;
+    if (user >= 0) t = user;
+    else if (n <= 1024) t = 1 << 30;
+    else if (med < 0) t = 16;  // no dependencies at all
+    else if (med <= 5) t = 1 << 30;
+    else if (med <= 9) t = 2;
+    else if (med <= 12) t = 6;
+    else t = 20;
+    out->threshold = t;
+}
+
+// exclusive scan of the per-block task / thread-group counts (one CTA, any number of blocks):
+// blk_offset[b] = tasks before block b; out->n_tasks / n_tgroups = the totals
+__global__ void __launch_bounds__(1024) k_plan_scan(const int32_t *__restrict__ blk_tasks,
+                                                    const int32_t *__restrict__ blk_tgroups, int32_t nb,
+                                                    int32_t *blk_offset, AnalyseOut *out) {
+    __shared__ int s_warp[33];
+    long long carry = 0, carry_g = 0;
+    for (int b0 = 0; b0 < nb; b0 += blockDim.x) {
+        const int b = b0 + threadIdx.x;
+        const int v = b < nb ? blk_tasks[b] : 0;
+        const int g = b < nb ? blk_tgroups[b] : 0;
+        int tot, totg;
+        const int ex = block_exclusive_scan(v, s_warp, &tot);
+        block_exclusive_scan(g, s_warp, &totg);
+        if (b < nb) blk_offset[b] = (int32_t)(carry + ex);
+        carry += tot;
+        carry_g += totg;
+    }
+    if (threadIdx.x == 0) {
+        out->n_tasks = (int32_t)carry;
+        out->n_tgroups = (int32_t)carry_g;
     }
 }
 

@@ -33,12 +33,18 @@ constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the
 // engines (SPTRSV_OPT_ENGINE values, include/sptrsv.h)
 enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_CHAINP = 8 };
 
+// The handle's workspace is ONE device allocation (analyse is O(nnz) work plus a fixed handful of
+// runtime calls), carved in 256-byte aligned pieces: the 16-byte FUSED records, the FLAGS words,
+// in-degrees, the task list (at most n tasks), the solve state and the analyse results / scratch.
 struct Workspace {
+    void *base = nullptr;          // the single allocation below
     uint32_t *flags = nullptr;     // n      (PROTO_FLAGS)
-    unsigned long long *rec = nullptr;  // 2n (PROTO_FUSED, lazy)
+    unsigned long long *rec = nullptr;  // 2n (PROTO_FUSED)
     int32_t *indeg = nullptr;      // n
-    int32_t *tasks = nullptr;      // n_tasks (PLAN_LIST only)
+    int32_t *tasks = nullptr;      // n (PLAN_LIST uses n_tasks <= n of them)
     SolveState *st = nullptr;      // 1
+    AnalyseOut *aout = nullptr;    // 1: analyse results (one D2H copy)
+    int32_t *blk = nullptr;        // 3 * nb: plan block counts / thread groups / offsets
     uint32_t *lvl = nullptr;       // n (levels diagnostic, lazy)
     double *b_stage = nullptr;     // n (solve_host, lazy)
     SolveState *mst = nullptr;     // multi-RHS: own solve state (own epoch sequence)
@@ -215,11 +221,7 @@ int set_kernel_attrs() {
 }
 
 void free_ws(Workspace &w) {
-    cudaFree(w.flags);
-    cudaFree(w.rec);
-    cudaFree(w.indeg);
-    cudaFree(w.tasks);
-    cudaFree(w.st);
+    cudaFree(w.base);
     cudaFree(w.lvl);
     cudaFree(w.b_stage);
     cudaFree(w.mst);
@@ -233,77 +235,44 @@ void free_ws(Workspace &w) {
     w = Workspace();
 }
 
-// Build the row-ordered task list for the current mode/threshold (synchronous).
-int build_plan(sptrsv_handle_s *h) {
+// Enqueue the plan kernels (AUTO threshold, per-block counts, one-CTA scan, task list) on stream
+// s: the plan is built on the device from rowptr alone (sec.4.4's nnz-per-row pass, no level
+// analysis); the host reads AnalyseOut afterwards.
+int enqueue_plan(sptrsv_handle_s *h, cudaStream_t s) {
     const int32_t n = h->n;
     const int32_t ngroups = (n + 31) / 32;
-    if (ngroups == 0) {
-        h->n_tasks = 0;
-        h->n_thread_groups = 0;
-        h->n_warp_rows = 0;
-        h->plan = PLAN_THREAD;
-        return SPTRSV_OK;
-    }
+    if (ngroups == 0) return SPTRSV_OK;
     const int nb = (ngroups + 1023) / 1024;
-    int32_t *d_bt = nullptr, *d_bg = nullptr, *d_off = nullptr;
-    std::vector<int32_t> bt(nb), bg(nb), off(nb);
-    int rc = SPTRSV_OK;
-    do {
-        if (cudaMalloc(&d_bt, sizeof(int32_t) * nb) != cudaSuccess ||
-            cudaMalloc(&d_bg, sizeof(int32_t) * nb) != cudaSuccess ||
-            cudaMalloc(&d_off, sizeof(int32_t) * nb) != cudaSuccess) {
-            rc = SPTRSV_ERR_ALLOC;
-            break;
-        }
-        const bool rev = h->tri & SPTRSV_TRI_UPPER;  // f4 upper: plan over logical (reversed) rows
-        k_plan_count<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_bt, d_bg, rev);
-        if (cudaGetLastError() != cudaSuccess ||
-            cudaMemcpy(bt.data(), d_bt, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(bg.data(), d_bg, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess) {
-            rc = SPTRSV_ERR_CUDA;
-            break;
-        }
-        int64_t tot = 0, tg = 0;
-        for (int b = 0; b < nb; ++b) {
-            off[b] = (int32_t)tot;
-            tot += bt[b];
-            tg += bg[b];
-        }
-        h->n_tasks = (int32_t)tot;
-        h->n_thread_groups = (int32_t)tg;
-        h->n_warp_rows = (int32_t)(tot - tg);  // every warp-level group contributes one task per row
-        if (tg == ngroups) {
-            h->plan = PLAN_THREAD;  // implicit mapping: task t = rows [32t, 32t+32)
-        } else if (tg == 0) {
-            h->plan = PLAN_WARP;    // implicit mapping: task t = row t
-        } else {
-            h->plan = PLAN_LIST;
-            if (h->n_tasks > h->n_tasks_cap) {
-                cudaFree(h->ws.tasks);
-                h->ws.tasks = nullptr;
-                if (cudaMalloc(&h->ws.tasks, sizeof(int32_t) * (size_t)h->n_tasks) != cudaSuccess) {
-                    h->n_tasks_cap = 0;
-                    rc = SPTRSV_ERR_ALLOC;
-                    break;
-                }
-                h->n_tasks_cap = h->n_tasks;
-            }
-            if (cudaMemcpy(d_off, off.data(), sizeof(int32_t) * nb, cudaMemcpyHostToDevice) != cudaSuccess) {
-                rc = SPTRSV_ERR_CUDA;
-                break;
-            }
-            k_plan_write<<<nb, 1024>>>(h->rowptr, n, ngroups, h->mode, h->threshold, d_off, h->ws.tasks, rev);
-            if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
-                rc = SPTRSV_ERR_CUDA;
-                break;
-            }
-        }
-    } while (0);
-    if (rc != SPTRSV_OK) (void)cudaGetLastError();
-    cudaFree(d_bt);
-    cudaFree(d_bg);
-    cudaFree(d_off);
-    return rc;
+    const bool rev = h->tri & SPTRSV_TRI_UPPER;  // f4 upper: plan over logical (reversed) rows
+    int32_t *bt = h->ws.blk, *bg = bt + nb, *off = bg + nb;
+    k_auto_threshold<<<1, 1, 0, s>>>(h->ws.aout, n, h->threshold_user ? h->threshold : -1);
+    k_plan_count<<<nb, 1024, 0, s>>>(h->rowptr, n, ngroups, h->mode, h->ws.aout, bt, bg, rev);
+    k_plan_scan<<<1, 1024, 0, s>>>(bt, bg, nb, off, h->ws.aout);
+    k_plan_write<<<nb, 1024, 0, s>>>(h->rowptr, n, ngroups, h->mode, h->ws.aout, off, h->ws.tasks, rev);
+    CK(cudaGetLastError());
+    return SPTRSV_OK;
+}
+
+// the plan's shape from the read-back results
+void adopt_plan(sptrsv_handle_s *h, const AnalyseOut &o) {
+    const int32_t ngroups = (h->n + 31) / 32;
+    h->threshold = o.threshold;
+    h->dmin_log2 = o.med_log2;
+    h->n_tasks = ngroups ? o.n_tasks : 0;
+    h->n_thread_groups = ngroups ? o.n_tgroups : 0;
+    h->n_warp_rows = h->n_tasks - h->n_thread_groups;  // a warp-level group contributes one task per row
+    h->plan = (h->n_thread_groups == ngroups) ? PLAN_THREAD : (h->n_thread_groups == 0 ? PLAN_WARP : PLAN_LIST);
+}
+
+// Re-plan after a MODE / WARP_THRESHOLD change (synchronous: one D2H copy).
+int build_plan(sptrsv_handle_s *h) {
+    if (h->n == 0) return SPTRSV_OK;
+    int rc = enqueue_plan(h, 0);
+    if (rc) return rc;
+    AnalyseOut o;
+    CK(cudaMemcpy(&o, h->ws.aout, sizeof(o), cudaMemcpyDeviceToHost));
+    adopt_plan(h, o);
+    return SPTRSV_OK;
 }
 
 // discard.global.L2 over [p, p + bytes) (whole 128-B lines inside the range): drops a dead window's
@@ -331,7 +300,7 @@ int reset_state(sptrsv_handle_s *h, cudaStream_t s) {
     // flags / records := 0 (no epoch matches), counters := 0 under a new generation; the next
     // solve has epoch 1
     CK(cudaMemsetAsync(h->ws.flags, 0, sizeof(uint32_t) * (size_t)(h->n > 0 ? h->n : 1), s));
-    if (h->ws.rec) CK(cudaMemsetAsync(h->ws.rec, 0, 16 * (size_t)(h->n > 0 ? h->n : 1), s));
+    CK(cudaMemsetAsync(h->ws.rec, 0, 16 * (size_t)(h->n > 0 ? h->n : 1), s));
     h->gen = (h->gen + 1) & 0xFFFFFFu;
     h->since_reset = 0;
     return init_state(h->ws.st, h->gen, s);
@@ -375,18 +344,6 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, 
 }
 
 void size_l2_window(sptrsv_handle_s *h);
-// AUTO's per-32-row-group warp threshold (mean nnz/row above which a group runs warp-level), from
-// floor(log2) of the median distance to a row's nearest dependency -- on leveled matrices about the
-// level width, which moves the thread/warp crossover (profiles/r01_ablation_final.md,
-// tools/dispatch_probe.py): < 64 rows: in-CTA / in-warp resolution wins, thread level only;
-// 64..1023: warp from 2 nnz/row; 1024..8191: from 6; wider: from 20.
-int auto_warp_threshold(int med_log2) {
-    if (med_log2 < 0) return 16;  // no dependencies at all
-    if (med_log2 <= 5) return 1 << 30;
-    if (med_log2 <= 9) return 2;
-    if (med_log2 <= 12) return 6;
-    return 20;
-}
 
 
 int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
@@ -396,7 +353,7 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
     *out = nullptr;
     if (n < 0 || (tri_flags & ~(SPTRSV_TRI_UPPER | SPTRSV_TRI_UNIT_DIAG))) return SPTRSV_ERR_INVALID_ARG;
     if (n > 0x7FFFFFFE) return SPTRSV_ERR_TOO_LARGE;
-    // colidx / val may be NULL only when nnz == 0 (unit-diagonal identity), checked below
+    // colidx / val may be NULL only when nnz == 0 (unit-diagonal identity), checked on the device
     if (!rowptr || (n > 0 && !(tri_flags & SPTRSV_TRI_UNIT_DIAG) && (!colidx || !val)))
         return SPTRSV_ERR_INVALID_ARG;
     int rc = set_kernel_attrs();
@@ -412,98 +369,68 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
     h->colidx = colidx;
     h->val = val;
     h->tri = tri_flags;
-    unsigned long long *d_status = nullptr, *d_near = nullptr;
-    int32_t *d_maxrow = nullptr;
+    // O(nnz) setup as ONE allocation, ONE memset, a fixed handful of kernels on the legacy stream
+    // and ONE device->host copy of the results (Alg.5 l.1 "MALLOC(get_value, m)", PAPER.md:307;
+    // "no preprocessing", :248): validation + in-degree + AUTO statistics (k_validate), the AUTO
+    // warp threshold, the thread/warp plan (count, scan, write), the solve state.
     do {
-        int32_t ends[2] = {0, 0};
-        if (cudaMemcpy(&ends[0], rowptr, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(&ends[1], rowptr + n, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
-            rc = SPTRSV_ERR_CUDA;
-            break;
-        }
-        if (ends[0] != 0 || ends[1] < 0) {
-            rc = SPTRSV_ERR_BAD_ROWPTR;
-            break;
-        }
-        h->nnz = ends[1];
-        if (h->nnz > 0 && (!colidx || !val)) {
-            rc = SPTRSV_ERR_INVALID_ARG;
-            break;
-        }
         const size_t nn = (size_t)(n > 0 ? n : 1);
-        if (cudaMalloc(&h->ws.flags, sizeof(uint32_t) * nn) != cudaSuccess ||
-            (h->proto == PROTO_FUSED && cudaMalloc(&h->ws.rec, 16 * nn) != cudaSuccess) ||
-            cudaMalloc(&h->ws.indeg, sizeof(int32_t) * nn) != cudaSuccess ||
-            cudaMalloc(&h->ws.st, sizeof(SolveState)) != cudaSuccess ||
-            cudaMalloc(&d_status, sizeof(unsigned long long)) != cudaSuccess ||
-            cudaMalloc(&d_maxrow, sizeof(int32_t)) != cudaSuccess ||
-            cudaMalloc(&d_near, 34 * sizeof(unsigned long long)) != cudaSuccess) {
+        const size_t ngroups = ((size_t)n + 31) / 32;
+        const size_t nb = (ngroups + 1023) / 1024;
+        auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
+        const size_t o_rec = 0, o_flags = o_rec + al(16 * nn), o_indeg = o_flags + al(4 * nn),
+                     o_tasks = o_indeg + al(4 * nn), o_st = o_tasks + al(4 * nn),
+                     o_out = o_st + al(sizeof(SolveState)), o_blk = o_out + al(sizeof(AnalyseOut)),
+                     total = o_blk + al(4 * 3 * (nb ? nb : 1));
+        if (cudaMalloc(&h->ws.base, total) != cudaSuccess) {
             rc = SPTRSV_ERR_ALLOC;
             break;
         }
-        if (cudaMemset(d_status, 0xff, sizeof(unsigned long long)) != cudaSuccess ||
-            cudaMemset(d_maxrow, 0, sizeof(int32_t)) != cudaSuccess ||
-            cudaMemset(d_near, 0, 34 * sizeof(unsigned long long)) != cudaSuccess) {
+        char *b = static_cast<char *>(h->ws.base);
+        h->ws.rec = reinterpret_cast<unsigned long long *>(b + o_rec);
+        h->ws.flags = reinterpret_cast<uint32_t *>(b + o_flags);
+        h->ws.indeg = reinterpret_cast<int32_t *>(b + o_indeg);
+        h->ws.tasks = reinterpret_cast<int32_t *>(b + o_tasks);
+        h->ws.st = reinterpret_cast<SolveState *>(b + o_st);
+        h->ws.aout = reinterpret_cast<AnalyseOut *>(b + o_out);
+        h->ws.blk = reinterpret_cast<int32_t *>(b + o_blk);
+        // everything zero (ready words: no epoch matches; counters; results), then status := ~0
+        if (cudaMemsetAsync(h->ws.base, 0, total, 0) != cudaSuccess ||
+            cudaMemsetAsync(&h->ws.aout->status, 0xff, sizeof(unsigned long long), 0) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
         if (n > 0) {
-            k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->nnz, h->ws.indeg, d_status,
-                                                 d_maxrow, d_near, tri_flags);
+            k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->ws.indeg, h->ws.aout, tri_flags);
             if (cudaGetLastError() != cudaSuccess) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
             }
+            rc = enqueue_plan(h, 0);
+            if (rc) break;
         }
-        unsigned long long status = 0;
-        if (cudaMemcpy(&status, d_status, sizeof(status), cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(&h->max_row, d_maxrow, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(&h->near_deps, d_near, sizeof(int64_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
-            cudaMemcpy(&h->prev_deps, d_near + 1, sizeof(int64_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+        h->gen = 1;
+        rc = init_state(h->ws.st, h->gen, 0);
+        if (rc) break;
+        AnalyseOut o;
+        if (cudaMemcpy(&o, h->ws.aout, sizeof(o), cudaMemcpyDeviceToHost) != cudaSuccess) {
             rc = SPTRSV_ERR_CUDA;
             break;
         }
-        h->warp_deps = (int64_t)((uint64_t)h->near_deps >> 32);
-        h->near_deps &= 0xFFFFFFFFll;
-        h->near_rows = (int64_t)((uint64_t)h->prev_deps >> 32);
-        h->prev_deps &= 0xFFFFFFFFll;
-        {   // the AUTO warp threshold from the median nearest-dependency distance (f2)
-            unsigned long long hist[32];
-            if (cudaMemcpy(hist, d_near + 2, sizeof(hist), cudaMemcpyDeviceToHost) != cudaSuccess) {
-                rc = SPTRSV_ERR_CUDA;
-                break;
-            }
-            unsigned long long tot = 0, acc = 0;
-            for (int k = 0; k < 32; ++k) tot += hist[k];
-            int med = -1;
-            for (int k = 0; k < 32 && tot; ++k) {
-                acc += hist[k];
-                if (2 * acc >= tot) {
-                    med = k;
-                    break;
-                }
-            }
-            h->dmin_log2 = med;
-            // a system that fits one 1024-thread one-shot CTA resolves everything in shared memory:
-            // thread level only (c1: 28.2 us vs 32.9 us with warp rows)
-            if (!h->threshold_user) h->threshold = h->n <= 1024 ? (1 << 30) : auto_warp_threshold(med);
-        }
-        if (status != ~0ull) {
-            rc = -(int)(status & 0xff);
+        if (o.status != ~0ull) {
+            rc = -(int)(o.status & 0xff);
             break;
         }
-        rc = build_plan(h);
-        if (rc) break;
-        rc = reset_state(h, 0);
-        if (rc) break;
-        if (cudaDeviceSynchronize() != cudaSuccess) {
-            rc = SPTRSV_ERR_CUDA;
-            break;
-        }
+        h->nnz = n > 0 ? o.nnz : 0;
+        h->max_row = o.max_row;
+        h->near_deps = (int64_t)(o.near & 0xFFFFFFFFull);
+        h->warp_deps = (int64_t)(o.near >> 32);
+        h->prev_deps = (int64_t)(o.prev & 0xFFFFFFFFull);
+        h->near_rows = (int64_t)(o.prev >> 32);
+        if (n > 0) adopt_plan(h, o);
+        else h->plan = PLAN_THREAD;
+        h->since_reset = 0;
     } while (0);
-    cudaFree(d_status);
-    cudaFree(d_maxrow);
-    cudaFree(d_near);
     if (rc != SPTRSV_OK) {
         (void)cudaGetLastError();
         free_ws(h->ws);
@@ -635,12 +562,13 @@ lean_fn chain_kernel(int proto, int tri, int K) {
 
 lean_fn chainp_kernel(int proto, int tri, int K) {
 #define CHAINP_ROW(U_, N_)                                                                             \
-    {{k_solve_chainp<PROTO_FLAGS, 1, U_, N_>, k_solve_chainp<PROTO_FUSED, 1, U_, N_>},                 \
-     {k_solve_chainp<PROTO_FLAGS, 2, U_, N_>, k_solve_chainp<PROTO_FUSED, 2, U_, N_>}}
-    static const lean_fn tab[4][2][2] = {CHAINP_ROW(false, false), CHAINP_ROW(true, false),
+    {{k_solve_chainp<PROTO_FLAGS, 2, U_, N_>, k_solve_chainp<PROTO_FUSED, 2, U_, N_>},                 \
+     {k_solve_chainp<PROTO_FLAGS, 4, U_, N_>, k_solve_chainp<PROTO_FUSED, 4, U_, N_>},                 \
+     {k_solve_chainp<PROTO_FLAGS, 8, U_, N_>, k_solve_chainp<PROTO_FUSED, 8, U_, N_>}}
+    static const lean_fn tab[4][3][2] = {CHAINP_ROW(false, false), CHAINP_ROW(true, false),
                                          CHAINP_ROW(false, true), CHAINP_ROW(true, true)};
 #undef CHAINP_ROW
-    return tab[tri & 3][K - 1][proto ? 1 : 0];
+    return tab[tri & 3][K == 2 ? 0 : K == 4 ? 1 : 2][proto ? 1 : 0];
 }
 
 int plan_launch(sptrsv_handle_s *h, Launch *L) {
@@ -674,7 +602,7 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         }
     }
     if (L->engine == ENG_CHAIN) {  // warp-sequential in-warp chains (solve_chain.cuh): 64..256 threads
-        const int K = h->rows_per_lane == 1 ? 1 : 2;
+        const int K = h->rows_per_lane == 1 ? 1 : 2;  // other values: the default 2
         const int cta = (user == 64 || user == 128 || user == 256) ? user : kChainCta;
         const int warps = cta / 32;
         const long long rows_per_cta = (long long)warps * 32 * K;
@@ -693,7 +621,7 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         return SPTRSV_OK;
     }
     if (L->engine == ENG_CHAINP) {  // chain warps with poller warps (solve_chainp.cuh): 1..4 pairs per CTA
-        const int K = h->rows_per_lane == 1 ? 1 : 2;
+        const int K = (h->rows_per_lane == 2 || h->rows_per_lane == 4) ? h->rows_per_lane : 8;
         const int cta = (user == 64 || user == 128 || user == 256) ? user : 64 * kChainPPairs;
         const int pairs = cta / 64;
         const long long rows_per_cta = (long long)pairs * 32 * K;
@@ -703,6 +631,11 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
         L->block = dim3((unsigned)cta);
         L->smem = (size_t)pairs * chainp_pair_smem_bytes(K);
+        if (L->smem > 48 * 1024 &&
+            cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_CUDA;
+        }
         L->key = (8500000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta) ^ (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
@@ -1134,15 +1067,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             return SPTRSV_OK;
         case SPTRSV_OPT_PROTOCOL:
             if (value != PROTO_FLAGS && value != PROTO_FUSED) return SPTRSV_ERR_INVALID_ARG;
-            if (value == PROTO_FUSED && !h->ws.rec && h->n > 0) {
-                // records are epoch-tagged like the flags: zeroed once, valid for any later epoch
-                if (cudaMalloc(&h->ws.rec, 16 * (size_t)h->n) != cudaSuccess) {
-                    (void)cudaGetLastError();
-                    return SPTRSV_ERR_ALLOC;
-                }
-                CK(cudaMemset(h->ws.rec, 0, 16 * (size_t)h->n));
-            }
-            h->proto = (int)value;
+            h->proto = (int)value;  // both kinds of ready words live in the workspace; the next solve re-zeroes
             size_l2_window(h);
             return SPTRSV_OK;
         case SPTRSV_OPT_LOCAL:
@@ -1156,7 +1081,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE:
-            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 8) return SPTRSV_ERR_INVALID_ARG;
             h->rows_per_lane = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT:

@@ -57,4 +57,23 @@ if (tc[g:] > 0).mean() > 0.5:
     ok = tc.reshape(g, g)[1:, :] > 0
     out["north_seen_us_p10_50_90"] = q(seen[ok])
     out["north_consumed_to_publish_us_p10_50_90"] = q(pub[ok])
+    # CHAINP: [2n+i] = when the chain warp started a run at row i (0 = not a run start)
+    rs = tr.cpu().numpy().astype(np.int64)[2 * s.n: 3 * s.n]
+    if (rs > 0).any():
+        rsu = ((rs - t0) / 1e3).reshape(g, g)
+        okr = (rs.reshape(g, g) > 0) & (tc.reshape(g, g) > 0)
+        okr[0, :] = False
+        out["run_starts_per_row"] = round(float(okr.sum() / (g - 1)), 2)
+        out["handover_us_p10_50_90"] = q((rsu - tcu)[okr])
+        out["runstart_to_publish_us_p10_50_90"] = q((t - rsu)[okr])
+        ho = tr.cpu().numpy().astype(np.int64)[3 * s.n + 3: 4 * s.n + 3]
+        if (ho > 0).any():
+            hou = ((ho - t0) / 1e3).reshape(g, g)
+            okh = okr & (ho.reshape(g, g) > 0)
+            out["consumed_to_handed_us_p10_50_90"] = q((hou - tcu)[okh])
+            out["handed_to_runstart_us_p10_50_90"] = q((rsu - hou)[okh])
+        c0 = okr[:, 0]
+        out["col0_seen_handover_publish_us"] = [round(float(np.median(seen[:, 0])), 3),
+                                                 round(float(np.median((rsu - tcu)[c0, 0])), 3),
+                                                 round(float(np.median((t - rsu)[c0, 0])), 3)]
 print(json.dumps(out))
