@@ -162,7 +162,8 @@ __global__ void __launch_bounds__(256) k_solve_chainp(SolveParams p) {
             // for the previous pair's last row while the rows after it consume their norths)
             int cnt = 0;
             bool found = false;
-            for (int base = lo; base < rows && cnt < 64; base += 32) {
+            const int wmax = p.poll_one ? 32 : 64;  // window: 2 rows per lane, or 1 (SPTRSV_OPT_POLL_ONE)
+            for (int base = lo; base < rows && cnt < wmax; base += 32) {
                 const int t = base + lane;
                 const bool pend = t < rows && p_nc[t] >= 0;
                 const unsigned m = __ballot_sync(FULL, pend);
@@ -176,7 +177,7 @@ __global__ void __launch_bounds__(256) k_solve_chainp(SolveParams p) {
                 }
                 if (pend) {
                     const int r = cnt + __popc(m & ((1u << lane) - 1u));
-                    if (r < 64) win[r] = t;
+                    if (r < wmax) win[r] = t;
                 }
                 cnt += __popc(m);
             }
@@ -186,7 +187,7 @@ __global__ void __launch_bounds__(256) k_solve_chainp(SolveParams p) {
             unsigned long long w0[2], w1[2];
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
-                tt[u] = lane + 32 * u < cnt ? win[lane + 32 * u] : -1;
+                tt[u] = lane + 32 * u < min(cnt, wmax) ? win[lane + 32 * u] : -1;
                 cc[u] = tt[u] >= 0 ? p_nc[tt[u]] : -1;
                 w0[u] = 0;
                 w1[u] = 0;
@@ -280,7 +281,8 @@ __global__ void __launch_bounds__(256) k_solve_chainp(SolveParams p) {
                     q = g.cand(a);
                     // the guard (Diag::ok) leaves the loop instead of branching around __ddiv_rn:
                     // no reconvergence point in the loop body
-                    if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0), 0)) break;
+                    if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0 && Diag::exact(a, dv, q)), 0))
+                        break;
                 }
                 s_x[t] = q;  // every lane stores the same value (each lane re-reads its own store)
                 if (PROTO == PROTO_FUSED) {
