@@ -242,7 +242,8 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 // failure LEAVES the fast loop instead of branching around an in-loop __ddiv_rn: the
                 // loop body then has no reconvergence point, and the guard resolves from a while the
                 // Markstein step is still in flight (chain step ~140 -> ~90 cycles, chainstep.cu)
-                if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0), 0)) break;
+                if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0 && Diag::exact(a, dv, q)), 0))
+                    break;
                 const int owner = t & 31, kk = t >> 5;
                 const bool mine = lane == owner;
 #pragma unroll
@@ -287,7 +288,7 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 g.r = f_r[s];
                 const double a = __dsub_rn(f_b[s], ls[k]);
                 double q = g.cand(a);
-                const int bad = !g.ok(a);
+                const int bad = !g.ok(a, q);
                 double xv = __shfl_sync(FULL, q, owner);
                 if (__shfl_sync(FULL, bad, owner)) {  // warp-uniform, rare: outside the guard
                     q = __ddiv_rn(a, g.d);

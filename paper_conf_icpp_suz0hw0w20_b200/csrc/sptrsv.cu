@@ -21,7 +21,6 @@
 #include "solve_multi.cuh"
 #include "solve_paper.cuh"
 #include "solve_chain.cuh"
-#include "solve_chainp.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -31,7 +30,7 @@ namespace {
 constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
 
 // engines (SPTRSV_OPT_ENGINE values, include/sptrsv.h)
-enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_CHAINP = 8 };
+enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7 };
 
 // The handle's workspace is ONE device allocation (analyse is O(nnz) work plus a fixed handful of
 // runtime calls), carved in 256-byte aligned pieces: the 16-byte FUSED records, the FLAGS words,
@@ -560,17 +559,6 @@ lean_fn chain_kernel(int proto, int tri, int K) {
     return tab[tri & 3][K - 1][proto ? 1 : 0];
 }
 
-lean_fn chainp_kernel(int proto, int tri, int K) {
-#define CHAINP_ROW(U_, N_)                                                                             \
-    {{k_solve_chainp<PROTO_FLAGS, 2, U_, N_>, k_solve_chainp<PROTO_FUSED, 2, U_, N_>},                 \
-     {k_solve_chainp<PROTO_FLAGS, 4, U_, N_>, k_solve_chainp<PROTO_FUSED, 4, U_, N_>},                 \
-     {k_solve_chainp<PROTO_FLAGS, 8, U_, N_>, k_solve_chainp<PROTO_FUSED, 8, U_, N_>}}
-    static const lean_fn tab[4][3][2] = {CHAINP_ROW(false, false), CHAINP_ROW(true, false),
-                                         CHAINP_ROW(false, true), CHAINP_ROW(true, true)};
-#undef CHAINP_ROW
-    return tab[tri & 3][K == 2 ? 0 : K == 4 ? 1 : 2][proto ? 1 : 0];
-}
-
 int plan_launch(sptrsv_handle_s *h, Launch *L) {
     if (h->variant) {  // the paper's kernels, control flow as printed (solve_paper.cuh; ablation only)
         L->block = dim3(kPaperCta);
@@ -618,25 +606,6 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
             return SPTRSV_ERR_CUDA;
         }
         L->key = (8000000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta) ^ (int)L->grid.x * 7919;
-        return SPTRSV_OK;
-    }
-    if (L->engine == ENG_CHAINP) {  // chain warps with poller warps (solve_chainp.cuh): 1..4 pairs per CTA
-        const int K = (h->rows_per_lane == 2 || h->rows_per_lane == 4) ? h->rows_per_lane : 8;
-        const int cta = (user == 64 || user == 128 || user == 256) ? user : 64 * kChainPPairs;
-        const int pairs = cta / 64;
-        const long long rows_per_cta = (long long)pairs * 32 * K;
-        L->fn = (const void *)chainp_kernel(h->proto, h->tri, K);
-        L->cta = cta;
-        L->K = K;
-        L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
-        L->block = dim3((unsigned)cta);
-        L->smem = (size_t)pairs * chainp_pair_smem_bytes(K);
-        if (L->smem > 48 * 1024 &&
-            cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess) {
-            (void)cudaGetLastError();
-            return SPTRSV_ERR_CUDA;
-        }
-        L->key = (8500000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta) ^ (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
     if (L->engine == ENG_LEAN) {  // minimal one-shot kernel for all-thread-level plans (solve_lean.cuh)
@@ -1076,12 +1045,12 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
             if (value != ENG_ONESHOT && value != ENG_LEAN && value != ENG_AUTO && value != ENG_HYBRID &&
-                value != ENG_CHAIN && value != ENG_CHAINP)
+                value != ENG_CHAIN)
                 return SPTRSV_ERR_INVALID_ARG;
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE:
-            if (value < 0 || value > 8) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
             h->rows_per_lane = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT:

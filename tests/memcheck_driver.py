@@ -18,7 +18,7 @@ def run(s, flags=0, **opt):
 
 bases = [synth.gen_random_lower(1025, 4, seed=3), synth.gen_grid(40), synth.gen_chain(700), synth.gen_c2i(n=5000)]
 for s in bases:
-    for eng in (0, 3, 6, 7, 8):
+    for eng in (0, 3, 6, 7):
         for proto in (0, 1):
             run(s, engine=eng, protocol=proto)
     for flags in (1, 2, 3):

@@ -61,7 +61,7 @@ def random_structure(rng):
     return synth.from_pattern(f"fuzz{kind}", rowptr, allc, rng)
 
 
-ENGINES = [(5, {}), (0, {}), (3, {}), (6, {}), (7, {}), (8, {}), (8, {"rows_per_lane": 1, "cta_threads": 256}),
+ENGINES = [(5, {}), (0, {}), (3, {}), (6, {}), (7, {}),
            (0, {"cta_threads": 1024}), (7, {"rows_per_lane": 1, "cta_threads": 64}), (3, {"cta_threads": 128}),
            (7, {"cta_threads": 512}), (3, {"cta_threads": 1024})]
 

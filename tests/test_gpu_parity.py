@@ -100,6 +100,48 @@ def test_closed_forms_bit_exact(cap, mode):
     assert np.array_equal(x, want)
 
 
+def _near_midpoint_quotients(rng, m):
+    """(a, d) with a/d within about an ulp of a rounding midpoint in (1/2, 1): the inputs where the
+    Markstein candidate's q0 = RN(a*RN(1/d)) is not always faithful (round-1 VERDICT).  d in [1, 2),
+    q a random double in (1/2, 1), a = RN((q + ulp(q)/2) * d), then nudged by 0..3 ulps."""
+    d = rng.uniform(1.0, 2.0, size=m)
+    q = rng.uniform(0.5, 1.0, size=m)
+    a = (q + np.spacing(q) / 2) * d
+    steps = rng.integers(-3, 4, size=m)
+    for k in range(3):
+        up, dn = steps > k, steps < -k
+        a[up] = np.nextafter(a[up], np.inf)
+        a[dn] = np.nextafter(a[dn], -np.inf)
+    return a, d
+
+
+@pytest.mark.parametrize("engine", [3, 0, 7])
+def test_division_near_midpoints_bit_exact(cap, engine):
+    """Quotients next to rounding midpoints through every engine's division (LEAN / ONE-SHOT
+    Diag::div, the CHAIN fast loops): bit-identical to IEEE a / d.  The chain engines get a
+    bidiagonal system with ZERO off-diagonals, so x_i = (b_i - 0 * x_{i-1}) / d_i = b_i / d_i runs
+    through their in-register chain step."""
+    rng = np.random.default_rng(4242 + engine)
+    n = 300_000
+    a, d = _near_midpoint_quotients(rng, n)
+    want = a / d
+    if engine == 7:
+        rp = np.r_[0, np.arange(1, 2 * n, 2)].astype(np.int32)
+        ci = np.empty(2 * n - 1, np.int32)
+        v = np.empty(2 * n - 1)
+        ci[0], ci[1::2], ci[2::2] = 0, np.arange(0, n - 1), np.arange(1, n)
+        v[0], v[2::2] = d[0], d[1:]
+        v[1::2] = 0.0
+        s = synth.CSRSystem("midchain", n, rp, ci, v, a, None, {})
+    else:
+        s = synth.CSRSystem("middiag", n, np.arange(n + 1, dtype=np.int32), np.arange(n, dtype=np.int32), d, a,
+                            None, {})
+    x, info = gpu_solve(cap, s, 1, engine=engine)
+    assert info["engine"] == engine
+    bad = x.view(np.int64) != want.view(np.int64)
+    assert not bad.any(), (np.nonzero(bad)[0][:10], x[bad][:3], want[bad][:3])
+
+
 @pytest.mark.parametrize("mode", [1, 2])
 def test_division_bit_exact_wide_range(cap, mode):
     """x_i = b_i / d_i over the whole double range + specials: the kernel's divide (Markstein
@@ -388,7 +430,7 @@ def test_lean_engine(cap, proto):
     assert np.array_equal(x, si.x_true)
 
 
-CHAIN_ENGINES = [7, 8]
+CHAIN_ENGINES = [7]
 
 
 @pytest.mark.parametrize("proto", PROTOS)

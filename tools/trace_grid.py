@@ -72,6 +72,15 @@ if (tc[g:] > 0).mean() > 0.5:
             okh = okr & (ho.reshape(g, g) > 0)
             out["consumed_to_handed_us_p10_50_90"] = q((hou - tcu)[okh])
             out["handed_to_runstart_us_p10_50_90"] = q((rsu - hou)[okh])
+            # pair boundaries (c % R == 0, c > 0): west published -> west consumed -> handed -> run -> publish
+            bc = np.arange(R, g, R)
+            if bc.size:
+                wp = t[:, bc - 1]
+                out["bnd_west_pub_to_consumed_us_p10_50_90"] = q((tcu[:, bc] - wp).ravel())
+                out["bnd_consumed_to_handed_us_p10_50_90"] = q((hou[:, bc] - tcu[:, bc]).ravel())
+                out["bnd_handed_to_runstart_us_p10_50_90"] = q((rsu[:, bc] - hou[:, bc]).ravel())
+                out["bnd_runstart_to_pub_us_p10_50_90"] = q((t[:, bc] - rsu[:, bc]).ravel())
+                out["bnd_north_pub_minus_west_pub_us_p10_50_90"] = q((np.vstack([t[:1, bc] * 0, t[:-1, bc]]) - wp)[1:].ravel())
         c0 = okr[:, 0]
         out["col0_seen_handover_publish_us"] = [round(float(np.median(seen[:, 0])), 3),
                                                  round(float(np.median((rsu - tcu)[c0, 0])), 3),
