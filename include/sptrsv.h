@@ -59,7 +59,9 @@ typedef enum sptrsv_status {
  * beyond fp64 summation order (warp mode sums lane-strided partials). */
 typedef enum sptrsv_option {
     SPTRSV_OPT_MODE = 1,           /* 0 AUTO (default), 1 THREAD (every row thread-level,
-                                      Alg.5), 2 WARP (every row warp-level, Alg.3).
+                                      Alg.5), 2 WARP (every row warp-level, Alg.3), 3 SUB-WARP
+                                      (every 32-row group at the sub-warp width its mean
+                                      nnz/row gives, see SPTRSV_OPT_SUBWARP).
                                       Setting it re-plans (synchronous).                    */
     SPTRSV_OPT_WARP_THRESHOLD = 2, /* AUTO: a 32-row group goes warp-level when its mean
                                       nnz/row exceeds this.  Default: derived at analyse from
@@ -110,14 +112,22 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_ROWS_PER_LANE = 15, /* CHAIN: K = 1 or 2 (0 = default 2) rows per lane       */
     SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 6)
                                       resident 256-thread CTAs per SM                       */
-    SPTRSV_OPT_PREFETCH = 18,      /* L2 bulk prefetch (cp.async.bulk.prefetch.L2) of the
-                                      CSR range of the CTA this many logical blocks ahead:
-                                      -1 (default) = the engine's measured choice, 0 = off.
-                                      A cache hint only; never changes a result            */
+    /* 18: retired (the L2 bulk prefetch of LEAN measured no gain and left in round 2)   */
     SPTRSV_OPT_POLL_GAP_NS = 19,   /* LEAN: __nanosleep after a pass that progressed but left
                                       lanes waiting (0 = default, none)                    */
     SPTRSV_OPT_POLL_ONE = 20,      /* LEAN: 1 = poll one dependency per lane per pass
                                       (default 0: the next two, DESIGN G21)                 */
+    SPTRSV_OPT_SUBWARP = 24,       /* sub-warp rows (the thread-vs-warp granularity
+                                      of sec.4.4): a 32-row group that AUTO
+                                      takes beyond thread level runs W lanes per row, W the
+                                      smallest power of two in [2, 32] with W * value >= its
+                                      mean off-diagonals per row (32 / W rows per warp task,
+                                      segmented lane tree).  value = target off-diagonals per
+                                      lane, 1..64; 0 = one warp per row (Alg.3) for every
+                                      such group.  Default: AUTO picks it (and the threshold)
+                                      from the median nearest-dependency distance (DESIGN.md
+                                      section 6); AUTO caps W at 16.  Setting it re-plans
+                                      (synchronous).                                        */
     SPTRSV_OPT_HOST_IO = 23,       /* sptrsv_solve_host with pinned buffers on LEAN: bit 0 =
                                       b copied in chunks on a second stream, each CTA waiting
                                       for its own chunk only (needs cuStreamWriteValue32);
@@ -143,7 +153,8 @@ typedef struct sptrsv_info {
     int32_t n_thread_groups;  /* 32-row groups solved thread-level                       */
     int64_t nnz;              /* rowptr[n]                                                */
     int32_t n_warp_rows;      /* rows solved warp-level                                   */
-    int32_t n_tasks;          /* warp tasks per solve = n_thread_groups + n_warp_rows     */
+    int32_t n_tasks;          /* warp tasks per solve = n_thread_groups + n_warp_rows +
+                                 n_sub_tasks                                               */
     int32_t max_row_nnz;      /* longest row (incl. diagonal)                             */
     int32_t device;           /* CUDA ordinal the handle is bound to                      */
     float analyse_ms;         /* wall time of sptrsv_analyse_csr (Table 1 analogue)        */
@@ -156,6 +167,8 @@ typedef struct sptrsv_info {
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
     int64_t prev_deps;        /* dependencies on the previous row in solve order (i - 1;
                                  i + 1 for upper handles): AUTO's CHAIN criterion           */
+    int32_t n_sub_tasks;      /* warp tasks holding 32/W sub-warp rows (W = 2..16 lanes per row) */
+    int32_t pad_;
     int64_t near_rows;        /* rows whose nearest dependency is < 256 rows away: AUTO's
                                  LEAN criterion (LEAN when < n/4)                          */
 } sptrsv_info;

@@ -201,10 +201,10 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
             "rows_per_lane": _lib.OPT_ROWS_PER_LANE,
             "variant": _lib.OPT_VARIANT, "lean_occupancy": _lib.OPT_LEAN_OCCUPANCY,
-            "prefetch": _lib.OPT_PREFETCH, "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
+            "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
             "poll_one": _lib.OPT_POLL_ONE,
             "warp_split_last": _lib.OPT_WARP_SPLIT_LAST,
-            "host_io": _lib.OPT_HOST_IO}
+            "host_io": _lib.OPT_HOST_IO, "subwarp": _lib.OPT_SUBWARP}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

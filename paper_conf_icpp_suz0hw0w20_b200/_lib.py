@@ -52,14 +52,14 @@ OPT_ENGINE = 11
 OPT_ROWS_PER_LANE = 15
 OPT_VARIANT = 16
 OPT_LEAN_OCCUPANCY = 17
-OPT_PREFETCH = 18
 OPT_POLL_GAP_NS = 19
 OPT_POLL_ONE = 20
 OPT_WARP_SPLIT_LAST = 22
 OPT_HOST_IO = 23
+OPT_SUBWARP = 24
 ENGINE_ONESHOT, ENGINE_LEAN, ENGINE_AUTO, ENGINE_HYBRID, ENGINE_CHAIN = 0, 3, 5, 6, 7
 PROTO_FLAGS, PROTO_FUSED = 0, 1
-MODE_AUTO, MODE_THREAD, MODE_WARP = 0, 1, 2
+MODE_AUTO, MODE_THREAD, MODE_WARP, MODE_SUBWARP = 0, 1, 2, 3
 
 
 class sptrsv_info(ctypes.Structure):
@@ -79,6 +79,8 @@ class sptrsv_info(ctypes.Structure):
         ("cta_threads", ctypes.c_int32),
         ("rows_per_lane", ctypes.c_int32),
         ("prev_deps", ctypes.c_int64),
+        ("n_sub_tasks", ctypes.c_int32),
+        ("pad_", ctypes.c_int32),
         ("near_rows", ctypes.c_int64),
     ]
 

@@ -112,19 +112,6 @@ __device__ __forceinline__ double ld_stream_f64(const double *p, uint64_t pol) {
     return v;
 }
 
-// Bulk L2 prefetch (TMA unit, no shared memory, no completion to wait for) of the
-// byte range [lo, hi), shrunk inward to 16-byte boundaries so it never touches a
-// byte outside the caller's arrays.  A hint only: it changes no result.
-__device__ __forceinline__ void bulk_prefetch_l2(const void *lo, const void *hi) {
-    uintptr_t a = ((uintptr_t)lo + 15) & ~(uintptr_t)15;
-    const uintptr_t e = (uintptr_t)hi & ~(uintptr_t)15;
-    while (a < e) {
-        const uintptr_t c = (e - a) > 65536 ? 65536 : (e - a);
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((unsigned)c) : "memory");
-        a += c;
-    }
-}
-
 __device__ __forceinline__ void nanosleep_ns(uint32_t ns) {
     asm volatile("nanosleep.u32 %0;" ::"r"(ns));
 }
@@ -133,49 +120,6 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
-}
-
-// ---------------------------------------------------------------- mbarrier + TMA bulk copy
-// (the shared-memory ring of the pipelined engine, solve_pipe.cuh)
-
-__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(unsigned bar, unsigned count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive(unsigned bar) {
-    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(bar) : "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive_expect_tx(unsigned bar, unsigned bytes) {
-    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(bar),
-                 "r"(bytes)
-                 : "memory");
-}
-
-// true once the phase with the given parity has completed
-__device__ __forceinline__ bool mbar_try_wait(unsigned bar, unsigned parity) {
-    unsigned ok;
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(ok)
-        : "r"(bar), "r"(parity)
-        : "memory");
-    return ok != 0;
-}
-
-// 1-D TMA bulk copy global -> shared, completion counted on an mbarrier
-// (sizes and both addresses multiples of 16 bytes).
-__device__ __forceinline__ void bulk_g2s(unsigned dst, const void *src, unsigned bytes, unsigned bar, uint64_t pol) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(dst),
-        "l"(src), "r"(bytes), "r"(bar), "l"(pol)
-        : "memory");
-}
-
-__device__ __forceinline__ void fence_mbar_init() {
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
 
 }  // namespace sptrsv_dev

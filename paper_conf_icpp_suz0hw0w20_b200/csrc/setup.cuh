@@ -27,7 +27,9 @@ struct AnalyseOut {
     int32_t threshold;           // AUTO warp threshold the plan used (sec.4.4)
     int32_t med_log2;            // floor(log2(median nearest-dependency distance)), -1 = none
     int32_t n_tasks, n_tgroups;  // plan: warp tasks, 32-row thread groups
-    int32_t pad;
+    int32_t n_subtasks;          // plan: tasks with 2..16 lanes per row (sub-warp rows)
+    int32_t epl;                 // sub-warp target off-diagonals per lane (0: warp rows only)
+    int32_t pad2;
     unsigned long long near;     // near_deps | warp_deps << 32
     unsigned long long prev;     // prev_deps | near_rows << 32
     unsigned long long hist[32]; // rows by floor(log2(nearest-dependency distance))
@@ -116,19 +118,36 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
         atomicAdd(near_deps + 1, (unsigned long long)pdep | ((unsigned long long)nrow << 32));
 }
 
-// mode: 0 auto, 1 all thread-level, 2 all warp-level.
-// A group of `rows` rows goes warp-level in auto mode when its nnz (diagonals
-// included) exceeds threshold * rows, i.e. mean nnz/row > threshold.
+// mode: 0 auto, 1 all thread-level, 2 all warp-level, 3 all sub-warp (width from the group's mean).
+// A group of `rows` rows goes beyond thread level in auto mode when its nnz (diagonals
+// included) exceeds threshold * rows, i.e. mean nnz/row > threshold (sec.4.4).
+// Its width W (lanes per row) is then 32 (a warp per row, Alg.3), or -- with sub-warp rows enabled
+// (epl = target off-diagonals per lane) -- the smallest power of two in [2, 32] with
+// W * epl >= mean off-diagonals per row: 32 / W rows share one warp task.
 // rev (f4 UPPER): groups are over LOGICAL rows r -> row n-1-r (the solve order).
+// Returns the group's tasks; *width = 0 (thread level: one task), 32 (one task per row) or W.
 __device__ __forceinline__ int group_tasks(const int32_t *rowptr, int32_t n, int g, int mode,
-                                           int threshold, bool *is_warp, bool rev) {
+                                           int threshold, int epl, int *width, bool rev) {
     const int r0 = g * 32;
     const int rows = min(32, n - r0);
     const long long gnnz = rev ? (long long)rowptr[n - r0] - rowptr[n - r0 - rows]
                                : (long long)rowptr[r0 + rows] - rowptr[r0];
-    const bool w = (mode == 2) || (mode == 0 && gnnz > (long long)threshold * rows);
-    *is_warp = w;
-    return w ? rows : 1;
+    const bool beyond = (mode >= 2) || (mode == 0 && gnnz > (long long)threshold * rows);
+    if (!beyond) {
+        *width = 0;
+        return 1;
+    }
+    int w = 32;
+    if (mode == 3 || (mode == 0 && epl > 0)) {
+        const long long off = gnnz - rows;  // off-diagonals in the group (approx. for unit forms)
+        const int e = max(1, epl > 0 ? epl : 4);
+        const int wmax = mode == 3 ? 32 : 16;  // AUTO keeps sub-warp rows at <= 16 lanes
+        w = 2;
+        while (w < wmax && (long long)w * e * rows < off) w <<= 1;
+    }
+    *width = w;
+    const int per = 32 / w;  // rows per task
+    return (rows + per - 1) / per;
 }
 
 __device__ __forceinline__ int block_exclusive_scan(int v, int *s_warp, int *total) {
@@ -162,51 +181,66 @@ __global__ void __launch_bounds__(1024) k_plan_count(const int32_t *__restrict__
                                                      int32_t ngroups, int mode, const AnalyseOut *out,
                                                      int32_t *blk_tasks, int32_t *blk_tgroups, bool rev) {
     __shared__ int s_warp[33];
-    const int threshold = out->threshold;
+    const int threshold = out->threshold, epl = out->epl;
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
-    int t = 0, tg = 0;
+    int t = 0, tg = 0, ts = 0;
     if (g < ngroups) {
-        bool w;
-        t = group_tasks(rowptr, n, g, mode, threshold, &w, rev);
-        tg = w ? 0 : 1;
+        int w;
+        t = group_tasks(rowptr, n, g, mode, threshold, epl, &w, rev);
+        tg = w == 0 ? 1 : 0;
+        ts = (w > 0 && w < 32) ? t : 0;
     }
-    int tot_t, tot_g;
+    int tot_t, tot_g, tot_s;
     block_exclusive_scan(t, s_warp, &tot_t);
     block_exclusive_scan(tg, s_warp, &tot_g);
+    block_exclusive_scan(ts, s_warp, &tot_s);
     if (threadIdx.x == 0) {
         blk_tasks[blockIdx.x] = tot_t;
         blk_tgroups[blockIdx.x] = tot_g;
+        if (tot_s) atomicAdd(&((AnalyseOut *)out)->n_subtasks, tot_s);  // zeroed by k_auto_threshold
     }
 }
 
 __global__ void __launch_bounds__(1024) k_plan_write(const int32_t *__restrict__ rowptr, int32_t n,
                                                      int32_t ngroups, int mode, const AnalyseOut *out,
                                                      const int32_t *__restrict__ blk_offset,
-                                                     int32_t *tasks, bool rev) {
+                                                     int32_t *tasks, uint8_t *task_w, bool rev) {
     __shared__ int s_warp[33];
-    const int threshold = out->threshold;
+    const int threshold = out->threshold, epl = out->epl;
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
-    int t = 0;
-    bool w = false;
-    if (g < ngroups) t = group_tasks(rowptr, n, g, mode, threshold, &w, rev);
+    int t = 0, w = 0;
+    if (g < ngroups) t = group_tasks(rowptr, n, g, mode, threshold, epl, &w, rev);
     int tot;
     const int off = block_exclusive_scan(t, s_warp, &tot) + blk_offset[blockIdx.x];
     if (g < ngroups) {
-        if (w) {
-            for (int k = 0; k < t; ++k) tasks[off + k] = ~(g * 32 + k);  // warp task: row
+        if (w == 0) {
+            tasks[off] = g * 32;  // thread task: the group's first (logical) row
+            task_w[off] = 0;
         } else {
-            tasks[off] = g * 32;  // thread task: first row of the group
+            const int per = 32 / w;  // w = 32: one warp task per row (Alg.3); else 32/w rows per task
+            for (int k = 0; k < t; ++k) {
+                tasks[off + k] = ~(g * 32 + k * per);
+                task_w[off + k] = (uint8_t)w;
+            }
         }
     }
 }
 
-// AUTO's per-32-row-group warp threshold (mean nnz/row above which a group runs warp-level), from
-// floor(log2) of the median distance to a row's nearest dependency -- on leveled matrices about the
-// level width, which moves the thread/warp crossover (f2 sweep): < 64 rows:
-// thread level only; 64..1023: warp from 2 nnz/row; 1024..8191: from 6; wider: from 20.  A system
-// that fits one 1024-thread one-shot CTA resolves in shared memory: thread level only.
-// user >= 0: SPTRSV_OPT_WARP_THRESHOLD was set, use it.  One thread.
-__global__ void k_auto_threshold(AnalyseOut *out, int32_t n, int32_t user) {
+// AUTO's per-32-row-group dispatch (sec.4.4, PAPER.md:329-335 leaves it as future work; SURVEY
+// f2): from floor(log2) of the median distance to a row's nearest dependency -- on leveled matrices
+// about the level width, which moves the crossover -- the mean nnz/row above which a group leaves
+// thread level (threshold) and how many lanes its rows get (epl: target off-diagonals per lane,
+// W = smallest power of two with W * epl >= mean off-diagonals, capped at 16; 0 = a warp per row).
+// Measured on B200 (profiles/r02_f2_sweep.md, n = 2e5 leveled synthetics + c2 / c4 / c5):
+//   < 64 rows            thread level only (in-CTA / in-warp resolution wins)
+//   64 .. 511            threshold 2, warp rows (Alg.3)
+//   512 .. 1023          threshold 2, sub-warp rows, epl 4   (c4: 16 lanes per 64-entry row)
+//   1024 .. 8191         threshold 2, sub-warp rows, epl 2
+//   >= 8192              threshold 3, sub-warp rows, epl 8   (c2 / c5 at 2.8 nnz/row stay thread)
+//   n <= 1024            thread level only (one 1024-thread one-shot CTA resolves it in smem)
+// user >= 0 / user_epl >= 0: SPTRSV_OPT_WARP_THRESHOLD / SPTRSV_OPT_SUBWARP were set.  One thread.
+__global__ void k_auto_threshold(AnalyseOut *out, int32_t n, int32_t user, int32_t user_epl) {
+    out->n_subtasks = 0;
     unsigned long long tot = 0, acc = 0;
     for (int k = 0; k < 32; ++k) tot += out->hist[k];
     int med = -1;
@@ -218,15 +252,16 @@ __global__ void k_auto_threshold(AnalyseOut *out, int32_t n, int32_t user) {
         }
     }
     out->med_log2 = med;
-    int t;
-    if (user >= 0) t = user;
-    else if (n <= 1024) t = 1 << 30;
-    else if (med < 0) t = 16;  // no dependencies at all
-    else if (med <= 5) t = 1 << 30;
-    else if (med <= 9) t = 2;
-    else if (med <= 12) t = 6;
-    else t = 20;
-    out->threshold = t;
+    int t, e;
+    if (n <= 1024) t = 1 << 30, e = 0;
+    else if (med < 0) t = 16, e = 0;  // no dependencies at all
+    else if (med <= 5) t = 1 << 30, e = 0;
+    else if (med <= 8) t = 2, e = 0;
+    else if (med <= 9) t = 2, e = 4;
+    else if (med <= 12) t = 2, e = 2;
+    else t = 3, e = 8;
+    out->threshold = user >= 0 ? user : t;
+    out->epl = user_epl >= 0 ? user_epl : e;
 }
 
 // exclusive scan of the per-block task / thread-group counts (one CTA, any number of blocks):

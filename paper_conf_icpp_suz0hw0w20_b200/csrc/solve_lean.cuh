@@ -23,16 +23,6 @@
 namespace sptrsv_dev {
 
 constexpr int kLeanCta = 256;
-constexpr int kLeanPrefetchDefault = 0;  // SPTRSV_OPT_PREFETCH = -1 resolves to this (CTAs ahead)
-
-// L2 bulk prefetch of the physical rows [A, B): rowptr[A..B], b[A..B) and the
-// entries [pa, pb) = [rowptr[A], rowptr[B]) of colidx and val.
-__device__ __forceinline__ void prefetch_rows_l2(const SolveParams &p, int A, int B, int pa, int pb) {
-    bulk_prefetch_l2(p.rowptr + A, p.rowptr + B + 1);
-    bulk_prefetch_l2(p.b + A, p.b + B);
-    bulk_prefetch_l2(p.colidx + pa, p.colidx + pb);
-    bulk_prefetch_l2(p.val + pa, p.val + pb);
-}
 
 // One warp, one row per lane (Alg.5 l.3-18): lane's row i (act: i is a real row), its
 // bounds [rs, re) and b_i already loaded.  Returns when every lane of the warp has
@@ -150,19 +140,6 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         re = ld_stream_i32(p.rowptr + i + 1, pol);
         if (!bgate) bi = ld_b(p, i, pol);
     }
-    // ---- L2 bulk prefetch of the block pf_dist logical blocks ahead (speculatively
-    // blockIdx.x + pf_dist): its bounds load overlaps the ticket, the copy is issued after it
-    int pfA = 0, pfB = 0, pfa = 0, pfb = 0;
-    if (p.pf_dist > 0 && tid == 32) {
-        const long long r0 = ((long long)blockIdx.x + p.pf_dist) * CT;
-        if (r0 < p.n) {
-            const int r1 = (int)min((long long)p.n, r0 + CT);
-            pfA = UPPER ? p.n - r1 : (int)r0;
-            pfB = UPPER ? p.n - (int)r0 : r1;
-            pfa = ld_stream_i32(p.rowptr + pfA, pol);
-            pfb = ld_stream_i32(p.rowptr + pfB, pol);
-        }
-    }
     if (tid == 0) {
         if (p.trace) {
             atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
@@ -177,7 +154,6 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     __syncthreads();
     if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
-    if (pfB > pfA) prefetch_rows_l2(p, pfA, pfB, pfa, pfb);
     if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
         i = (int)s_blk * CT + tid;
         if (UPPER) i = p.n - 1 - i;

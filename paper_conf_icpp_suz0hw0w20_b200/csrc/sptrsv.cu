@@ -41,6 +41,7 @@ struct Workspace {
     unsigned long long *rec = nullptr;  // 2n (PROTO_FUSED)
     int32_t *indeg = nullptr;      // n
     int32_t *tasks = nullptr;      // n (PLAN_LIST uses n_tasks <= n of them)
+    uint8_t *task_w = nullptr;     // n: lanes per row of each task (0 thread group, 32 warp row, 2..16)
     SolveState *st = nullptr;      // 1
     AnalyseOut *aout = nullptr;    // 1: analyse results (one D2H copy)
     int32_t *blk = nullptr;        // 3 * nb: plan block counts / thread groups / offsets
@@ -91,6 +92,9 @@ struct sptrsv_handle_s {
     int32_t n_tasks_cap = 0;
     int32_t n_thread_groups = 0;
     int32_t n_warp_rows = 0;
+    int32_t n_sub_tasks = 0;  // tasks of 2..16 lanes per row (sub-warp rows)
+    int subwarp_epl = -1;     // SPTRSV_OPT_SUBWARP: off-diagonals per lane of a sub-warp row (-1 AUTO, 0 off)
+    int epl_eff = 0;          // the value the current plan used
     int32_t max_row = 0;
     int64_t near_deps = 0;  // dependencies within 256 rows (analyse statistic for ENGINE_AUTO)
     int64_t warp_deps = 0;  // dependencies inside the row's own 32-row group (ditto)
@@ -115,7 +119,6 @@ struct sptrsv_handle_s {
     int rows_per_lane = 0;  // CHAIN: K rows per lane (0 = 2)
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
     int lean_minb = 6;      // LEAN: resident 256-thread CTAs per SM the register budget targets (5..8)
-    int pf_dist = -1;       // L2 bulk prefetch lookahead in CTAs (-1 = engine default, 0 = off)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
     int host_io = 3;        // sptrsv_solve_host on LEAN with pinned buffers (SPTRSV_OPT_HOST_IO)
@@ -244,10 +247,11 @@ int enqueue_plan(sptrsv_handle_s *h, cudaStream_t s) {
     const int nb = (ngroups + 1023) / 1024;
     const bool rev = h->tri & SPTRSV_TRI_UPPER;  // f4 upper: plan over logical (reversed) rows
     int32_t *bt = h->ws.blk, *bg = bt + nb, *off = bg + nb;
-    k_auto_threshold<<<1, 1, 0, s>>>(h->ws.aout, n, h->threshold_user ? h->threshold : -1);
+    k_auto_threshold<<<1, 1, 0, s>>>(h->ws.aout, n, h->threshold_user ? h->threshold : -1, h->subwarp_epl);
     k_plan_count<<<nb, 1024, 0, s>>>(h->rowptr, n, ngroups, h->mode, h->ws.aout, bt, bg, rev);
     k_plan_scan<<<1, 1024, 0, s>>>(bt, bg, nb, off, h->ws.aout);
-    k_plan_write<<<nb, 1024, 0, s>>>(h->rowptr, n, ngroups, h->mode, h->ws.aout, off, h->ws.tasks, rev);
+    k_plan_write<<<nb, 1024, 0, s>>>(h->rowptr, n, ngroups, h->mode, h->ws.aout, off, h->ws.tasks, h->ws.task_w,
+                                     rev);
     CK(cudaGetLastError());
     return SPTRSV_OK;
 }
@@ -259,8 +263,12 @@ void adopt_plan(sptrsv_handle_s *h, const AnalyseOut &o) {
     h->dmin_log2 = o.med_log2;
     h->n_tasks = ngroups ? o.n_tasks : 0;
     h->n_thread_groups = ngroups ? o.n_tgroups : 0;
-    h->n_warp_rows = h->n_tasks - h->n_thread_groups;  // a warp-level group contributes one task per row
-    h->plan = (h->n_thread_groups == ngroups) ? PLAN_THREAD : (h->n_thread_groups == 0 ? PLAN_WARP : PLAN_LIST);
+    h->n_sub_tasks = ngroups ? o.n_subtasks : 0;
+    h->epl_eff = o.epl;
+    // rows beyond thread level: warp rows are one task each, sub-warp tasks hold 32/W rows
+    h->n_warp_rows = h->n_tasks - h->n_thread_groups - h->n_sub_tasks;
+    h->plan = (h->n_thread_groups == ngroups) ? PLAN_THREAD
+              : (h->n_thread_groups == 0 && h->n_sub_tasks == 0) ? PLAN_WARP : PLAN_LIST;
 }
 
 // Re-plan after a MODE / WARP_THRESHOLD change (synchronous: one D2H copy).
@@ -378,7 +386,7 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         const size_t nb = (ngroups + 1023) / 1024;
         auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
         const size_t o_rec = 0, o_flags = o_rec + al(16 * nn), o_indeg = o_flags + al(4 * nn),
-                     o_tasks = o_indeg + al(4 * nn), o_st = o_tasks + al(4 * nn),
+                     o_tasks = o_indeg + al(4 * nn), o_tw = o_tasks + al(4 * nn), o_st = o_tw + al(nn),
                      o_out = o_st + al(sizeof(SolveState)), o_blk = o_out + al(sizeof(AnalyseOut)),
                      total = o_blk + al(4 * 3 * (nb ? nb : 1));
         if (cudaMalloc(&h->ws.base, total) != cudaSuccess) {
@@ -390,6 +398,7 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         h->ws.flags = reinterpret_cast<uint32_t *>(b + o_flags);
         h->ws.indeg = reinterpret_cast<int32_t *>(b + o_indeg);
         h->ws.tasks = reinterpret_cast<int32_t *>(b + o_tasks);
+        h->ws.task_w = reinterpret_cast<uint8_t *>(b + o_tw);
         h->ws.st = reinterpret_cast<SolveState *>(b + o_st);
         h->ws.aout = reinterpret_cast<AnalyseOut *>(b + o_out);
         h->ws.blk = reinterpret_cast<int32_t *>(b + o_blk);
@@ -453,7 +462,6 @@ struct Launch {
     dim3 grid, block;
     size_t smem = 0;
     int key = 0;      // configuration identity (the epoch arithmetic needs a fixed grid per key)
-    int pf_dist = 0;  // SolveParams::pf_dist (LEAN's optional L2 prefetch)
     int engine = 0;   // engine launched (ENG_*; 30 + v for the paper's Alg. v)
     int cta = 0;      // threads per CTA
     int K = 1;        // thread-level rows per lane
@@ -503,7 +511,8 @@ void size_l2_window(sptrsv_handle_s *h) {
 int resolve_engine(const sptrsv_handle_s *h) {
     const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;  // unit handles store no diagonal
     const bool chains = offdiag > 0 && 4 * h->prev_deps >= offdiag;
-    if (h->plan != PLAN_THREAD) return (h->engine == ENG_ONESHOT && !h->tri) ? ENG_ONESHOT : ENG_HYBRID;
+    if (h->plan != PLAN_THREAD)  // ONE-SHOT has no sub-warp rows
+        return (h->engine == ENG_ONESHOT && !h->tri && h->n_sub_tasks == 0) ? ENG_ONESHOT : ENG_HYBRID;
     if (h->engine != ENG_AUTO) return (h->tri && h->engine == ENG_ONESHOT) ? ENG_LEAN : h->engine;
     if (h->tri) return chains ? ENG_CHAIN : ENG_LEAN;
     if (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n) return ENG_LEAN;
@@ -618,7 +627,6 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
             if (user == 128 || user == 512) ct = user;
             L->fn = (const void *)lean_lower_kernel(h->proto, h->lean_minb, ct);
             if (!L->fn) return SPTRSV_ERR_INVALID_ARG;
-            L->pf_dist = h->pf_dist < 0 ? kLeanPrefetchDefault : h->pf_dist;
         }
         L->cta = ct;
         L->grid = dim3((unsigned)((h->n + ct - 1) / ct));
@@ -683,6 +691,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.flags = h->ws.flags;
     p.rec = h->ws.rec;
     p.tasks = h->ws.tasks;
+    p.task_w = h->ws.task_w;
     p.st = h->ws.st;
     p.nnz = h->nnz;
     p.n = h->n;
@@ -695,7 +704,6 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.spin_limit = h->spin_limit;
     p.stage = h->stage;
     p.local = h->local;
-    p.pf_dist = L.pf_dist;
     p.poll_gap = h->poll_gap;
     p.poll_one = h->poll_one;
     p.split_last = h->split_last;
@@ -1000,7 +1008,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
     DeviceGuard g(h->device);
     switch (key) {
         case SPTRSV_OPT_MODE:
-            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
+            if (value < 0 || value > 3) return SPTRSV_ERR_INVALID_ARG;
             h->mode = (int)value;
             return build_plan(h);
         case SPTRSV_OPT_WARP_THRESHOLD:
@@ -1061,10 +1069,6 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             if (value < 5 || value > 8) return SPTRSV_ERR_INVALID_ARG;
             h->lean_minb = (int)value;
             return SPTRSV_OK;
-        case SPTRSV_OPT_PREFETCH:
-            if (value < -1 || value > (1 << 24)) return SPTRSV_ERR_INVALID_ARG;
-            h->pf_dist = (int)value;
-            return SPTRSV_OK;
         case SPTRSV_OPT_POLL_GAP_NS:
             if (value < 0 || value > 1000000) return SPTRSV_ERR_INVALID_ARG;
             h->poll_gap = (uint32_t)value;
@@ -1078,6 +1082,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
                 return SPTRSV_ERR_INVALID_ARG;
             h->host_io = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_SUBWARP:
+            if (value < 0 || value > 64) return SPTRSV_ERR_INVALID_ARG;
+            h->subwarp_epl = (int)value;
+            return build_plan(h);
         case SPTRSV_OPT_WARP_SPLIT_LAST:
             if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
             h->split_last = (int)value;
@@ -1104,11 +1112,11 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_ROWS_PER_LANE: *value = h->rows_per_lane; return SPTRSV_OK;
         case SPTRSV_OPT_VARIANT: *value = h->variant; return SPTRSV_OK;
         case SPTRSV_OPT_LEAN_OCCUPANCY: *value = h->lean_minb; return SPTRSV_OK;
-        case SPTRSV_OPT_PREFETCH: *value = h->pf_dist; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_GAP_NS: *value = h->poll_gap; return SPTRSV_OK;
         case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST: *value = h->split_last; return SPTRSV_OK;
         case SPTRSV_OPT_HOST_IO: *value = h->host_io; return SPTRSV_OK;
+        case SPTRSV_OPT_SUBWARP: *value = h->subwarp_epl >= 0 ? h->subwarp_epl : h->epl_eff; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
 }
@@ -1119,6 +1127,7 @@ int sptrsv_get_info(sptrsv_handle_t h, sptrsv_info *out) {
     out->nnz = h->nnz;
     out->n_thread_groups = h->n_thread_groups;
     out->n_warp_rows = h->n_warp_rows;
+    out->n_sub_tasks = h->n_sub_tasks;
     out->n_tasks = h->n_tasks;
     out->max_row_nnz = h->max_row;
     out->device = h->device;

@@ -120,3 +120,27 @@ def test_f4_forms_full(cfg, flags):
         assert np.max(np.abs(got - ref) / np.abs(ref)) <= TOL
     else:
         assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("cfg", ["c2", "c3", "c4"])
+def test_levels_full_size_bit_exact(cfg):
+    """a10 at full BASELINE size: the GPU level diagnostic (sptrsv_levels) against the oracle's Kahn
+    BFS -- every component's level, the level count and every per-level count, bit for bit (beta =
+    n / levels of Table 6) -- and the generator's closed form (10 x 1e5; 4095 with
+    min(k+1, 4095-k) per anti-diagonal; 1000 x 1000)."""
+    import paper_conf_icpp_suz0hw0w20_b200 as cap
+    s = {"c2": synth.gen_c2, "c3": synth.gen_c3, "c4": synth.gen_c4}[cfg]()
+    d = torch.device("cuda:0")
+    rp, ci, v = (torch.from_numpy(a).to(d) for a in (s.rowptr, s.colidx, s.val))
+    with cap.analyse(rp, ci, v) as h:
+        lv, nl, counts = h.levels()
+        deg = h.indegree().cpu().numpy()
+    olv = oracle.levels_bfs(s.rowptr, s.colidx)
+    onl, ocounts = oracle.level_counts(olv)
+    assert nl == onl
+    assert np.array_equal(lv.cpu().numpy(), olv)
+    assert np.array_equal(counts.cpu().numpy(), ocounts)
+    assert np.array_equal(deg, oracle.indegree(s.rowptr, s.colidx))
+    want = {"c2": [100_000] * 10, "c4": [1000] * 1000,
+            "c3": [min(k + 1, 4095 - k) for k in range(4095)]}[cfg]
+    assert ocounts.tolist() == want

@@ -62,7 +62,7 @@ def test_random_small_sizes(cap, n, mode, proto, local, engine):
     s = synth.gen_random_lower(n, 4, seed=n)
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     x, info = gpu_solve(cap, s, mode, protocol=proto, local=local, engine=engine)
-    if mode == 1:
+    if info["n_warp_rows"] == 0 and info["n_sub_tasks"] == 0:  # an all-thread-level plan: Alg.1's arithmetic
         assert np.array_equal(x, ref)
     else:
         assert relerr(x, ref) <= TOL
@@ -515,7 +515,8 @@ def test_hybrid_engine(cap, proto, mode):
         s = synth.gen_random_lower(n, 24, seed=n + 17)
         x, info = gpu_solve(cap, s, mode, protocol=proto, engine=6)
         ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
-        assert info["engine"] == 6
+        # an all-thread-level plan has no warp tasks: HYBRID runs its thread-group path as LEAN
+        assert info["engine"] == (6 if info["n_warp_rows"] + info["n_sub_tasks"] else 3)
         if mode == 1:
             assert np.array_equal(x, ref), n
         else:
@@ -528,6 +529,51 @@ def test_hybrid_engine(cap, proto, mode):
     si = synth.integerize(synth.gen_leveled(50_000, 20, 1, 30, 4, "l"))
     x, _ = gpu_solve(cap, si, mode, protocol=proto, engine=6)
     assert np.array_equal(x, si.x_true)
+
+
+@pytest.mark.parametrize("proto", PROTOS)
+@pytest.mark.parametrize("epl", [1, 2, 4, 8, 16])
+def test_subwarp_rows(cap, proto, epl):
+    """Sub-warp rows (SPTRSV_OPT_SUBWARP): W = 2..16 lanes per row, 32/W rows per warp
+    task, segmented lane tree -- within the warp-mode bound of the oracle; exact-integer systems
+    bit-exact; ragged tails (n not a multiple of 32 or of 32/W); every f4 form."""
+    for n in (1, 31, 33, 257, 4099):
+        s = synth.gen_random_lower(n, 12, seed=n + 29)
+        x, info = gpu_solve(cap, s, 0, protocol=proto, subwarp=epl, warp_threshold=2)
+        assert relerr(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)) <= TOL, n
+    for gen in (lambda: synth.gen_leveled(100_000, 100, 1, 8, 5, "l8"), lambda: synth.gen_leveled(60_000, 60, 1, 20, 6, "l20"),
+                lambda: synth.gen_c4(n=40_000, nlevels=80), lambda: synth.gen_dense_lower(200)):
+        s = gen()
+        x, info = gpu_solve(cap, s, 3, protocol=proto, subwarp=epl)  # MODE_SUBWARP: every group
+        assert info["n_sub_tasks"] > 0 or info["n_warp_rows"] > 0, info
+        assert relerr(x, oracle.solve(s.rowptr, s.colidx, s.val, s.b)) <= TOL, s.name
+    si = synth.integerize(synth.gen_leveled(50_000, 20, 1, 10, 4, "l"))
+    x, info = gpu_solve(cap, si, 3, protocol=proto, subwarp=epl)
+    assert info["n_sub_tasks"] > 0, info
+    assert np.array_equal(x, si.x_true)
+    for flags in (1, 2, 3):
+        t = synth.gen_leveled(30_000, 30, 1, 10, 7, "lt")
+        t = synth.to_upper(t) if flags & 1 else t
+        t = synth.to_unit(t, upper=bool(flags & 1)) if flags & 2 else t
+        rp, ci, v, b = dev_csr(t)
+        with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2), mode=3, subwarp=epl) as h:
+            x = torch.full_like(b, float("nan"))
+            h.solve(b, x)
+            h.check()
+            assert h.info()["engine"] == 6
+            ref = oracle.solve_tri(t.rowptr, t.colidx, t.val, t.b, flags)
+            assert relerr(x.cpu().numpy(), ref) <= TOL, flags
+
+
+def test_subwarp_plan_widths(cap):
+    """The plan gives a 32-row group W = the smallest power of two with W * epl >= its mean
+    off-diagonals per row (capped at 32 = a warp row): checked through the task counts."""
+    s = synth.gen_leveled(64_000, 64, 1, 15, 8, "l16")  # 16 off-diagonals per row
+    for epl, w in ((1, 16), (2, 8), (4, 4), (8, 2), (16, 2)):
+        _, info = gpu_solve(cap, s, 3, subwarp=epl)
+        groups = (s.n + 31) // 32 - 32  # level 0 (1000 rows, diagonal only) stays mixed; count the rest
+        assert info["n_sub_tasks"] >= groups * w, (epl, info)
+        assert info["n_sub_tasks"] <= ((s.n + 31) // 32) * w, (epl, info)
 
 
 @pytest.mark.parametrize("nrhs", [1, 2, 3, 4, 7, 8, 16, 32])
@@ -604,3 +650,90 @@ def test_flag_latency_runs(cap):
     for proto in (0, 1, 2, 3, 4):
         t = cap.flag_latency(2000, proto)
         assert 10.0 < t < 100_000.0
+
+
+# ------------------------------------------------------------------ failure detection (watchdog, stale graphs)
+
+@pytest.mark.parametrize("engine,gen", [(3, "chain"), (7, "grid"), (6, "dense"), (0, "chain")])
+def test_watchdog_fires_and_next_solve_is_exact(cap, engine, gen):
+    """SPTRSV_OPT_SPIN_LIMIT = 1: the first warp that idles 64 passes raises the sticky error and
+    the abort word, every spinning warp bails out, and sptrsv_check reports SPTRSV_ERR_TIMEOUT
+    (the failure mode of the method: Alg.5 only terminates at the diagonal).  The
+    check clears the condition; the next solve (default limit) re-zeroes the ready words and must
+    match the oracle exactly."""
+    s = {"chain": lambda: synth.gen_chain(60_000), "grid": lambda: synth.gen_grid(300),
+         "dense": lambda: synth.gen_dense_lower(1500)}[gen]()
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v, engine=engine, mode=1 if engine != 6 else 2) as h:
+        default = h.get_option(cap.OPT_SPIN_LIMIT)
+        h.set_option(cap.OPT_SPIN_LIMIT, 1)
+        x = torch.full_like(b, float("nan"))
+        h.solve(b, x)
+        with pytest.raises(cap.SptrsvError) as e:
+            h.check()
+        assert e.value.status == cap._lib.ERR_TIMEOUT
+        h.check()  # cleared
+        h.set_option(cap.OPT_SPIN_LIMIT, default)
+        x.fill_(float("nan"))
+        h.solve(b, x)
+        h.check()
+        got = x.cpu().numpy()
+        if engine == 6:
+            assert relerr(got, ref) <= TOL
+        else:
+            assert np.array_equal(got, ref)
+
+
+def test_stale_graph_replay_is_refused(cap):
+    """A CUDA graph captured under one launch configuration and replayed after the handle was
+    re-configured (here: another CTA size, so the ready words were re-zeroed under a new
+    generation) must not solve with stale epochs: sptrsv_check reports SPTRSV_ERR_STALE_LAUNCH,
+    and a re-captured graph solves exactly."""
+    s = synth.gen_c2i(n=40_000)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v, engine=3) as h:
+        st = torch.cuda.Stream()
+        x = torch.empty_like(b)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(st):
+            h.solve(b, x, stream=st)
+            st.synchronize()
+            with torch.cuda.graph(g, stream=st):
+                h.solve(b, x, stream=st)
+        g.replay()
+        torch.cuda.synchronize()
+        h.check(st)
+        assert np.array_equal(x.cpu().numpy(), ref)
+        h.set_option(cap.OPT_CTA_THREADS, 128)  # new launch configuration
+        with torch.cuda.stream(st):
+            h.solve(b, x, stream=st)  # resets the ready words under a new generation
+        h.check(st)
+        g.replay()  # stale: captured with the old grid / generation
+        torch.cuda.synchronize()
+        with pytest.raises(cap.SptrsvError) as e:
+            h.check(st)
+        assert e.value.status == cap._lib.ERR_STALE_LAUNCH
+        x.fill_(float("nan"))
+        g2 = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(st):
+            h.solve(b, x, stream=st)
+            st.synchronize()
+            with torch.cuda.graph(g2, stream=st):
+                h.solve(b, x, stream=st)
+        x.fill_(float("nan"))
+        g2.replay()
+        torch.cuda.synchronize()
+        h.check(st)
+        assert np.array_equal(x.cpu().numpy(), ref)
+
+
+def test_handle_rejects_tensors_on_another_device(cap):
+    """The binding checks the device of b / x against the handle's; the C ABI
+    rejects a solve whose handle device is not current."""
+    s = synth.gen_c1()
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        with pytest.raises((ValueError, TypeError)):
+            h.solve(b.cpu(), None)

@@ -35,6 +35,11 @@ def delta_table6(n_level, nnz_row):
 
 VARIANTS = {"alg3": dict(variant=3), "alg4": dict(variant=4), "alg5": dict(variant=5),
             "thread": dict(mode=1, engine=0), "warp": dict(mode=2, engine=0), "auto": dict()}
+if os.environ.get("ABLATION_SET") == "f2":  # thread / sub-warp widths / warp, and AUTO variants
+    VARIANTS = {"thread": dict(mode=1), "lean": dict(mode=1, engine=3), "warp": dict(mode=2),
+                "sub_e1": dict(mode=3, subwarp=1), "sub_e2": dict(mode=3, subwarp=2), "sub_e4": dict(mode=3, subwarp=4),
+                "sub_e8": dict(mode=3, subwarp=8), "auto": dict(), "auto_e2": dict(subwarp=2),
+                "auto_e4": dict(subwarp=4), "auto_e8": dict(subwarp=8)}
 
 
 def timeit(h, b, x, reps=5, limit_s=20.0):
@@ -77,10 +82,13 @@ for levels in (10, 100, 1000, 10000):
                 assert err <= 1e-12, (name, err)
                 rec["gflops"][name] = round(2 * s.nnz / t / 1e9, 3)
         g = rec["gflops"]
-        rec["alg5_over_alg4"] = round(g["alg5"] / g["alg4"], 2)
-        rec["alg5_over_alg3"] = round(g["alg5"] / g["alg3"], 2)
-        rec["ours_over_alg5"] = round(g["auto"] / g["alg5"], 2)
+        if "alg5" in g:
+            rec["alg5_over_alg4"] = round(g["alg5"] / g["alg4"], 2)
+            rec["alg5_over_alg3"] = round(g["alg5"] / g["alg3"], 2)
+            rec["ours_over_alg5"] = round(g["auto"] / g["alg5"], 2)
         rec["thread_over_warp"] = round(g["thread"] / g["warp"], 2)
+        ours = [v for k, v in g.items() if not k.startswith("alg")]
+        rec["auto_over_best"] = round(g["auto"] / max(ours), 3)
         print(json.dumps(rec), flush=True)
         if out:
             out.write(json.dumps(rec) + "\n")
