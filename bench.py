@@ -618,22 +618,59 @@ def run_single(args):
 
 # ------------------------------------------------------------------ N > 1: batches over devices / ranks
 
-def run_batch(args, rank, world, dist=None):
-    """C5 (or replicas of another config) over N GPUs.  world > 1: this process is one rank of
-    torchrun and drives GPU LOCAL_RANK; world == 1: this process drives args.gpus devices."""
-    import torch
-    from paper_conf_icpp_suz0hw0w20_b200.batch import MultiDeviceBatch, max_over_ranks, shard, sum_over_ranks
+class CudaEnv:
+    """What run_batch needs from the machine: devices, the batch runner, L2 flushes, pinned host
+    buffers, clock sampling.  (tests/test_multiproc.py swaps in a CPU stand-in to run the same
+    rank / shard / max-over-ranks path under gloo without a GPU.)"""
 
-    ndev = torch.cuda.device_count()
-    if world > 1:
-        local = int(os.environ.get("LOCAL_RANK", "0"))
-        if local >= ndev:
-            raise SystemExit(f"bench.py: rank {rank} needs GPU {local} but only {ndev} visible")
-        devices = [local]
-    else:
+    def __init__(self):
+        import torch
+        self.torch = torch
+
+    def devices(self, args, rank, world):
+        ndev = self.torch.cuda.device_count()
+        if world > 1:
+            local = int(os.environ.get("LOCAL_RANK", "0"))
+            if local >= ndev:
+                raise SystemExit(f"bench.py: rank {rank} needs GPU {local} but only {ndev} visible")
+            return [local]
         if args.gpus > ndev:
             raise SystemExit(f"bench.py --gpus {args.gpus}: only {ndev} CUDA device(s) visible")
-        devices = list(range(args.gpus))
+        return list(range(args.gpus))
+
+    def make_batch(self, systems, devices, opts):
+        from paper_conf_icpp_suz0hw0w20_b200.batch import MultiDeviceBatch
+        return MultiDeviceBatch([(s.rowptr, s.colidx, s.val, s.b) for s in systems], devices, **opts)
+
+    def make_flush(self, batch):
+        torch = self.torch
+        bufs = []
+        for d in batch.devices:
+            with torch.cuda.device(d):
+                bufs.append(torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=d))
+        return lambda g: bufs[g].zero_()
+
+    def host_buffers(self, systems):
+        torch = self.torch
+        return ([torch.from_numpy(s.b).pin_memory() for s in systems],
+                [torch.empty(s.n, dtype=torch.float64).pin_memory() for s in systems])
+
+    @staticmethod
+    def numpy(t):
+        return t.cpu().numpy()
+
+    def clocks(self, devices):
+        return ClockSampler(devices)
+
+
+def run_batch(args, rank, world, dist=None, env=None):
+    """C5 (or replicas of another config) over N GPUs.  world > 1: this process is one rank of
+    torchrun and drives GPU LOCAL_RANK; world == 1: this process drives args.gpus devices.
+    Every collective below (barrier, max / sum over ranks) runs on every rank."""
+    from paper_conf_icpp_suz0hw0w20_b200.batch import max_over_ranks, shard, sum_over_ranks
+
+    env = env or CudaEnv()
+    devices = env.devices(args, rank, world)
     n_gpus = args.gpus if world == 1 else world
     opts = {"mode": args.mode, "protocol": 1}
     for kv in args.opt:
@@ -647,19 +684,12 @@ def run_batch(args, rank, world, dist=None):
         owned = list(range(len(devices)))
         systems = [make_system(args.config, rank * len(devices) + k) for k in range(len(devices))]
         scaling = "weak"
-    batch = MultiDeviceBatch([(s.rowptr, s.colidx, s.val, s.b) for s in systems], devices, **opts)
-    flushes = []
-    for d in batch.devices:
-        with torch.cuda.device(d):
-            flushes.append(torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=d))
-
-    def flush(g):
-        flushes[g].zero_()
-
+    batch = env.make_batch(systems, devices, opts)
+    flush = env.make_flush(batch)
     for _ in range(args.warmup):
         batch.timed_solve(flush)
     batch.check()
-    sampler = ClockSampler(devices)
+    sampler = env.clocks(devices)
     sampler.__enter__()
     if dist is not None:
         dist.barrier()
@@ -679,8 +709,7 @@ def run_batch(args, rank, world, dist=None):
     value = 2.0 * nnz_all * args.steps / tot_s / 1e9
 
     # e2e through the public API: pinned host b -> device -> solve -> host x, every step
-    hb = [torch.from_numpy(s.b).pin_memory() for s in systems]
-    hx = [torch.empty(s.n, dtype=torch.float64).pin_memory() for s in systems]
+    hb, hx = env.host_buffers(systems)
     batch.solve_host(hb, hx)
     if dist is not None:
         dist.barrier()
@@ -690,14 +719,15 @@ def run_batch(args, rank, world, dist=None):
         batch.solve_host(hb, hx)
         e_t.append(time.perf_counter() - t0)
     et = max_over_ranks(float(np.sum(e_t)), dist)
-    ok = all(np.array_equal(hx[k].numpy(), batch.x(k).cpu().numpy()) for k in range(len(systems)))
+    ok = all(np.array_equal(env.numpy(hx[k]), env.numpy(batch.x(k))) for k in range(len(systems)))
+    ok = sum_over_ranks(0.0 if ok else 1.0, dist) == 0.0
+    h2d = int(sum_over_ranks(float(sum(8 * s.n for s in systems)), dist))
     e2e = {"value": 2.0 * nnz_all * args.steps / et / 1e9, "unit": UNIT,
-           "h2d_bytes_per_step": int(sum_over_ranks(float(sum(8 * s.n for s in systems)), dist)),
-           "d2h_bytes_per_step": int(sum_over_ranks(float(sum(8 * s.n for s in systems)), dist)),
-           "matches_device_path": bool(ok),
+           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d, "matches_device_path": bool(ok),
            "timing": "host wall clock per step around sptrsv_solve_host of every owned system (one host thread "
                      "per device), max over ranks"}
     launches = int(sum_over_ranks(float(args.steps * len(systems)), dist))
+    systems_total = int(sum_over_ranks(float(len(systems)), dist))
     info = batch.handles[0].info()
     if rank == 0:
         line = {
@@ -706,12 +736,12 @@ def run_batch(args, rank, world, dist=None):
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": f"{args.config}: {WORKLOADS[args.config]}",
-                       "systems_total": 8 if args.config == "c5" else int(sum_over_ranks(len(systems), dist)),
+                       "systems_total": systems_total,
                        "n_per_system": systems[0].n, "nnz_per_system": systems[0].nnz,
                        "engine": ENGINES.get(info["engine"], str(info["engine"])),
                        "parallelism": (f"{n_gpus} GPUs, system s on GPU s mod {n_gpus}, one stream per device, "
                                        "no inter-GPU exchange (no NCCL)") + (
-                           f"; torchrun ranks, gloo control plane" if world > 1 else "; one host process"),
+                           "; torchrun ranks, gloo control plane" if world > 1 else "; one host process"),
                        "timing": "per-device CUDA events around each device's solves on its stream; step = max over "
                                  "devices; L2 flushed before every step outside the events",
                        "options": opts},

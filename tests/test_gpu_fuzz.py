@@ -85,7 +85,7 @@ def test_fuzz_engines_vs_oracle(seed):
                 h.check()
                 got = x.cpu().numpy()
                 info = h.info()
-                if info["n_warp_rows"] == 0:
+                if info["n_warp_rows"] == 0 and info["n_sub_tasks"] == 0:
                     assert np.array_equal(got, ref), (s.name, s.n, engine, proto, extra, info)
                 else:
                     err = float(np.max(np.abs(got - ref) / np.abs(ref))) if s.n else 0.0

@@ -65,3 +65,138 @@ def test_shard_single_rank_and_errors():
     assert b.shard(8, 7, 8) == [7]
     with pytest.raises(ValueError):
         b.shard(8, 2, 2)
+
+
+# ------------------------------------------------------------------ the bench's own N>1 rank path
+
+class _CpuBatch:
+    """CPU stand-in for MultiDeviceBatch with the same interface: every 'device' solves its systems
+    with the oracle (wall clock as its event span) -- so bench.run_batch's rank / shard / timing /
+    max-over-ranks path runs under gloo without a GPU."""
+
+    def __init__(self, systems, devices):
+        import oracle
+        self.oracle = oracle
+        self.systems = systems
+        self.devices = devices
+        self.owner = [s % len(devices) for s in range(len(systems))]
+        self.xs = [np.zeros(s.n) for s in systems]
+        self.solved = 0
+
+    class _H:
+        @staticmethod
+        def info():
+            return {"engine": 3}
+
+    @property
+    def handles(self):
+        return [self._H()]
+
+    def timed_solve(self, before=None):
+        ms = []
+        for g in range(len(self.devices)):
+            if before:
+                before(g)
+            t0 = time.perf_counter()
+            for s, o in enumerate(self.owner):
+                if o == g:
+                    sy = self.systems[s]
+                    self.xs[s] = self.oracle.solve(sy.rowptr, sy.colidx, sy.val, sy.b)
+                    self.solved += 1
+            ms.append((time.perf_counter() - t0) * 1e3)
+        return ms
+
+    def solve_host(self, hb, hx):
+        for s, sy in enumerate(self.systems):
+            hx[s][:] = self.oracle.solve(sy.rowptr, sy.colidx, sy.val, hb[s])
+
+    def synchronize(self):
+        pass
+
+    def check(self):
+        pass
+
+    def x(self, s):
+        return self.xs[s]
+
+    def close(self):
+        pass
+
+
+class _CpuEnv:
+    def devices(self, args, rank, world):
+        return [0] if world > 1 else list(range(args.gpus))
+
+    def make_batch(self, systems, devices, opts):
+        return _CpuBatch(systems, devices)
+
+    def make_flush(self, batch):
+        return lambda g: None
+
+    def host_buffers(self, systems):
+        return [s.b.copy() for s in systems], [np.zeros(s.n) for s in systems]
+
+    @staticmethod
+    def numpy(t):
+        return t
+
+    def clocks(self, devices):
+        class _S:
+            def __enter__(self):
+                return self
+
+            def __exit__(self, *a):
+                pass
+
+            def summary(self):
+                return {"sm_mhz": None, "reasons": ["cpu stand-in"]}
+        return _S()
+
+
+def _bench_worker(rank, world, port, q, config):
+    import contextlib
+    import io
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update({"RANK": str(rank), "WORLD_SIZE": str(world), "LOCAL_RANK": "0"})
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    import bench
+    args = bench.parse(["--gpus", str(world), "--steps", "2", "--warmup", "1", "--config", config])
+    env = _CpuEnv()
+    out = io.StringIO()
+    with contextlib.redirect_stdout(out):
+        bench.run_batch(args, rank, world, dist, env=env)
+    dist.destroy_process_group()
+    q.put((rank, out.getvalue()))
+
+
+import time  # noqa: E402
+
+import numpy as np  # noqa: E402
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_bench_rank_path_gloo(world):
+    """bench.py's N>1 path itself (run_batch, as torchrun launches it), with a CPU stand-in for the
+    device batch: the C5 systems are sharded s -> rank s mod N (each exactly once), only rank 0
+    prints, the line reports n_gpus = N, all 8 systems' launches, and a value equal to
+    (8 systems' 2*nnz * steps) / (max over ranks of the summed step times)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bench_worker, args=(r, world, port, q, "c5")) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=600) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    import json
+    assert all(not out[r].strip() for r in range(1, world))  # only rank 0 prints
+    line = json.loads(out[0].strip().splitlines()[-1])
+    assert line["n_gpus"] == world and line["scaling"] == "strong"
+    assert line["gpu_launches"] == 8 * 2 and line["config"]["systems_total"] == 8
+    assert line["e2e"]["matches_device_path"] is True
+    assert line["e2e"]["h2d_bytes_per_step"] == 8 * 8 * 2_000_000
+    nnz = 8 * 5_600_000
+    assert abs(line["value"] - 2.0 * nnz * 2 / (line["ms_per_step"] * 2 * 1e-3) / 1e9) <= 1e-3 * line["value"]
