@@ -48,6 +48,10 @@ typedef enum sptrsv_status {
     SPTRSV_ERR_CUDA = -9,         /* a CUDA runtime call failed (launch, copy, ...)         */
     SPTRSV_ERR_ALLOC = -10,       /* device / pinned allocation failed                      */
     SPTRSV_ERR_TIMEOUT = -11,     /* watchdog: a solve spun past SPTRSV_OPT_SPIN_LIMIT      */
+    SPTRSV_ERR_INEXACT = -13,     /* a CHAIN solve found a quotient that failed its exactness
+                                     proof (never observed): the solve
+                                     was aborted and the handle switched to in-loop proofs
+                                     (SPTRSV_OPT_CHAIN_DIV = 1); re-solve                   */
     SPTRSV_ERR_STALE_LAUNCH = -12 /* a solve captured in a CUDA graph was replayed after the
                                      handle's launch configuration changed (an option
                                      change or a watchdog reset re-zeroes the ready words
@@ -128,6 +132,13 @@ typedef enum sptrsv_option {
                                       from the median nearest-dependency distance (DESIGN.md
                                       section 6); AUTO caps W at 16.  Setting it re-plans
                                       (synchronous).                                        */
+    SPTRSV_OPT_CHAIN_DIV = 25,     /* CHAIN's division proof (Diag::exact, DESIGN.md section
+                                      6): 0 (default) = the chain runs the Markstein candidate
+                                      and proves each run's quotients right after it, all
+                                      lanes in parallel (a failure aborts the solve with
+                                      SPTRSV_ERR_INEXACT); 1 = prove every quotient before the
+                                      chain uses it (+~25 cycles per chain step); 2 = test
+                                      hook: every post-run proof fails                      */
     SPTRSV_OPT_HOST_IO = 23,       /* sptrsv_solve_host with pinned buffers on LEAN: bit 0 =
                                       b copied in chunks on a second stream, each CTA waiting
                                       for its own chunk only (needs cuStreamWriteValue32);

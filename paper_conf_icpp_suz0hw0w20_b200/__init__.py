@@ -204,7 +204,7 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "poll_gap_ns": _lib.OPT_POLL_GAP_NS,
             "poll_one": _lib.OPT_POLL_ONE,
             "warp_split_last": _lib.OPT_WARP_SPLIT_LAST,
-            "host_io": _lib.OPT_HOST_IO, "subwarp": _lib.OPT_SUBWARP}
+            "host_io": _lib.OPT_HOST_IO, "subwarp": _lib.OPT_SUBWARP, "chain_div": _lib.OPT_CHAIN_DIV}
     for k, v in options.items():
         h.set_option(keys[k], v)
     return h

@@ -36,6 +36,7 @@ ERR_CUDA = -9
 ERR_ALLOC = -10
 ERR_TIMEOUT = -11
 ERR_STALE_LAUNCH = -12
+ERR_INEXACT = -13
 
 # options
 OPT_MODE = 1
@@ -57,6 +58,7 @@ OPT_POLL_ONE = 20
 OPT_WARP_SPLIT_LAST = 22
 OPT_HOST_IO = 23
 OPT_SUBWARP = 24
+OPT_CHAIN_DIV = 25
 ENGINE_ONESHOT, ENGINE_LEAN, ENGINE_AUTO, ENGINE_HYBRID, ENGINE_CHAIN = 0, 3, 5, 6, 7
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP, MODE_SUBWARP = 0, 1, 2, 3

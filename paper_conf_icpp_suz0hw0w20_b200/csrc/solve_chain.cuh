@@ -51,7 +51,13 @@ __host__ __device__ constexpr int chain_warp_smem_bytes(int K) {
 // off-diagonals are walked earliest-solved first (descending physical column for upper), its
 // diagonal is the first entry (upper), the last (lower) or implicit 1 (unit).  Loads of CSR
 // entries, polls and publication use physical indices.
-template <int PROTO, int K, bool UPPER = false, bool UNIT = false>
+// SAFE (SPTRSV_OPT_CHAIN_DIV = 1): the fast loop proves every quotient before using it (Diag::exact
+// in the loop condition, +~25 cycles per chain step).  Otherwise (default) the fast loop runs the
+// Markstein candidate at full speed and the rows of each run are proven right after the run, all
+// lanes in parallel; a candidate that is not RN(a/d) -- never observed --
+// aborts the solve with kErrInexact, sptrsv_check reports SPTRSV_ERR_INEXACT and switches the
+// handle to SAFE, so no solve ever returns an unproven quotient.
+template <int PROTO, int K, bool UPPER = false, bool UNIT = false, bool SAFE = false>
 __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams p) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint32_t s_blk, s_epoch;
@@ -154,6 +160,8 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
     const bool tracing = p.trace != nullptr;
     int s = 0;  // next row (warp-relative) to finalize; rows < s are published
     uint32_t backoff = p.backoff_min, idle = 0;
+    // the fast loop's rows of the current pass, proven after the run (!SAFE)
+    int vf0 = 0, vf1 = 0;
     while (true) {
         bool prog = false;
         // ---- A. external dependencies: one poll per unfinished row, K in flight
@@ -221,19 +229,33 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                 f_has[t] = prev ? 1 : 0;
             }
         }
+        vf0 = vf1 = s;
         if (run_end > s && __all_sync(FULL, el)) {
             __syncwarp();
             double xp = 0.0;  // x of row t - 1 (read only when row t has that entry)
-            // The division of row t is verified ONE STEP LATE (Diag::exact, the remainder proof):
-            // the test for row t-1 runs while row t's chain is in flight, and row t-1 is only
-            // committed -- owner registers, its record published -- once it passed.  A failed row
-            // is redone by the exact loop below.  The chain itself never waits for the test.
-            double xc = 0.0;                              // x of row t - 2 (committed)
-            double pa = 0.0, pd = 1.0, pq = 0.0;          // the pending row t-1: numerator, divisor, candidate
-            int ph = 0;                                   // ... and whether it had the previous-row entry
-            bool pending = false;
-            auto commit = [&](int tt, double q) {
-                const int owner = tt & 31, kk = tt >> 5;
+            // operands of row t are loaded one iteration ahead, off the dependency chain
+            double lsv = f_ls[s], bv = f_b[s], vv = f_v[s], dv = f_d[s], rv = f_r[s];
+            int hv = f_has[s];
+            int t = s;
+            for (; t < run_end; ++t) {
+                const int tn = min(t + 1, run_end - 1);
+                const double lsn = f_ls[tn], bn = f_b[tn], vn = f_v[tn], dn = f_d[tn], rn = f_r[tn];
+                const int hn = f_has[tn];
+                const double u = hv ? __dadd_rn(lsv, __dmul_rn(vv, xp)) : lsv;
+                const double a = __dsub_rn(bv, u);
+                Diag g;
+                g.d = dv;
+                g.r = rv;
+                const double q = g.cand(a);
+                // guard (Diag::ok) in integer ops, warp-uniform here (every lane holds the same a).  A
+                // failure LEAVES the fast loop instead of branching around an in-loop __ddiv_rn: the
+                // loop body then has no reconvergence point, and the guard resolves from a while the
+                // Markstein step is still in flight (chain step ~140 -> ~90 cycles, chainstep.cu)
+                if (__builtin_expect(!(Diag::in_range(a) && __double2hiint(rv) != 0 &&
+                                       (!SAFE || Diag::exact(a, dv, q))), 0))
+                    break;
+                if (!SAFE) f_ls[t] = a;  // the numerator, for the proof after the run (own store, all lanes)
+                const int owner = t & 31, kk = t >> 5;
                 const bool mine = lane == owner;
 #pragma unroll
                 for (int k = 0; k < K; ++k) {
@@ -246,54 +268,13 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                     unsigned long long bits = (unsigned long long)__double_as_longlong(q);
                     bits = bits == kSentinel ? kCanonNaN : bits;
                     const unsigned long long e = (unsigned long long)epoch << 32;
-                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)phys(r0 + tt), e | (bits & 0xffffffffull), e | (bits >> 32));
-                    if (tracing) st_u64_if(mine, p.trace + phys(r0 + tt), globaltimer_ns());
+                    st_relaxed_v2_u64_if(mine, p.rec + 2 * (size_t)phys(r0 + t), e | (bits & 0xffffffffull), e | (bits >> 32));
+                    if (tracing) st_u64_if(mine, p.trace + phys(r0 + t), globaltimer_ns());
                 }
-            };
-            // operands of row t are loaded one iteration ahead, off the dependency chain
-            double lsv = f_ls[s], bv = f_b[s], vv = f_v[s], dv = f_d[s], rv = f_r[s];
-            int hv = f_has[s];
-            int t = s;
-            for (; t < run_end; ++t) {
-                const int tn = min(t + 1, run_end - 1);
-                const double lsn = f_ls[tn], bn = f_b[tn], vn = f_v[tn], dn = f_d[tn], rn = f_r[tn];
-                const int hn = f_has[tn];
-                const bool pok = !pending || Diag::exact(pa, pd, pq);  // row t-1's proof
-                const double u = hv ? __dadd_rn(lsv, __dmul_rn(vv, xp)) : lsv;
-                const double a = __dsub_rn(bv, u);
-                Diag g;
-                g.d = dv;
-                g.r = rv;
-                const double q = g.cand(a);
-                // range guard (Diag::ok) in integer ops, warp-uniform here (every lane holds the same a).
-                // A failure LEAVES the fast loop instead of branching around an in-loop __ddiv_rn: the
-                // loop body then has no reconvergence point (chain step ~140 -> ~90 cycles, chainstep.cu)
-                const bool gok = Diag::in_range(a) && __double2hiint(rv) != 0;
-                if (__builtin_expect(!pok, 0)) {  // row t-1's candidate was not RN: redo it exactly
-                    --t;
-                    xp = xc;
-                    hv = ph;
-                    pending = false;
-                    break;
-                }
-                if (pending) commit(t - 1, pq);
-                pending = false;
-                if (__builtin_expect(!gok, 0)) break;
-                pending = true;
-                pa = a, pd = dv, pq = q, ph = hv;
-                xc = xp;
                 xp = q;
                 lsv = lsn, bv = bn, vv = vn, dv = dn, rv = rn, hv = hn;
             }
-            if (pending) {  // the run's last row: its proof, then commit or redo
-                if (Diag::exact(pa, pd, pq)) {
-                    commit(t - 1, pq);
-                } else {
-                    --t;
-                    xp = xc;
-                    hv = ph;
-                }
-            }
+            vf1 = t;
             if (t < run_end && hv) {
                 // the guard failed at row t: the exact loop below finishes the run from t.  Row t's
                 // previous-row entry is consumed first, by its owner, with the same mul and add as the
@@ -343,6 +324,23 @@ __global__ void __launch_bounds__(256, K == 1 ? 4 : 3) k_solve_chain(SolveParams
                     ls[m] = c ? t : ls[m];
                     if (c) advance(m);
                 }
+            }
+        }
+        if (!SAFE && !UNIT && vf1 > vf0) {
+            // the proof of the fast loop's quotients (Diag::exact), one row per owner lane: row t's
+            // numerator is f_ls[t], its quotient the owner's xm
+            bool bad = false;
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+                const int t = lane + 32 * k;
+                if (t >= vf0 && t < vf1) bad |= (p.chain_div == 2) | !Diag::exact(f_ls[t], f_d[t], xm[k]);
+            }
+            if (__any_sync(FULL, bad)) {
+                if (lane == 0) {
+                    atomicCAS(&p.st->error.v, 0u, kErrInexact);
+                    st_relaxed_u32(&p.st->abort.v, 1u);
+                }
+                return;
             }
         }
         if (s > s0) {

@@ -24,28 +24,49 @@ namespace sptrsv_dev {
 
 constexpr int kLeanCta = 256;
 
-// One warp, one row per lane (Alg.5 l.3-18): lane's row i (act: i is a real row), its
-// bounds [rs, re) and b_i already loaded.  Returns when every lane of the warp has
-// published, or on abort.  Shared by k_solve_lean and the f4 list kernel (solve_tri.cuh).
-template <int PROTO, bool UPPER, bool UNIT>
-__device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, int rs, int re, double bi,
-                                          uint32_t epoch, int lane, uint64_t pol) {
+// A lane's row once its second-level loads are issued: the off-diagonals [lo, hi) walked from j
+// (earliest-solved first), the next two dependencies (column, value) and L_ii.
+struct LeanRow {
+    int lo, hi, j, nc, nc2;
+    double nv, nv2, dv;
+};
+
+// Second-level loads of row i with bounds [rs, re): L_ii and the first two dependencies.  Split from
+// lean_rows so that k_solve_lean can issue them BEFORE the CTA barrier that waits for the start
+// ticket: the ticket's same-address atomic then overlaps both load phases.
+template <bool UPPER, bool UNIT>
+__device__ __forceinline__ LeanRow lean_load(const SolveParams &p, bool act, int rs, int re, uint64_t pol) {
     // off-diagonal entries [lo, hi); the diagonal is last (lower), first (upper) or implicit
     // (unit).  They are consumed earliest-solved first: ascending for lower (Alg.1 l.3-4),
     // DESCENDING for upper (G25) -- the nearest, latest dependency is waited for last.
-    const int lo = (UPPER && !UNIT) ? rs + 1 : rs;
-    const int hi = (UPPER || UNIT) ? re : re - 1;
+    LeanRow r;
+    r.lo = (UPPER && !UNIT) ? rs + 1 : rs;
+    r.hi = (UPPER || UNIT) ? re : re - 1;
     constexpr int dir = UPPER ? -1 : 1;
-    auto inr = [&](int k) { return UPPER ? k >= lo : k < hi; };
-    int j = UPPER ? hi - 1 : lo;
-    // ---- second-level loads: L_ii and the next two dependencies
-    double dv = (act && !UNIT) ? ld_stream_f64(p.val + (UPPER ? rs : re - 1), pol) : 1.0;
-    int nc = (act && inr(j)) ? ld_stream_i32(p.colidx + j, pol) : -1;
-    double nv = (act && inr(j)) ? ld_stream_f64(p.val + j, pol) : 0.0;
-    int nc2 = (act && inr(j + dir)) ? ld_stream_i32(p.colidx + j + dir, pol) : -1;
+    auto inr = [&](int k) { return UPPER ? k >= r.lo : k < r.hi; };
+    r.j = UPPER ? r.hi - 1 : r.lo;
+    r.dv = (act && !UNIT) ? ld_stream_f64(p.val + (UPPER ? rs : re - 1), pol) : 1.0;
+    r.nc = (act && inr(r.j)) ? ld_stream_i32(p.colidx + r.j, pol) : -1;
+    r.nv = (act && inr(r.j)) ? ld_stream_f64(p.val + r.j, pol) : 0.0;
+    r.nc2 = (act && inr(r.j + dir)) ? ld_stream_i32(p.colidx + r.j + dir, pol) : -1;
     // the second dependency's VALUE is preloaded too: consuming both dependencies in one pass
     // (the common case when the earlier one is long solved) then never waits on a reload
-    double nv2 = (act && inr(j + dir)) ? ld_stream_f64(p.val + j + dir, pol) : 0.0;
+    r.nv2 = (act && inr(r.j + dir)) ? ld_stream_f64(p.val + r.j + dir, pol) : 0.0;
+    return r;
+}
+
+// One warp, one row per lane (Alg.5 l.3-18): lane's row i (act: i is a real row), b_i and its
+// second-level loads (lean_load) already issued.  Returns when every lane of the warp has
+// published, or on abort.  Shared by k_solve_lean and the f4 list kernel (solve_tri.cuh).
+template <int PROTO, bool UPPER, bool UNIT>
+__device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, const LeanRow &lr, double bi,
+                                          uint32_t epoch, int lane, uint64_t pol) {
+    const int lo = lr.lo, hi = lr.hi;
+    constexpr int dir = UPPER ? -1 : 1;
+    auto inr = [&](int k) { return UPPER ? k >= lo : k < hi; };
+    int j = lr.j, nc = lr.nc, nc2 = lr.nc2;
+    double nv = lr.nv, nv2 = lr.nv2;
+    const double dv = lr.dv;
     Diag dg;
     dg.init(dv);
     if (p.trace && act && nc != -2) p.trace[2 * (size_t)p.n + i] = globaltimer_ns();  // loads landed
@@ -128,7 +149,11 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint64_t pol = policy_evict_first();
-    // ---- speculative first-level loads for logical block == blockIdx.x
+    // ---- the start ticket's atomic is issued first; its result is only needed at the barrier, so
+    // it overlaps the speculative loads (logical block == blockIdx.x, the common case) of both
+    // levels: rowptr / b, then L_ii and the first two dependencies
+    unsigned long long tk = 0;
+    if (tid == 0) tk = atomicAdd(&p.st->tk.v, 1ull);
     int i = (int)blockIdx.x * CT + tid;
     if (UPPER) i = p.n - 1 - i;
     int rs = 0, re = 1;
@@ -140,12 +165,13 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         re = ld_stream_i32(p.rowptr + i + 1, pol);
         if (!bgate) bi = ld_b(p, i, pol);
     }
+    LeanRow lr = lean_load<UPPER, UNIT>(p, i >= 0 && i < p.n, rs, re, pol);
     if (tid == 0) {
         if (p.trace) {
             atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
             atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
         }
-        cta_ticket(p, s_blk, s_epoch);
+        cta_ticket_decode(p, tk, s_blk, s_epoch);
         if (bgate) {  // wait until the b chunks of this CTA's (physical) rows have landed
             const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
             wait_b_chunks(p, UPPER ? p.n - lr1 : lr0, UPPER ? p.n - lr0 : lr1);
@@ -163,11 +189,12 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
             re = ld_stream_i32(p.rowptr + i + 1, pol);
             bi = ld_b(p, i, pol);
         }
+        lr = lean_load<UPPER, UNIT>(p, i >= 0 && i < p.n, rs, re, pol);
     } else if (bgate && i >= 0 && i < p.n) {
         bi = ld_b(p, i, pol);
     }
     const bool act = i >= 0 && i < p.n;
-    lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);
+    lean_rows<PROTO, UPPER, UNIT>(p, i, act, lr, bi, epoch, lane, pol);
     if (p.trace && lane == 0) atomicMax(&p.trace[3 * (size_t)p.n + 1], globaltimer_ns());  // last warp exit
     if (p.x_host) {
         // sptrsv_solve_host: the CTA's finished rows go to pinned host memory over PCIe as one

@@ -210,15 +210,15 @@ __device__ __forceinline__ void subwarp_task(SolveParams &p, int r0, int w, uint
 // PLAN_WARP: task t = logical row t.  PLAN_LIST: tasks[t] >= 0 is a 32-row thread-level
 // group starting at that logical row (one row per lane, lean_rows), ~row a warp-level row;
 // the list is in logical (ticket) order, built by build_plan over reversed rows for UPPER.
-template <int PROTO, bool UPPER, bool UNIT, int PLAN>
-__global__ void __launch_bounds__(kTriWarpCta) k_solve_tri_warp(SolveParams p) {
+template <int PROTO, bool UPPER, bool UNIT, int PLAN, int CT = kTriWarpCta>
+__global__ void __launch_bounds__(CT) k_solve_tri_warp(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         cta_ticket(p, s_blk, s_epoch);
         if (p.bflag) {  // sptrsv_solve_host: the b chunks of this CTA's tasks' (physical) rows
             int lo = p.n, hi = 0;  // logical row range of the CTA's tasks
-            for (int t = (int)s_blk * (kTriWarpCta / 32); t < min(p.n_tasks, ((int)s_blk + 1) * (kTriWarpCta / 32)); ++t) {
+            for (int t = (int)s_blk * (CT / 32); t < min(p.n_tasks, ((int)s_blk + 1) * (CT / 32)); ++t) {
                 int r0 = t, r1 = t + 1;
                 if (PLAN == PLAN_LIST) {
                     const int v = p.tasks[t];
@@ -235,7 +235,7 @@ __global__ void __launch_bounds__(kTriWarpCta) k_solve_tri_warp(SolveParams p) {
     __syncthreads();
     if (s_blk == kStaleBlk) return;
     const uint32_t epoch = s_epoch;
-    const int task = (int)s_blk * (kTriWarpCta / 32) + warp;
+    const int task = (int)s_blk * (CT / 32) + warp;
     if (task >= p.n_tasks) return;
     const uint64_t pol = policy_evict_first();
     p.local = 0;
@@ -262,7 +262,7 @@ __global__ void __launch_bounds__(kTriWarpCta) k_solve_tri_warp(SolveParams p) {
         re = ld_stream_i32(p.rowptr + i + 1, pol);
         bi = ld_b(p, i, pol);
     }
-    lean_rows<PROTO, UPPER, UNIT>(p, i, act, rs, re, bi, epoch, lane, pol);
+    lean_rows<PROTO, UPPER, UNIT>(p, i, act, lean_load<UPPER, UNIT>(p, act, rs, re, pol), bi, epoch, lane, pol);
 }
 
 }  // namespace sptrsv_dev

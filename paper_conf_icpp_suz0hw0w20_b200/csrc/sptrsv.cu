@@ -118,12 +118,13 @@ struct sptrsv_handle_s {
     int engine = ENG_AUTO;  // SPTRSV_OPT_ENGINE: ENG_AUTO or a forced engine (resolve_engine)
     int rows_per_lane = 0;  // CHAIN: K rows per lane (0 = 2)
     int variant = 0;        // 0 product path; 3 / 4 / 5 = the paper's Alg.3 / Alg.4 / Alg.5 (ablation)
-    int lean_minb = 6;      // LEAN: resident 256-thread CTAs per SM the register budget targets (5..8)
+    int lean_minb = 5;      // LEAN: resident 256-thread CTAs per SM the register budget targets (5..8)
     uint32_t poll_gap = 0;  // LEAN: sleep after a progressing pass (SPTRSV_OPT_POLL_GAP_NS)
     int poll_one = 0;       // LEAN: one poll per lane per pass (SPTRSV_OPT_POLL_ONE)
     int host_io = 3;        // sptrsv_solve_host on LEAN with pinned buffers (SPTRSV_OPT_HOST_IO)
     uint32_t host_seq = 0;  // solve_host: sequence number of the chunked-b flags
     int split_last = 2;     // warp rows: last off-diagonal outside the lane tree (SPTRSV_OPT_WARP_SPLIT_LAST)
+    int chain_div = 0;      // SPTRSV_OPT_CHAIN_DIV: 0 proof after each run, 1 in-loop proof, 2 test hook
     int tri = 0;            // SPTRSV_TRI_* flags of sptrsv_analyse_csr_ex (f4): 1 UPPER, 2 UNIT_DIAG
     int grid_cache_key = -1;
     int grid_cache = 0;
@@ -339,6 +340,9 @@ const char *sptrsv_strerror(int status) {
         case SPTRSV_ERR_CUDA: return "CUDA runtime error";
         case SPTRSV_ERR_ALLOC: return "allocation failed";
         case SPTRSV_ERR_TIMEOUT: return "watchdog timeout in solve";
+        case SPTRSV_ERR_INEXACT:
+            return "a chain quotient failed its exactness proof; the solve was aborted and the handle now proves "
+                   "every quotient in-loop (re-solve)";
         case SPTRSV_ERR_STALE_LAUNCH:
             return "a captured solve was replayed after the handle's launch configuration changed (re-capture)";
         default: return "unknown status";
@@ -548,24 +552,29 @@ lean_fn lean_tri_kernel(int proto, int tri) {
     return tab[tri & 3][proto ? 1 : 0];
 }
 
-lean_fn tri_warp_kernel(int proto, int tri, int plan) {
-#define TRI_ROW(U, N)                                                                              \
-    {k_solve_tri_warp<PROTO_FLAGS, U, N, PLAN_WARP>, k_solve_tri_warp<PROTO_FUSED, U, N, PLAN_WARP>, \
-     k_solve_tri_warp<PROTO_FLAGS, U, N, PLAN_LIST>, k_solve_tri_warp<PROTO_FUSED, U, N, PLAN_LIST>}
-    static const lean_fn tab[4][4] = {TRI_ROW(false, false), TRI_ROW(true, false), TRI_ROW(false, true),
-                                      TRI_ROW(true, true)};
+lean_fn tri_warp_kernel(int proto, int tri, int plan, int ct) {
+#define TRI_ROW(U, N, C)                                                                                 \
+    {k_solve_tri_warp<PROTO_FLAGS, U, N, PLAN_WARP, C>, k_solve_tri_warp<PROTO_FUSED, U, N, PLAN_WARP, C>, \
+     k_solve_tri_warp<PROTO_FLAGS, U, N, PLAN_LIST, C>, k_solve_tri_warp<PROTO_FUSED, U, N, PLAN_LIST, C>}
+    static const lean_fn tab[2][4][4] = {
+        {TRI_ROW(false, false, 64), TRI_ROW(true, false, 64), TRI_ROW(false, true, 64), TRI_ROW(true, true, 64)},
+        {TRI_ROW(false, false, 256), TRI_ROW(true, false, 256), TRI_ROW(false, true, 256),
+         TRI_ROW(true, true, 256)}};
 #undef TRI_ROW
-    return tab[tri & 3][(plan == PLAN_LIST ? 2 : 0) + (proto ? 1 : 0)];
+    return tab[ct == 256 ? 1 : 0][tri & 3][(plan == PLAN_LIST ? 2 : 0) + (proto ? 1 : 0)];
 }
 
-lean_fn chain_kernel(int proto, int tri, int K) {
-#define CHAIN_ROW(U_, N_)                                                                              \
-    {{k_solve_chain<PROTO_FLAGS, 1, U_, N_>, k_solve_chain<PROTO_FUSED, 1, U_, N_>},                   \
-     {k_solve_chain<PROTO_FLAGS, 2, U_, N_>, k_solve_chain<PROTO_FUSED, 2, U_, N_>}}
-    static const lean_fn tab[4][2][2] = {CHAIN_ROW(false, false), CHAIN_ROW(true, false),
-                                         CHAIN_ROW(false, true), CHAIN_ROW(true, true)};
+lean_fn chain_kernel(int proto, int tri, int K, bool safe) {
+#define CHAIN_ROW(U_, N_, S_)                                                                          \
+    {{k_solve_chain<PROTO_FLAGS, 1, U_, N_, S_>, k_solve_chain<PROTO_FUSED, 1, U_, N_, S_>},           \
+     {k_solve_chain<PROTO_FLAGS, 2, U_, N_, S_>, k_solve_chain<PROTO_FUSED, 2, U_, N_, S_>}}
+    static const lean_fn tab[2][4][2][2] = {
+        {CHAIN_ROW(false, false, false), CHAIN_ROW(true, false, false), CHAIN_ROW(false, true, false),
+         CHAIN_ROW(true, true, false)},
+        {CHAIN_ROW(false, false, true), CHAIN_ROW(true, false, true), CHAIN_ROW(false, true, true),
+         CHAIN_ROW(true, true, true)}};
 #undef CHAIN_ROW
-    return tab[tri & 3][K - 1][proto ? 1 : 0];
+    return tab[safe ? 1 : 0][tri & 3][K - 1][proto ? 1 : 0];
 }
 
 int plan_launch(sptrsv_handle_s *h, Launch *L) {
@@ -587,14 +596,15 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
     const int user = h->cta_threads;
     L->engine = engine;
     if (engine == ENG_HYBRID) {  // warp-level rows: one task per warp (solve_tri.cuh), any triangular form
-        L->fn = (const void *)tri_warp_kernel(h->proto, h->tri, h->plan == PLAN_THREAD ? PLAN_LIST : h->plan);
         if (h->plan == PLAN_THREAD) {  // HYBRID forced on an all-thread plan: run it as LEAN
             L->engine = ENG_LEAN;
         } else {
-            L->cta = kTriWarpCta;
-            L->grid = dim3((unsigned)((h->n_tasks + kTriWarpCta / 32 - 1) / (kTriWarpCta / 32)));
-            L->block = dim3((unsigned)kTriWarpCta);
-            L->key = (7500000 + h->proto * 100000 + h->tri * 10000 + h->plan * 1000) ^ (int)L->grid.x * 7919;
+            const int ct = user == 256 ? 256 : kTriWarpCta;  // 64 (default) or 256 threads
+            L->fn = (const void *)tri_warp_kernel(h->proto, h->tri, h->plan, ct);
+            L->cta = ct;
+            L->grid = dim3((unsigned)((h->n_tasks + ct / 32 - 1) / (ct / 32)));
+            L->block = dim3((unsigned)ct);
+            L->key = (7500000 + h->proto * 100000 + h->tri * 10000 + h->plan * 1000 + ct / 64) ^ (int)L->grid.x * 7919;
             return SPTRSV_OK;
         }
     }
@@ -603,7 +613,7 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         const int cta = (user == 64 || user == 128 || user == 256) ? user : kChainCta;
         const int warps = cta / 32;
         const long long rows_per_cta = (long long)warps * 32 * K;
-        L->fn = (const void *)chain_kernel(h->proto, h->tri, K);
+        L->fn = (const void *)chain_kernel(h->proto, h->tri, K, h->chain_div == 1);
         L->cta = cta;
         L->K = K;
         L->grid = dim3((unsigned)((h->n + rows_per_cta - 1) / rows_per_cta));
@@ -614,7 +624,8 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
             (void)cudaGetLastError();
             return SPTRSV_ERR_CUDA;
         }
-        L->key = (8000000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta) ^ (int)L->grid.x * 7919;
+        L->key = (8000000 + h->proto * 100000 + K * 10000 + h->tri * 1000 + cta + (h->chain_div == 1 ? 500 : 0)) ^
+                 (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
     if (L->engine == ENG_LEAN) {  // minimal one-shot kernel for all-thread-level plans (solve_lean.cuh)
@@ -707,6 +718,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.poll_gap = h->poll_gap;
     p.poll_one = h->poll_one;
     p.split_last = h->split_last;
+    p.chain_div = h->chain_div;
     p.x_host = x_host;
     p.bflag = bflag;
     p.bseq = bseq;
@@ -1082,6 +1094,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
                 return SPTRSV_ERR_INVALID_ARG;
             h->host_io = (int)value;
             return SPTRSV_OK;
+        case SPTRSV_OPT_CHAIN_DIV:
+            if (value < 0 || value > 2) return SPTRSV_ERR_INVALID_ARG;
+            h->chain_div = (int)value;
+            return SPTRSV_OK;
         case SPTRSV_OPT_SUBWARP:
             if (value < 0 || value > 64) return SPTRSV_ERR_INVALID_ARG;
             h->subwarp_epl = (int)value;
@@ -1116,6 +1132,7 @@ int sptrsv_get_option(sptrsv_handle_t h, int key, int64_t *value) {
         case SPTRSV_OPT_POLL_ONE: *value = h->poll_one; return SPTRSV_OK;
         case SPTRSV_OPT_WARP_SPLIT_LAST: *value = h->split_last; return SPTRSV_OK;
         case SPTRSV_OPT_HOST_IO: *value = h->host_io; return SPTRSV_OK;
+        case SPTRSV_OPT_CHAIN_DIV: *value = h->chain_div; return SPTRSV_OK;
         case SPTRSV_OPT_SUBWARP: *value = h->subwarp_epl >= 0 ? h->subwarp_epl : h->epl_eff; return SPTRSV_OK;
         default: return SPTRSV_ERR_INVALID_ARG;
     }
@@ -1210,6 +1227,10 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
     }
     const uint32_t e = err ? err : merr;
     if (e == kErrStale) return SPTRSV_ERR_STALE_LAUNCH;
+    if (e == kErrInexact) {  // a CHAIN quotient failed its proof: prove every quotient in-loop from now on
+        h->chain_div = 1;
+        return SPTRSV_ERR_INEXACT;
+    }
     return e ? SPTRSV_ERR_TIMEOUT : SPTRSV_OK;
 }
 

@@ -115,7 +115,8 @@ def test_fuzz_triangular_forms_vs_oracle(seed):
                 h.solve(b, x)
                 h.check()
                 got = x.cpu().numpy()
-                if h.info()["n_warp_rows"] == 0:
+                inf = h.info()
+                if inf["n_warp_rows"] == 0 and inf["n_sub_tasks"] == 0:
                     assert np.array_equal(got, ref), (s.name, s.n, flags, opts, proto)
                 else:
                     err = float(np.max(np.abs(got - ref) / np.abs(ref))) if s.n else 0.0

@@ -654,7 +654,16 @@ def test_flag_latency_runs(cap):
 
 # ------------------------------------------------------------------ failure detection (watchdog, stale graphs)
 
-@pytest.mark.parametrize("engine,gen", [(3, "chain"), (7, "grid"), (6, "dense"), (0, "chain")])
+def _chain_with_waiting_tail(m, tail):
+    """Rows 0..m-1 a bidiagonal chain, rows m..m+tail-1 depend on row m-1 only: the tail's warps
+    wait m hops without any progress (what a watchdog test needs)."""
+    rows = list(range(1, m)) + list(range(m, m + tail))
+    cols = list(range(0, m - 1)) + [m - 1] * tail
+    rp, ci = synth._assemble(m + tail, (np.array(rows, np.int64), np.array(cols, np.int64)))
+    return synth.from_pattern("tail", rp, ci, np.random.default_rng(3))
+
+
+@pytest.mark.parametrize("engine,gen", [(3, "chain"), (7, "grid"), (6, "tail"), (0, "chain")])
 def test_watchdog_fires_and_next_solve_is_exact(cap, engine, gen):
     """SPTRSV_OPT_SPIN_LIMIT = 1: the first warp that idles 64 passes raises the sticky error and
     the abort word, every spinning warp bails out, and sptrsv_check reports SPTRSV_ERR_TIMEOUT
@@ -662,7 +671,7 @@ def test_watchdog_fires_and_next_solve_is_exact(cap, engine, gen):
     check clears the condition; the next solve (default limit) re-zeroes the ready words and must
     match the oracle exactly."""
     s = {"chain": lambda: synth.gen_chain(60_000), "grid": lambda: synth.gen_grid(300),
-         "dense": lambda: synth.gen_dense_lower(1500)}[gen]()
+         "tail": lambda: _chain_with_waiting_tail(3000, 64)}[gen]()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     rp, ci, v, b = dev_csr(s)
     with cap.analyse(rp, ci, v, engine=engine, mode=1 if engine != 6 else 2) as h:
@@ -737,3 +746,31 @@ def test_handle_rejects_tensors_on_another_device(cap):
     with cap.analyse(rp, ci, v) as h:
         with pytest.raises((ValueError, TypeError)):
             h.solve(b.cpu(), None)
+
+
+@pytest.mark.parametrize("proto", PROTOS)
+def test_chain_division_proof_modes(cap, proto):
+    """CHAIN's division proof (SPTRSV_OPT_CHAIN_DIV): the in-loop proof (1) is bit-exact like the
+    default post-run proof (0); the test hook (2) makes every post-run proof fail -> the solve is
+    aborted with SPTRSV_ERR_INEXACT, the handle switches itself to in-loop proofs, and the next
+    solve is bit-exact."""
+    for s in (synth.gen_grid(300), synth.gen_chain(20_000)):
+        ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+        rp, ci, v, b = dev_csr(s)
+        with cap.analyse(rp, ci, v, engine=7, protocol=proto) as h:
+            for mode in (0, 1):
+                h.set_option(cap._lib.OPT_CHAIN_DIV, mode)
+                x = torch.full_like(b, float("nan"))
+                h.solve(b, x)
+                h.check()
+                assert np.array_equal(x.cpu().numpy(), ref), (s.name, mode)
+            h.set_option(cap._lib.OPT_CHAIN_DIV, 2)
+            h.solve(b, x)
+            with pytest.raises(cap.SptrsvError) as e:
+                h.check()
+            assert e.value.status == cap._lib.ERR_INEXACT
+            assert h.get_option(cap._lib.OPT_CHAIN_DIV) == 1
+            x.fill_(float("nan"))
+            h.solve(b, x)
+            h.check()
+            assert np.array_equal(x.cpu().numpy(), ref), s.name
