@@ -287,7 +287,7 @@ def hop_placements(cap):
     every SM pair (0, b) is measured (one CTA per SM, sptrsv_hop_scan) and split into the two
     latency modes (same die / cross die; the B200 has two dies of 74 SMs)."""
     try:
-        sms, ns = cap.hop_scan(4000, 1)
+        sms, ns = cap.hop_scan(1500, 1)
     except Exception as e:  # pragma: no cover - diagnostics only
         return {"error": str(e)}
     ns = np.asarray(ns)

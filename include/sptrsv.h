@@ -357,7 +357,9 @@ int sptrsv_flag_latency(int32_t iters, int32_t protocol, double *ns_per_hop, dou
  * hop): one CTA per SM on the current device; the CTAs on SM sm_a (the
  * lowest SM id present) and on each other SM b ping-pong `iters` rounds through the solve's
  * publish / poll pair (protocol 0 FLAGS: st.release flag, ld.acquire poll + x load; 1 FUSED:
- * 16-byte epoch record, relaxed store / poll) and the mean one-way hop in ns is reported per b.
+ * 16-byte epoch record, relaxed store / poll) and the mean one-way hop in ns is reported per b,
+ * the fastest over 8 ready-word addresses 4 KB apart (the word's L2 slice, and its die, follow the
+ * address).
  *   capacity    entries sm_b_out / ns_out can hold (host arrays).
  *   sm_a_out    host int32, receives sm_a.   count  host int32, receives the pairs measured.
  * Synchronous.  The two dies of a B200 show as two latency modes over b.

@@ -149,11 +149,9 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint64_t pol = policy_evict_first();
-    // ---- the start ticket's atomic is issued first; its result is only needed at the barrier, so
-    // it overlaps the speculative loads (logical block == blockIdx.x, the common case) of both
-    // levels: rowptr / b, then L_ii and the first two dependencies
-    unsigned long long tk = 0;
-    if (tid == 0) tk = atomicAdd(&p.st->tk.v, 1ull);
+    // ---- speculative first-level loads for logical block == blockIdx.x (the common case), overlapped
+    // with the start ticket (round 2 also issued the second-level loads before the barrier: c5 53 ->
+    // 60 us, reverted)
     int i = (int)blockIdx.x * CT + tid;
     if (UPPER) i = p.n - 1 - i;
     int rs = 0, re = 1;
@@ -165,13 +163,12 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
         re = ld_stream_i32(p.rowptr + i + 1, pol);
         if (!bgate) bi = ld_b(p, i, pol);
     }
-    LeanRow lr = lean_load<UPPER, UNIT>(p, i >= 0 && i < p.n, rs, re, pol);
     if (tid == 0) {
         if (p.trace) {
             atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
             atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
         }
-        cta_ticket_decode(p, tk, s_blk, s_epoch);
+        cta_ticket(p, s_blk, s_epoch);
         if (bgate) {  // wait until the b chunks of this CTA's (physical) rows have landed
             const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
             wait_b_chunks(p, UPPER ? p.n - lr1 : lr0, UPPER ? p.n - lr0 : lr1);
@@ -189,12 +186,11 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
             re = ld_stream_i32(p.rowptr + i + 1, pol);
             bi = ld_b(p, i, pol);
         }
-        lr = lean_load<UPPER, UNIT>(p, i >= 0 && i < p.n, rs, re, pol);
     } else if (bgate && i >= 0 && i < p.n) {
         bi = ld_b(p, i, pol);
     }
     const bool act = i >= 0 && i < p.n;
-    lean_rows<PROTO, UPPER, UNIT>(p, i, act, lr, bi, epoch, lane, pol);
+    lean_rows<PROTO, UPPER, UNIT>(p, i, act, lean_load<UPPER, UNIT>(p, act, rs, re, pol), bi, epoch, lane, pol);
     if (p.trace && lane == 0) atomicMax(&p.trace[3 * (size_t)p.n + 1], globaltimer_ns());  // last warp exit
     if (p.x_host) {
         // sptrsv_solve_host: the CTA's finished rows go to pinned host memory over PCIe as one
