@@ -272,7 +272,10 @@ def roofline(s, mean_s, peak, peak_src, kernel, traffic=None):
 def latency_bound(levels, hops, mean_s, alg_bytes, peak):
     """T_lat = (levels - 1) * t_hop per die placement; t / max(T_bw, T_lat)."""
     t_bw = alg_bytes / (peak * 1e9)
-    out = {"levels": int(levels), "t_bw_us": round(t_bw * 1e6, 3)}
+    out = {"levels": int(levels), "t_bw_us": round(t_bw * 1e6, 3),
+           "model": "(levels - 1) * t_hop with the cross-SM record hop: a bound when every level boundary crosses "
+                    "SMs; CHAIN resolves in-warp levels in registers (~0.1 us per step), so for chains and grids it "
+                    "is a model, not a bound"}
     for place, hop in hops.items():
         if hop is None:
             continue

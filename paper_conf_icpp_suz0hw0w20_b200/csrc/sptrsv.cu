@@ -544,10 +544,10 @@ lean_fn lean_lower_kernel(int proto, int occ, int ct) {
 
 lean_fn lean_tri_kernel(int proto, int tri) {
     static const lean_fn tab[4][2] = {
-        {k_solve_lean<PROTO_FLAGS, 6>, k_solve_lean<PROTO_FUSED, 6>},
-        {k_solve_lean<PROTO_FLAGS, 6, true, false>, k_solve_lean<PROTO_FUSED, 6, true, false>},
-        {k_solve_lean<PROTO_FLAGS, 6, false, true>, k_solve_lean<PROTO_FUSED, 6, false, true>},
-        {k_solve_lean<PROTO_FLAGS, 6, true, true>, k_solve_lean<PROTO_FUSED, 6, true, true>},
+        {k_solve_lean<PROTO_FLAGS, 5>, k_solve_lean<PROTO_FUSED, 5>},
+        {k_solve_lean<PROTO_FLAGS, 5, true, false>, k_solve_lean<PROTO_FUSED, 5, true, false>},
+        {k_solve_lean<PROTO_FLAGS, 5, false, true>, k_solve_lean<PROTO_FUSED, 5, false, true>},
+        {k_solve_lean<PROTO_FLAGS, 5, true, true>, k_solve_lean<PROTO_FUSED, 5, true, true>},
     };
     return tab[tri & 3][proto ? 1 : 0];
 }
