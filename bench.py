@@ -14,8 +14,11 @@ c4, one C5 system; plus the aux pure chain) under the same rules, each with its 
 fraction (measured and nominal HBM peak), critical-path latency bound, t / max(T_bw, T_lat) and
 the ncu-measured DRAM bytes of one cold launch (``--no-ncu`` to skip).
 
-N > 1: the workload is C5 (BASELINE.json configs[4]): 8 independent n=2e6 systems, system s on
-GPU s mod N (``paper_conf_icpp_suz0hw0w20_b200.batch``).  No data is exchanged, so no NCCL:
+N > 1: ``value`` is WEAK scaling of the headline: every GPU solves its own c2-shaped system (seed + GPU),
+so the driver's per-N values compare like for like; ``c5_batch_leg`` is BASELINE.json configs[4]: the 8
+fixed C5 systems, system s on GPU s mod N (strong scaling; ``--config c5`` makes it the value).  The
+N = 1 line carries the same 8-system batch on one GPU (``configs.c5batch``).  No data is exchanged, so
+no NCCL (``paper_conf_icpp_suz0hw0w20_b200.batch``):
   * without torchrun, this one process drives N devices, one stream each;
   * under torchrun (WORLD_SIZE > 1), each rank drives its own GPU and the barrier / max over
     ranks go through a CPU (gloo) process group -- control plane only.
@@ -69,7 +72,7 @@ def parse(argv=None):
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default=None, choices=sorted(WORKLOADS),
-                    help="workload (default: c2 at N=1, c5 at N>1)")
+                    help="workload (default c2; N > 1: c2 on every GPU, plus the C5 batch leg)")
     ap.add_argument("--impl", default="cuda", choices=["cuda", "reference"])
     ap.add_argument("--mode", type=int, default=0, help="0 auto, 1 thread, 2 warp")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="cpu_baseline sample budget")
@@ -82,10 +85,11 @@ def parse(argv=None):
     ap.add_argument("--no-flags-leg", action="store_true", help="skip the FLAGS-protocol / no-window legs")
     ap.add_argument("--no-tri-leg", action="store_true", help="skip the upper / unit-diagonal (f4) leg")
     ap.add_argument("--nrhs", type=int, default=8, help="right-hand sides of the multi-RHS leg (0 = skip)")
+    ap.add_argument("--no-c5-leg", action="store_true", help="N > 1: skip the C5 strong-scaling leg")
     ap.add_argument("--ncu-child", default=None, help=argparse.SUPPRESS)
     a = ap.parse_args(argv)
     if a.config is None:
-        a.config = "c5" if a.gpus > 1 else "c2"
+        a.config = "c2"
     return a
 
 
@@ -561,6 +565,27 @@ def run_single(args):
             del t, x
             torch.cuda.empty_cache()
 
+    # ---- BASELINE configs[4] at N = 1: the 8 C5 systems back to back on this GPU (the N = 1 point of
+    # the C5 strong-scaling leg of the N > 1 lines)
+    if not args.no_configs and not args.profile:
+        from paper_conf_icpp_suz0hw0w20_b200.batch import MultiDeviceBatch
+        c5 = c5_systems(range(8))
+        batch = MultiDeviceBatch([(t.rowptr, t.colidx, t.val, t.b) for t in c5], [0], **opts)
+        fl = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+        for _ in range(args.warmup):
+            batch.timed_solve(lambda g: fl.zero_())
+        per = np.array([batch.timed_solve(lambda g: fl.zero_())[0] for _ in range(args.steps)])
+        batch.check()
+        m = float(per.mean()) * 1e-3
+        configs["c5batch"] = {"workload": WORKLOADS["c5"], "systems": 8, "n_per_system": c5[0].n,
+                              "value": round(2.0 * sum(t.nnz for t in c5) / m / 1e9, 3), "unit": UNIT,
+                              "ms_per_step": round(m * 1e3, 5), "steps": args.steps,
+                              "engine": ENGINES.get(batch.handles[0].info()["engine"]),
+                              "timing": "one step = the 8 solves back to back on one stream (CUDA events)"}
+        batch.close()
+        del c5, fl
+        torch.cuda.empty_cache()
+
     # ---- roofline of the headline kernel (mean step), latency bound, ncu-measured DRAM traffic
     traffic, ncu_err = ({}, "skipped")
     if not args.no_ncu and not args.profile:
@@ -666,11 +691,61 @@ class CudaEnv:
         return ClockSampler(devices)
 
 
+def _measure_batch(args, env, systems, devices, opts, dist, e2e=True):
+    """One workload through MultiDeviceBatch: warm-up, K timed steps (per-device CUDA events, step =
+    max over devices, L2 flushed before each step outside the events), max / sum over ranks, and the
+    end-to-end leg.  Every collective runs on every rank."""
+    from paper_conf_icpp_suz0hw0w20_b200.batch import max_over_ranks, sum_over_ranks
+
+    batch = env.make_batch(systems, devices, opts)
+    flush = env.make_flush(batch)
+    for _ in range(args.warmup):
+        batch.timed_solve(flush)
+    batch.check()
+    if dist is not None:
+        dist.barrier()
+    batch.synchronize()
+    per_dev = np.array([batch.timed_solve(flush) for _ in range(args.steps)])  # [steps, devices] ms
+    batch.synchronize()
+    if dist is not None:
+        dist.barrier()
+    batch.check()
+    step_ms = per_dev.max(axis=1)  # a step ends when the last device is done
+    tot_s = max_over_ranks(float(step_ms.sum()) * 1e-3, dist)
+    nnz_all = sum_over_ranks(float(sum(s.nnz for s in systems)), dist)
+    out = {"value": 2.0 * nnz_all * args.steps / tot_s / 1e9, "tot_s": tot_s, "per_dev": per_dev,
+           "launches": int(sum_over_ranks(float(args.steps * len(systems)), dist)),
+           "systems_total": int(sum_over_ranks(float(len(systems)), dist)),
+           "info": batch.handles[0].info()}
+    if e2e:  # pinned host b -> device -> solve -> host x, every step, through the public API
+        hb, hx = env.host_buffers(systems)
+        batch.solve_host(hb, hx)
+        if dist is not None:
+            dist.barrier()
+        e_t = []
+        for _ in range(args.steps):
+            t0 = time.perf_counter()
+            batch.solve_host(hb, hx)
+            e_t.append(time.perf_counter() - t0)
+        et = max_over_ranks(float(np.sum(e_t)), dist)
+        ok = all(np.array_equal(env.numpy(hx[k]), env.numpy(batch.x(k))) for k in range(len(systems)))
+        ok = sum_over_ranks(0.0 if ok else 1.0, dist) == 0.0
+        h2d = int(sum_over_ranks(float(sum(8 * s.n for s in systems)), dist))
+        out["e2e"] = {"value": 2.0 * nnz_all * args.steps / et / 1e9, "unit": UNIT,
+                      "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d, "matches_device_path": bool(ok),
+                      "timing": "host wall clock per step around sptrsv_solve_host of every owned system (one host "
+                                "thread per device), max over ranks"}
+    batch.close()
+    return out
+
+
 def run_batch(args, rank, world, dist=None, env=None):
-    """C5 (or replicas of another config) over N GPUs.  world > 1: this process is one rank of
+    """N > 1 (or --config c5): independent systems over N GPUs.  world > 1: this process is one rank of
     torchrun and drives GPU LOCAL_RANK; world == 1: this process drives args.gpus devices.
-    Every collective below (barrier, max / sum over ranks) runs on every rank."""
-    from paper_conf_icpp_suz0hw0w20_b200.batch import max_over_ranks, shard, sum_over_ranks
+    The line's `value` is WEAK scaling of the headline config (every GPU solves its own c2-shaped
+    system, seed + GPU), comparable with the N = 1 line; `c5_batch_leg` is BASELINE configs[4]: the 8
+    fixed C5 systems, s -> GPU s mod N (strong scaling).  `--config c5` makes C5 the value."""
+    from paper_conf_icpp_suz0hw0w20_b200.batch import shard
 
     env = env or CudaEnv()
     devices = env.devices(args, rank, world)
@@ -679,68 +754,34 @@ def run_batch(args, rank, world, dist=None, env=None):
     for kv in args.opt:
         k, v = kv.split("=")
         opts[k] = int(v)
+    c5 = c5_systems(shard(8, rank, world))  # ranks own systems s = rank (mod world); devices split them further
     if args.config == "c5":
-        owned = shard(8, rank, world)  # ranks own systems s = rank (mod world); devices split them further
-        systems = c5_systems(owned)
-        scaling = "strong"
+        main_sys, scaling = c5, "strong"
     else:
-        owned = list(range(len(devices)))
-        systems = [make_system(args.config, rank * len(devices) + k) for k in range(len(devices))]
+        main_sys = [make_system(args.config, rank * len(devices) + k) for k in range(len(devices))]
         scaling = "weak"
-    batch = env.make_batch(systems, devices, opts)
-    flush = env.make_flush(batch)
-    for _ in range(args.warmup):
-        batch.timed_solve(flush)
-    batch.check()
     sampler = env.clocks(devices)
     sampler.__enter__()
-    if dist is not None:
-        dist.barrier()
-    batch.synchronize()
-    per_dev = []
-    for _ in range(args.steps):
-        per_dev.append(batch.timed_solve(flush))
-    batch.synchronize()
-    if dist is not None:
-        dist.barrier()
+    m = _measure_batch(args, env, main_sys, devices, opts, dist)
     sampler.__exit__(None, None, None)
-    batch.check()
-    per_dev = np.array(per_dev)                  # [steps, devices] ms
-    step_ms = per_dev.max(axis=1)                # a step ends when the last device is done
-    tot_s = max_over_ranks(float(step_ms.sum()) * 1e-3, dist)
-    nnz_all = sum_over_ranks(float(sum(s.nnz for s in systems)), dist)
-    value = 2.0 * nnz_all * args.steps / tot_s / 1e9
-
-    # e2e through the public API: pinned host b -> device -> solve -> host x, every step
-    hb, hx = env.host_buffers(systems)
-    batch.solve_host(hb, hx)
-    if dist is not None:
-        dist.barrier()
-    e_t = []
-    for _ in range(args.steps):
-        t0 = time.perf_counter()
-        batch.solve_host(hb, hx)
-        e_t.append(time.perf_counter() - t0)
-    et = max_over_ranks(float(np.sum(e_t)), dist)
-    ok = all(np.array_equal(env.numpy(hx[k]), env.numpy(batch.x(k))) for k in range(len(systems)))
-    ok = sum_over_ranks(0.0 if ok else 1.0, dist) == 0.0
-    h2d = int(sum_over_ranks(float(sum(8 * s.n for s in systems)), dist))
-    e2e = {"value": 2.0 * nnz_all * args.steps / et / 1e9, "unit": UNIT,
-           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d, "matches_device_path": bool(ok),
-           "timing": "host wall clock per step around sptrsv_solve_host of every owned system (one host thread "
-                     "per device), max over ranks"}
-    launches = int(sum_over_ranks(float(args.steps * len(systems)), dist))
-    systems_total = int(sum_over_ranks(float(len(systems)), dist))
-    info = batch.handles[0].info()
+    leg = None
+    if args.config != "c5" and not args.no_c5_leg:
+        c = _measure_batch(args, env, c5, devices, opts, dist, e2e=False)
+        leg = {"workload": f"c5: {WORKLOADS['c5']}", "value": round(c["value"], 3), "unit": UNIT,
+               "ms_per_step": round(c["tot_s"] / args.steps * 1e3, 5), "scaling": "strong",
+               "systems_total": c["systems_total"], "gpu_launches": c["launches"],
+               "per_device_ms_mean": [round(float(v), 5) for v in c["per_dev"].mean(axis=0)]}
+    info = m["info"]
     if rank == 0:
         line = {
-            "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": n_gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot_s / args.steps * 1e3, 5),
+            "metric": METRIC, "value": round(m["value"], 3), "unit": UNIT, "n_gpus": n_gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(m["tot_s"] / args.steps * 1e3, 5),
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": f"{args.config}: {WORKLOADS[args.config]}",
-                       "systems_total": systems_total,
-                       "n_per_system": systems[0].n, "nnz_per_system": systems[0].nnz,
+            "config": {"workload": f"{args.config}: {WORKLOADS[args.config]}"
+                       + ("" if args.config == "c5" else f" -- one per GPU (seed + GPU), weak scaling"),
+                       "systems_total": m["systems_total"],
+                       "n_per_system": main_sys[0].n, "nnz_per_system": main_sys[0].nnz,
                        "engine": ENGINES.get(info["engine"], str(info["engine"])),
                        "parallelism": (f"{n_gpus} GPUs, system s on GPU s mod {n_gpus}, one stream per device, "
                                        "no inter-GPU exchange (no NCCL)") + (
@@ -748,14 +789,14 @@ def run_batch(args, rank, world, dist=None, env=None):
                        "timing": "per-device CUDA events around each device's solves on its stream; step = max over "
                                  "devices; L2 flushed before every step outside the events",
                        "options": opts},
-            "per_device_ms_mean": [round(float(v), 5) for v in per_dev.mean(axis=0)],
-            "e2e": e2e,
-            "gpu_launches": launches,
+            "per_device_ms_mean": [round(float(v), 5) for v in m["per_dev"].mean(axis=0)],
+            "c5_batch_leg": leg,
+            "e2e": m["e2e"],
+            "gpu_launches": m["launches"],
             "cpu_baseline": None,
             "clocks": sampler.summary(),
         }
         print(json.dumps(line), flush=True)
-    batch.close()
 
 
 def main():

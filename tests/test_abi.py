@@ -103,6 +103,6 @@ def test_bench_defaults():
     sys.path.insert(0, ROOT)
     import bench
     assert bench.parse([]).config == "c2" and bench.parse([]).gpus == 1
-    assert bench.parse(["--gpus", "4"]).config == "c5"
+    assert bench.parse(["--gpus", "4"]).config == "c2"  # N > 1: c2 on every GPU (weak) + the C5 leg
     a = bench.parse(["--gpus", "2", "--config", "c2"])
     assert a.config == "c2"

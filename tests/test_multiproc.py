@@ -161,7 +161,7 @@ def _bench_worker(rank, world, port, q, config):
     os.environ.update({"RANK": str(rank), "WORLD_SIZE": str(world), "LOCAL_RANK": "0"})
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
     import bench
-    args = bench.parse(["--gpus", str(world), "--steps", "2", "--warmup", "1", "--config", config])
+    args = bench.parse(["--gpus", str(world), "--steps", "2", "--warmup", "1", "--config", config, "--no-c5-leg"])
     env = _CpuEnv()
     out = io.StringIO()
     with contextlib.redirect_stdout(out):
@@ -200,3 +200,42 @@ def test_bench_rank_path_gloo(world):
     assert line["e2e"]["h2d_bytes_per_step"] == 8 * 8 * 2_000_000
     nnz = 8 * 5_600_000
     assert abs(line["value"] - 2.0 * nnz * 2 / (line["ms_per_step"] * 2 * 1e-3) / 1e9) <= 1e-3 * line["value"]
+
+
+def _bench_worker_weak(rank, world, port, q):
+    import contextlib
+    import io
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update({"RANK": str(rank), "WORLD_SIZE": str(world), "LOCAL_RANK": "0"})
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    import bench
+    args = bench.parse(["--gpus", str(world), "--steps", "2", "--warmup", "1"])
+    out = io.StringIO()
+    with contextlib.redirect_stdout(out):
+        bench.run_batch(args, rank, world, dist, env=_CpuEnv())
+    dist.destroy_process_group()
+    q.put((rank, out.getvalue()))
+
+
+def test_bench_default_n2_is_weak_scaling_with_c5_leg():
+    """The default N > 1 line (as the driver launches it): value = weak scaling of the c2 headline
+    (one c2-shaped system per rank, seed + rank), plus the C5 strong-scaling leg over the same ranks."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bench_worker_weak, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=900) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    import json
+    line = json.loads(out[0].strip().splitlines()[-1])
+    assert line["scaling"] == "weak" and line["n_gpus"] == world
+    assert line["config"]["systems_total"] == world and line["config"]["n_per_system"] == 1_000_000
+    assert line["gpu_launches"] == world * 2
+    leg = line["c5_batch_leg"]
+    assert leg["scaling"] == "strong" and leg["systems_total"] == 8 and leg["gpu_launches"] == 16
