@@ -37,6 +37,7 @@ enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 
 // in-degrees, the task list (at most n tasks), the solve state and the analyse results / scratch.
 struct Workspace {
     void *base = nullptr;          // the single allocation below
+    bool pooled = false;           // from the library's memory pool (ws_pool) rather than cudaMalloc
     uint32_t *flags = nullptr;     // n      (PROTO_FLAGS)
     unsigned long long *rec = nullptr;  // 2n (PROTO_FUSED)
     int32_t *indeg = nullptr;      // n
@@ -223,8 +224,41 @@ int set_kernel_attrs() {
     return rc;
 }
 
+// Handle workspaces come from a library-private stream-ordered memory pool per device: a destroyed
+// handle's workspace is kept (up to kPoolKeepBytes) and handed to the next analyse without a
+// cudaMalloc / cudaFree pair -- the warm analyse is then a memset, six kernels and one copy.
+constexpr unsigned long long kPoolKeepBytes = 1ull << 30;
+std::mutex g_pool_mu;
+cudaMemPool_t g_pool[256] = {};
+
+cudaMemPool_t ws_pool(int dev) {
+    std::lock_guard<std::mutex> lk(g_pool_mu);
+    cudaMemPool_t &p = g_pool[dev & 255];
+    if (!p) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+            (void)cudaGetLastError();
+            p = nullptr;
+            return nullptr;
+        }
+        unsigned long long keep = kPoolKeepBytes;
+        (void)cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &keep);
+        (void)cudaGetLastError();
+    }
+    return p;
+}
+
 void free_ws(Workspace &w) {
-    cudaFree(w.base);
+    if (w.base) {
+        if (w.pooled) {
+            (void)cudaFreeAsync(w.base, 0);
+        } else {
+            cudaFree(w.base);
+        }
+    }
     cudaFree(w.lvl);
     cudaFree(w.b_stage);
     cudaFree(w.mst);
@@ -393,9 +427,16 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
                      o_tasks = o_indeg + al(4 * nn), o_tw = o_tasks + al(4 * nn), o_st = o_tw + al(nn),
                      o_out = o_st + al(sizeof(SolveState)), o_blk = o_out + al(sizeof(AnalyseOut)),
                      total = o_blk + al(4 * 3 * (nb ? nb : 1));
-        if (cudaMalloc(&h->ws.base, total) != cudaSuccess) {
-            rc = SPTRSV_ERR_ALLOC;
-            break;
+        cudaMemPool_t pool = ws_pool(h->device);
+        if (pool && cudaMallocFromPoolAsync(&h->ws.base, total, pool, 0) == cudaSuccess) {
+            h->ws.pooled = true;
+        } else {
+            (void)cudaGetLastError();
+            h->ws.base = nullptr;
+            if (cudaMalloc(&h->ws.base, total) != cudaSuccess) {
+                rc = SPTRSV_ERR_ALLOC;
+                break;
+            }
         }
         char *b = static_cast<char *>(h->ws.base);
         h->ws.rec = reinterpret_cast<unsigned long long *>(b + o_rec);
