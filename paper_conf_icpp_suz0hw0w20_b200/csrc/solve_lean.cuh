@@ -58,15 +58,9 @@ __device__ __forceinline__ LeanRow lean_load(const SolveParams &p, bool act, int
 // One warp, one row per lane (Alg.5 l.3-18): lane's row i (act: i is a real row), b_i and its
 // second-level loads (lean_load) already issued.  Returns when every lane of the warp has
 // published, or on abort.  Shared by k_solve_lean and the f4 list kernel (solve_tri.cuh).
-// give_up(): polled in every pass that made no progress; true ends the loop early (LEAN's speculative
-// rows when the CTA's ticket names another block).  Returns false when it ended early or on abort.
-struct NeverGiveUp {
-    __device__ __forceinline__ bool operator()() const { return false; }
-};
-
-template <int PROTO, bool UPPER, bool UNIT, class GiveUp = NeverGiveUp>
-__device__ __forceinline__ bool lean_rows(SolveParams &p, int i, bool act, const LeanRow &lr, double bi,
-                                          uint32_t epoch, int lane, uint64_t pol, GiveUp give_up = GiveUp()) {
+template <int PROTO, bool UPPER, bool UNIT>
+__device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, const LeanRow &lr, double bi,
+                                          uint32_t epoch, int lane, uint64_t pol) {
     const int lo = lr.lo, hi = lr.hi;
     constexpr int dir = UPPER ? -1 : 1;
     auto inr = [&](int k) { return UPPER ? k >= lo : k < hi; };
@@ -129,7 +123,6 @@ __device__ __forceinline__ bool lean_rows(SolveParams &p, int i, bool act, const
             if (p.poll_gap) nanosleep_ns(p.poll_gap);
             continue;
         }
-        if (give_up()) return false;
         if (backoff) nanosleep_ns(backoff);
         backoff = min(max(backoff * 2u, 32u), p.backoff_max);
         if ((++idle & 63u) == 0) {
@@ -141,135 +134,63 @@ __device__ __forceinline__ bool lean_rows(SolveParams &p, int i, bool act, const
                 }
                 ab = ld_relaxed_u32(&p.st->abort.v);
             }
-            if (__shfl_sync(FULL, ab, 0)) return false;
+            if (__shfl_sync(FULL, ab, 0)) break;
         }
     }
-    return true;
 }
 
 // UPPER / UNIT: upper-triangular rows (diagonal first, dependencies
 // j > i) are taken in REVERSE order -- logical row r is row n-1-r, so the ticket
 // order is again a topological order; UNIT: the diagonal is implicitly 1 and
 // not stored.
-constexpr uint32_t kUnknownBlk = 0xFFFFFFFEu;  // s_tkv before thread 0's ticket has returned
-
-// Warp helper: the rows of logical block `blk` for this thread (upper: reversed), first-level loads.
-template <bool UPPER, int CT>
-__device__ __forceinline__ void lean_rows_of(const SolveParams &p, uint32_t blk, int tid, uint64_t pol, int &i, int &rs,
-                                             int &re, double &bi, bool load_b) {
-    i = (int)blk * CT + tid;
-    if (UPPER) i = p.n - 1 - i;
-    rs = 0, re = 1, bi = 0.0;
-    if (i >= 0 && i < p.n) {
-        rs = ld_stream_i32(p.rowptr + i, pol);
-        re = ld_stream_i32(p.rowptr + i + 1, pol);
-        if (load_b) bi = ld_b(p, i, pol);
-    }
-}
-
-// UPPER / UNIT: upper-triangular rows (diagonal first, dependencies
-// j > i) are taken in REVERSE order -- logical row r is row n-1-r, so the ticket
-// order is again a topological order; UNIT: the diagonal is implicitly 1 and
-// not stored.
-//
-// Start of a solve (round 2).  No warp waits for the CTA start ticket: the epoch comes from the
-// handle's `ep` word (generation-tagged; the previous solve's last CTA bumped it), every warp starts
-// on the rows of logical block blockIdx.x at once, and the ticket -- whose atomic is still taken, by
-// thread 0 -- only VERIFIES that block.  Dispatch is in blockIdx order in practice, so the ticket
-// almost always equals blockIdx.x; if it does not, the warps give up their speculative rows the
-// first time they would wait (a row they already published is correct: the CTA holding that
-// ticket publishes the same value under the same epoch) and solve the ticket's block instead, whose
-// dependencies all belong to CTAs that started earlier -- the forward-progress argument of
-// DESIGN.md G11 is unchanged.  The CTA that completes the solve (the G-th exit, counted on `done`)
-// writes the next solve's epoch.  With sptrsv_solve_host's chunked b (bflag) the round-1 start is
-// used: wait for the ticket, then for the CTA's b chunks.
 template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false, int CT = kLeanCta>
 __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     __shared__ uint32_t s_blk, s_epoch;
-    __shared__ volatile uint32_t s_tkv;  // the ticket's logical block (kUnknownBlk until known)
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint64_t pol = policy_evict_first();
+    // ---- speculative first-level loads for logical block == blockIdx.x (the common case), overlapped
+    // with the start ticket (round 2 also issued the second-level loads before the barrier: c5 53 ->
+    // 60 us, reverted)
+    int i = (int)blockIdx.x * CT + tid;
+    if (UPPER) i = p.n - 1 - i;
+    int rs = 0, re = 1;
+    double bi = 0.0;
     const bool bgate = p.bflag != nullptr;  // b still arriving in chunks (sptrsv_solve_host)
-    int i, rs, re;
-    double bi;
-    if (p.trace && tid == 0) {
-        atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());  // first CTA entry
-        atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);          // CTAs started
+    if (i >= 0 && i < p.n) {
+        if (p.trace) p.trace[3 * (size_t)p.n + 3 + i] = globaltimer_ns();  // CTA entry
+        rs = ld_stream_i32(p.rowptr + i, pol);
+        re = ld_stream_i32(p.rowptr + i + 1, pol);
+        if (!bgate) bi = ld_b(p, i, pol);
     }
-    if (bgate) {
-        // ---- round-1 start: speculative first-level loads, ticket, b chunks, barrier
-        lean_rows_of<UPPER, CT>(p, blockIdx.x, tid, pol, i, rs, re, bi, false);
-        if (tid == 0) {
-            cta_ticket(p, s_blk, s_epoch);
-            if (s_blk != kStaleBlk) {  // wait until the b chunks of this CTA's (physical) rows have landed
-                const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
-                wait_b_chunks(p, UPPER ? p.n - lr1 : lr0, UPPER ? p.n - lr0 : lr1);
-            }
+    if (tid == 0) {
+        if (p.trace) {
+            atomicMin(&p.trace[3 * (size_t)p.n], globaltimer_ns());                  // first CTA entry
+            atomicAdd(&p.trace[3 * (size_t)p.n + 2], 1ull);                          // CTAs started
         }
-        __syncthreads();
-        if (s_blk == kStaleBlk) return;
-        if (s_blk != blockIdx.x) {
-            lean_rows_of<UPPER, CT>(p, s_blk, tid, pol, i, rs, re, bi, true);
-        } else if (i >= 0 && i < p.n) {
+        cta_ticket(p, s_blk, s_epoch);
+        if (bgate) {  // wait until the b chunks of this CTA's (physical) rows have landed
+            const int lr0 = (int)s_blk * CT, lr1 = min(p.n, lr0 + CT);
+            wait_b_chunks(p, UPPER ? p.n - lr1 : lr0, UPPER ? p.n - lr0 : lr1);
+        }
+    }
+    __syncthreads();
+    if (s_blk == kStaleBlk) return;
+    const uint32_t epoch = s_epoch;
+    if (s_blk != blockIdx.x) {  // rare: re-load for the block the ticket assigned
+        i = (int)s_blk * CT + tid;
+        if (UPPER) i = p.n - 1 - i;
+        rs = 0, re = 1, bi = 0.0;
+        if (i >= 0 && i < p.n) {
+            rs = ld_stream_i32(p.rowptr + i, pol);
+            re = ld_stream_i32(p.rowptr + i + 1, pol);
             bi = ld_b(p, i, pol);
         }
-        const bool act = i >= 0 && i < p.n;
-        lean_rows<PROTO, UPPER, UNIT>(p, i, act, lean_load<UPPER, UNIT>(p, act, rs, re, pol), bi, s_epoch, lane, pol);
-        __syncthreads();  // every solve, whichever start it used, bumps `ep` exactly once (below)
-        if (tid == 0) {
-            const unsigned long long d = atomicAdd(&p.st->done.v, 1ull);
-            if ((d + 1) % p.grid == 0)
-                st_relaxed_u64(&p.st->ep.v, ((unsigned long long)p.gen << kGenShift) | (s_epoch + 1u));
-        }
-    } else {
-        if (tid == 0) s_tkv = kUnknownBlk;
-        __syncthreads();  // (launch skew only: nothing to wait for)
-        unsigned long long tk = 0;
-        if (tid == 0) tk = atomicAdd(&p.st->tk.v, 1ull);  // verified below, never waited for up front
-        lean_rows_of<UPPER, CT>(p, blockIdx.x, tid, pol, i, rs, re, bi, true);
-        if (p.trace && i >= 0 && i < p.n) p.trace[3 * (size_t)p.n + 3 + i] = globaltimer_ns();  // CTA entry
-        // the epoch: one L2 load per warp, in flight with the row loads
-        unsigned long long epw = 0;
-        if (lane == 0) epw = ld_relaxed_u64(&p.st->ep.v);
-        epw = __shfl_sync(FULL, epw, 0);
-        if ((uint32_t)(epw >> kGenShift) != p.gen) {  // a stale launch (graph of an older configuration)
-            if (lane == 0) {
-                atomicCAS(&p.st->error.v, 0u, kErrStale);
-                st_relaxed_u32(&p.st->abort.v, 1u);
-            }
-            return;
-        }
-        const uint32_t epoch = (uint32_t)epw;
-        if (tid == 0) {  // the ticket (warp 0 waits for it here; the other warps are already solving)
-            uint32_t blk, e;
-            cta_ticket_decode(p, tk, blk, e);
-            s_tkv = blk;
-        }
-        const bool act = i >= 0 && i < p.n;
-        // speculative rows: give up at a wait once the ticket names another block
-        auto give_up = [&]() -> bool {
-            const uint32_t t = s_tkv;
-            return t != kUnknownBlk && t != blockIdx.x;
-        };
-        lean_rows<PROTO, UPPER, UNIT>(p, i, act, lean_load<UPPER, UNIT>(p, act, rs, re, pol), bi, epoch, lane, pol,
-                                      give_up);
-        uint32_t t;
-        while ((t = s_tkv) == kUnknownBlk) {}  // the ticket is one atomic away
-        if (t == kStaleBlk) return;
-        if (t != blockIdx.x) {  // rare: dispatch out of blockIdx order -- solve the ticket's block
-            lean_rows_of<UPPER, CT>(p, t, tid, pol, i, rs, re, bi, true);
-            const bool a2 = i >= 0 && i < p.n;
-            lean_rows<PROTO, UPPER, UNIT>(p, i, a2, lean_load<UPPER, UNIT>(p, a2, rs, re, pol), bi, epoch, lane, pol);
-        }
-        s_blk = t;  // (every thread writes the same value; read after the barrier below)
-        // the CTA that completes the solve writes the next solve's epoch
-        __syncthreads();
-        if (tid == 0) {
-            const unsigned long long d = atomicAdd(&p.st->done.v, 1ull);
-            if ((d + 1) % p.grid == 0) st_relaxed_u64(&p.st->ep.v, ((unsigned long long)p.gen << kGenShift) | (epoch + 1u));
-        }
+    } else if (bgate && i >= 0 && i < p.n) {
+        bi = ld_b(p, i, pol);
     }
+    const bool act = i >= 0 && i < p.n;
+    lean_rows<PROTO, UPPER, UNIT>(p, i, act, lean_load<UPPER, UNIT>(p, act, rs, re, pol), bi, epoch, lane, pol);
     if (p.trace && lane == 0) atomicMax(&p.trace[3 * (size_t)p.n + 1], globaltimer_ns());  // last warp exit
     if (p.x_host) {
         // sptrsv_solve_host: the CTA's finished rows go to pinned host memory over PCIe as one

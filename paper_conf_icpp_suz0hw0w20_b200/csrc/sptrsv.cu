@@ -329,7 +329,6 @@ __global__ void k_l2_discard(char *p, size_t bytes) {
 // a host copy, so that a reset inside a stream capture is capturable.
 __global__ void k_state_init(SolveState *st, uint32_t gen) {
     st->tk.v = (unsigned long long)gen << kGenShift;
-    st->ep.v = ((unsigned long long)gen << kGenShift) | 1ull;
 }
 
 int init_state(SolveState *st, uint32_t gen, cudaStream_t s) {
