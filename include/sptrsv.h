@@ -74,8 +74,10 @@ typedef enum sptrsv_option {
                                       n <= 1024: never; sec.4.4, DESIGN G10).  Setting it
                                       overrides that and re-plans (synchronous).            */
     SPTRSV_OPT_CTA_THREADS = 3,    /* threads per CTA, or 0 (default) = the engine's measured
-                                      best.  ONE-SHOT: 64..1024; LEAN (lower): 128, 256, 512;
-                                      CHAIN: 64, 128, 256; other values / engines: default  */
+                                      best: 32, 64, 128, 256, 512 or 1024.  ONE-SHOT: 64..1024;
+                                      LEAN (lower): 128, 256, 512; CHAIN: 64, 128, 256;
+                                      HYBRID: 64, 256; SMALL: any (capped at n rounded up to
+                                      a warp); other values / engines: default             */
     SPTRSV_OPT_BACKOFF_MIN_NS = 4, /* __nanosleep after a pass where no lane progressed     */
     SPTRSV_OPT_BACKOFF_MAX_NS = 5, /* exponential backoff cap                               */
     SPTRSV_OPT_SPIN_LIMIT = 6,     /* watchdog: idle passes per warp before TIMEOUT (0=off) */
@@ -95,7 +97,11 @@ typedef enum sptrsv_option {
     SPTRSV_OPT_LOCAL = 10,         /* 1 (default): dependencies produced inside the same CTA
                                       are read from a shared-memory copy of x               */
     SPTRSV_OPT_ENGINE = 11,        /* 5 (default) AUTO, from analyse's statistics (DESIGN.md
-                                      section 6): HYBRID for plans with warp-level rows; for
+                                      section 6): SMALL for systems of <= 4096 rows with
+                                      near dependencies that are not pure chains and whose
+                                      CSR, b and x fit one CTA's shared memory (24 B per
+                                      row + 12 B per entry <= 226 KB);
+                                      else HYBRID for plans with warp-level rows; for
                                       all-thread-level plans LEAN when < 1/4 of the rows wait
                                       on a row < 256 away, CHAIN when >= 1/4 of the
                                       dependencies are on the previous row, else ONE-SHOT.
@@ -107,14 +113,17 @@ typedef enum sptrsv_option {
                                       6 HYBRID: one task per warp -- a warp-level row (Alg.3)
                                       or a 32-row thread group (LEAN's per-lane loop);
                                       7 CHAIN: in-warp dependency chains resolved in
-                                      registers / shared memory, external ones by polling.
+                                      registers / shared memory, external ones by polling;
+                                      8 SMALL: one CTA, the whole system in shared memory
+                                      (any plan, any triangular form; INVALID_ARG when it
+                                      does not fit; CTA_THREADS: 32..1024, multiple of 32).
                                       LEAN and CHAIN need an all-thread-level plan; a plan
                                       with warp-level rows runs HYBRID (ONE-SHOT if forced on
                                       a lower handle).  sptrsv_info.engine reports the engine
                                       that runs.  Other values: INVALID_ARG                 */
     /* 12, 13, 14: retired (the PIPE ablation engine left the library in round 2)       */
     SPTRSV_OPT_ROWS_PER_LANE = 15, /* CHAIN: K = 1 or 2 (0 = default 2) rows per lane       */
-    SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 6)
+    SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 5)
                                       resident 256-thread CTAs per SM                       */
     /* 18: retired (the L2 bulk prefetch of LEAN measured no gain and left in round 2)   */
     SPTRSV_OPT_POLL_GAP_NS = 19,   /* LEAN: __nanosleep after a pass that progressed but left
@@ -138,7 +147,9 @@ typedef enum sptrsv_option {
                                       lanes in parallel (a failure aborts the solve with
                                       SPTRSV_ERR_INEXACT); 1 = prove every quotient before the
                                       chain uses it (+~25 cycles per chain step); 2 = test
-                                      hook: every post-run proof fails                      */
+                                      hook: every post-run proof fails.  SMALL always proves
+                                      after its sweep and, on a failure, re-runs the sweep
+                                      with the verified division (no error; 2 forces it)    */
     SPTRSV_OPT_HOST_IO = 23,       /* sptrsv_solve_host with pinned buffers on LEAN: bit 0 =
                                       b copied in chunks on a second stream, each CTA waiting
                                       for its own chunk only (needs cuStreamWriteValue32);
@@ -173,7 +184,8 @@ typedef struct sptrsv_info {
     int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
     int64_t warp_deps;        /* dependencies inside the row's own 32-row group            */
     int32_t engine;           /* engine the next solve launches (0 ONE-SHOT, 3 LEAN,
-                                 6 HYBRID, 7 CHAIN; 33/34/35 the paper's Alg.3/4/5)        */
+                                 6 HYBRID, 7 CHAIN, 8 SMALL; 33/34/35 the paper's
+                                 Alg.3/4/5)                                                */
     int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
     int64_t prev_deps;        /* dependencies on the previous row in solve order (i - 1;
@@ -241,11 +253,12 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
  * earliest-solved first: ascending column (lower), descending column (upper).
  * sptrsv_solve, sptrsv_solve_multi (column by column), sptrsv_solve_host,
  * sptrsv_get_indegree, sptrsv_check and the
- * options work as for lower handles (ENGINE: only 3 LEAN and 7 CHAIN are
- * honoured, for all-thread-level plans);
+ * options work as for lower handles (ENGINE: 3 LEAN and 7 CHAIN are honoured
+ * for all-thread-level plans, 8 SMALL for systems that fit one CTA);
  * sptrsv_levels and VARIANT != 0 return SPTRSV_ERR_INVALID_ARG.  Thread-level rows are bit-exact with that fp64
  * substitution (one rounded multiply and add each); warp rows are within the
- * warp-mode bound, as for lower handles.  sptrsv_info.engine: 3 LEAN, 6 warp.
+ * warp-mode bound, as for lower handles.  sptrsv_info.engine: 3 LEAN, 6 warp,
+ * 7 CHAIN, 8 SMALL (bit-exact: every row is thread-level there).
  */
 int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx,
                           const double *val, int32_t tri_flags, sptrsv_handle_t *out);
@@ -288,6 +301,8 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
  *     finished rows of x to x_host as one contiguous block -- both transfers
  *     overlap the solve (x also lands in handle-owned device staging).
  *     SPTRSV_OPT_HOST_IO selects the variants.
+ *   - Both pinned and the handle runs SMALL: the kernel reads b from b_host
+ *     and writes x to x_host through the UVA mapping (no copy launches).
  *   - Otherwise: b is copied to handle-owned device staging, solved, and x is
  *     copied back (cudaMemcpyAsync; pageable buffers are staged by the driver).
  */

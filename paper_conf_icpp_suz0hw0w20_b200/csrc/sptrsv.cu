@@ -21,6 +21,7 @@
 #include "solve_multi.cuh"
 #include "solve_paper.cuh"
 #include "solve_chain.cuh"
+#include "solve_small.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -30,7 +31,14 @@ namespace {
 constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
 
 // engines (SPTRSV_OPT_ENGINE values, include/sptrsv.h)
-enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7 };
+enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_SMALL = 8 };
+
+// ENGINE_SMALL (solve_small.cuh): the whole system in one CTA's shared memory.  Usable when it fits
+// (kSmallSmemMax bytes of dynamic shared memory, sm_100a allows 227 KB per CTA); AUTO picks it up to
+// kSmallAutoN rows (measured against LEAN / ONE-SHOT / CHAIN on c1-shaped systems).
+constexpr size_t kSmallSmemMax = 226 * 1024;
+constexpr int kSmallAutoN = 4096;
+constexpr int kSmallCta = 256;
 
 // The handle's workspace is ONE device allocation (analyse is O(nnz) work plus a fixed handful of
 // runtime calls), carved in 256-byte aligned pieces: the 16-byte FUSED records, the FLAGS words,
@@ -548,14 +556,31 @@ void size_l2_window(sptrsv_handle_s *h) {
 }
 
 // ENGINE_AUTO, from analyse's O(nnz) statistics:
+//   near-dependency systems that are not pure chains, <= kSmallAutoN rows, fitting one CTA's
+//   shared memory (c1, small grids)                              -> SMALL (any plan, any form)
 //   plans with warp-level rows                                   -> HYBRID
 //   all-thread plans, < 1/4 of the rows waiting on a row < 256 away -> LEAN
 //   all-thread plans, >= 1/4 of the dependencies on row i-1 (chains, grids) -> CHAIN
 //   other near-dependency plans (small levels, c1)               -> ONE-SHOT (in-CTA smem copy of x)
 // f4 (upper / unit) handles: HYBRID for warp rows, else CHAIN (chains) or LEAN.
+bool small_fits(const sptrsv_handle_s *h) {
+    return h->n > 0 && h->n <= (1 << 20) && small_smem_bytes(h->n, h->nnz) <= kSmallSmemMax;
+}
+
 int resolve_engine(const sptrsv_handle_s *h) {
+    if (h->engine == ENG_SMALL && small_fits(h)) return ENG_SMALL;
     const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;  // unit handles store no diagonal
     const bool chains = offdiag > 0 && 4 * h->prev_deps >= offdiag;
+    const bool near = offdiag > 0 && 4 * h->near_rows >= (int64_t)h->n;
+    // a pure chain: almost every row waits on its predecessor and little else (critical path ~ n rows;
+    // CHAIN's in-register hop beats SMALL's shared-memory pass there: 1024-row chain 111 vs 200 us)
+    const bool pure_chain = 10 * h->prev_deps >= 9 * (int64_t)h->n && 4 * offdiag <= 5 * (int64_t)h->n;
+    // AUTO: small near-dependency systems that fit one CTA (c1, small grids, short dense-ish rows) ->
+    // SMALL, whatever the plan (measured: c1 18 vs 29 us ONE-SHOT, 32x32 grid 22 vs 169 us CHAIN,
+    // 600 rows x 20 entries 38 vs 99 us)
+    // (not when the user asked for warp-level rows: MODE 2 / 3 plans keep their warp engine)
+    if (h->engine == ENG_AUTO && h->mode <= 1 && near && !pure_chain && h->n <= kSmallAutoN && small_fits(h))
+        return ENG_SMALL;
     if (h->plan != PLAN_THREAD)  // ONE-SHOT has no sub-warp rows
         return (h->engine == ENG_ONESHOT && !h->tri && h->n_sub_tasks == 0) ? ENG_ONESHOT : ENG_HYBRID;
     if (h->engine != ENG_AUTO) return (h->tri && h->engine == ENG_ONESHOT) ? ENG_LEAN : h->engine;
@@ -636,6 +661,34 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
     const int engine = resolve_engine(h);
     const int user = h->cta_threads;
     L->engine = engine;
+    if (engine == ENG_SMALL) {  // one CTA, the system in shared memory (solve_small.cuh)
+        static const lean_fn tab[4] = {k_solve_small<false, false>, k_solve_small<true, false>,
+                                       k_solve_small<false, true>, k_solve_small<true, true>};
+        // the dynamic shared memory limit is raised to what this launch needs (per device: the attribute
+        // is per context), not to the 226 KB maximum
+        static int attr_set[64][4] = {};
+        const int t = h->tri & 3, dv = h->device & 63;
+        const size_t need = small_smem_bytes(h->n, h->nnz);
+        L->fn = (const void *)tab[t];
+        if ((size_t)attr_set[dv][t] < need) {
+            if (cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)need) != cudaSuccess) {
+                (void)cudaGetLastError();
+                return SPTRSV_ERR_CUDA;
+            }
+            attr_set[dv][t] = (int)need;
+        }
+        // 256 threads (default): measured best on c1 / 32x32 grids (fewer spinning warps leave the
+        // issue slots to the ones on the critical path; 1024 threads: c1 32.8 us, 256: 18.5 us)
+        const int rows32 = (int)std::min<long long>(kSmallCtaMax, ((long long)h->n + 31) / 32 * 32);
+        int ct = std::min(kSmallCta, rows32);
+        if (user >= 32 && user <= kSmallCtaMax && user % 32 == 0) ct = std::min(user, rows32);
+        L->cta = ct;
+        L->grid = dim3(1u);
+        L->block = dim3((unsigned)ct);
+        L->smem = small_smem_bytes(h->n, h->nnz);
+        L->key = (9000000 + h->tri * 10000 + ct) ^ h->n * 7919;
+        return SPTRSV_OK;
+    }
     if (engine == ENG_HYBRID) {  // warp-level rows: one task per warp (solve_tri.cuh), any triangular form
         if (h->plan == PLAN_THREAD) {  // HYBRID forced on an all-thread plan: run it as LEAN
             L->engine = ENG_LEAN;
@@ -690,7 +743,7 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
     // x.  64-thread CTAs on plans with warp-level rows; 1024 for small (n <= 32768) thread-level systems
     // (more dependencies resolved in-CTA: c1 29.7 -> 26.7 us); else 256.
     int cta = h->plan != PLAN_THREAD ? 64 : h->n <= 32768 ? 1024 : 256;
-    if (user) cta = user;
+    if (user >= 64) cta = user;  // (32: SMALL only)
     const int warps = cta / 32;
     L->engine = ENG_ONESHOT;
     L->fn = (const void *)solve_kernel(h->plan, h->proto);
@@ -972,6 +1025,14 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
     // engines that take the chunked b (wait_b_chunks) and, for LEAN / CHAIN, write x per CTA / warp
     const int eng = L0.engine;
     const bool gated = eng == ENG_LEAN || eng == ENG_CHAIN || eng == ENG_HYBRID;
+    if (pinned && io && eng == ENG_SMALL) {
+        // SMALL: the one CTA reads b straight from the mapped pinned buffer (one coalesced pass over
+        // PCIe, no copy launch) and writes x to both x_stage and the mapped pinned x
+        int rc = solve_impl(h, (const double *)ab.devicePointer, h->ws.x_stage, (double *)ax.devicePointer, stream);
+        if (rc) return rc;
+        CK(cudaStreamSynchronize(s));
+        return SPTRSV_OK;
+    }
     if (!(eng == ENG_LEAN || eng == ENG_CHAIN)) io &= ~2;
     if (pinned && io && gated) {
         const uint32_t *bflag = nullptr;
@@ -1070,7 +1131,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             h->threshold_user = true;
             return build_plan(h);
         case SPTRSV_OPT_CTA_THREADS:
-            if (value != 0 && value != 64 && value != 128 && value != 256 && value != 512 && value != 1024)
+            if (value != 0 && value != 32 && value != 64 && value != 128 && value != 256 && value != 512 && value != 1024)
                 return SPTRSV_ERR_INVALID_ARG;
             h->cta_threads = (int)value;
             return SPTRSV_OK;
@@ -1106,8 +1167,9 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
             if (value != ENG_ONESHOT && value != ENG_LEAN && value != ENG_AUTO && value != ENG_HYBRID &&
-                value != ENG_CHAIN)
+                value != ENG_CHAIN && value != ENG_SMALL)
                 return SPTRSV_ERR_INVALID_ARG;
+            if (value == ENG_SMALL && !small_fits(h)) return SPTRSV_ERR_INVALID_ARG;  // does not fit one CTA
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE:

@@ -63,7 +63,15 @@ def random_structure(rng):
 
 ENGINES = [(5, {}), (0, {}), (3, {}), (6, {}), (7, {}),
            (0, {"cta_threads": 1024}), (7, {"rows_per_lane": 1, "cta_threads": 64}), (3, {"cta_threads": 128}),
-           (7, {"cta_threads": 512}), (3, {"cta_threads": 1024})]
+           (7, {"cta_threads": 512}), (3, {"cta_threads": 1024}), (8, {}), (8, {"cta_threads": 64})]
+
+
+def small_fits(s):
+    """ENGINE_SMALL accepts systems whose CSR, b and x fit one CTA's shared memory (sptrsv.cu)."""
+    n, nnz = s.n, int(s.rowptr[-1])
+    up = lambda v: (v + 15) // 16 * 16
+    z = max(nnz, 1)
+    return n <= (1 << 20) and 3 * up(8 * n) + up(8 * z) + up(4 * (n + 1)) + up(4 * z) + 64 <= 226 * 1024
 
 
 @pytest.mark.parametrize("seed", range(int(os.environ.get("SPTRSV_FUZZ_SEEDS", "100"))))
@@ -78,6 +86,8 @@ def test_fuzz_engines_vs_oracle(seed):
     for k in picks:
         engine, extra = ENGINES[k]
         proto = int(rng.integers(0, 2))
+        if engine == 8 and (s.n == 0 or not small_fits(s)):
+            continue
         with cap.analyse(rp, ci, v, engine=engine, protocol=proto, **extra) as h:
             for _ in range(2):  # two solves: the epoch path
                 x = torch.full_like(b, float("nan"))
@@ -107,8 +117,10 @@ def test_fuzz_triangular_forms_vs_oracle(seed):
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     d = torch.device("cuda:0")
     rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
-    for opts in ({}, {"engine": 3, "mode": 1}, {"engine": 7, "mode": 1}):
+    for opts in ({}, {"engine": 3, "mode": 1}, {"engine": 7, "mode": 1}, {"engine": 8}):
         proto = int(rng.integers(0, 2))
+        if opts.get("engine") == 8 and (s.n == 0 or not small_fits(s)):
+            continue
         with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2), protocol=proto, **opts) as h:
             for _ in range(2):
                 x = torch.full_like(b, float("nan"))

@@ -492,12 +492,13 @@ def test_chain_engine_division_guard_exits(cap, proto, K, eng):
 
 
 def test_engine_auto_choice(cap):
-    """ENGINE_AUTO: far dependencies -> LEAN (3); chains / grid wavefronts (>= 1/4 of the dependencies
-    on the previous row) -> CHAIN (7); other near-dependency plans (small levels, c1) -> staged one-shot
-    (0); plans with warp-level rows -> HYBRID (6)."""
+    """ENGINE_AUTO: small near-dependency systems that fit one CTA and are not pure chains (c1, a 32x32
+    grid) -> SMALL (8); far dependencies -> LEAN (3); chains / grid wavefronts (>= 1/4 of the
+    dependencies on the previous row) -> CHAIN (7); other near-dependency plans (small levels) ->
+    staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""
     for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 7, 128, 2),
                               (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
-                              (lambda: synth.gen_c1(), 0, 1024, 1),
+                              (lambda: synth.gen_c1(), 8, 256, 1), (lambda: synth.gen_grid(32), 8, 256, 1),
                               (lambda: synth.gen_c4(n=5000, nlevels=50), 6, 64, 1),
                               (lambda: synth.gen_leveled(20_000, 1000, 1, 3, 77, "lev_small"), 0, 1024, 1)):
         s = gen()

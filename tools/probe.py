@@ -1,7 +1,7 @@
 """Scratch perf probe over systems x option sets (CUDA events, L2 flushed between solves).
 
 usage: python tools/probe.py SYS[,SYS...] [OPTS_JSON_LIST]
-  SYS: c1..c5 | chain | grid:G | stride:N:S (row i depends on i-S only) | lev:N:L:KANY | diag:N
+  SYS: c1..c5 | chain | grid:G | stride:N:S (row i depends on i-S only) | lev:N:L:KANY | diag:N | rand:N:K
   OPTS_JSON_LIST: JSON list of option dicts (default [{}]), e.g. '[{}, {"backoff_max": 64}]'
 Prints one JSON line per (system, options): median / mean solve time, GFLOPS, engine, parity vs x_true."""
 import json, os, sys
@@ -23,6 +23,8 @@ def build(spec):
         return synth.from_pattern(spec, rp, ci, rng, {"levels": (n + S - 1) // S})
     if p[0] == "lev":
         return synth.gen_leveled(int(p[1]), int(p[2]), 1, int(p[3]), 9, spec)
+    if p[0] == "rand":  # rand:N:K -- row i: min(K, i) distinct columns uniform in [0, i) (c1's recipe)
+        return synth.gen_random_lower(int(p[1]), int(p[2]), 11, spec)
     if p[0] == "diag":
         return synth.gen_diag(int(p[1]))
     return synth.make(spec)
