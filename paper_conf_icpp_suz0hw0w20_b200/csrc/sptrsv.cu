@@ -695,6 +695,11 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         } else {
             const int ct = user == 256 ? 256 : kTriWarpCta;  // 64 (default) or 256 threads
             L->fn = (const void *)tri_warp_kernel(h->proto, h->tri, h->plan, ct);
+#ifdef SPTRSV_MEASURE_HYBRID_SMEM  // measurement builds only (tools/): cap residency with padding
+            L->smem = SPTRSV_MEASURE_HYBRID_SMEM;
+            if (cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess)
+                return SPTRSV_ERR_CUDA;
+#endif
             L->cta = ct;
             L->grid = dim3((unsigned)((h->n_tasks + ct / 32 - 1) / (ct / 32)));
             L->block = dim3((unsigned)ct);
