@@ -65,6 +65,9 @@ __device__ __forceinline__ void subwarp_rows(SolveParams &p, int r0, uint32_t ep
     const bool act = r < p.n;
     const bool leader = act && sl == 0;
     const int i = UPPER ? p.n - 1 - r : r;
+#ifdef SPTRSV_MEASURE_ROWSTART  // measurement builds only (tools/trace_polls.py): task start per row
+    if (p.trace && leader) p.trace[2 * (size_t)p.n + i] = globaltimer_ns();
+#endif
     int rs = 0, re = 0;
     if (act) {
         rs = ld_stream_i32(p.rowptr + i, pol);
@@ -113,6 +116,9 @@ __device__ __forceinline__ void subwarp_rows(SolveParams &p, int r0, uint32_t ep
     bool lane_done = mm == 0, reduced = false, published = !leader;
     const unsigned segmask = W == 32 ? FULL : ((1u << W) - 1u) << (lane & ~(W - 1));
     uint32_t backoff = p.backoff_min, idle = 0;
+#ifdef SPTRSV_MEASURE_POLLS
+    unsigned long long np_ = 0, tl_ = 0;
+#endif
     while (true) {
         bool prog = false;
         if (!lane_done) {  // poll the batch, consume its ready prefix in order
@@ -157,12 +163,24 @@ __device__ __forceinline__ void subwarp_rows(SolveParams &p, int r0, uint32_t ep
             bool go = true;
             if (has_last) {
                 unsigned long long w0, w1;
+#ifdef SPTRSV_MEASURE_POLLS  // measurement builds only (tools/trace_polls.py): wait start, last poll, polls
+                if (p.trace) {
+#ifndef SPTRSV_MEASURE_ROWSTART
+                    if (np_ == 0) p.trace[2 * (size_t)p.n + i] = globaltimer_ns();
+#endif
+                    tl_ = globaltimer_ns();
+                }
+                ++np_;
+#endif
                 poll1<PROTO>(p, c_last, w0, w1);
                 go = ready1<PROTO>(w0, w1, epoch);
                 if (go) tot = __dadd_rn(tot, __dmul_rn(v_last, value1<PROTO>(p, c_last, w0, w1)));
             }
             if (go) {
                 if (p.trace) p.trace[p.n + i] = globaltimer_ns();
+#ifdef SPTRSV_MEASURE_POLLS
+                if (p.trace && has_last) p.trace[3 * (size_t)p.n + 3 + i] = (np_ << 40) | (tl_ & ((1ull << 40) - 1));
+#endif
                 Cta nocta;
                 nocta.R0 = nocta.R1 = 0;
                 nocta.xc = nullptr;

@@ -1,0 +1,5 @@
+python paper_conf_icpp_suz0hw0w20_b200/build.py --force -DSPTRSV_MEASURE_POLLS > gpurun_out/exp56_build.txt 2>&1
+cd tools
+timeout 300 python trace_polls.py 1000000 1000 62 > ../gpurun_out/exp56.txt 2>&1
+timeout 300 python trace_polls.py 100000 1000 62 >> ../gpurun_out/exp56.txt 2>&1
+timeout 300 python trace_polls.py 1000000 1000 62 subwarp=0 >> ../gpurun_out/exp56.txt 2>&1
