@@ -59,9 +59,9 @@ WORKLOADS = {
     "chain": "bidiagonal chain n=100,000 (pure dependency chain, aux)",
 }
 ENGINES = {0: "one-shot (staged, in-CTA x copy)", 3: "lean", 6: "hybrid (warp tasks + 32-row thread groups)",
-           7: "chain (in-warp chains)",
+           7: "chain (in-warp chains)", 8: "small (one CTA, shared memory)",
            33: "paper Alg.3", 34: "paper Alg.4", 35: "paper Alg.5"}
-KERNELS = {0: "k_solve", 3: "k_solve_lean", 6: "k_solve_tri_warp", 7: "k_solve_chain",
+KERNELS = {0: "k_solve", 3: "k_solve_lean", 6: "k_solve_tri_warp", 7: "k_solve_chain", 8: "k_solve_small",
            33: "k_paper_alg3", 34: "k_paper_alg4", 35: "k_paper_alg5"}
 EXTRA_CONFIGS = ["c1", "c3", "c4", "c5sys", "chain"]
 
@@ -273,13 +273,16 @@ def roofline(s, mean_s, peak, peak_src, kernel, traffic=None):
             "alg_bytes_per_launch": alg, "alg_bytes_formula": "4(n+1) + 12*nnz + 8n (b) + 8n (x) + 4n (flags)"}
 
 
-def latency_bound(levels, hops, mean_s, alg_bytes, peak):
+def latency_bound(levels, hops, mean_s, alg_bytes, peak, engine=None):
     """T_lat = (levels - 1) * t_hop per die placement; t / max(T_bw, T_lat)."""
     t_bw = alg_bytes / (peak * 1e9)
     out = {"levels": int(levels), "t_bw_us": round(t_bw * 1e6, 3),
            "model": "(levels - 1) * t_hop with the cross-SM record hop: a bound when every level boundary crosses "
                     "SMs; CHAIN resolves in-warp levels in registers (~0.1 us per step), so for chains and grids it "
                     "is a model, not a bound"}
+    if engine == 8:
+        out["model"] = ("SMALL solves the whole system in ONE SM's shared memory: no level boundary crosses SMs, so "
+                        "the cross-SM hop figures below are a reference scale only, not a bound")
     for place, hop in hops.items():
         if hop is None:
             continue
@@ -556,7 +559,7 @@ def run_single(args):
                 "engine": ENGINES.get(inf["engine"], str(inf["engine"])), "cta_threads": inf["cta_threads"],
                 "rows_per_lane": inf["rows_per_lane"], "analyse_ms": round(inf["analyse_ms"], 3),
                 "roofline": roofline(s, m, peak, peak_src, KERNELS.get(inf["engine"], "?")),
-                "latency_bound": latency_bound(nlev, hops, m, s.alg_bytes(), peak),
+                "latency_bound": latency_bound(nlev, hops, m, s.alg_bytes(), peak, inf["engine"]),
                 "levels_gpu": int(nlev), "levels_generator": generator_levels(s),
                 "max_rel_err_vs_x_true": (float(np.max(np.abs(xt - ref) / np.abs(ref))) if ref is not None
                                           else None)}

@@ -10,6 +10,6 @@ $NCU --set full --clock-control none --import-source on -k regex:k_solve_tri_war
     python tools/run_one.py c4 5 > gpurun_out/r02prof/hybrid_c4.log 2>&1
 $NCU --set full --clock-control none --import-source on -k regex:k_solve_chain -s 3 -c 1 -o gpurun_out/r02prof/chain_c3 \
     python tools/run_one.py c3 5 > gpurun_out/r02prof/chain_c3.log 2>&1
-$NCU --set full --clock-control none --import-source on -k regex:k_solve -s 3 -c 1 -o gpurun_out/r02prof/oneshot_c1 \
-    python tools/run_one.py c1 5 > gpurun_out/r02prof/oneshot_c1.log 2>&1
+$NCU --set full --clock-control none --import-source on -k regex:k_solve_small -s 3 -c 1 -o gpurun_out/r02prof/small_c1 \
+    python tools/run_one.py c1 5 > gpurun_out/r02prof/small_c1.log 2>&1
 ls -la gpurun_out/r02prof
