@@ -59,9 +59,10 @@ WORKLOADS = {
     "chain": "bidiagonal chain n=100,000 (pure dependency chain, aux)",
 }
 ENGINES = {0: "one-shot (staged, in-CTA x copy)", 3: "lean", 6: "hybrid (warp tasks + 32-row thread groups)",
-           7: "chain (in-warp chains)", 8: "small (one CTA, shared memory)",
+           7: "chain (in-warp chains)", 8: "small (one CTA, shared memory)", 9: "leanp (persistent, pipelined)",
            33: "paper Alg.3", 34: "paper Alg.4", 35: "paper Alg.5"}
 KERNELS = {0: "k_solve", 3: "k_solve_lean", 6: "k_solve_tri_warp", 7: "k_solve_chain", 8: "k_solve_small",
+           9: "k_solve_leanp",
            33: "k_paper_alg3", 34: "k_paper_alg4", 35: "k_paper_alg5"}
 EXTRA_CONFIGS = ["c1", "c3", "c4", "c5sys", "chain"]
 

@@ -102,9 +102,11 @@ typedef enum sptrsv_option {
                                       CSR, b and x fit one CTA's shared memory (24 B per
                                       row + 12 B per entry <= 226 KB);
                                       else HYBRID for plans with warp-level rows; for
-                                      all-thread-level plans LEAN when < 1/4 of the rows wait
-                                      on a row < 256 away, CHAIN when >= 1/4 of the
-                                      dependencies are on the previous row, else ONE-SHOT.
+                                      all-thread-level plans LEANP when < 1/4 of the rows
+                                      wait on a row < 256 away, CHAIN for long runs of
+                                      previous-row dependencies (>= 1/4 of the dependencies,
+                                      mean run >= 2048 rows, runs starting on 64-row
+                                      boundaries), else ONE-SHOT.
                                       Forced engines:
                                       0 ONE-SHOT (lower): one CTA per row range, ticketed,
                                       smem-staged CSR slices, in-CTA x copy in smem;
@@ -116,11 +118,15 @@ typedef enum sptrsv_option {
                                       registers / shared memory, external ones by polling;
                                       8 SMALL: one CTA, the whole system in shared memory
                                       (any plan, any triangular form; INVALID_ARG when it
-                                      does not fit; CTA_THREADS: 32..1024, multiple of 32).
-                                      LEAN and CHAIN need an all-thread-level plan; a plan
-                                      with warp-level rows runs HYBRID (ONE-SHOT if forced on
-                                      a lower handle).  sptrsv_info.engine reports the engine
-                                      that runs.  Other values: INVALID_ARG                 */
+                                      does not fit; CTA_THREADS: 32..1024, multiple of 32);
+                                      9 LEANP: LEAN's row loop in persistent warps (a
+                                      cooperative launch of what fits on the device, static
+                                      round-robin blocks) with the next chunks' loads in
+                                      flight during the current chunk's waits.
+                                      LEAN, LEANP and CHAIN need an all-thread-level plan; a
+                                      plan with warp-level rows runs HYBRID (ONE-SHOT if
+                                      forced on a lower handle).  sptrsv_info.engine reports
+                                      the engine that runs.  Other values: INVALID_ARG      */
     /* 12, 13, 14: retired (the PIPE ablation engine left the library in round 2)       */
     SPTRSV_OPT_ROWS_PER_LANE = 15, /* CHAIN: K = 1 or 2 (0 = default 2) rows per lane       */
     SPTRSV_OPT_LEAN_OCCUPANCY = 17,/* LEAN engine register budget: 5..8 (default 5)
@@ -184,8 +190,8 @@ typedef struct sptrsv_info {
     int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
     int64_t warp_deps;        /* dependencies inside the row's own 32-row group            */
     int32_t engine;           /* engine the next solve launches (0 ONE-SHOT, 3 LEAN,
-                                 6 HYBRID, 7 CHAIN, 8 SMALL; 33/34/35 the paper's
-                                 Alg.3/4/5)                                                */
+                                 6 HYBRID, 7 CHAIN, 8 SMALL, 9 LEANP; 33/34/35 the
+                                 paper's Alg.3/4/5)                                        */
     int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
     int64_t prev_deps;        /* dependencies on the previous row in solve order (i - 1;
@@ -295,7 +301,7 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
  * sptrsv_solve_host -- end-to-end convenience from host buffers; synchronises
  * `stream` before returning.  b_host/x_host: host double[n].
  *   - Both pinned (page-locked, UVA-mapped; e.g. cudaHostAlloc or torch
- *     pin_memory) and the handle runs LEAN: b is copied to device staging in
+ *     pin_memory) and the handle runs LEAN or LEANP: b is copied to device staging in
  *     about four chunks on a handle-owned second stream, each CTA of the solve
  *     waiting only for the chunk of its own rows, and every CTA writes its
  *     finished rows of x to x_host as one contiguous block -- both transfers

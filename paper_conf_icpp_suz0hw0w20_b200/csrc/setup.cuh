@@ -29,7 +29,8 @@ struct AnalyseOut {
     int32_t n_tasks, n_tgroups;  // plan: warp tasks, 32-row thread groups
     int32_t n_subtasks;          // plan: tasks with 2..16 lanes per row (sub-warp rows)
     int32_t epl;                 // sub-warp target off-diagonals per lane (0: warp rows only)
-    int32_t pad2;
+    int32_t mid_breaks;          // rows not at a 64-row boundary (logical order) without a previous-row
+                                 // dependency: where CHAIN's in-warp order would serialise independent runs
     unsigned long long near;     // near_deps | warp_deps << 32
     unsigned long long prev;     // prev_deps | near_rows << 32
     unsigned long long hist[32]; // rows by floor(log2(nearest-dependency distance))
@@ -60,7 +61,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
     }
     if (nnz > 0 && (!colidx || (!val && !unit))) return;
     int len = 0;
-    unsigned near = 0, wdep = 0, pdep = 0, nrow = 0;
+    unsigned near = 0, wdep = 0, pdep = 0, nrow = 0, mbrk = 0;
     int dmin = 0x7fffffff;  // the row's nearest dependency (distance in rows)
     if (i < n) {
         const int64_t s = rowptr[i], e = rowptr[i + 1];
@@ -92,6 +93,7 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
             }
         }
         if (!code && dmin < 256) nrow = 1;  // the row's latest-solved dependency is near
+        if (!code && pdep == 0 && ((upper ? n - 1 - i : i) & 63) != 0) mbrk = 1;
         if (!code && dmin != 0x7fffffff) {  // histogram of floor(log2(nearest-dependency distance))
             const int bk = 31 - __clz(dmin);
             const unsigned same = __match_any_sync(__activemask(), bk);
@@ -108,7 +110,9 @@ __global__ void __launch_bounds__(256) k_validate(const int32_t *__restrict__ ro
         wdep += __shfl_xor_sync(0xffffffffu, wdep, off);
         pdep += __shfl_xor_sync(0xffffffffu, pdep, off);
         nrow += __shfl_xor_sync(0xffffffffu, nrow, off);
+        mbrk += __shfl_xor_sync(0xffffffffu, mbrk, off);
     }
+    if ((threadIdx.x & 31) == 0 && mbrk) atomicAdd(&out->mid_breaks, (int)mbrk);
     if ((threadIdx.x & 31) == 0 && len > 0) atomicMax(max_row, len);
     // both totals are < nnz < 2^31: near in the low word, wdep in the high word
     if ((threadIdx.x & 31) == 0 && (near | wdep))

@@ -205,4 +205,70 @@ __global__ void __launch_bounds__(CT, MINB) k_solve_lean(SolveParams p) {
     }
 }
 
+
+// ENGINE_LEANP: LEAN with PERSISTENT warps and a software pipeline.  The grid is
+// exactly what fits on the device at once (cooperative launch: every CTA is co-resident), CTA c
+// (its logical id from the start ticket) owns blocks c, c + G, c + 2G, ... of 256 logical rows, and
+// warp w of the CTA owns the 32-row slice w of each: a static round-robin that needs no work
+// tickets.  Each warp keeps three chunks in flight: the first-level loads (rowptr, b) of chunk k+2,
+// the second-level loads (L_ii, first two dependencies) of chunk k+1 and the solve of chunk k, so the
+// two dependent DRAM round trips of a chunk overlap the previous chunk's dependency waits instead of
+// adding to them.  Forward progress: the lowest unsolved row's chunk is the current chunk of its
+// warp (the warp's earlier chunks are lower, hence solved) and every warp is resident.
+template <int PROTO, int MINB, bool UPPER = false, bool UNIT = false>
+__global__ void __launch_bounds__(kLeanCta, MINB) k_solve_leanp(SolveParams p) {
+    constexpr int CT = kLeanCta;
+    __shared__ uint32_t s_blk, s_epoch;
+    const int tid = threadIdx.x;
+    const int lane = tid & 31, warp = tid >> 5;
+    const uint64_t pol = policy_evict_first();
+    if (tid == 0) cta_ticket(p, s_blk, s_epoch);
+    __syncthreads();
+    if (s_blk == kStaleBlk) return;
+    const uint32_t epoch = s_epoch;
+    const long long G = p.grid, c = s_blk;
+    const long long nblk = ((long long)p.n + CT - 1) / CT;
+    // logical row of this lane in its k-th chunk (>= n: past the end)
+    auto row_of = [&](long long k) -> long long { return (c + k * G) * CT + warp * 32 + lane; };
+    auto phys = [&](long long r) -> int { return UPPER ? p.n - 1 - (int)r : (int)r; };
+    auto first = [&](long long k, int &rs, int &re, double &bi) {
+        const long long r = row_of(k);
+        rs = 0, re = 1, bi = 0.0;
+        if (r < p.n) {
+            const int i = phys(r);
+            rs = ld_stream_i32(p.rowptr + i, pol);
+            re = ld_stream_i32(p.rowptr + i + 1, pol);
+        }
+        if (p.bflag) {  // sptrsv_solve_host's chunked b: lane 0 waits for the chunk(s) of the warp's rows
+            const long long r0 = row_of(k) - lane;
+            if (lane == 0 && r0 < p.n) {
+                const int a = (int)r0, e = (int)min((long long)p.n, r0 + 32);
+                wait_b_chunks(p, UPPER ? p.n - e : a, UPPER ? p.n - a : e);
+            }
+            __syncwarp();
+        }
+        if (r < p.n) bi = ld_b(p, phys(r), pol);
+    };
+    if (c >= nblk) return;
+    int rs1, re1, rs2, re2;
+    double bi0, bi1, bi2;
+    first(0, rs1, re1, bi0);
+    bool act0 = row_of(0) < p.n;
+    LeanRow lr0 = lean_load<UPPER, UNIT>(p, act0, rs1, re1, pol);
+    first(1, rs1, re1, bi1);
+    for (long long k = 0; c + k * G < nblk; ++k) {
+        const bool act1 = row_of(k + 1) < p.n;
+        const LeanRow lr1 = lean_load<UPPER, UNIT>(p, act1, rs1, re1, pol);  // chunk k+1: second level
+        first(k + 2, rs2, re2, bi2);                                           // chunk k+2: first level
+        const long long r0 = row_of(k);
+        lean_rows<PROTO, UPPER, UNIT>(p, r0 < p.n ? phys(r0) : 0, act0, lr0, bi0, epoch, lane, pol);
+        // sptrsv_solve_host: the warp's finished rows to pinned host memory (UVA), 256 contiguous bytes
+        if (p.x_host && act0) p.x_host[phys(r0)] = __ldcg(p.x + phys(r0));
+        lr0 = lr1;
+        act0 = act1;
+        bi0 = bi1;
+        rs1 = rs2, re1 = re2, bi1 = bi2;
+    }
+}
+
 }  // namespace sptrsv_dev

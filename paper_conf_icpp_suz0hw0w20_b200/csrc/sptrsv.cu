@@ -31,7 +31,7 @@ namespace {
 constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
 
 // engines (SPTRSV_OPT_ENGINE values, include/sptrsv.h)
-enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_SMALL = 8 };
+enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_SMALL = 8, ENG_LEANP = 9 };
 
 // ENGINE_SMALL (solve_small.cuh): the whole system in one CTA's shared memory.  Usable when it fits
 // (kSmallSmemMax bytes of dynamic shared memory, sm_100a allows 227 KB per CTA); AUTO picks it up to
@@ -108,6 +108,7 @@ struct sptrsv_handle_s {
     int64_t near_deps = 0;  // dependencies within 256 rows (analyse statistic for ENGINE_AUTO)
     int64_t warp_deps = 0;  // dependencies inside the row's own 32-row group (ditto)
     int64_t prev_deps = 0;  // dependencies on the previous row in solve order (ditto: chains)
+    int64_t mid_breaks = 0; // rows off a 64-row boundary without a previous-row dependency (ditto)
     int64_t near_rows = 0;  // rows whose nearest dependency is < 256 rows away (ditto)
     // options
     int mode = 0;
@@ -487,6 +488,7 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         h->near_deps = (int64_t)(o.near & 0xFFFFFFFFull);
         h->warp_deps = (int64_t)(o.near >> 32);
         h->prev_deps = (int64_t)(o.prev & 0xFFFFFFFFull);
+        h->mid_breaks = o.mid_breaks;
         h->near_rows = (int64_t)(o.prev >> 32);
         if (n > 0) adopt_plan(h, o);
         else h->plan = PLAN_THREAD;
@@ -518,6 +520,7 @@ struct Launch {
     int engine = 0;   // engine launched (ENG_*; 30 + v for the paper's Alg. v)
     int cta = 0;      // threads per CTA
     int K = 1;        // thread-level rows per lane
+    bool coop = false;  // cooperative launch (every CTA co-resident: LEANP's static work assignment)
 };
 
 // Size the device's persisting L2 set-aside for the handle's ready-word window (SPTRSV_OPT_L2_WINDOW):
@@ -570,7 +573,18 @@ bool small_fits(const sptrsv_handle_s *h) {
 int resolve_engine(const sptrsv_handle_s *h) {
     if (h->engine == ENG_SMALL && small_fits(h)) return ENG_SMALL;
     const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;  // unit handles store no diagonal
-    const bool chains = offdiag > 0 && 4 * h->prev_deps >= offdiag;
+    // chains: >= 1/4 of the dependencies on the previous row AND runs of such rows long enough for
+    // CHAIN's in-warp steps to pay (mean run n / (rows without one) >= 64 rows, one CHAIN warp): with
+    // short runs CHAIN serialises its warps through every run that crosses a warp boundary (c2i,
+    // runs of 10: 11.5 ms on CHAIN, 74 us on LEAN)
+    // ... and runs that CHAIN's warps can take whole: CHAIN solves a warp's 64 rows in row order, so a
+    // run starting inside a warp waits for the previous run's tail -- on grids whose side is not a
+    // multiple of 64 that serialises whole grid lines (1000^2 grid: 94 ms on CHAIN, 2.9 ms on
+    // ONE-SHOT; 500^2: 24.6 vs 0.84 ms on LEAN).  Mean run >= 2048 rows (1024^2 grid: LEANP 1.73 ms
+    // beats CHAIN's 2.33; 2048^2: CHAIN 5.1 ms, the rest >= 13 ms) and <= 1 run start per 4096 rows
+    // off a warp boundary.
+    const bool chains = offdiag > 0 && 4 * h->prev_deps >= offdiag &&
+                        2048 * ((int64_t)h->n - h->prev_deps) <= (int64_t)h->n && 4096 * h->mid_breaks <= (int64_t)h->n;
     const bool near = offdiag > 0 && 4 * h->near_rows >= (int64_t)h->n;
     // a pure chain: almost every row waits on its predecessor and little else (critical path ~ n rows;
     // CHAIN's in-register hop beats SMALL's shared-memory pass there: 1024-row chain 111 vs 200 us)
@@ -584,8 +598,8 @@ int resolve_engine(const sptrsv_handle_s *h) {
     if (h->plan != PLAN_THREAD)  // ONE-SHOT has no sub-warp rows
         return (h->engine == ENG_ONESHOT && !h->tri && h->n_sub_tasks == 0) ? ENG_ONESHOT : ENG_HYBRID;
     if (h->engine != ENG_AUTO) return (h->tri && h->engine == ENG_ONESHOT) ? ENG_LEAN : h->engine;
-    if (h->tri) return chains ? ENG_CHAIN : ENG_LEAN;
-    if (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n) return ENG_LEAN;
+    if (h->tri) return chains ? ENG_CHAIN : ENG_LEANP;
+    if (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n) return ENG_LEANP;
     return chains ? ENG_CHAIN : ENG_ONESHOT;
 }
 
@@ -727,6 +741,32 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
                  (int)L->grid.x * 7919;
         return SPTRSV_OK;
     }
+    if (L->engine == ENG_LEANP) {  // persistent pipelined LEAN (solve_lean.cuh), experimental
+#ifndef SPTRSV_LEANP_MINB
+#define SPTRSV_LEANP_MINB 3
+#endif
+        constexpr int MB = SPTRSV_LEANP_MINB;
+        static const lean_fn tab[4][2] = {
+            {k_solve_leanp<PROTO_FLAGS, MB>, k_solve_leanp<PROTO_FUSED, MB>},
+            {k_solve_leanp<PROTO_FLAGS, MB, true, false>, k_solve_leanp<PROTO_FUSED, MB, true, false>},
+            {k_solve_leanp<PROTO_FLAGS, MB, false, true>, k_solve_leanp<PROTO_FUSED, MB, false, true>},
+            {k_solve_leanp<PROTO_FLAGS, MB, true, true>, k_solve_leanp<PROTO_FUSED, MB, true, true>}};
+        L->fn = (const void *)tab[h->tri & 3][h->proto ? 1 : 0];
+        int per_sm = 0, sms = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, L->fn, kLeanCta, 0) != cudaSuccess ||
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device) != cudaSuccess || per_sm < 1) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_CUDA;
+        }
+        const long long nblk = ((long long)h->n + kLeanCta - 1) / kLeanCta;
+        const long long g = std::min<long long>(nblk, (long long)per_sm * sms);
+        L->cta = kLeanCta;
+        L->grid = dim3((unsigned)g);
+        L->block = dim3((unsigned)kLeanCta);
+        L->coop = true;
+        L->key = (9500000 + h->proto * 100000 + h->tri * 10) ^ (int)L->grid.x * 7919;
+        return SPTRSV_OK;
+    }
     if (L->engine == ENG_LEAN) {  // minimal one-shot kernel for all-thread-level plans (solve_lean.cuh)
         int ct = kLeanCta;
         if (h->tri) {
@@ -828,8 +868,13 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     cfg.blockDim = L.block;
     cfg.dynamicSmemBytes = L.smem;
     cfg.stream = s;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     cfg.numAttrs = 0;
+    if (L.coop) {
+        cudaLaunchAttribute &a = attr[cfg.numAttrs++];
+        a.id = cudaLaunchAttributeCooperative;
+        a.val.cooperative = 1;
+    }
     cfg.attrs = attr;
     // The ready words (FLAGS: flags, FUSED: records) in a persisting L2 window -- north_star's
     // "L2 access-policy window pinning the flags".  They are the handle's workspace, re-read by
@@ -1029,7 +1074,7 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
     if ((io & 1) && !write_value32()) io &= ~1;
     // engines that take the chunked b (wait_b_chunks) and, for LEAN / CHAIN, write x per CTA / warp
     const int eng = L0.engine;
-    const bool gated = eng == ENG_LEAN || eng == ENG_CHAIN || eng == ENG_HYBRID;
+    const bool gated = eng == ENG_LEAN || eng == ENG_LEANP || eng == ENG_CHAIN || eng == ENG_HYBRID;
     if (pinned && io && eng == ENG_SMALL) {
         // SMALL: the one CTA reads b straight from the mapped pinned buffer (one coalesced pass over
         // PCIe, no copy launch) and writes x to both x_stage and the mapped pinned x
@@ -1038,7 +1083,7 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         CK(cudaStreamSynchronize(s));
         return SPTRSV_OK;
     }
-    if (!(eng == ENG_LEAN || eng == ENG_CHAIN)) io &= ~2;
+    if (!(eng == ENG_LEAN || eng == ENG_LEANP || eng == ENG_CHAIN)) io &= ~2;
     if (pinned && io && gated) {
         const uint32_t *bflag = nullptr;
         uint32_t seq = 0;
@@ -1172,7 +1217,7 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
             if (value != ENG_ONESHOT && value != ENG_LEAN && value != ENG_AUTO && value != ENG_HYBRID &&
-                value != ENG_CHAIN && value != ENG_SMALL)
+                value != ENG_CHAIN && value != ENG_SMALL && value != ENG_LEANP)
                 return SPTRSV_ERR_INVALID_ARG;
             if (value == ENG_SMALL && !small_fits(h)) return SPTRSV_ERR_INVALID_ARG;  // does not fit one CTA
             h->engine = (int)value;

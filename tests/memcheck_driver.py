@@ -18,13 +18,13 @@ def run(s, flags=0, **opt):
 
 bases = [synth.gen_random_lower(1025, 4, seed=3), synth.gen_grid(40), synth.gen_chain(700), synth.gen_c2i(n=2000)]
 for s in bases:
-    for eng in (0, 3, 6, 7, 8):
+    for eng in (0, 3, 6, 7, 8, 9):
         for proto in (0, 1):
             run(s, engine=eng, protocol=proto)
     for flags in (1, 2, 3):
         s2 = synth.to_upper(s) if flags & 1 else s
         s2 = synth.to_unit(s2, upper=bool(flags & 1)) if flags & 2 else s2
-        for eng in (3, 7, 8):
+        for eng in (3, 7, 8, 9):
             run(s2, flags, engine=eng)
     run(s, engine=8, chain_div=2)  # SMALL's verified re-run
 print("memcheck_small ok")

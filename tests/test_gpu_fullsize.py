@@ -27,7 +27,7 @@ def _run(s, **opt):
         return x1, x.cpu().numpy(), h.info()
 
 
-@pytest.mark.parametrize("proto,engine", [(0, 0), (1, 0), (0, 3), (1, 3), (1, 5)])
+@pytest.mark.parametrize("proto,engine", [(0, 0), (1, 0), (0, 3), (1, 3), (0, 9), (1, 9), (1, 5)])
 def test_c2_full(proto, engine):
     s = synth.gen_c2()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
@@ -75,11 +75,11 @@ def test_chain_full_closed_form(proto):
 
 @pytest.mark.parametrize("proto", [0, 1])
 def test_c2_full_default_launch(proto):
-    """c2 in exactly the bench.py configuration: default options, AUTO -> LEAN."""
+    """c2 in exactly the bench.py configuration: default options, AUTO -> LEANP."""
     s = synth.gen_c2()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     x1, x2, info = _run(s, protocol=proto)
-    assert info["engine"] == 3
+    assert info["engine"] == 9
     assert np.array_equal(x1, ref) and np.array_equal(x2, ref)
 
 
@@ -115,7 +115,7 @@ def test_f4_forms_full(cfg, flags):
         h.check()
         info = h.info()
         got = x.cpu().numpy()
-    assert info["engine"] == {"c2": 3, "c3": 7, "c4": 6}[cfg], info
+    assert info["engine"] == {"c2": 9, "c3": 7, "c4": 6}[cfg], info
     if cfg == "c4":
         assert np.max(np.abs(got - ref) / np.abs(ref)) <= TOL
     else:

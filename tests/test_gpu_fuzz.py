@@ -63,7 +63,7 @@ def random_structure(rng):
 
 ENGINES = [(5, {}), (0, {}), (3, {}), (6, {}), (7, {}),
            (0, {"cta_threads": 1024}), (7, {"rows_per_lane": 1, "cta_threads": 64}), (3, {"cta_threads": 128}),
-           (7, {"cta_threads": 512}), (3, {"cta_threads": 1024}), (8, {}), (8, {"cta_threads": 64})]
+           (7, {"cta_threads": 512}), (3, {"cta_threads": 1024}), (8, {}), (8, {"cta_threads": 64}), (9, {})]
 
 
 def small_fits(s):
@@ -117,7 +117,7 @@ def test_fuzz_triangular_forms_vs_oracle(seed):
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     d = torch.device("cuda:0")
     rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
-    for opts in ({}, {"engine": 3, "mode": 1}, {"engine": 7, "mode": 1}, {"engine": 8}):
+    for opts in ({}, {"engine": 3, "mode": 1}, {"engine": 7, "mode": 1}, {"engine": 8}, {"engine": 9, "mode": 1}):
         proto = int(rng.integers(0, 2))
         if opts.get("engine") == 8 and (s.n == 0 or not small_fits(s)):
             continue

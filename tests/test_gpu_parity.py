@@ -48,7 +48,7 @@ def relerr(a, ref):
 
 MODES = [0, 1, 2]
 PROTOS = [0, 1]  # 0 FLAGS (release/acquire), 1 FUSED (epoch-tagged value records)
-ENGINES = [0, 3]  # 0 one-shot k_solve (staged, in-CTA x copy), 3 LEAN
+ENGINES = [0, 3, 9]  # 0 one-shot k_solve (staged, in-CTA x copy), 3 LEAN, 9 LEANP (persistent, pipelined)
 
 
 # ------------------------------------------------------------------ small, many tiles + ragged tails
@@ -309,7 +309,10 @@ def test_solve_host_e2e_chain_hybrid(cap, proto, host_io, case):
         s = synth.to_unit(s)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags) if flags else oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     rp, ci, v, _ = dev_csr(s)
-    with cap.analyse(rp, ci, v, protocol=proto, host_io=host_io, upper=bool(flags & 1), unit_diag=bool(flags & 2)) as h:
+    # (CHAIN forced on the grids: AUTO keeps a 600^2 grid, whose lines do not align with CHAIN's warps, off it)
+    extra = {"engine": 7} if "grid" in case else {}
+    with cap.analyse(rp, ci, v, protocol=proto, host_io=host_io, upper=bool(flags & 1), unit_diag=bool(flags & 2),
+                     **extra) as h:
         eng = h.info()["engine"]
         assert eng == (7 if "grid" in case else 6), (case, eng)
         bh = torch.from_numpy(s.b).pin_memory()
@@ -336,7 +339,7 @@ def test_solve_host_e2e_f4_lean(cap, flags, host_io):
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     rp, ci, v, _ = dev_csr(s)
     with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2), host_io=host_io) as h:
-        assert h.info()["engine"] == 3
+        assert h.info()["engine"] == 9  # LEANP: far dependencies
         bh = torch.from_numpy(s.b).pin_memory()
         xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
         for _ in range(2):
@@ -493,11 +496,13 @@ def test_chain_engine_division_guard_exits(cap, proto, K, eng):
 
 def test_engine_auto_choice(cap):
     """ENGINE_AUTO: small near-dependency systems that fit one CTA and are not pure chains (c1, a 32x32
-    grid) -> SMALL (8); far dependencies -> LEAN (3); chains / grid wavefronts (>= 1/4 of the
-    dependencies on the previous row) -> CHAIN (7); other near-dependency plans (small levels) ->
-    staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""
-    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 3, 256, 1), (lambda: synth.gen_grid(100), 7, 128, 2),
-                              (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 3, 256, 1),
+    grid) -> SMALL (8); far dependencies -> LEANP (9); long, warp-aligned runs of previous-row
+    dependencies (chains; grids whose side is a multiple of 64 and >= 2048) -> CHAIN (7); other
+    near-dependency plans (small levels, unaligned grids) -> staged one-shot (0); plans with
+    warp-level rows -> HYBRID (6)."""
+    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 9, 256, 1), (lambda: synth.gen_grid(100), 0, 1024, 1),
+                              (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 9, 256, 1),
+                              (lambda: synth.gen_c2i(n=100_000), 0, 256, 1),
                               (lambda: synth.gen_c1(), 8, 256, 1), (lambda: synth.gen_grid(32), 8, 256, 1),
                               (lambda: synth.gen_c4(n=5000, nlevels=50), 6, 64, 1),
                               (lambda: synth.gen_leveled(20_000, 1000, 1, 3, 77, "lev_small"), 0, 1024, 1)):
@@ -612,7 +617,7 @@ def test_multi_rhs_chain_plans_by_column(cap, nrhs):
         B = rng.uniform(-1, 1, (s.n, nrhs))
         ref = oracle.solve_multi(s.rowptr, s.colidx, s.val, B)
         rp, ci, v, _ = dev_csr(s)
-        with cap.analyse(rp, ci, v) as h:
+        with cap.analyse(rp, ci, v, engine=7) as h:  # (AUTO keeps a 300^2 grid off CHAIN: 300 % 64 != 0)
             assert h.info()["engine"] == 7
             X = h.solve_multi(torch.from_numpy(B).cuda())
             h.check()

@@ -147,7 +147,7 @@ def test_small_auto_choice(cap):
     above 4096 rows on the multi-CTA engines.  Forcing SMALL on a system that does not fit fails."""
     for gen, want in ((synth.gen_c1, SMALL), (lambda: synth.gen_grid(32), SMALL),
                       (lambda: synth.gen_random_lower(600, 20, seed=3), SMALL),
-                      (lambda: synth.gen_chain(3000), 7), (lambda: synth.gen_diag(4000), 3),
+                      (lambda: synth.gen_chain(3000), 7), (lambda: synth.gen_diag(4000), 9),
                       (lambda: synth.gen_random_lower(5000, 3, seed=4), None),
                       (lambda: synth.gen_random_lower(4000, 6, seed=4), None)):
         s = gen()

@@ -68,10 +68,10 @@ def test_tri_random_sizes_bit_exact(cap, n, gen, flags, proto):
     s = form(GENS[gen](n), flags)
     ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
     x, info = gpu_solve(cap, s, flags, protocol=proto, mode=1)  # thread level: bit-exact
-    # LEAN, CHAIN when >= 1/4 of the dependencies are on the previous row, SMALL for small near-dependency systems
-    assert info["engine"] in (3, 7, 8)
+    # LEANP, CHAIN for long aligned previous-row runs, SMALL for small near-dependency systems
+    assert info["engine"] in (7, 8, 9)
     assert np.array_equal(x, ref)
-    for engine in (3, 7, 8):  # the thread-level engines, forced (SMALL where the system fits one CTA)
+    for engine in (3, 7, 8, 9):  # the thread-level engines, forced (SMALL where the system fits one CTA)
         if engine == 8 and (s.n > 4096 or 24 * s.n + 12 * int(s.rowptr[-1]) > 220 * 1024):
             continue
         x, info = gpu_solve(cap, s, flags, protocol=proto, engine=engine, mode=1)
@@ -310,14 +310,15 @@ def test_tri_chain_engine_bit_exact(cap, which, flags, proto, K, cta):
 
 @pytest.mark.parametrize("flags", FORMS)
 def test_tri_chain_auto_choice_and_closed_forms(cap, flags):
-    """AUTO sends f4 grids and chains to CHAIN; the f4 bidiagonal closed forms stay exact."""
+    """AUTO sends f4 chains to CHAIN (a 200^2 grid, whose lines do not align with CHAIN's 64-row
+    warps, to LEANP); the f4 bidiagonal closed forms stay exact."""
     s = form(synth.gen_grid(200), flags)
     x, info = gpu_solve(cap, s, flags)
-    assert info["engine"] == 7, info
+    assert info["engine"] == 9, info
     assert np.array_equal(x, oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags))
     s = form(synth.gen_c2(n=100_000), flags)
     _, info = gpu_solve(cap, s, flags)
-    assert info["engine"] == 3, info  # far dependencies stay on LEAN
+    assert info["engine"] == 9, info  # far dependencies: LEANP
     n = 100_000  # upper bidiagonal U_ii = 2, U_{i,i+1} = -1, b = 1 (as test_upper_bidiagonal_closed_form)
     rp = np.r_[np.arange(0, 2 * n, 2), 2 * n - 1].astype(np.int32)
     ci = np.empty(2 * n - 1, np.int32)

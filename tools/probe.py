@@ -61,7 +61,7 @@ def main():
             t = float(np.median(ts))
             inf = h.info()
             print(json.dumps({"sys": spec, "opts": opts, "n": s.n, "nnz": s.nnz, "t_us": round(t * 1e6, 2),
-                              "mean_us": round(float(np.mean(ts)) * 1e6, 2), "gflops": round(2 * s.nnz / t / 1e9, 2),
+                              "mean_us": round(float(np.mean(ts)) * 1e6, 2), "p90_us": round(float(np.percentile(ts, 90)) * 1e6, 2), "gflops": round(2 * s.nnz / t / 1e9, 2),
                               "engine": inf["engine"], "cta": inf["cta_threads"], "K": inf["rows_per_lane"],
                               "err": err}), flush=True)
             h.close()
