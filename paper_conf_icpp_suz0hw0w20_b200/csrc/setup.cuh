@@ -240,7 +240,11 @@ __global__ void __launch_bounds__(1024) k_plan_write(const int32_t *__restrict__
 //   64 .. 511            threshold 2, warp rows (Alg.3)
 //   512 .. 1023          threshold 2, sub-warp rows, epl 4   (c4: 16 lanes per 64-entry row)
 //   1024 .. 8191         threshold 2, sub-warp rows, epl 2
-//   >= 8192              threshold 3, sub-warp rows, epl 8   (c2 / c5 at 2.8 nnz/row stay thread)
+//   8192 .. 65535        threshold 3, sub-warp rows, epl 8
+//   >= 65536             threshold 7, sub-warp rows, epl 8   (c2 / c5 at 2.8 nnz/row stay thread; at
+//                        n = 1e6 with 10 levels the persistent thread engine LEANP beats sub-warp rows
+//                        up to ~7 nnz/row: 4 nnz/row 41 vs 72 us, 6 nnz/row 56 vs 72 us --
+//                        profiles/r02_auto/lev_1m_sweep.txt)
 //   n <= 1024            thread level only (one 1024-thread one-shot CTA resolves it in smem)
 // user >= 0 / user_epl >= 0: SPTRSV_OPT_WARP_THRESHOLD / SPTRSV_OPT_SUBWARP were set.  One thread.
 __global__ void k_auto_threshold(AnalyseOut *out, int32_t n, int32_t user, int32_t user_epl) {
@@ -263,7 +267,8 @@ __global__ void k_auto_threshold(AnalyseOut *out, int32_t n, int32_t user, int32
     else if (med <= 8) t = 2, e = 0;
     else if (med <= 9) t = 2, e = 4;
     else if (med <= 12) t = 2, e = 2;
-    else t = 3, e = 8;
+    else if (med <= 15) t = 3, e = 8;
+    else t = 7, e = 8;  // >= 65536 rows: very wide levels, thread rows (LEANP) win up to ~7 nnz/row
     out->threshold = user >= 0 ? user : t;
     out->epl = user_epl >= 0 ? user_epl : e;
 }
