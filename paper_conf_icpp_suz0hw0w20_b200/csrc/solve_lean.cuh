@@ -60,7 +60,7 @@ __device__ __forceinline__ LeanRow lean_load(const SolveParams &p, bool act, int
 // published, or on abort.  Shared by k_solve_lean and the f4 list kernel (solve_tri.cuh).
 template <int PROTO, bool UPPER, bool UNIT>
 __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, const LeanRow &lr, double bi,
-                                          uint32_t epoch, int lane, uint64_t pol) {
+                                          uint32_t epoch, int lane, uint64_t pol, double *xout = nullptr) {
     const int lo = lr.lo, hi = lr.hi;
     constexpr int dir = UPPER ? -1 : 1;
     auto inr = [&](int k) { return UPPER ? k >= lo : k < hi; };
@@ -91,7 +91,9 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, const
         bool prog = false;
         if (!done) {
             if (nc < 0) {  // reached the diagonal (Alg.5 l.12-16)
-                publish<PROTO>(p, nocta, i, UNIT ? __dsub_rn(bi, ls) : dg.div(__dsub_rn(bi, ls)), epoch);
+                const double xi = UNIT ? __dsub_rn(bi, ls) : dg.div(__dsub_rn(bi, ls));
+                publish<PROTO>(p, nocta, i, xi, epoch);
+                if (xout) *xout = xi;
                 done = true;
                 prog = true;
             } else {
@@ -110,7 +112,9 @@ __device__ __forceinline__ void lean_rows(SolveParams &p, int i, bool act, const
                         advance();
                     }
                     if (nc < 0) {
-                        publish<PROTO>(p, nocta, i, UNIT ? __dsub_rn(bi, ls) : dg.div(__dsub_rn(bi, ls)), epoch);
+                        const double xi = UNIT ? __dsub_rn(bi, ls) : dg.div(__dsub_rn(bi, ls));
+                publish<PROTO>(p, nocta, i, xi, epoch);
+                if (xout) *xout = xi;
                         done = true;
                     }
                 }
@@ -239,14 +243,17 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_leanp(SolveParams p) {
             rs = ld_stream_i32(p.rowptr + i, pol);
             re = ld_stream_i32(p.rowptr + i + 1, pol);
         }
-        if (p.bflag) {  // sptrsv_solve_host's chunked b: lane 0 waits for the chunk(s) of the warp's rows
-            const long long r0 = row_of(k) - lane;
-            if (lane == 0 && r0 < p.n) {
-                const int a = (int)r0, e = (int)min((long long)p.n, r0 + 32);
-                wait_b_chunks(p, UPPER ? p.n - e : a, UPPER ? p.n - a : e);
-            }
-            __syncwarp();
+        // (with sptrsv_solve_host's chunked b, b is loaded just before the chunk's solve instead: a
+        // prefetch would wait for b two chunks ahead of the solve)
+        if (r < p.n && !p.bflag) bi = ld_b(p, phys(r), pol);
+    };
+    auto gated_b = [&](long long k, double &bi) {  // lane 0 waits for the chunk(s) of the warp's rows
+        const long long r = row_of(k), r0 = r - lane;
+        if (lane == 0 && r0 < p.n) {
+            const int a = (int)r0, e = (int)min((long long)p.n, r0 + 32);
+            wait_b_chunks(p, UPPER ? p.n - e : a, UPPER ? p.n - a : e);
         }
+        __syncwarp();
         if (r < p.n) bi = ld_b(p, phys(r), pol);
     };
     if (c >= nblk) return;
@@ -261,9 +268,12 @@ __global__ void __launch_bounds__(kLeanCta, MINB) k_solve_leanp(SolveParams p) {
         const LeanRow lr1 = lean_load<UPPER, UNIT>(p, act1, rs1, re1, pol);  // chunk k+1: second level
         first(k + 2, rs2, re2, bi2);                                           // chunk k+2: first level
         const long long r0 = row_of(k);
-        lean_rows<PROTO, UPPER, UNIT>(p, r0 < p.n ? phys(r0) : 0, act0, lr0, bi0, epoch, lane, pol);
-        // sptrsv_solve_host: the warp's finished rows to pinned host memory (UVA), 256 contiguous bytes
-        if (p.x_host && act0) p.x_host[phys(r0)] = __ldcg(p.x + phys(r0));
+        if (p.bflag) gated_b(k, bi0);
+        double xi = 0.0;
+        lean_rows<PROTO, UPPER, UNIT>(p, r0 < p.n ? phys(r0) : 0, act0, lr0, bi0, epoch, lane, pol, &xi);
+        // sptrsv_solve_host: the warp's finished rows to pinned host memory (UVA), 256 contiguous bytes,
+        // from the registers (no read-back of x on the pipeline)
+        if (p.x_host && act0) p.x_host[phys(r0)] = xi;
         lr0 = lr1;
         act0 = act1;
         bi0 = bi1;

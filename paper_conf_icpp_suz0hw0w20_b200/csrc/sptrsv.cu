@@ -57,6 +57,12 @@ struct Workspace {
     uint32_t *lvl = nullptr;       // n (levels diagnostic, lazy)
     double *b_stage = nullptr;     // n (solve_host, lazy)
     SolveState *mst = nullptr;     // multi-RHS: own solve state (own epoch sequence)
+    // sptrsv_solve_host on a LEANP handle runs the LEAN kernel (its per-CTA b gating and x write-back
+    // overlap the PCIe copies better: c2 e2e 270 vs 305 us) on its OWN ready words and epoch sequence,
+    // so host and device solves interleave without re-zeroing each other's state (lazy)
+    SolveState *hst = nullptr;
+    unsigned long long *hrec = nullptr;  // 2n
+    uint32_t *hflags = nullptr;          // n
     uint32_t *mflags = nullptr;    // multi-RHS: n * mcap flags (FLAGS)
     unsigned long long *mrec = nullptr;  // multi-RHS: n * mcap records (FUSED)
     int64_t mcap = 0;              // right-hand sides the multi buffers hold
@@ -142,6 +148,8 @@ struct sptrsv_handle_s {
     long long mlaunch_key = -1;  // same for sptrsv_solve_multi
     uint32_t msince_reset = 0;
     uint32_t gen = 0, mgen = 0;  // configuration generations of the solve / multi-RHS state (cta_ticket)
+    uint32_t hgen = 0, hsince_reset = 0;  // the host-path state (Workspace::hst)
+    int hlaunch_key = -1;
     unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
@@ -271,6 +279,9 @@ void free_ws(Workspace &w) {
     cudaFree(w.lvl);
     cudaFree(w.b_stage);
     cudaFree(w.mst);
+    cudaFree(w.hst);
+    cudaFree(w.hrec);
+    cudaFree(w.hflags);
     cudaFree(w.mflags);
     cudaFree(w.mrec);
     cudaFree(w.x_stage);
@@ -347,15 +358,6 @@ int init_state(SolveState *st, uint32_t gen, cudaStream_t s) {
     return SPTRSV_OK;
 }
 
-int reset_state(sptrsv_handle_s *h, cudaStream_t s) {
-    // flags / records := 0 (no epoch matches), counters := 0 under a new generation; the next
-    // solve has epoch 1
-    CK(cudaMemsetAsync(h->ws.flags, 0, sizeof(uint32_t) * (size_t)(h->n > 0 ? h->n : 1), s));
-    CK(cudaMemsetAsync(h->ws.rec, 0, 16 * (size_t)(h->n > 0 ? h->n : 1), s));
-    h->gen = (h->gen + 1) & 0xFFFFFFu;
-    h->since_reset = 0;
-    return init_state(h->ws.st, h->gen, s);
-}
 
 // a reset is due before the next launch: new configuration, epoch about to wrap, or the 40-bit
 // ticket count of this generation about to overflow
@@ -803,7 +805,8 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
 }  // namespace
 
 static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream,
-                      const uint32_t *bflag = nullptr, uint32_t bseq = 0, int bshift = kBChunkShift);
+                      const uint32_t *bflag = nullptr, uint32_t bseq = 0, int bshift = kBChunkShift,
+                      bool host_state = false);
 
 int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t stream) {
     return solve_impl(h, b, x, nullptr, stream);
@@ -811,7 +814,7 @@ int sptrsv_solve(sptrsv_handle_t h, const double *b, double *x, sptrsv_stream_t 
 
 // x_host (LEAN only, from sptrsv_solve_host): device-mapped pinned host copy target of x
 static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_host, sptrsv_stream_t stream,
-                      const uint32_t *bflag, uint32_t bseq, int bshift) {
+                      const uint32_t *bflag, uint32_t bseq, int bshift, bool host_state) {
     if (!h) return SPTRSV_ERR_INVALID_ARG;
     if (h->n == 0) return SPTRSV_OK;
     if (!b || !x || b == x) return SPTRSV_ERR_INVALID_ARG;
@@ -824,13 +827,48 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     Launch L;
     int rc = plan_launch(h, &L);
     if (rc) return rc;
+    // host_state (sptrsv_solve_host on a LEANP plan): the LEAN kernel on the host-path state set
+    host_state = host_state && L.engine == ENG_LEANP;
+    if (host_state) {
+        const int saved = h->engine;
+        h->engine = ENG_LEAN;
+        L = Launch();
+        rc = plan_launch(h, &L);
+        h->engine = saved;
+        if (rc) return rc;
+        Workspace &w = h->ws;
+        if (!w.hst) {
+            const size_t nn = (size_t)(h->n > 0 ? h->n : 1);
+            if (cudaMalloc(&w.hst, sizeof(SolveState)) != cudaSuccess || cudaMalloc(&w.hrec, 16 * nn) != cudaSuccess ||
+                cudaMalloc(&w.hflags, 4 * nn) != cudaSuccess) {
+                (void)cudaGetLastError();
+                cudaFree(w.hst);
+                cudaFree(w.hrec);
+                cudaFree(w.hflags);
+                w.hst = nullptr, w.hrec = nullptr, w.hflags = nullptr;
+                return SPTRSV_ERR_ALLOC;
+            }
+            h->hlaunch_key = -1;
+        }
+    }
+    SolveState *st = host_state ? h->ws.hst : h->ws.st;
+    unsigned long long *rec = host_state ? h->ws.hrec : h->ws.rec;
+    uint32_t *flags = host_state ? h->ws.hflags : h->ws.flags;
+    int &launch_key = host_state ? h->hlaunch_key : h->launch_key;
+    uint32_t &since_reset = host_state ? h->hsince_reset : h->since_reset;
+    uint32_t &gen = host_state ? h->hgen : h->gen;
     // The epoch of a solve is derived on the device from the start ticket and the
     // grid size (solve.cuh SolveState); a new launch configuration, or an epoch
     // about to wrap, re-zeroes the flags / records and the counters first.
-    if (L.key != h->launch_key || reset_due(h->since_reset, L.grid.x)) {
-        rc = reset_state(h, s);
+    if (L.key != launch_key || reset_due(since_reset, L.grid.x)) {
+        const size_t nn = (size_t)(h->n > 0 ? h->n : 1);
+        CK(cudaMemsetAsync(flags, 0, sizeof(uint32_t) * nn, s));
+        CK(cudaMemsetAsync(rec, 0, 16 * nn, s));
+        gen = (gen + 1) & 0xFFFFFFu;
+        since_reset = 0;
+        rc = init_state(st, gen, s);
         if (rc) return rc;
-        h->launch_key = L.key;
+        launch_key = L.key;
     }
     SolveParams p{};
     p.rowptr = h->rowptr;
@@ -838,16 +876,16 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.val = h->val;
     p.b = b;
     p.x = x;
-    p.flags = h->ws.flags;
-    p.rec = h->ws.rec;
+    p.flags = flags;
+    p.rec = rec;
     p.tasks = h->ws.tasks;
     p.task_w = h->ws.task_w;
-    p.st = h->ws.st;
+    p.st = st;
     p.nnz = h->nnz;
     p.n = h->n;
     p.n_tasks = h->n_tasks;
     p.epoch0 = 1;
-    p.gen = h->gen;
+    p.gen = gen;
     p.grid = L.grid.x;
     p.backoff_min = h->backoff_min;
     p.backoff_max = h->backoff_max;
@@ -883,7 +921,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     // polls of not-yet-published dependencies and the publishes hit L2 (c2 41.0 -> 32.8 us).
     // The device's persisting set-aside is grown to the window (size_l2_window, at analyse time and
     // on option changes -- never inside a stream capture); a window it cannot hold whole is not used.
-    void *wbase = h->proto == PROTO_FLAGS ? (void *)h->ws.flags : (void *)h->ws.rec;
+    void *wbase = host_state ? nullptr : h->proto == PROTO_FLAGS ? (void *)h->ws.flags : (void *)h->ws.rec;
     const size_t wbytes = (h->proto == PROTO_FLAGS ? sizeof(uint32_t) : 16) * (size_t)h->n;
     if (h->l2_window && wbase && h->l2_hit == 0.f) size_l2_window(h);  // normally done at analyse / set_option
     if (h->l2_window && wbase && h->l2_hit > 0.f) {
@@ -901,7 +939,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
         return SPTRSV_ERR_CUDA;
     }
     h->solves++;
-    h->since_reset++;
+    since_reset++;
     return SPTRSV_OK;
 }
 
@@ -1125,7 +1163,7 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
             CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
         }
         int rc = solve_impl(h, h->ws.b_stage, h->ws.x_stage, (io & 2) ? (double *)ax.devicePointer : nullptr, stream,
-                            bflag, seq, sh);
+                            bflag, seq, sh, /*host_state=*/true);
         if (rc) return rc;
         if (io & 1) {  // the stream also orders after the copies (they finish before the solve does)
             CK(cudaEventRecord(h->ws.ev_b, h->ws.s2));
@@ -1371,6 +1409,13 @@ int sptrsv_check(sptrsv_handle_t h, sptrsv_stream_t stream) {
         if (merr) {
             CK(cudaMemset(h->ws.mst, 0, sizeof(SolveState)));
             h->mlaunch_key = -1;
+        }
+    }
+    if (h->ws.hst && !merr) {  // the host-path state of a LEANP handle (its own epoch sequence)
+        CK(cudaMemcpy(&merr, &h->ws.hst->error.v, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+        if (merr) {
+            CK(cudaMemset(h->ws.hst, 0, sizeof(SolveState)));
+            h->hlaunch_key = -1;
         }
     }
     if (err) {

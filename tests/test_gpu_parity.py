@@ -780,3 +780,34 @@ def test_chain_division_proof_modes(cap, proto):
             h.solve(b, x)
             h.check()
             assert np.array_equal(x.cpu().numpy(), ref), s.name
+
+
+def test_leanp_host_path_interleaves_with_graph_replays(cap):
+    """A LEANP handle's sptrsv_solve_host runs the LEAN kernel on its own ready words and epoch sequence
+    (sptrsv.cu Workspace::hst): device solves -- here a captured CUDA graph -- and host solves interleave
+    on one handle, every result bit-exact, no stale-launch report and no re-zeroing between them."""
+    s = synth.gen_c2(n=300_000)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev_csr(s)
+    with cap.analyse(rp, ci, v) as h:
+        assert h.info()["engine"] == 9
+        st = torch.cuda.Stream()
+        x = torch.empty_like(b)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(st):
+            h.solve(b, x, stream=st)
+            st.synchronize()
+            with torch.cuda.graph(g, stream=st):
+                h.solve(b, x, stream=st)
+        bh = torch.from_numpy(s.b).pin_memory()
+        xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
+        for _ in range(3):
+            x.fill_(float("nan"))
+            g.replay()
+            torch.cuda.synchronize()
+            h.check(st)
+            assert np.array_equal(x.cpu().numpy(), ref)
+            xh.fill_(float("nan"))
+            h.solve_host(bh, xh)
+            h.check()
+            assert np.array_equal(xh.numpy(), ref)
