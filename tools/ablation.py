@@ -36,7 +36,8 @@ def delta_table6(n_level, nnz_row):
 VARIANTS = {"alg3": dict(variant=3), "alg4": dict(variant=4), "alg5": dict(variant=5),
             "thread": dict(mode=1, engine=0), "warp": dict(mode=2, engine=0), "auto": dict()}
 if os.environ.get("ABLATION_SET") == "f2":  # thread / sub-warp widths / warp, and AUTO variants
-    VARIANTS = {"thread": dict(mode=1), "lean": dict(mode=1, engine=3), "warp": dict(mode=2),
+    VARIANTS = {"thread": dict(mode=1), "lean": dict(mode=1, engine=3), "leanp": dict(mode=1, engine=9),
+                "warp": dict(mode=2),
                 "sub_e1": dict(mode=3, subwarp=1), "sub_e2": dict(mode=3, subwarp=2), "sub_e4": dict(mode=3, subwarp=4),
                 "sub_e8": dict(mode=3, subwarp=8), "auto": dict(), "auto_e2": dict(subwarp=2),
                 "auto_e4": dict(subwarp=4), "auto_e8": dict(subwarp=8)}
@@ -62,7 +63,8 @@ def timeit(h, b, x, reps=5, limit_s=20.0):
 
 
 rows = []
-for levels in (10, 100, 1000, 10000):
+LEVELS = [int(v) for v in os.environ.get("ABLATION_LEVELS", "10,100,1000,10000").split(",")]
+for levels in LEVELS:
     W = n // levels
     for deps in (2, 4, 8, 16, 32, 64):
         if deps - 1 >= W:
