@@ -761,6 +761,9 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
             return SPTRSV_ERR_CUDA;
         }
         const long long nblk = ((long long)h->n + kLeanCta - 1) / kLeanCta;
+#ifdef SPTRSV_MEASURE_LEANP_PER_SM  // measurement builds only: fewer resident CTAs than fit
+        per_sm = std::min(per_sm, SPTRSV_MEASURE_LEANP_PER_SM);
+#endif
         const long long g = std::min<long long>(nblk, (long long)per_sm * sms);
         L->cta = kLeanCta;
         L->grid = dim3((unsigned)g);
