@@ -71,6 +71,7 @@ struct Workspace {
     int32_t bflag_n = 0;
     cudaStream_t s2 = nullptr;     // solve_host: copy stream for the chunked b
     cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+    cudaEvent_t ev_done = nullptr;  // solve_host: completion (spin_sync)
 };
 
 // cuStreamWriteValue32 through the runtime's driver entry point (no link-time libcuda
@@ -90,6 +91,20 @@ write_value32_fn write_value32() {
     return fn;
 }
 constexpr int kBChunkShift = 16;  // solve_host: smallest b chunk, 2^16 rows (512 KB)
+
+// sptrsv_solve_host's completion wait: an event on the stream polled by the calling thread (a
+// blocking cudaStreamSynchronize may yield the thread and add its wake-up to every end-to-end step)
+int spin_sync(cudaStream_t s, cudaEvent_t &ev) {
+    if (!ev && cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return cudaStreamSynchronize(s) == cudaSuccess ? 0 : -1;
+    }
+    if (cudaEventRecord(ev, s) != cudaSuccess) return -1;
+    cudaError_t e;
+    while ((e = cudaEventQuery(ev)) == cudaErrorNotReady) {
+    }
+    return e == cudaSuccess ? 0 : -1;
+}
 
 }  // namespace
 
@@ -289,6 +304,7 @@ void free_ws(Workspace &w) {
     if (w.s2) cudaStreamDestroy(w.s2);
     if (w.ev_a) cudaEventDestroy(w.ev_a);
     if (w.ev_b) cudaEventDestroy(w.ev_b);
+    if (w.ev_done) cudaEventDestroy(w.ev_done);
     w = Workspace();
 }
 
@@ -1121,7 +1137,7 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
         // PCIe, no copy launch) and writes x to both x_stage and the mapped pinned x
         int rc = solve_impl(h, (const double *)ab.devicePointer, h->ws.x_stage, (double *)ax.devicePointer, stream);
         if (rc) return rc;
-        CK(cudaStreamSynchronize(s));
+        if (spin_sync(s, h->ws.ev_done)) return SPTRSV_ERR_CUDA;
         return SPTRSV_OK;
     }
     if (!(eng == ENG_LEAN || eng == ENG_LEANP || eng == ENG_CHAIN)) io &= ~2;
@@ -1173,14 +1189,14 @@ int sptrsv_solve_host(sptrsv_handle_t h, const double *b_host, double *x_host, s
             CK(cudaStreamWaitEvent(s, h->ws.ev_b, 0));
         }
         if (!(io & 2)) CK(cudaMemcpyAsync(x_host, h->ws.x_stage, bytes, cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
+        if (spin_sync(s, h->ws.ev_done)) return SPTRSV_ERR_CUDA;
         return SPTRSV_OK;
     }
     CK(cudaMemcpyAsync(h->ws.b_stage, b_host, bytes, cudaMemcpyHostToDevice, s));
     int rc = sptrsv_solve(h, h->ws.b_stage, h->ws.x_stage, stream);
     if (rc) return rc;
     CK(cudaMemcpyAsync(x_host, h->ws.x_stage, bytes, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
+    if (spin_sync(s, h->ws.ev_done)) return SPTRSV_ERR_CUDA;
     return SPTRSV_OK;
 }
 
