@@ -299,7 +299,8 @@ int sptrsv_solve_multi(sptrsv_handle_t h, const double *B, double *X, int32_t nr
 
 /*
  * sptrsv_solve_host -- end-to-end convenience from host buffers; synchronises
- * `stream` before returning.  b_host/x_host: host double[n].
+ * `stream` before returning (the calling thread polls an event: it spins for
+ * the duration of the solve rather than sleeping in a blocking sync).  b_host/x_host: host double[n].
  *   - Both pinned (page-locked, UVA-mapped; e.g. cudaHostAlloc or torch
  *     pin_memory) and the handle runs LEAN or LEANP: b is copied to device staging in
  *     about four chunks on a handle-owned second stream, each CTA of the solve
