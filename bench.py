@@ -587,7 +587,28 @@ def run_single(args):
                               "engine": ENGINES.get(batch.handles[0].info()["engine"]),
                               "timing": "one step = the 8 solves back to back on one stream (CUDA events)"}
         batch.close()
-        del c5, fl
+        # the same 8 systems as block-diagonal BATCH handles (sptrsv_analyse_csr_batch): one launch per
+        # group of g systems -- 8 x 1 (= the leg above, through one handle each), 4 x 2, 1 x 8
+        stream = torch.cuda.current_stream()
+        grouped = {}
+        dsys = [tuple(torch.from_numpy(a).to(dev) for a in (t.rowptr, t.colidx, t.val)) for t in c5]
+        for g in (2, 8):
+            hs = [cap.analyse_batch(dsys[k:k + g], **opts) for k in range(0, 8, g)]
+            bs = [torch.from_numpy(np.concatenate([t.b for t in c5[k:k + g]])).to(dev) for k in range(0, 8, g)]
+            xs = [torch.empty_like(b) for b in bs]
+            ms = time_steps(torch, lambda: [h.solve(b, x, stream=stream) for h, b, x in zip(hs, bs, xs)], stream,
+                            fl, args.steps, args.warmup)
+            for h in hs:
+                h.check(stream)
+            mg = float(ms.mean()) * 1e-3
+            grouped[f"{g}_per_launch"] = {"launches": len(hs), "value": round(2.0 * sum(t.nnz for t in c5) / mg / 1e9, 3),
+                                          "ms_per_step": round(mg * 1e3, 5),
+                                          "engine": ENGINES.get(hs[0].info()["engine"])}
+            for h in hs:
+                h.close()
+            del hs, bs, xs
+        configs["c5batch"]["one_launch_groups"] = grouped
+        del c5, fl, dsys
         torch.cuda.empty_cache()
 
     # ---- roofline of the headline kernel (mean step), latency bound, ncu-measured DRAM traffic

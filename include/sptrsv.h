@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define SPTRSV_ABI_VERSION 3
+#define SPTRSV_ABI_VERSION 4
 
 typedef struct sptrsv_handle_s *sptrsv_handle_t;
 typedef void *sptrsv_stream_t; /* cudaStream_t */
@@ -264,10 +264,36 @@ int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx,
  * sptrsv_levels and VARIANT != 0 return SPTRSV_ERR_INVALID_ARG.  Thread-level rows are bit-exact with that fp64
  * substitution (one rounded multiply and add each); warp rows are within the
  * warp-mode bound, as for lower handles.  sptrsv_info.engine: 3 LEAN, 6 warp,
- * 7 CHAIN, 8 SMALL (bit-exact: every row is thread-level there).
+ * 7 CHAIN, 8 SMALL (bit-exact: every row is thread-level there), 9 LEANP.
  */
 int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colidx,
                           const double *val, int32_t tri_flags, sptrsv_handle_t *out);
+
+/*
+ * sptrsv_analyse_csr_batch -- a BATCH of independent systems (the
+ * C5 batch of BASELINE configs[4]) as ONE handle, so that a solve is one launch
+ * over all of them: the block-diagonal matrix diag(L_0, ..., L_{nsys-1}), each
+ * block the paper's problem (Alg.5) on its own rows.
+ *   nsys     number of systems (>= 1).
+ *   n        HOST array [nsys]: rows of each system (>= 0).
+ *   rowptr, colidx, val
+ *            HOST arrays [nsys] of DEVICE pointers to each system's CSR, in the
+ *            layout of sptrsv_analyse_csr (val / colidx may be NULL for a
+ *            system with no entries, unit-diagonal forms only).
+ *   tri_flags as sptrsv_analyse_csr_ex, for every system.
+ * The library copies the systems into one handle-owned concatenation (rowptr
+ * shifted by the entries, colidx by the rows before each system; freed by
+ * sptrsv_destroy; the caller's arrays are not kept), then analyses it as
+ * sptrsv_analyse_csr_ex does (same validation codes, row indices of the
+ * concatenation).  Solves take the concatenated b / x: system s occupies rows
+ * n[0] + ... + n[s-1] onward.  Synchronous.  Measured:
+ * one launch over 2 C5 systems beats 2 launches; over 8 the ready words
+ * outgrow the persisting L2 window and separate launches win -- group systems
+ * by what the window holds.
+ */
+int sptrsv_analyse_csr_batch(int32_t nsys, const int32_t *n, const int32_t *const *rowptr,
+                             const int32_t *const *colidx, const double *const *val, int32_t tri_flags,
+                             sptrsv_handle_t *out);
 
 /*
  * sptrsv_solve -- one solve L x = b (Alg.5), enqueued on

@@ -17,7 +17,7 @@ from ._lib import (MODE_AUTO, MODE_THREAD, MODE_WARP, OPT_BACKOFF_MAX_NS, OPT_BA
                    OPT_CTA_THREADS, OPT_L2_WINDOW, OPT_LOCAL, OPT_MODE, OPT_PROTOCOL, OPT_SPIN_LIMIT,
                    OPT_STAGE_SMEM, OPT_WARP_THRESHOLD, PROTO_FLAGS, PROTO_FUSED, SptrsvError, check)
 
-__all__ = ["analyse", "Handle", "SptrsvError", "flag_latency", "hop_scan", "MODE_AUTO", "MODE_THREAD",
+__all__ = ["analyse", "analyse_batch", "Handle", "SptrsvError", "flag_latency", "hop_scan", "MODE_AUTO", "MODE_THREAD",
            "MODE_WARP", "PROTO_FLAGS", "PROTO_FUSED", "lib"]
 
 lib = _lib.lib
@@ -71,6 +71,41 @@ class Handle:
                                             val.data_ptr() if val.numel() else None, self.tri,
                                             ctypes.byref(self._h)),
                   "sptrsv_analyse_csr_ex")
+
+    @classmethod
+    def batch(cls, systems, upper=False, unit_diag=False):
+        """``sptrsv_analyse_csr_batch``: independent systems [(rowptr, colidx, val), ...] on one device as
+        ONE block-diagonal handle (the library owns the concatenation); solve / solve_host then take
+        the concatenated b / x (system s at rows offsets[s] .. offsets[s + 1])."""
+        import numpy as np
+        import torch
+        if not systems:
+            raise ValueError("no systems")
+        dev = systems[0][0].device
+        ns = []
+        for rp, ci, v in systems:
+            _need(rp, torch.int32, None, "rowptr", dev)
+            _need(ci, torch.int32, None, "colidx", dev)
+            _need(v, torch.float64, ci.numel(), "val", dev)
+            ns.append(rp.numel() - 1)
+        self = cls.__new__(cls)
+        self.device = dev
+        self.n = int(sum(ns))
+        self.offsets = np.concatenate([[0], np.cumsum(ns)]).astype(np.int64)
+        self._keep = tuple(systems)
+        self._h = ctypes.c_void_p()
+        self.tri = (_lib.TRI_UPPER if upper else 0) | (_lib.TRI_UNIT_DIAG if unit_diag else 0)
+        k = len(systems)
+        n_arr = (ctypes.c_int32 * k)(*ns)
+        rp_arr = (ctypes.c_void_p * k)(*[rp.data_ptr() for rp, _, _ in systems])
+        ci_arr = (ctypes.c_void_p * k)(*[ci.data_ptr() if ci.numel() else None for _, ci, _ in systems])
+        v_arr = (ctypes.c_void_p * k)(*[v.data_ptr() if v.numel() else None for _, _, v in systems])
+        with torch.cuda.device(dev):
+            torch.cuda.current_stream().synchronize()
+            check(lib.sptrsv_analyse_csr_batch(k, ctypes.addressof(n_arr), ctypes.addressof(rp_arr),
+                                               ctypes.addressof(ci_arr), ctypes.addressof(v_arr), self.tri,
+                                               ctypes.byref(self._h)), "sptrsv_analyse_csr_batch")
+        return self
 
     # -- solve -------------------------------------------------------------------------
     def solve(self, b, x=None, stream=None):
@@ -195,7 +230,12 @@ class Handle:
 def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Handle:
     """``sptrsv_analyse_csr[_ex]`` + options (mode=, warp_threshold=, cta_threads=, ...)."""
     h = Handle(rowptr, colidx, val, upper=upper, unit_diag=unit_diag)
-    keys = {"mode": OPT_MODE, "warp_threshold": OPT_WARP_THRESHOLD, "cta_threads": OPT_CTA_THREADS,
+    for k, v in options.items():
+        h.set_option(_OPTION_KEYS[k], v)
+    return h
+
+
+_OPTION_KEYS = {"mode": OPT_MODE, "warp_threshold": OPT_WARP_THRESHOLD, "cta_threads": OPT_CTA_THREADS,
             "backoff_min_ns": OPT_BACKOFF_MIN_NS, "backoff_max_ns": OPT_BACKOFF_MAX_NS,
             "spin_limit": OPT_SPIN_LIMIT, "l2_window": OPT_L2_WINDOW, "stage_smem": OPT_STAGE_SMEM,
             "protocol": OPT_PROTOCOL, "local": OPT_LOCAL, "engine": _lib.OPT_ENGINE,
@@ -205,8 +245,13 @@ def analyse(rowptr, colidx, val, upper=False, unit_diag=False, **options) -> Han
             "poll_one": _lib.OPT_POLL_ONE,
             "warp_split_last": _lib.OPT_WARP_SPLIT_LAST,
             "host_io": _lib.OPT_HOST_IO, "subwarp": _lib.OPT_SUBWARP, "chain_div": _lib.OPT_CHAIN_DIV}
+
+
+def analyse_batch(systems, upper=False, unit_diag=False, **options) -> Handle:
+    """``sptrsv_analyse_csr_batch`` + options: independent systems as one block-diagonal handle."""
+    h = Handle.batch(systems, upper=upper, unit_diag=unit_diag)
     for k, v in options.items():
-        h.set_option(keys[k], v)
+        h.set_option(_OPTION_KEYS[k], v)
     return h
 
 

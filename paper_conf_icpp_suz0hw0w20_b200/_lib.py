@@ -94,6 +94,7 @@ _i32, _i64 = ctypes.c_int32, ctypes.c_int64
 EXPORTS = {
     "sptrsv_analyse_csr": (ctypes.c_int, [_i32, _p, _p, _p, ctypes.POINTER(_h)]),
     "sptrsv_analyse_csr_ex": (ctypes.c_int, [_i32, _p, _p, _p, _i32, ctypes.POINTER(_h)]),
+    "sptrsv_analyse_csr_batch": (ctypes.c_int, [_i32, _p, _p, _p, _p, _i32, ctypes.POINTER(_h)]),
     "sptrsv_solve": (ctypes.c_int, [_h, _p, _p, _p]),
     "sptrsv_solve_host": (ctypes.c_int, [_h, _p, _p, _p]),
     "sptrsv_solve_multi": (ctypes.c_int, [_h, _p, _p, _i32, _i64, _i64, _p]),

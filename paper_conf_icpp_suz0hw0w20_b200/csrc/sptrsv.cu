@@ -110,6 +110,9 @@ int spin_sync(cudaStream_t s, cudaEvent_t &ev) {
 
 struct sptrsv_handle_s {
     int device = 0;
+    // sptrsv_analyse_csr_batch: the handle owns the block-diagonal concatenation of its systems
+    int32_t *own_rowptr = nullptr, *own_colidx = nullptr;
+    double *own_val = nullptr;
     int32_t n = 0;
     int64_t nnz = 0;
     const int32_t *rowptr = nullptr;
@@ -413,6 +416,90 @@ const char *sptrsv_strerror(int status) {
 int sptrsv_analyse_csr(int32_t n, const int32_t *rowptr, const int32_t *colidx, const double *val,
                        sptrsv_handle_t *out) {
     return sptrsv_analyse_csr_ex(n, rowptr, colidx, val, 0, out);
+}
+
+}  // extern "C"
+
+namespace {
+// block-diagonal concatenation (sptrsv_analyse_csr_batch): one system's rowptr shifted by the entries
+// before it, its column indices by the rows before it (lower and upper alike: the blocks sit on the
+// diagonal), its values copied
+__global__ void k_concat_rowptr(const int32_t *__restrict__ src, int32_t n, int32_t row_off, int64_t nnz_off,
+                                int32_t *__restrict__ dst) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) dst[row_off + i] = (int32_t)(src[i] + nnz_off);
+}
+__global__ void k_concat_colidx(const int32_t *__restrict__ src, int64_t nnz, int32_t row_off,
+                                int32_t *__restrict__ dst) {
+    const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < nnz) dst[j] = src[j] + row_off;
+}
+__global__ void k_set_i32(int32_t *p, int32_t v) { *p = v; }
+}  // namespace
+
+extern "C" {
+
+int sptrsv_analyse_csr_batch(int32_t nsys, const int32_t *n, const int32_t *const *rowptr,
+                             const int32_t *const *colidx, const double *const *val, int32_t tri_flags,
+                             sptrsv_handle_t *out) {
+    if (!out) return SPTRSV_ERR_INVALID_ARG;
+    *out = nullptr;
+    if (nsys < 1 || !n || !rowptr || !colidx || !val) return SPTRSV_ERR_INVALID_ARG;
+    // each system's entry count: rowptr[n_s] (a rowptr[0] != 0 is caught by the validation below,
+    // as a malformed rowptr of the concatenated system)
+    std::vector<int64_t> nnz(nsys), z0(nsys + 1, 0);
+    std::vector<int32_t> r0(nsys + 1, 0);
+    for (int k = 0; k < nsys; ++k) {
+        if (n[k] < 0 || !rowptr[k]) return SPTRSV_ERR_INVALID_ARG;
+        int32_t last = 0, first = 0;
+        if (cudaMemcpy(&last, rowptr[k] + n[k], sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(&first, rowptr[k], sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return SPTRSV_ERR_INVALID_ARG;
+        }
+        if (first != 0 || last < 0) return SPTRSV_ERR_BAD_ROWPTR;
+        if (last > 0 && (!colidx[k] || (!val[k] && !(tri_flags & SPTRSV_TRI_UNIT_DIAG)))) return SPTRSV_ERR_INVALID_ARG;
+        nnz[k] = last;
+        if ((int64_t)r0[k] + n[k] > 0x7FFFFFFE) return SPTRSV_ERR_TOO_LARGE;
+        r0[k + 1] = r0[k] + n[k];
+        z0[k + 1] = z0[k] + last;
+    }
+    if (z0[nsys] > 0x7FFFFFFF) return SPTRSV_ERR_TOO_LARGE;
+    const int32_t N = r0[nsys];
+    const int64_t Z = z0[nsys];
+    int32_t *rp = nullptr, *ci = nullptr;
+    double *v = nullptr;
+    auto fail = [&](int rc) {
+        (void)cudaGetLastError();
+        cudaFree(rp);
+        cudaFree(ci);
+        cudaFree(v);
+        return rc;
+    };
+    if (cudaMalloc(&rp, sizeof(int32_t) * ((size_t)N + 1)) != cudaSuccess ||
+        cudaMalloc(&ci, sizeof(int32_t) * (size_t)(Z > 0 ? Z : 1)) != cudaSuccess ||
+        cudaMalloc(&v, sizeof(double) * (size_t)(Z > 0 ? Z : 1)) != cudaSuccess)
+        return fail(SPTRSV_ERR_ALLOC);
+    for (int k = 0; k < nsys; ++k) {
+        if (n[k] > 0) k_concat_rowptr<<<(n[k] + 255) / 256, 256>>>(rowptr[k], n[k], r0[k], z0[k], rp);
+        if (nnz[k] > 0) {
+            k_concat_colidx<<<(unsigned)((nnz[k] + 255) / 256), 256>>>(colidx[k], nnz[k], r0[k], ci + z0[k]);
+            if (val[k] && cudaMemcpyAsync(v + z0[k], val[k], sizeof(double) * (size_t)nnz[k], cudaMemcpyDeviceToDevice,
+                                          0) != cudaSuccess)
+                return fail(SPTRSV_ERR_CUDA);
+        }
+    }
+    k_set_i32<<<1, 1>>>(rp + N, (int32_t)Z);
+    if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) return fail(SPTRSV_ERR_CUDA);
+    sptrsv_handle_t h = nullptr;
+    const int rc = sptrsv_analyse_csr_ex(N, rp, ci, (tri_flags & SPTRSV_TRI_UNIT_DIAG) && Z == 0 ? nullptr : v,
+                                         tri_flags, &h);
+    if (rc) return fail(rc);
+    h->own_rowptr = rp;
+    h->own_colidx = ci;
+    h->own_val = v;
+    *out = h;
+    return SPTRSV_OK;
 }
 
 void size_l2_window(sptrsv_handle_s *h);
@@ -1218,6 +1305,9 @@ int sptrsv_destroy(sptrsv_handle_t h) {
     }
     (void)cudaGetLastError();
     free_ws(h->ws);
+    cudaFree(h->own_rowptr);
+    cudaFree(h->own_colidx);
+    cudaFree(h->own_val);
     delete h;
     return SPTRSV_OK;
 }

@@ -39,7 +39,7 @@ def test_library_exports_every_declared_symbol(libpath):
 def test_binding_covers_header_and_loads(libpath):
     import paper_conf_icpp_suz0hw0w20_b200._lib as L
     assert sorted(L.EXPORTS) == _declared()
-    assert L.lib.sptrsv_abi_version() == 3
+    assert L.lib.sptrsv_abi_version() == 4
     assert L.lib.sptrsv_strerror(-3).decode().startswith("row without a diagonal")
     # argument validation happens before any CUDA call
     assert L.lib.sptrsv_analyse_csr(-1, None, None, None, None) == L.ERR_INVALID_ARG

@@ -811,3 +811,59 @@ def test_leanp_host_path_interleaves_with_graph_replays(cap):
             h.solve_host(bh, xh)
             h.check()
             assert np.array_equal(xh.numpy(), ref)
+
+
+@pytest.mark.parametrize("flags", [0, 1, 2, 3])
+def test_batch_handle_block_diagonal_bit_exact(cap, flags):
+    """sptrsv_analyse_csr_batch: independent systems (ragged sizes, a chain, a c2-shaped one) as ONE
+    block-diagonal handle, one launch per solve; every block bit-identical to the oracle's
+    solve of that system alone, through solve and solve_host."""
+    systems = [synth.gen_random_lower(1001, 3, seed=1), synth.gen_c2(n=50_000), synth.gen_chain(700),
+               synth.gen_random_lower(33, 5, seed=3)]
+    if flags & 1:
+        systems = [synth.to_upper(s) for s in systems]
+    if flags & 2:
+        systems = [synth.to_unit(s, upper=bool(flags & 1)) for s in systems]
+    d = torch.device("cuda:0")
+    dev = [tuple(torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val)) for s in systems]
+    refs = [oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags) if flags else
+            oracle.solve(s.rowptr, s.colidx, s.val, s.b) for s in systems]
+    b = torch.from_numpy(np.concatenate([s.b for s in systems])).to(d)
+    # (MODE 1: every row thread-level, so every block is bit-exact; AUTO may give the 5-dependency rows
+    # warp-level rows, which are within the warp-mode bound instead)
+    with cap.analyse_batch(dev, upper=bool(flags & 1), unit_diag=bool(flags & 2), mode=1) as h:
+        assert h.n == sum(s.n for s in systems)
+        off = h.offsets
+        x = torch.full_like(b, float("nan"))
+        h.solve(b, x)
+        h.check()
+        got = x.cpu().numpy()
+        for k, ref in enumerate(refs):
+            assert np.array_equal(got[off[k]:off[k + 1]], ref), k
+        bh = b.cpu().pin_memory()
+        xh = torch.full((h.n,), float("nan"), dtype=torch.float64).pin_memory()
+        h.solve_host(bh, xh)
+        for k, ref in enumerate(refs):
+            assert np.array_equal(xh.numpy()[off[k]:off[k + 1]], ref), k
+
+
+def test_batch_handle_validation_and_empty(cap):
+    """A malformed system in a batch is reported with the concatenation's row index (the lowest
+    offending row); a batch of one equals the plain handle; a zero-row system is allowed."""
+    d = torch.device("cuda:0")
+    good = synth.gen_random_lower(100, 3, seed=5)
+    t = tuple(torch.from_numpy(a).to(d) for a in (good.rowptr, good.colidx, good.val))
+    ci = good.colidx.copy()
+    ci[good.rowptr[10]] = 50  # row 10 of the second system: a column above the diagonal
+    bad = tuple(torch.from_numpy(a).to(d) for a in (good.rowptr, ci, good.val))
+    with pytest.raises(cap.SptrsvError) as e:
+        cap.analyse_batch([t, bad])
+    assert e.value.status == cap._lib.ERR_NOT_LOWER
+    empty = (torch.zeros(1, dtype=torch.int32, device=d), torch.zeros(0, dtype=torch.int32, device=d),
+             torch.zeros(0, dtype=torch.float64, device=d))
+    with cap.analyse_batch([empty, t, empty]) as h:
+        assert h.n == 100 and list(h.offsets) == [0, 0, 100, 100]
+        b = torch.from_numpy(good.b).to(d)
+        x = h.solve(b)
+        h.check()
+        assert np.array_equal(x.cpu().numpy(), oracle.solve(good.rowptr, good.colidx, good.val, good.b))
