@@ -168,6 +168,7 @@ struct sptrsv_handle_s {
     uint32_t gen = 0, mgen = 0;  // configuration generations of the solve / multi-RHS state (cta_ticket)
     uint32_t hgen = 0, hsince_reset = 0;  // the host-path state (Workspace::hst)
     int hlaunch_key = -1;
+    bool no_coop = false;  // a cooperative launch was refused (shared GPU, MPS): AUTO falls back to LEAN
     unsigned long long *trace = nullptr;
     // bookkeeping
     uint32_t solves = 0;
@@ -703,8 +704,9 @@ int resolve_engine(const sptrsv_handle_s *h) {
     if (h->plan != PLAN_THREAD)  // ONE-SHOT has no sub-warp rows
         return (h->engine == ENG_ONESHOT && !h->tri && h->n_sub_tasks == 0) ? ENG_ONESHOT : ENG_HYBRID;
     if (h->engine != ENG_AUTO) return (h->tri && h->engine == ENG_ONESHOT) ? ENG_LEAN : h->engine;
-    if (h->tri) return chains ? ENG_CHAIN : ENG_LEANP;
-    if (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n) return ENG_LEANP;
+    const int lean_auto = h->no_coop ? ENG_LEAN : ENG_LEANP;  // LEANP needs a cooperative launch
+    if (h->tri) return chains ? ENG_CHAIN : lean_auto;
+    if (offdiag <= 0 || 4 * h->near_rows < (int64_t)h->n) return lean_auto;
     return chains ? ENG_CHAIN : ENG_ONESHOT;
 }
 
@@ -1042,6 +1044,12 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     const cudaError_t e = cudaLaunchKernelEx(&cfg, (void (*)(SolveParams))L.fn, p);
     if (e != cudaSuccess) {
         (void)cudaGetLastError();
+        if (L.coop && h->engine == ENG_AUTO && !h->no_coop) {
+            // the device would not co-schedule the persistent grid (another process holds SMs, MPS
+            // limits ...): AUTO falls back to the non-persistent LEAN for this handle from now on
+            h->no_coop = true;
+            return solve_impl(h, b, x, x_host, stream, bflag, bseq, bshift, host_state);
+        }
         return SPTRSV_ERR_CUDA;
     }
     h->solves++;
