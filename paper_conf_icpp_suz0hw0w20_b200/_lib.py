@@ -59,7 +59,8 @@ OPT_WARP_SPLIT_LAST = 22
 OPT_HOST_IO = 23
 OPT_SUBWARP = 24
 OPT_CHAIN_DIV = 25
-ENGINE_ONESHOT, ENGINE_LEAN, ENGINE_AUTO, ENGINE_HYBRID, ENGINE_CHAIN, ENGINE_SMALL, ENGINE_LEANP = 0, 3, 5, 6, 7, 8, 9
+(ENGINE_ONESHOT, ENGINE_LEAN, ENGINE_AUTO, ENGINE_HYBRID, ENGINE_CHAIN, ENGINE_SMALL, ENGINE_LEANP,
+ ENGINE_GRID) = 0, 3, 5, 6, 7, 8, 9, 10
 PROTO_FLAGS, PROTO_FUSED = 0, 1
 MODE_AUTO, MODE_THREAD, MODE_WARP, MODE_SUBWARP = 0, 1, 2, 3
 

@@ -34,6 +34,13 @@ struct AnalyseOut {
     unsigned long long near;     // near_deps | warp_deps << 32
     unsigned long long prev;     // prev_deps | near_rows << 32
     unsigned long long hist[32]; // rows by floor(log2(nearest-dependency distance))
+    // ENGINE_GRID eligibility (solve_grid.cuh k_grid_probe / k_grid_check): the line length m the
+    // probe proposes (0 = none), and over every row for that m: rows violating the band order,
+    // north / west entries (register / shuffle operands), far entries (polled)
+    int32_t grid_m;
+    int32_t grid_viol;
+    long long grid_fast;
+    long long grid_far;
 };
 
 // status: 64-bit min over (row << 8 | code) -> the lowest offending row wins,

@@ -1,0 +1,495 @@
+// solve_grid.cuh -- ENGINE_GRID: wavefront bands for stencil-shaped lower factors.
+//
+// The same per-row method as every engine -- Alg.5's row: the off-diagonals
+// consumed in column order with separately rounded mul / add, the division at the diagonal, the
+// publish -- mapped onto the shape of the paper's low-parallelism regime (Table 6, PAPER.md:421-437:
+// small beta = n / levels): lower factors of structured grids, where row r = y*m + x (line y,
+// column x) depends on its west neighbour r-1 and its north neighbour r-m (5-point stencil), plus at
+// most one far row (7-point: the plane below).  CHAIN walks such a matrix in row order, so each grid
+// line waits for the line above through the global protocol (c3, 2048^2: ~2.4 us per line).
+//
+// GRID cuts the matrix into BANDS of 32 columns: band k = columns [32k, 32k+32) of every line.  Lane
+// l of band k's warp owns column x = 32k + l and walks the lines with a skew of one step per lane
+// (step s: lane l solves line y = s - l).  Then
+//   north (r - m)  = the lane's own result of the previous step       (a register)
+//   west  (r - 1)  = lane l-1's result of the previous step           (one __shfl_up_sync)
+//   lane 0's west  = band k-1's lane 31, through the global protocol: a RING of polls -- lane
+//                    (y & 31) issues line y's poll kGridRing steps before lane 0 needs it
+//   a far entry    = the global protocol (its poll issued one step ahead)
+// so a step costs one shuffle and the row's dependent fp64 operations, and band k waits on band k-1
+// through lane 0 only: one global hop per 32 columns instead of one per line.  The critical path is
+// the grid's wavefront, lines + 32 * bands steps, plus one hop per band.
+//
+// Eligibility (k_grid_check, every row, for the m k_grid_probe proposes): each off-diagonal is the
+// west neighbour (c = r - 1 with x >= 1), the north neighbour (c = r - m), or a far entry c < r - m
+// that lies in an earlier band, or in the same band at an earlier step; at most one far entry.
+// That is exactly when no step waits on a later step of its own band or on a later band (forward
+// progress: bands take the CTA start ticket, so band k only waits on bands started before it).
+// Accumulation far -> north -> west is column order with separately rounded mul and add, as Alg.1
+// (PAPER.md:82-92): x is bit-identical to the oracle.  Division: Diag (solve.cuh) -- the Markstein
+// candidate, proven by its remainder either in the loop (SAFE) or off the chain with the failure
+// reported as SPTRSV_ERR_INEXACT (the CHAIN contract, SPTRSV_OPT_CHAIN_DIV).
+#pragma once
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "setup.cuh"
+#include "solve.cuh"
+
+namespace sptrsv_dev {
+
+#ifndef SPTRSV_GRID_RING
+#define SPTRSV_GRID_RING 8
+#endif
+constexpr int kGridRing = SPTRSV_GRID_RING;  // steps between lane 0's west poll and its use (< 32)
+
+// ---------------------------------------------------------------- analyse: is the matrix a grid?
+
+// One warp proposes the line length m: each lane samples one row and takes the distance to its
+// nearest off-diagonal that is not the previous row (the north neighbour of a grid row); the most
+// frequent candidate (>= 2 votes) wins.  Lower non-unit handles only (tri == 0).
+__global__ void k_grid_probe(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ colidx, int32_t n,
+                             AnalyseOut *out, int tri) {
+    const int lane = threadIdx.x;
+    int cand = 0;
+    const bool valid = out->status == ~0ull && tri == 0 && n >= 2;
+    if (valid) {
+        const int r = (int)((long long)(lane + 1) * n / 33);
+        const int s = rowptr[r], e = rowptr[r + 1];
+        int j = e - 2;  // the last off-diagonal (the diagonal is last)
+        if (j >= s && colidx[j] == r - 1) --j;
+        if (j >= s) cand = r - colidx[j];
+    }
+    const unsigned same = __match_any_sync(0xffffffffu, cand);
+    const unsigned cnt = cand > 1 ? (unsigned)__popc(same) : 0u;
+    unsigned long long key = ((unsigned long long)cnt << 32) | (unsigned)cand;
+    for (int off = 16; off; off >>= 1) {
+        const unsigned long long o = __shfl_xor_sync(0xffffffffu, key, off);
+        key = o > key ? o : key;
+    }
+    if (lane == 0) out->grid_m = (valid && (key >> 32) >= 2) ? (int)(key & 0xffffffffu) : 0;
+}
+
+// Every row against the m of k_grid_probe: violations of the band order (see the header), fast
+// entries (north / west) and far entries.
+__global__ void __launch_bounds__(256) k_grid_check(const int32_t *__restrict__ rowptr,
+                                                    const int32_t *__restrict__ colidx, int32_t n, AnalyseOut *out) {
+    const int m = out->grid_m;
+    if (m < 2 || out->status != ~0ull) return;
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned viol = 0, fast = 0, far = 0;
+    if (r < n) {
+        const int y = r / m, x = r - y * m, k = x >> 5, l = x & 31;
+        const int s = rowptr[r], e = rowptr[r + 1] - 1;  // off-diagonals [s, e)
+        for (int j = s; j < e; ++j) {
+            const int c = colidx[j];
+            if ((c == r - 1 && x >= 1) || c == r - m) {
+                ++fast;
+            } else if (c < r - m) {
+                const int y2 = c / m, x2 = c - y2 * m, k2 = x2 >> 5, l2 = x2 & 31;
+                if (!(k2 < k || (k2 == k && y2 + l2 < y + l))) viol = 1;
+                ++far;
+            } else {
+                viol = 1;  // between the north and the west neighbour, or r-1 across a line start
+            }
+        }
+        if (far > 1) viol = 1;
+    }
+    for (int off = 16; off; off >>= 1) {
+        viol += __shfl_xor_sync(0xffffffffu, viol, off);
+        fast += __shfl_xor_sync(0xffffffffu, fast, off);
+        far += __shfl_xor_sync(0xffffffffu, far, off);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (viol) atomicAdd(&out->grid_viol, (int)viol);
+        if (fast) atomicAdd((unsigned long long *)&out->grid_fast, (unsigned long long)fast);
+        if (far) atomicAdd((unsigned long long *)&out->grid_far, (unsigned long long)far);
+    }
+}
+
+// ---------------------------------------------------------------- the solve
+//
+// One band per CTA of four warps: warp 0, the CONSUMER, runs the band's chain (the skewed steps
+// above) and nothing else; warps 1..3, the PRODUCERS, keep it fed:
+//   - raw CSR staging: the rows of one line of a band are contiguous, so rowptr / b / entries of a
+//     line are copied into a shared-memory ring (kGridRaw lines) by cp.async, coalesced, kGridA1 /
+//     kGridA2 blocks before they are needed;
+//   - classification: each staged row becomes a DESCRIPTOR (ls0 = its far entry's product already
+//     summed when the far row was published, north / west coefficients, b, d, RN(1/d), flags) in a
+//     second ring (kGridDesc lines).
+// The CTA meets at a barrier every kGridBlk consumer steps: block b runs steps [B*b, B*b + B) and
+// produces the descriptors of lines [B*b + B + 1, B*b + 2B] (B = kGridBlk), so the consumer always
+// finds the next B + 1 lines ready and its step is one shuffle, the row's dependent fp64 operations,
+// two stores and one-step-ahead shared-memory loads.
+constexpr int kGridProd = 3;              // producer warps (one per remaining SM sub-partition)
+constexpr int kGridBlk = 2 * kGridProd;   // consumer steps per block (each producer: 2 lines per block)
+constexpr int kGridDesc = 48;             // descriptor ring (lines): line y is read until step y + 30
+constexpr int kGridRaw = 64;              // raw CSR ring (lines)
+constexpr int kGridA1 = 8;                // rowptr / b staged this many blocks before production
+constexpr int kGridA2 = 4;                // entries staged this many blocks before production
+constexpr int kGridSlack = 16;  // a band that found lane 0's west operand missing resumes only once
+                                // the line this far ahead is published (so its next polls find their
+                                // records: a band tracking its predecessor at the minimum lag would
+                                // pay a round trip on every step)
+static_assert(kGridA1 == 2 * kGridA2, "one cp.async wait covers both staging distances");
+static_assert(kGridBlk * (kGridA1 + 1) <= kGridRaw, "raw ring too small");
+
+enum : int { kDescAct = 1, kDescN = 2, kDescW = 4, kDescFar = 8 /* far entry not folded: poll it */ };
+
+__host__ __device__ constexpr size_t grid_smem_bytes(int ecap) {
+    return (size_t)kGridDesc * 32 * (6 * 8 + 2 * 4) + (size_t)kGridRaw * (64 * 4 + 32 * 8 + (size_t)ecap * 12);
+}
+
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+#ifdef SPTRSV_GRID_NOASYNC  // measurement builds only: synchronous staging through registers
+__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
+    *reinterpret_cast<int32_t *>(dst) = __ldcg(reinterpret_cast<const int32_t *>(src));
+}
+__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+    *reinterpret_cast<double *>(dst) = __ldcg(reinterpret_cast<const double *>(src));
+}
+#else
+__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+#endif
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+#ifdef SPTRSV_GRID_DEBUG_OOB  // measurement builds only: the first out-of-range index, clamped
+__device__ __forceinline__ long long gchk(const SolveParams &p, long long i, long long lim, int tag) {
+    if (i < 0 || i >= lim) {
+        unsigned long long *t = p.trace + p.n;  // after the publish timestamps
+        if (p.trace && atomicCAS(t + 32, 0ull, 1ull) == 0ull) {
+            t[33] = tag; t[34] = i; t[35] = lim; t[36] = blockIdx.x; t[37] = threadIdx.x;
+        }
+        return 0;
+    }
+    return i;
+}
+#define GCHK(i, lim, tag) gchk(p, (i), (lim), (tag))
+#else
+#define GCHK(i, lim, tag) (i)
+#endif
+
+template <int PROTO, bool SAFE>
+__global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolveParams p) {
+    extern __shared__ __align__(16) unsigned char gsm[];
+    __shared__ uint32_t s_blk, s_epoch, s_stop;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        cta_ticket(p, s_blk, s_epoch);
+        s_stop = 0;
+    }
+    __syncthreads();
+    if (s_blk == kStaleBlk) return;
+    const uint32_t epoch = s_epoch;
+    const int m = p.grid_m, lines = p.grid_lines, E = p.grid_ecap;
+    const unsigned n = (unsigned)p.n;
+    const int band = (int)s_blk;
+    const int x0 = band * 32;
+    const int nl = min(32, m - x0);  // lanes owning a column (>= 1: the grid is ceil(m / 32) bands)
+    const int steps = lines + nl - 1;
+    const int nblocks = (steps + kGridBlk - 1) / kGridBlk;
+    // ---- shared memory: descriptor ring, then raw ring
+    double *d_ls0 = reinterpret_cast<double *>(gsm);  // [desc][32]: far product summed (or vf if pending)
+    double *d_vn = d_ls0 + kGridDesc * 32, *d_vw = d_vn + kGridDesc * 32, *d_b = d_vw + kGridDesc * 32;
+    double *d_d = d_b + kGridDesc * 32, *d_rc = d_d + kGridDesc * 32;
+    int32_t *d_meta = reinterpret_cast<int32_t *>(d_rc + kGridDesc * 32), *d_fc = d_meta + kGridDesc * 32;
+    int32_t *s_rp = d_fc + kGridDesc * 32;                                   // [raw][64]
+    double *s_b = reinterpret_cast<double *>(s_rp + kGridRaw * 64);          // [raw][32]
+    double *s_val = s_b + kGridRaw * 32;                                     // [raw][E]
+    int32_t *s_col = reinterpret_cast<int32_t *>(s_val + (size_t)kGridRaw * E);  // [raw][E]
+
+    if (warp > 0) {
+        // ================================================================ producers
+        const int w = warp - 1;
+        auto line_rows = [&](int y, unsigned &row0) -> int {  // rows of line y in this band (0: none)
+            row0 = (unsigned)y * (unsigned)m + (unsigned)x0;
+            if (y < 0 || y >= lines || row0 >= n) return 0;
+            return min(nl, (int)(n - row0));
+        };
+        auto stage_rp = [&](int y) {  // rowptr[row0 .. row0 + k] and b[row0 .. row0 + k)
+            unsigned row0;
+            const int k = line_rows(y, row0);
+            if (k == 0) return;
+            int32_t *rp = s_rp + (y & (kGridRaw - 1)) * 64;
+            if (lane <= k) cp_async4(rp + lane, p.rowptr + GCHK((long long)row0 + lane, (long long)n + 1, 1));
+            if (lane == 0 && k == 32) cp_async4(rp + 32, p.rowptr + GCHK((long long)row0 + 32, (long long)n + 1, 2));
+            if (lane < k) cp_async8(s_b + (y & (kGridRaw - 1)) * 32 + lane, p.b + GCHK((long long)row0 + lane, (long long)n, 3));
+        };
+        auto stage_ent = [&](int y) {  // entries of line y (its rowptr slice complete in the ring)
+            unsigned row0;
+            const int k = line_rows(y, row0);
+            if (k == 0) return;
+            const int sl = y & (kGridRaw - 1);
+            const int lo = s_rp[sl * 64], hi = s_rp[sl * 64 + k];
+            for (int e = lo + lane; e < hi; e += 32) {
+                cp_async4(s_col + (size_t)sl * E + GCHK(e - lo, E, 6), p.colidx + GCHK(e, p.nnz, 4));
+                cp_async8(s_val + (size_t)sl * E + GCHK(e - lo, E, 7), p.val + GCHK(e, p.nnz, 5));
+            }
+        };
+        auto produce = [&](int y) {  // descriptors of line y from its staged raw rows
+            unsigned row0;
+            const int k = line_rows(y, row0);
+            if (y >= lines) return;
+            const int sl = y & (kGridRaw - 1), ds = (y % kGridDesc) * 32 + lane;
+            const bool act = lane < k;
+            const int r = (int)(row0 + lane);
+            int meta = 0, fc = 0;
+            double ls0 = 0.0, vn = 0.0, vw = 0.0, bv = 0.0, dv = 1.0, rc = 1.0;
+            if (act) {
+                const int base = s_rp[sl * 64];
+                const int lo = s_rp[sl * 64 + lane] - base, hi = s_rp[sl * 64 + lane + 1] - base;
+                const double *v = s_val + (size_t)sl * E;
+                const int32_t *c = s_col + (size_t)sl * E;
+                const int len = hi - lo;
+                const bool hw = len > 1 && c[hi - 2] == r - 1;  // (row 0 has no west: no -1 sentinel)
+                const int jn = hi - 2 - (int)hw;
+                const bool hn = jn >= lo && c[jn] == r - m;
+                const int jf = jn - (int)hn;
+                meta = kDescAct | (hn ? kDescN : 0) | (hw ? kDescW : 0);
+                vw = hw ? v[hi - 2] : 0.0;
+                vn = hn ? v[jn] : 0.0;
+                if (jf >= lo) {  // the far entry (at most one: k_grid_check)
+                    fc = c[jf];
+                    const double vf = v[jf];
+                    unsigned long long f0, f1;
+                    poll1<PROTO>(p, (int)GCHK(fc, (long long)n, 8), f0, f1);
+                    if (ready1<PROTO>(f0, f1, epoch)) {
+                        ls0 = __dadd_rn(0.0, __dmul_rn(vf, value1<PROTO>(p, fc, f0, f1)));
+                    } else {
+                        ls0 = vf;
+                        meta |= kDescFar;
+                    }
+                }
+                bv = s_b[sl * 32 + lane];
+                Diag g;
+                g.init(v[hi - 1]);
+                dv = g.d;
+                rc = g.r;
+            }
+            d_ls0[ds] = ls0;
+            d_vn[ds] = vn;
+            d_vw[ds] = vw;
+            d_b[ds] = bv;
+            d_d[ds] = dv;
+            d_rc[ds] = rc;
+            d_meta[ds] = meta;
+            d_fc[ds] = fc;
+        };
+        // prologue: the raw rows of the first lines, then the descriptors of lines [0, kGridBlk]
+        for (int y = w; y < kGridBlk + 1 + kGridBlk * kGridA1; y += kGridProd) stage_rp(y);
+        cp_async_commit();
+        cp_async_wait<0>();
+        __syncwarp();
+        for (int y = w; y < kGridBlk + 1 + kGridBlk * kGridA2; y += kGridProd) stage_ent(y);
+        cp_async_commit();
+        cp_async_wait<0>();
+        __syncwarp();
+        for (int y = w; y <= kGridBlk; y += kGridProd) produce(y);
+        for (int b = 0; b < nblocks; ++b) {
+            __syncthreads();  // block b begins: lines <= B*b + B are in the descriptor ring
+            if (s_stop) continue;
+#ifdef SPTRSV_GRID_WAITALL  // measurement builds only
+            cp_async_wait<0>();
+#else
+            cp_async_wait<kGridA2 - 1>();
+#endif
+            __syncwarp();
+            const int y0 = kGridBlk * b + kGridBlk + 1;
+            for (int y = y0 + w; y < y0 + kGridBlk; y += kGridProd) {
+                stage_rp(y + kGridBlk * kGridA1);
+                stage_ent(y + kGridBlk * kGridA2);
+            }
+            cp_async_commit();
+            for (int y = y0 + w; y < y0 + kGridBlk; y += kGridProd) produce(y);
+        }
+        cp_async_wait<0>();
+        return;
+    }
+    // ==================================================================== consumer (warp 0)
+    const int x = x0 + lane;
+    const bool colok = lane < nl;
+    const bool ring_on = band > 0;
+    auto ring_row = [&](int y) -> int {  // lane 0's west neighbour on line y (band k-1, lane 31)
+        if (!ring_on || y >= lines) return -1;
+        const unsigned r = (unsigned)y * (unsigned)m + (unsigned)x0 - 1u;
+        return r < n ? (int)r : -1;
+    };
+    // the row of the next step (line s + 1 - lane), read from the descriptor ring one step ahead
+    int c_r = -1, c_meta = 0, c_fc = 0;
+    double c_ls0 = 0, c_vn = 0, c_vw = 0, c_b = 0, c_d = 1, c_rc = 1;
+    unsigned long long c_f0 = 0, c_f1 = 0;
+    auto fetch = [&](int s1) {
+        const int y = s1 - lane;
+        const unsigned r = (unsigned)y * (unsigned)m + (unsigned)x;
+        const bool act = colok && y >= 0 && y < lines && r < n;
+        const int ds = ((act ? y : 0) % kGridDesc) * 32 + lane;
+        c_meta = act ? d_meta[ds] : 0;
+        c_ls0 = d_ls0[ds];
+        c_vn = d_vn[ds];
+        c_vw = d_vw[ds];
+        c_b = d_b[ds];
+        c_d = d_d[ds];
+        c_rc = d_rc[ds];
+        c_fc = d_fc[ds];
+        c_r = act ? (int)r : -1;
+        if (c_meta & kDescFar) poll1<PROTO>(p, (int)GCHK(c_fc, (long long)n, 9), c_f0, c_f1);
+    };
+    // ---- the ring: the lane holding line y polls its record kGridRing steps before step y
+    unsigned long long rw0 = 0, rw1 = 0;
+    int rrow = -1, rline = -1;
+    if (lane < kGridRing) {
+        rline = lane;
+        rrow = ring_row(lane);
+        if (rrow >= 0) poll1<PROTO>(p, rrow, rw0, rw1);
+    }
+    double xl = 0.0;  // this lane's latest x (the north operand of its next row)
+    bool bad = false, stop = false;
+    uint32_t backoff = p.backoff_min, idle = 0;
+    for (int b = 0; b < nblocks; ++b) {
+        __syncthreads();
+        if (stop) continue;
+        if (b == 0) fetch(0);
+        const int s_end = min(steps, kGridBlk * (b + 1));
+        for (int s = kGridBlk * b; s < s_end; ++s) {
+            const int r = c_r;
+            const bool act = r >= 0;
+            const bool pend = (c_meta & kDescFar) != 0;
+            // ---- operands produced outside this warp: lane 0's west (the ring), pending far entries
+            const int hold = s & 31;
+            const bool ring_ok = lane != hold || rrow < 0 || ready1<PROTO>(rw0, rw1, epoch);
+            bool ok = ring_ok && (!pend || ready1<PROTO>(c_f0, c_f1, epoch));
+            if (__any_sync(FULL, !ok)) {  // not there yet: wait (warp-uniform, backoff, watchdog)
+                const bool late = __any_sync(FULL, !ring_ok);
+                const int trow = late && lane == 0 ? ring_row(min(s + kGridSlack, lines - 1)) : -1;
+                bool tok = trow < 0;
+                while (true) {
+                    if (lane == hold && rrow >= 0 && !ready1<PROTO>(rw0, rw1, epoch)) poll1<PROTO>(p, rrow, rw0, rw1);
+                    if (pend && !ready1<PROTO>(c_f0, c_f1, epoch)) poll1<PROTO>(p, c_fc, c_f0, c_f1);
+                    if (!tok) {
+                        unsigned long long t0, t1;
+                        poll1<PROTO>(p, (int)GCHK(trow, (long long)n, 10), t0, t1);
+                        tok = ready1<PROTO>(t0, t1, epoch);
+                    }
+                    ok = tok && (lane != hold || rrow < 0 || ready1<PROTO>(rw0, rw1, epoch)) &&
+                         (!pend || ready1<PROTO>(c_f0, c_f1, epoch));
+                    if (!__any_sync(FULL, !ok)) break;
+                    if (backoff) nanosleep_ns(backoff);
+                    backoff = min(max(backoff * 2u, 32u), p.backoff_max);
+                    ++idle;
+                    if ((idle & 63u) == 0 || (p.spin_limit && idle >= p.spin_limit)) {
+                        uint32_t ab = 0;
+                        if (lane == 0) {
+                            if (p.spin_limit && idle >= p.spin_limit) {
+                                atomicCAS(&p.st->error.v, 0u, kErrTimeout);
+                                st_relaxed_u32(&p.st->abort.v, 1u);
+                            }
+                            ab = ld_relaxed_u32(&p.st->abort.v);
+                        }
+                        if (__shfl_sync(FULL, ab, 0)) {
+                            stop = true;
+                            break;
+                        }
+                    }
+                }
+                if (stop) break;
+                // the polls in flight for the next lines predate the wait: issue them again
+                if (late && rrow >= 0 && rline > s) poll1<PROTO>(p, rrow, rw0, rw1);
+                backoff = p.backoff_min;
+                idle = 0;
+            }
+            double xw = __shfl_up_sync(FULL, xl, 1);
+            double rv = 0.0;
+            if (lane == hold && rrow >= 0) rv = value1<PROTO>(p, rrow, rw0, rw1);
+            rv = __shfl_sync(FULL, rv, hold);
+            if (lane == 0) xw = rv;
+            // ---- Alg.1's row: far (ls0), north, west (column order), then the division
+            double ls = pend ? __dadd_rn(0.0, __dmul_rn(c_ls0, value1<PROTO>(p, c_fc, c_f0, c_f1))) : c_ls0;
+            ls = (c_meta & kDescN) ? __dadd_rn(ls, __dmul_rn(c_vn, xl)) : ls;
+            ls = (c_meta & kDescW) ? __dadd_rn(ls, __dmul_rn(c_vw, xw)) : ls;
+            const double a = __dsub_rn(c_b, ls);
+            const double dd = c_d;
+            Diag g;
+            g.d = dd;
+            g.r = c_rc;
+            double q = g.cand(a);
+            const bool guard = Diag::in_range(a) && c_rc != 0.0;
+            if (SAFE) {
+                const bool fix = act && !(guard && Diag::exact(a, dd, q));
+                if (__any_sync(FULL, fix)) {
+                    if (fix) q = Diag::slow_div(a, dd);
+                }
+            } else {
+                // outside the guard (a zero numerator, extreme magnitudes): the full division, in-loop;
+                // inside it the candidate's proof runs off the chain and a failure fails the solve
+                const bool fix = act && !guard;
+                if (__any_sync(FULL, fix)) {
+                    if (fix) q = Diag::slow_div(a, dd);
+                }
+                bad |= act && guard && !Diag::exact(a, dd, q);
+            }
+            // ---- publish (Alg.5 l.13-16)
+            const int ri = act ? r : 0;
+            if (PROTO == PROTO_FUSED) {
+                unsigned long long bits = (unsigned long long)__double_as_longlong(q);
+                const unsigned long long xb = bits;
+                bits = bits == kSentinel ? kCanonNaN : bits;
+                const unsigned long long e = (unsigned long long)epoch << 32;
+                st_relaxed_v2_u64_if(act, p.rec + 2 * (size_t)ri, e | (bits & 0xffffffffull), e | (bits >> 32));
+#ifdef SPTRSV_GRID_PLAINX  // measurement builds only
+                if (act) p.x[ri] = q;
+                (void)xb;
+#else
+                st_u64_if(act, reinterpret_cast<unsigned long long *>(p.x) + ri, xb);
+#endif
+            } else if (act) {
+                p.x[r] = q;
+                st_release_u32(p.flags + r, epoch);
+            }
+#ifdef SPTRSV_GRID_DEBUG_NAN  // measurement builds only: the first NaN result and its operands
+            if (p.trace && act && q != q && atomicCAS(p.trace + p.n, 0ull, 1ull) == 0ull) {
+                unsigned long long *t = p.trace + p.n;
+                t[1] = s; t[2] = band; t[3] = lane; t[4] = r; t[5] = c_meta;
+                t[6] = __double_as_longlong(c_b); t[7] = __double_as_longlong(c_d); t[8] = __double_as_longlong(c_ls0);
+                t[9] = __double_as_longlong(xl); t[10] = __double_as_longlong(xw); t[11] = __double_as_longlong(c_vn);
+                t[12] = __double_as_longlong(c_vw); t[13] = __double_as_longlong(c_rc); t[14] = __double_as_longlong(a);
+                t[15] = b; t[16] = hold; t[17] = rrow;
+            }
+#elif defined(SPTRSV_GRID_TRACEX)  // measurement builds only: the value computed for row r
+            if (p.trace && act) p.trace[r] = (unsigned long long)__double_as_longlong(q);
+            if (p.trace && act && r == 0) {
+                unsigned long long *t = p.trace + p.n;
+                t[0] = __double_as_longlong(c_b); t[1] = __double_as_longlong(c_d); t[2] = __double_as_longlong(c_rc);
+                t[3] = __double_as_longlong(c_ls0); t[4] = c_meta; t[5] = __double_as_longlong(xl);
+                t[6] = __double_as_longlong(xw); t[7] = __double_as_longlong(a); t[8] = __double_as_longlong(ls);
+                t[9] = s; t[10] = epoch; t[11] = pend;
+            }
+#else
+            if (p.trace && act) p.trace[r] = globaltimer_ns();
+#endif
+            xl = act ? q : xl;
+            // ---- the ring: the lane holding line s + kGridRing polls it now
+            if (lane == ((s + kGridRing) & 31)) {
+                rline = s + kGridRing;
+                rrow = ring_row(rline);
+                if (rrow >= 0) poll1<PROTO>(p, rrow, rw0, rw1);
+            }
+            fetch(s + 1);
+        }
+        if (stop && lane == 0) s_stop = 1;  // the producers skip the remaining blocks
+    }
+    if (!stop && !SAFE && __any_sync(FULL, bad || p.chain_div == 2)) {
+        if (lane == 0) {
+            atomicCAS(&p.st->error.v, 0u, kErrInexact);
+            st_relaxed_u32(&p.st->abort.v, 1u);
+        }
+    }
+}
+
+}  // namespace sptrsv_dev

@@ -22,6 +22,7 @@
 #include "solve_paper.cuh"
 #include "solve_chain.cuh"
 #include "solve_small.cuh"
+#include "solve_grid.cuh"
 #include "sptrsv.h"
 
 using namespace sptrsv_dev;
@@ -31,7 +32,7 @@ namespace {
 constexpr uint32_t kEpochResetAt = 0xFFFFFF00u;  // re-zero the flags before the epoch wraps
 
 // engines (SPTRSV_OPT_ENGINE values, include/sptrsv.h)
-enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_SMALL = 8, ENG_LEANP = 9 };
+enum { ENG_ONESHOT = 0, ENG_LEAN = 3, ENG_AUTO = 5, ENG_HYBRID = 6, ENG_CHAIN = 7, ENG_SMALL = 8, ENG_LEANP = 9, ENG_GRID = 10 };
 
 // ENGINE_SMALL (solve_small.cuh): the whole system in one CTA's shared memory.  Usable when it fits
 // (kSmallSmemMax bytes of dynamic shared memory, sm_100a allows 227 KB per CTA); AUTO picks it up to
@@ -134,6 +135,9 @@ struct sptrsv_handle_s {
     int64_t prev_deps = 0;  // dependencies on the previous row in solve order (ditto: chains)
     int64_t mid_breaks = 0; // rows off a 64-row boundary without a previous-row dependency (ditto)
     int64_t near_rows = 0;  // rows whose nearest dependency is < 256 rows away (ditto)
+    int32_t grid_m = 0;     // ENGINE_GRID: line length found by analyse (0 = none), rows violating its
+    int32_t grid_viol = 0;  // band order, north / west entries and far entries (solve_grid.cuh)
+    int64_t grid_fast = 0, grid_far = 0;
     // options
     int mode = 0;
     int threshold = 16;
@@ -570,6 +574,8 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         }
         if (n > 0) {
             k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->ws.indeg, h->ws.aout, tri_flags);
+            k_grid_probe<<<1, 32>>>(rowptr, colidx, n, h->ws.aout, tri_flags);
+            k_grid_check<<<(n + 255) / 256, 256>>>(rowptr, colidx, n, h->ws.aout);
             if (cudaGetLastError() != cudaSuccess) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
@@ -596,6 +602,10 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         h->prev_deps = (int64_t)(o.prev & 0xFFFFFFFFull);
         h->mid_breaks = o.mid_breaks;
         h->near_rows = (int64_t)(o.prev >> 32);
+        h->grid_m = n > 0 ? o.grid_m : 0;
+        h->grid_viol = o.grid_viol;
+        h->grid_fast = o.grid_fast;
+        h->grid_far = o.grid_far;
         if (n > 0) adopt_plan(h, o);
         else h->plan = PLAN_THREAD;
         h->since_reset = 0;
@@ -676,8 +686,23 @@ bool small_fits(const sptrsv_handle_s *h) {
     return h->n > 0 && h->n <= (1 << 20) && small_smem_bytes(h->n, h->nnz) <= kSmallSmemMax;
 }
 
+// ENGINE_GRID (solve_grid.cuh): usable when analyse found a line length m under which every row
+// keeps the band order (lower non-unit handles); AUTO takes it for grid-shaped factors -- m >= 32
+// columns, >= 32 lines, >= 1/2 of the off-diagonals north / west neighbours, >= 1/4 west (the
+// wavefront runs along the lines).
+bool grid_ok(const sptrsv_handle_s *h) {
+    return h->tri == 0 && h->n > 0 && h->grid_m >= 2 && h->grid_viol == 0 && h->nnz > h->n;
+}
+bool grid_auto(const sptrsv_handle_s *h) {
+    if (!grid_ok(h) || h->proto != PROTO_FUSED) return false;
+    const long long offdiag = h->nnz - h->n;
+    const long long lines = ((long long)h->n + h->grid_m - 1) / h->grid_m;
+    return h->grid_m >= 32 && lines >= 32 && 2 * h->grid_fast >= offdiag && 4 * h->prev_deps >= offdiag;
+}
+
 int resolve_engine(const sptrsv_handle_s *h) {
     if (h->engine == ENG_SMALL && small_fits(h)) return ENG_SMALL;
+    if (h->engine == ENG_GRID && grid_ok(h)) return ENG_GRID;
     const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;  // unit handles store no diagonal
     // chains: >= 1/4 of the dependencies on the previous row AND runs of such rows long enough for
     // CHAIN's in-warp steps to pay (mean run n / (rows without one) >= 64 rows, one CHAIN warp): with
@@ -701,6 +726,7 @@ int resolve_engine(const sptrsv_handle_s *h) {
     // (not when the user asked for warp-level rows: MODE 2 / 3 plans keep their warp engine)
     if (h->engine == ENG_AUTO && h->mode <= 1 && near && !pure_chain && h->n <= kSmallAutoN && small_fits(h))
         return ENG_SMALL;
+    if (h->engine == ENG_AUTO && h->mode <= 1 && grid_auto(h)) return ENG_GRID;
     if (h->plan != PLAN_THREAD)  // ONE-SHOT has no sub-warp rows
         return (h->engine == ENG_ONESHOT && !h->tri && h->n_sub_tasks == 0) ? ENG_ONESHOT : ENG_HYBRID;
     if (h->engine != ENG_AUTO) return (h->tri && h->engine == ENG_ONESHOT) ? ENG_LEAN : h->engine;
@@ -827,6 +853,26 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
             L->key = (7500000 + h->proto * 100000 + h->tri * 10000 + h->plan * 1000 + ct / 64) ^ (int)L->grid.x * 7919;
             return SPTRSV_OK;
         }
+    }
+    if (engine == ENG_GRID) {  // wavefront bands of 32 columns, one CTA per band (solve_grid.cuh)
+        static const lean_fn tab[2][2] = {{k_solve_grid<PROTO_FLAGS, false>, k_solve_grid<PROTO_FUSED, false>},
+                                          {k_solve_grid<PROTO_FLAGS, true>, k_solve_grid<PROTO_FUSED, true>}};
+        L->fn = (const void *)tab[h->chain_div == 1 ? 1 : 0][h->proto ? 1 : 0];
+        L->smem = grid_smem_bytes(32 * std::max(1, h->max_row));
+        static size_t attr_set[64][4] = {};  // per device and kernel: the dynamic smem limit raised so far
+        size_t &cur = attr_set[h->device & 63][(h->chain_div == 1 ? 2 : 0) + (h->proto ? 1 : 0)];
+        if (cur < L->smem) {
+            if (cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess) {
+                (void)cudaGetLastError();
+                return SPTRSV_ERR_CUDA;
+            }
+            cur = L->smem;
+        }
+        L->cta = 32 * (1 + kGridProd);
+        L->grid = dim3((unsigned)((h->grid_m + 31) / 32));
+        L->block = dim3((unsigned)L->cta);
+        L->key = (10000000 + h->proto * 100000 + (h->chain_div == 1 ? 500 : 0)) ^ (int)L->grid.x * 7919;
+        return SPTRSV_OK;
     }
     if (L->engine == ENG_CHAIN) {  // warp-sequential in-warp chains (solve_chain.cuh): 64..256 threads
         const int K = h->rows_per_lane == 1 ? 1 : 2;  // other values: the default 2
@@ -1004,6 +1050,9 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.poll_one = h->poll_one;
     p.split_last = h->split_last;
     p.chain_div = h->chain_div;
+    p.grid_m = h->grid_m;
+    p.grid_lines = h->grid_m > 0 ? (int32_t)(((long long)h->n + h->grid_m - 1) / h->grid_m) : 0;
+    p.grid_ecap = 32 * std::max(1, h->max_row);
     p.x_host = x_host;
     p.bflag = bflag;
     p.bseq = bseq;
@@ -1372,9 +1421,10 @@ int sptrsv_set_option(sptrsv_handle_t h, int key, int64_t value) {
             return SPTRSV_OK;
         case SPTRSV_OPT_ENGINE:
             if (value != ENG_ONESHOT && value != ENG_LEAN && value != ENG_AUTO && value != ENG_HYBRID &&
-                value != ENG_CHAIN && value != ENG_SMALL && value != ENG_LEANP)
+                value != ENG_CHAIN && value != ENG_SMALL && value != ENG_LEANP && value != ENG_GRID)
                 return SPTRSV_ERR_INVALID_ARG;
             if (value == ENG_SMALL && !small_fits(h)) return SPTRSV_ERR_INVALID_ARG;  // does not fit one CTA
+            if (value == ENG_GRID && !grid_ok(h)) return SPTRSV_ERR_INVALID_ARG;    // not grid-shaped
             h->engine = (int)value;
             return SPTRSV_OK;
         case SPTRSV_OPT_ROWS_PER_LANE:

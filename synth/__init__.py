@@ -236,6 +236,30 @@ def gen_grid(g: int = 2048, seed: int = 3, ones: bool = False, name: str | None 
                         diag=4.0)
 
 
+def gen_stencil(nx: int, ny: int, nz: int = 1, seed: int = 12, rows: int | None = None,
+                name: str | None = None) -> CSRSystem:
+    """Lower factor pattern of an nx x ny (x nz) 5-point (7-point) grid, row-major
+    i = (z*ny + y)*nx + x: off-diagonals at i-1 (x > 0), i-nx (y > 0), i-nx*ny (z > 0); the
+    standard values (off-diagonals U[-0.5, 0.5], diag 1 + sum |L_ij|, x_true ~ U[1, 2]).
+    ``rows``: keep only the leading rows (a ragged last grid line)."""
+    rng = np.random.default_rng(seed)
+    n = nx * ny * nz
+    i = np.arange(n, dtype=np.int64)
+    x, y, z = i % nx, (i // nx) % ny, i // (nx * ny)
+    parts_r, parts_c = [i[x > 0]], [i[x > 0] - 1]
+    parts_r.append(i[y > 0]), parts_c.append(i[y > 0] - nx)
+    if nz > 1:
+        parts_r.append(i[z > 0]), parts_c.append(i[z > 0] - nx * ny)
+    r_all, c_all = np.concatenate(parts_r), np.concatenate(parts_c)
+    if rows is not None:
+        keep = r_all < rows
+        r_all, c_all, n = r_all[keep], c_all[keep], rows
+    order = np.lexsort((c_all, r_all))
+    rp, ci = _assemble(n, (r_all[order], c_all[order]))
+    return from_pattern(name or f"stencil{nx}x{ny}x{nz}", rp, ci, rng,
+                        {"seed": seed, "nx": nx, "ny": ny, "nz": nz})
+
+
 def gen_c3(seed: int = 3, ones: bool = False) -> CSRSystem:
     return gen_grid(2048, seed, ones, name="c3")
 
