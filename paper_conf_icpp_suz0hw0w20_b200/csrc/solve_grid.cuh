@@ -127,63 +127,67 @@ constexpr int kGridDesc = 48;             // descriptor ring (lines): line y is 
 constexpr int kGridRaw = 64;              // raw CSR ring (lines)
 constexpr int kGridA1 = 8;                // rowptr / b staged this many blocks before production
 constexpr int kGridA2 = 4;                // entries staged this many blocks before production
-constexpr int kGridSlack = 16;  // a band that found lane 0's west operand missing resumes only once
-                                // the line this far ahead is published (so its next polls find their
-                                // records: a band tracking its predecessor at the minimum lag would
-                                // pay a round trip on every step)
+constexpr int kGridWarps = 2 + kGridProd;  // consumer, producers, ring
 static_assert(kGridA1 == 2 * kGridA2, "one cp.async wait covers both staging distances");
 static_assert(kGridBlk * (kGridA1 + 1) <= kGridRaw, "raw ring too small");
 
-enum : int { kDescAct = 1, kDescN = 2, kDescW = 4, kDescFar = 8 /* far entry not folded: poll it */ };
+enum : int { kDescN = 2, kDescW = 4, kDescFar = 8 /* far entry not folded: poll it */ };
 
 __host__ __device__ constexpr size_t grid_smem_bytes(int ecap) {
-    return (size_t)kGridDesc * 32 * (6 * 8 + 2 * 4) + (size_t)kGridRaw * (64 * 4 + 32 * 8 + (size_t)ecap * 12);
+    return (size_t)kGridDesc * 32 * (6 * 8 + 3 * 4) + (size_t)kGridDesc * 8 +
+           (size_t)kGridRaw * (64 * 4 + 32 * 8 + (size_t)ecap * 12);
 }
 
 __device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
-#ifdef SPTRSV_GRID_NOASYNC  // measurement builds only: synchronous staging through registers
-__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
-    *reinterpret_cast<int32_t *>(dst) = __ldcg(reinterpret_cast<const int32_t *>(src));
-}
-__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
-    *reinterpret_cast<double *>(dst) = __ldcg(reinterpret_cast<const double *>(src));
-}
-#else
 __device__ __forceinline__ void cp_async4(void *dst, const void *src) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async8(void *dst, const void *src) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
-#endif
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-#ifdef SPTRSV_GRID_DEBUG_OOB  // measurement builds only: the first out-of-range index, clamped
-__device__ __forceinline__ long long gchk(const SolveParams &p, long long i, long long lim, int tag) {
-    if (i < 0 || i >= lim) {
-        unsigned long long *t = p.trace + p.n;  // after the publish timestamps
-        if (p.trace && atomicCAS(t + 32, 0ull, 1ull) == 0ull) {
-            t[33] = tag; t[34] = i; t[35] = lim; t[36] = blockIdx.x; t[37] = threadIdx.x;
-        }
-        return 0;
-    }
-    return i;
+
+// the consumer / producer barrier (named barrier 1, warps 0 .. kGridProd; the ring warp runs free)
+__device__ __forceinline__ void bar_sync_cp() {
+    asm volatile("bar.sync 1, %0;" ::"n"(32 * (1 + kGridProd)) : "memory");
 }
-#define GCHK(i, lim, tag) gchk(p, (i), (lim), (tag))
-#else
-#define GCHK(i, lim, tag) (i)
-#endif
+__device__ __forceinline__ int ld_volatile_s32(const int *a) {
+    int v;
+    asm volatile("ld.volatile.shared.s32 %0, [%1];" : "=r"(v) : "r"((unsigned)__cvta_generic_to_shared(a)) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_volatile_s32(int *a, int v) {
+    asm volatile("st.volatile.shared.s32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(a)), "r"(v) : "memory");
+}
+
+// a poll issued only when `go` holds: one predicated load for the FUSED records (no branch)
+template <int PROTO>
+__device__ __forceinline__ void poll1_if(bool go, const SolveParams &p, int c, unsigned long long &w0,
+                                         unsigned long long &w1) {
+    if (PROTO == PROTO_FUSED) {
+        asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];\n\t}"
+                     : "+l"(w0), "+l"(w1)
+                     : "l"(p.rec + 2 * (size_t)(go ? c : 0)), "r"((unsigned)go)
+                     : "memory");
+    } else if (go) {
+        poll1<PROTO>(p, c, w0, w1);
+    }
+}
 
 template <int PROTO, bool SAFE>
-__global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolveParams p) {
+__global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p) {
     extern __shared__ __align__(16) unsigned char gsm[];
     __shared__ uint32_t s_blk, s_epoch, s_stop;
+    __shared__ int s_ring, s_cons;  // lines whose west value is in s_west; the consumer's block start
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         cta_ticket(p, s_blk, s_epoch);
         s_stop = 0;
+        s_ring = 0;
+        s_cons = 0;
     }
     __syncthreads();
     if (s_blk == kStaleBlk) return;
@@ -200,11 +204,64 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
     double *d_vn = d_ls0 + kGridDesc * 32, *d_vw = d_vn + kGridDesc * 32, *d_b = d_vw + kGridDesc * 32;
     double *d_d = d_b + kGridDesc * 32, *d_rc = d_d + kGridDesc * 32;
     int32_t *d_meta = reinterpret_cast<int32_t *>(d_rc + kGridDesc * 32), *d_fc = d_meta + kGridDesc * 32;
-    int32_t *s_rp = d_fc + kGridDesc * 32;                                   // [raw][64]
+    int32_t *d_row = d_fc + kGridDesc * 32;                                  // [desc][32]: row, -1 = none
+    double *s_west = reinterpret_cast<double *>(d_row + kGridDesc * 32);     // [desc]: lane 0's west x
+    int32_t *s_rp = reinterpret_cast<int32_t *>(s_west + kGridDesc);        // [raw][64]
     double *s_b = reinterpret_cast<double *>(s_rp + kGridRaw * 64);          // [raw][32]
     double *s_val = s_b + kGridRaw * 32;                                     // [raw][E]
     int32_t *s_col = reinterpret_cast<int32_t *>(s_val + (size_t)kGridRaw * E);  // [raw][E]
 
+    const bool ring_on = band > 0;
+    if (warp == kGridWarps - 1) {
+        // ================================================================ the ring (band > 0)
+        // Lane 0's west operand is band k-1's lane 31: this warp polls those records 32 lines at a
+        // time (lane j: line base + j), stores the values of the ready prefix in s_west and advances
+        // s_ring, one round trip per pass -- the consumer only reads shared memory.  It stays within
+        // kGridDesc - 8 lines of the consumer's block start (s_west's slots).
+        if (!ring_on) return;
+        int base = 0;
+        uint32_t bo = p.backoff_min, idl = 0;
+        while (base < lines) {
+            const int y = base + lane;
+            const unsigned wr = (unsigned)y * (unsigned)m + (unsigned)x0 - 1u;
+            const bool need = y < lines && wr < n;
+            const bool room = y < ld_volatile_s32(&s_cons) + kGridDesc - 8;
+            unsigned long long w0 = 0, w1 = 0;
+            if (need && room) poll1<PROTO>(p, (int)wr, w0, w1);
+            const bool rdy = room && (!need || ready1<PROTO>(w0, w1, epoch));
+            const unsigned mask = __ballot_sync(FULL, rdy);
+            const int L = __ffs(~mask) - 1 < 0 ? 32 : __ffs(~mask) - 1;  // ready prefix
+            if (lane < L && need) s_west[y % kGridDesc] = value1<PROTO>(p, (int)wr, w0, w1);
+            __syncwarp();
+            if (L > 0) {
+                __threadfence_block();
+                if (lane == 0) st_volatile_s32(&s_ring, base + L);
+                base += L;
+                bo = p.backoff_min;
+                idl = 0;
+                continue;
+            }
+            if (ld_volatile_s32((const int *)&s_stop)) return;
+            if (bo) nanosleep_ns(bo);
+            bo = min(max(bo * 2u, 32u), p.backoff_max);
+            ++idl;
+            if ((idl & 63u) == 0 || (p.spin_limit && idl >= p.spin_limit)) {
+                uint32_t ab = 0;
+                if (lane == 0) {
+                    if (p.spin_limit && idl >= p.spin_limit) {
+                        atomicCAS(&p.st->error.v, 0u, kErrTimeout);
+                        st_relaxed_u32(&p.st->abort.v, 1u);
+                    }
+                    ab = ld_relaxed_u32(&p.st->abort.v);
+                }
+                if (__shfl_sync(FULL, ab, 0)) {
+                    if (lane == 0) st_volatile_s32((int *)&s_stop, 1);
+                    return;
+                }
+            }
+        }
+        return;
+    }
     if (warp > 0) {
         // ================================================================ producers
         const int w = warp - 1;
@@ -218,9 +275,9 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
             const int k = line_rows(y, row0);
             if (k == 0) return;
             int32_t *rp = s_rp + (y & (kGridRaw - 1)) * 64;
-            if (lane <= k) cp_async4(rp + lane, p.rowptr + GCHK((long long)row0 + lane, (long long)n + 1, 1));
-            if (lane == 0 && k == 32) cp_async4(rp + 32, p.rowptr + GCHK((long long)row0 + 32, (long long)n + 1, 2));
-            if (lane < k) cp_async8(s_b + (y & (kGridRaw - 1)) * 32 + lane, p.b + GCHK((long long)row0 + lane, (long long)n, 3));
+            if (lane <= k) cp_async4(rp + lane, p.rowptr + row0 + lane);
+            if (lane == 0 && k == 32) cp_async4(rp + 32, p.rowptr + row0 + 32);
+            if (lane < k) cp_async8(s_b + (y & (kGridRaw - 1)) * 32 + lane, p.b + row0 + lane);
         };
         auto stage_ent = [&](int y) {  // entries of line y (its rowptr slice complete in the ring)
             unsigned row0;
@@ -229,8 +286,8 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
             const int sl = y & (kGridRaw - 1);
             const int lo = s_rp[sl * 64], hi = s_rp[sl * 64 + k];
             for (int e = lo + lane; e < hi; e += 32) {
-                cp_async4(s_col + (size_t)sl * E + GCHK(e - lo, E, 6), p.colidx + GCHK(e, p.nnz, 4));
-                cp_async8(s_val + (size_t)sl * E + GCHK(e - lo, E, 7), p.val + GCHK(e, p.nnz, 5));
+                cp_async4(s_col + (size_t)sl * E + (e - lo), p.colidx + e);
+                cp_async8(s_val + (size_t)sl * E + (e - lo), p.val + e);
             }
         };
         auto produce = [&](int y) {  // descriptors of line y from its staged raw rows
@@ -252,14 +309,14 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
                 const int jn = hi - 2 - (int)hw;
                 const bool hn = jn >= lo && c[jn] == r - m;
                 const int jf = jn - (int)hn;
-                meta = kDescAct | (hn ? kDescN : 0) | (hw ? kDescW : 0);
+                meta = (hn ? kDescN : 0) | (hw ? kDescW : 0);
                 vw = hw ? v[hi - 2] : 0.0;
                 vn = hn ? v[jn] : 0.0;
                 if (jf >= lo) {  // the far entry (at most one: k_grid_check)
                     fc = c[jf];
                     const double vf = v[jf];
                     unsigned long long f0, f1;
-                    poll1<PROTO>(p, (int)GCHK(fc, (long long)n, 8), f0, f1);
+                    poll1<PROTO>(p, fc, f0, f1);
                     if (ready1<PROTO>(f0, f1, epoch)) {
                         ls0 = __dadd_rn(0.0, __dmul_rn(vf, value1<PROTO>(p, fc, f0, f1)));
                     } else {
@@ -281,6 +338,7 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
             d_rc[ds] = rc;
             d_meta[ds] = meta;
             d_fc[ds] = fc;
+            d_row[ds] = act ? r : -1;
         };
         // prologue: the raw rows of the first lines, then the descriptors of lines [0, kGridBlk]
         for (int y = w; y < kGridBlk + 1 + kGridBlk * kGridA1; y += kGridProd) stage_rp(y);
@@ -293,13 +351,9 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
         __syncwarp();
         for (int y = w; y <= kGridBlk; y += kGridProd) produce(y);
         for (int b = 0; b < nblocks; ++b) {
-            __syncthreads();  // block b begins: lines <= B*b + B are in the descriptor ring
-            if (s_stop) continue;
-#ifdef SPTRSV_GRID_WAITALL  // measurement builds only
-            cp_async_wait<0>();
-#else
+            bar_sync_cp();  // block b begins: lines <= B*b + B are in the descriptor ring
+            if (ld_volatile_s32((const int *)&s_stop)) continue;
             cp_async_wait<kGridA2 - 1>();
-#endif
             __syncwarp();
             const int y0 = kGridBlk * b + kGridBlk + 1;
             for (int y = y0 + w; y < y0 + kGridBlk; y += kGridProd) {
@@ -313,177 +367,132 @@ __global__ void __launch_bounds__(32 * (1 + kGridProd), 1) k_solve_grid(SolvePar
         return;
     }
     // ==================================================================== consumer (warp 0)
-    const int x = x0 + lane;
-    const bool colok = lane < nl;
-    const bool ring_on = band > 0;
-    auto ring_row = [&](int y) -> int {  // lane 0's west neighbour on line y (band k-1, lane 31)
-        if (!ring_on || y >= lines) return -1;
-        const unsigned r = (unsigned)y * (unsigned)m + (unsigned)x0 - 1u;
-        return r < n ? (int)r : -1;
+    // the row of a step (line s - lane) comes from the descriptor ring through a per-lane cursor
+    // (line fy, its ring slot fsl), advanced once per step; the NEXT step's row is fetched at the top
+    // of each step so its shared-memory loads overlap the current chain
+    int fy = -lane, fsl = lane == 0 ? 0 : kGridDesc - lane;
+    struct Row {
+        int r, meta, fc;
+        double ls0, vn, vw, b, d, rc;
     };
-    // the row of the next step (line s + 1 - lane), read from the descriptor ring one step ahead
-    int c_r = -1, c_meta = 0, c_fc = 0;
-    double c_ls0 = 0, c_vn = 0, c_vw = 0, c_b = 0, c_d = 1, c_rc = 1;
-    unsigned long long c_f0 = 0, c_f1 = 0;
-    auto fetch = [&](int s1) {
-        const int y = s1 - lane;
-        const unsigned r = (unsigned)y * (unsigned)m + (unsigned)x;
-        const bool act = colok && y >= 0 && y < lines && r < n;
-        const int ds = ((act ? y : 0) % kGridDesc) * 32 + lane;
-        c_meta = act ? d_meta[ds] : 0;
-        c_ls0 = d_ls0[ds];
-        c_vn = d_vn[ds];
-        c_vw = d_vw[ds];
-        c_b = d_b[ds];
-        c_d = d_d[ds];
-        c_rc = d_rc[ds];
-        c_fc = d_fc[ds];
-        c_r = act ? (int)r : -1;
-        if (c_meta & kDescFar) poll1<PROTO>(p, (int)GCHK(c_fc, (long long)n, 9), c_f0, c_f1);
+    auto fetch = [&](Row &o) {
+        const int ds = fsl * 32 + lane;
+        const int row = d_row[ds];
+        o.r = (unsigned)fy < (unsigned)lines ? row : -1;
+        o.meta = d_meta[ds];
+        o.ls0 = d_ls0[ds];
+        o.vn = d_vn[ds];
+        o.vw = d_vw[ds];
+        o.b = d_b[ds];
+        o.d = d_d[ds];
+        o.rc = d_rc[ds];
+        o.fc = d_fc[ds];
+        o.meta = o.r >= 0 ? o.meta : 0;
+        ++fy;
+        fsl = fsl == kGridDesc - 1 ? 0 : fsl + 1;
     };
-    // ---- the ring: the lane holding line y polls its record kGridRing steps before step y
-    unsigned long long rw0 = 0, rw1 = 0;
-    int rrow = -1, rline = -1;
-    if (lane < kGridRing) {
-        rline = lane;
-        rrow = ring_row(lane);
-        if (rrow >= 0) poll1<PROTO>(p, rrow, rw0, rw1);
-    }
+    Row cur, nxt;
     double xl = 0.0;  // this lane's latest x (the north operand of its next row)
     bool bad = false, stop = false;
-    uint32_t backoff = p.backoff_min, idle = 0;
+    int ring_have = ring_on ? 0 : 0x7fffffff;  // lines whose west value the ring warp has stored
+    const unsigned long long ep = (unsigned long long)epoch << 32;
+    // the rare cases wait here: the ring behind (lane 0's west not stored yet), or a far entry that was
+    // not published when its row was produced (polled in place); backoff and watchdog as everywhere
+    auto wait_for = [&](int s, bool pend, int fc, double &xf) -> bool {
+        uint32_t bo = p.backoff_min, idl = 0;
+        bool have_f = !pend;
+        while (true) {
+            if (ring_have <= s) ring_have = ld_volatile_s32(&s_ring);
+            if (!have_f) {
+                unsigned long long f0, f1;
+                poll1<PROTO>(p, fc, f0, f1);
+                if (ready1<PROTO>(f0, f1, epoch)) {
+                    xf = value1<PROTO>(p, fc, f0, f1);
+                    have_f = true;
+                }
+            }
+            if (!__any_sync(FULL, ring_have <= s || !have_f)) return true;
+            if (ld_volatile_s32((const int *)&s_stop)) return false;
+            if (bo) nanosleep_ns(bo);
+            bo = min(max(bo * 2u, 32u), p.backoff_max);
+            ++idl;
+            if ((idl & 63u) == 0 || (p.spin_limit && idl >= p.spin_limit)) {
+                uint32_t ab = 0;
+                if (lane == 0) {
+                    if (p.spin_limit && idl >= p.spin_limit) {
+                        atomicCAS(&p.st->error.v, 0u, kErrTimeout);
+                        st_relaxed_u32(&p.st->abort.v, 1u);
+                    }
+                    ab = ld_relaxed_u32(&p.st->abort.v);
+                }
+                if (__shfl_sync(FULL, ab, 0)) return false;
+            }
+        }
+    };
     for (int b = 0; b < nblocks; ++b) {
-        __syncthreads();
+        if (lane == 0) st_volatile_s32(&s_cons, kGridBlk * b);
+        bar_sync_cp();
         if (stop) continue;
-        if (b == 0) fetch(0);
+        if (b == 0) fetch(cur);
         const int s_end = min(steps, kGridBlk * (b + 1));
         for (int s = kGridBlk * b; s < s_end; ++s) {
-            const int r = c_r;
+            fetch(nxt);  // the next step's row (its lines were produced before this block)
+            const int r = cur.r;
             const bool act = r >= 0;
-            const bool pend = (c_meta & kDescFar) != 0;
-            // ---- operands produced outside this warp: lane 0's west (the ring), pending far entries
-            const int hold = s & 31;
-            const bool ring_ok = lane != hold || rrow < 0 || ready1<PROTO>(rw0, rw1, epoch);
-            bool ok = ring_ok && (!pend || ready1<PROTO>(c_f0, c_f1, epoch));
-            if (__any_sync(FULL, !ok)) {  // not there yet: wait (warp-uniform, backoff, watchdog)
-                const bool late = __any_sync(FULL, !ring_ok);
-                const int trow = late && lane == 0 ? ring_row(min(s + kGridSlack, lines - 1)) : -1;
-                bool tok = trow < 0;
-                while (true) {
-                    if (lane == hold && rrow >= 0 && !ready1<PROTO>(rw0, rw1, epoch)) poll1<PROTO>(p, rrow, rw0, rw1);
-                    if (pend && !ready1<PROTO>(c_f0, c_f1, epoch)) poll1<PROTO>(p, c_fc, c_f0, c_f1);
-                    if (!tok) {
-                        unsigned long long t0, t1;
-                        poll1<PROTO>(p, (int)GCHK(trow, (long long)n, 10), t0, t1);
-                        tok = ready1<PROTO>(t0, t1, epoch);
-                    }
-                    ok = tok && (lane != hold || rrow < 0 || ready1<PROTO>(rw0, rw1, epoch)) &&
-                         (!pend || ready1<PROTO>(c_f0, c_f1, epoch));
-                    if (!__any_sync(FULL, !ok)) break;
-                    if (backoff) nanosleep_ns(backoff);
-                    backoff = min(max(backoff * 2u, 32u), p.backoff_max);
-                    ++idle;
-                    if ((idle & 63u) == 0 || (p.spin_limit && idle >= p.spin_limit)) {
-                        uint32_t ab = 0;
-                        if (lane == 0) {
-                            if (p.spin_limit && idle >= p.spin_limit) {
-                                atomicCAS(&p.st->error.v, 0u, kErrTimeout);
-                                st_relaxed_u32(&p.st->abort.v, 1u);
-                            }
-                            ab = ld_relaxed_u32(&p.st->abort.v);
-                        }
-                        if (__shfl_sync(FULL, ab, 0)) {
-                            stop = true;
-                            break;
-                        }
-                    }
+            const bool pend = (cur.meta & kDescFar) != 0;
+            double xf = 0.0;
+            // lane 0's west (line s) from the ring warp; pending far entries (rare)
+            if (ring_have <= s && s < lines) ring_have = ld_volatile_s32(&s_ring);
+            if (__any_sync(FULL, (ring_have <= s && s < lines) || pend)) {
+                if (!wait_for(s < lines ? s : -1, pend, cur.fc, xf)) {
+                    stop = true;
+                    break;
                 }
-                if (stop) break;
-                // the polls in flight for the next lines predate the wait: issue them again
-                if (late && rrow >= 0 && rline > s) poll1<PROTO>(p, rrow, rw0, rw1);
-                backoff = p.backoff_min;
-                idle = 0;
             }
+            const double wv = s_west[(s < lines ? s : 0) % kGridDesc];
             double xw = __shfl_up_sync(FULL, xl, 1);
-            double rv = 0.0;
-            if (lane == hold && rrow >= 0) rv = value1<PROTO>(p, rrow, rw0, rw1);
-            rv = __shfl_sync(FULL, rv, hold);
-            if (lane == 0) xw = rv;
+            xw = lane == 0 ? wv : xw;
             // ---- Alg.1's row: far (ls0), north, west (column order), then the division
-            double ls = pend ? __dadd_rn(0.0, __dmul_rn(c_ls0, value1<PROTO>(p, c_fc, c_f0, c_f1))) : c_ls0;
-            ls = (c_meta & kDescN) ? __dadd_rn(ls, __dmul_rn(c_vn, xl)) : ls;
-            ls = (c_meta & kDescW) ? __dadd_rn(ls, __dmul_rn(c_vw, xw)) : ls;
-            const double a = __dsub_rn(c_b, ls);
-            const double dd = c_d;
+            double ls = pend ? __dadd_rn(0.0, __dmul_rn(cur.ls0, xf)) : cur.ls0;
+            ls = (cur.meta & kDescN) ? __dadd_rn(ls, __dmul_rn(cur.vn, xl)) : ls;
+            ls = (cur.meta & kDescW) ? __dadd_rn(ls, __dmul_rn(cur.vw, xw)) : ls;
+            const double a = __dsub_rn(cur.b, ls);
             Diag g;
-            g.d = dd;
-            g.r = c_rc;
+            g.d = cur.d;
+            g.r = cur.rc;
             double q = g.cand(a);
-            const bool guard = Diag::in_range(a) && c_rc != 0.0;
+            const bool guard = Diag::in_range(a) && cur.rc != 0.0;
             if (SAFE) {
-                const bool fix = act && !(guard && Diag::exact(a, dd, q));
+                const bool fix = act && !(guard && Diag::exact(a, cur.d, q));
                 if (__any_sync(FULL, fix)) {
-                    if (fix) q = Diag::slow_div(a, dd);
+                    if (fix) q = Diag::slow_div(a, cur.d);
                 }
             } else {
                 // outside the guard (a zero numerator, extreme magnitudes): the full division, in-loop;
                 // inside it the candidate's proof runs off the chain and a failure fails the solve
                 const bool fix = act && !guard;
                 if (__any_sync(FULL, fix)) {
-                    if (fix) q = Diag::slow_div(a, dd);
+                    if (fix) q = Diag::slow_div(a, cur.d);
                 }
-                bad |= act && guard && !Diag::exact(a, dd, q);
+                bad |= act && guard && !Diag::exact(a, cur.d, q);
             }
-            // ---- publish (Alg.5 l.13-16)
+            // ---- publish (Alg.5 l.13-16); GRID records are read by GRID warps only (no shared-
+            // memory sentinel to avoid)
             const int ri = act ? r : 0;
             if (PROTO == PROTO_FUSED) {
-                unsigned long long bits = (unsigned long long)__double_as_longlong(q);
-                const unsigned long long xb = bits;
-                bits = bits == kSentinel ? kCanonNaN : bits;
-                const unsigned long long e = (unsigned long long)epoch << 32;
-                st_relaxed_v2_u64_if(act, p.rec + 2 * (size_t)ri, e | (bits & 0xffffffffull), e | (bits >> 32));
-#ifdef SPTRSV_GRID_PLAINX  // measurement builds only
-                if (act) p.x[ri] = q;
-                (void)xb;
-#else
-                st_u64_if(act, reinterpret_cast<unsigned long long *>(p.x) + ri, xb);
-#endif
+                const unsigned long long bits = (unsigned long long)__double_as_longlong(q);
+                st_relaxed_v2_u64_if(act, p.rec + 2 * (size_t)ri, ep | (bits & 0xffffffffull), ep | (bits >> 32));
+                st_u64_if(act, reinterpret_cast<unsigned long long *>(p.x) + ri, bits);
             } else if (act) {
                 p.x[r] = q;
                 st_release_u32(p.flags + r, epoch);
             }
-#ifdef SPTRSV_GRID_DEBUG_NAN  // measurement builds only: the first NaN result and its operands
-            if (p.trace && act && q != q && atomicCAS(p.trace + p.n, 0ull, 1ull) == 0ull) {
-                unsigned long long *t = p.trace + p.n;
-                t[1] = s; t[2] = band; t[3] = lane; t[4] = r; t[5] = c_meta;
-                t[6] = __double_as_longlong(c_b); t[7] = __double_as_longlong(c_d); t[8] = __double_as_longlong(c_ls0);
-                t[9] = __double_as_longlong(xl); t[10] = __double_as_longlong(xw); t[11] = __double_as_longlong(c_vn);
-                t[12] = __double_as_longlong(c_vw); t[13] = __double_as_longlong(c_rc); t[14] = __double_as_longlong(a);
-                t[15] = b; t[16] = hold; t[17] = rrow;
-            }
-#elif defined(SPTRSV_GRID_TRACEX)  // measurement builds only: the value computed for row r
-            if (p.trace && act) p.trace[r] = (unsigned long long)__double_as_longlong(q);
-            if (p.trace && act && r == 0) {
-                unsigned long long *t = p.trace + p.n;
-                t[0] = __double_as_longlong(c_b); t[1] = __double_as_longlong(c_d); t[2] = __double_as_longlong(c_rc);
-                t[3] = __double_as_longlong(c_ls0); t[4] = c_meta; t[5] = __double_as_longlong(xl);
-                t[6] = __double_as_longlong(xw); t[7] = __double_as_longlong(a); t[8] = __double_as_longlong(ls);
-                t[9] = s; t[10] = epoch; t[11] = pend;
-            }
-#else
-            if (p.trace && act) p.trace[r] = globaltimer_ns();
-#endif
             xl = act ? q : xl;
-            // ---- the ring: the lane holding line s + kGridRing polls it now
-            if (lane == ((s + kGridRing) & 31)) {
-                rline = s + kGridRing;
-                rrow = ring_row(rline);
-                if (rrow >= 0) poll1<PROTO>(p, rrow, rw0, rw1);
-            }
-            fetch(s + 1);
+            cur = nxt;
         }
-        if (stop && lane == 0) s_stop = 1;  // the producers skip the remaining blocks
+        if (stop && lane == 0) st_volatile_s32((int *)&s_stop, 1);  // producers and ring skip the rest
     }
+    if (lane == 0) st_volatile_s32(&s_cons, 0x3fffffff);
     if (!stop && !SAFE && __any_sync(FULL, bad || p.chain_div == 2)) {
         if (lane == 0) {
             atomicCAS(&p.st->error.v, 0u, kErrInexact);

@@ -868,7 +868,7 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
             }
             cur = L->smem;
         }
-        L->cta = 32 * (1 + kGridProd);
+        L->cta = 32 * kGridWarps;
         L->grid = dim3((unsigned)((h->grid_m + 31) / 32));
         L->block = dim3((unsigned)L->cta);
         L->key = (10000000 + h->proto * 100000 + (h->chain_div == 1 ? 500 : 0)) ^ (int)L->grid.x * 7919;
