@@ -163,6 +163,23 @@ __device__ __forceinline__ void st_volatile_s32(int *a, int v) {
     asm volatile("st.volatile.shared.s32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(a)), "r"(v) : "memory");
 }
 
+// GRID's publishes: predicated stores WITHOUT a compiler memory clobber, so the scheduler may overlap
+// them with the next step's shared-memory loads (they only depend on the quotient)
+__device__ __forceinline__ void grid_st_rec_if(bool pr, unsigned long long *a, unsigned long long lo,
+                                               unsigned long long hi) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};\n\t}" ::"l"(a),
+                 "l"(lo), "l"(hi), "r"((unsigned)pr));
+}
+__device__ __forceinline__ void grid_st_x_if(bool pr, unsigned long long *a, unsigned long long v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.u64 [%0], %1;\n\t}" ::"l"(a), "l"(v),
+                 "r"((unsigned)pr));
+}
+__device__ __forceinline__ int ld_volatile_s32_nc(const int *a) {  // no compiler memory clobber
+    int v;
+    asm volatile("ld.volatile.shared.s32 %0, [%1];" : "=r"(v) : "r"((unsigned)__cvta_generic_to_shared(a)));
+    return v;
+}
+
 // a poll issued only when `go` holds: one predicated load for the FUSED records (no branch)
 template <int PROTO>
 __device__ __forceinline__ void poll1_if(bool go, const SolveParams &p, int c, unsigned long long &w0,
@@ -391,7 +408,6 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         ++fy;
         fsl = fsl == kGridDesc - 1 ? 0 : fsl + 1;
     };
-    Row cur, nxt;
     double xl = 0.0;  // this lane's latest x (the north operand of its next row)
     bool bad = false, stop = false;
     int ring_have = ring_on ? 0 : 0x7fffffff;  // lines whose west value the ring warp has stored
@@ -429,67 +445,102 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             }
         }
     };
+    const bool has_far = p.grid_far != 0;
+    // one step (line s - lane; lane 0's west value in s_west slot ws): Alg.1's row, the division, the
+    // publish.  `cur` is this step's row, `nxt` receives the next one (two register sets alternate)
+    auto step = [&](Row &cur, Row &nxt, int s, int ws) -> bool {
+        fetch(nxt);  // the next step's row (its lines were produced before this block)
+        const int r = cur.r;
+        const bool act = r >= 0;
+        const bool pend = has_far && (cur.meta & kDescFar) != 0;
+        double xf = 0.0;
+        if (has_far && __any_sync(FULL, pend)) {  // a far entry not published when its row was produced
+            if (!wait_for(-1, pend, cur.fc, xf)) return false;
+        }
+        const double wv = s_west[ws];
+        double xw = __shfl_up_sync(FULL, xl, 1);
+        xw = lane == 0 ? wv : xw;
+        // ---- Alg.1's row: far (ls0), north, west (column order), then the division
+        double ls = pend ? __dadd_rn(0.0, __dmul_rn(cur.ls0, xf)) : cur.ls0;
+        ls = (cur.meta & kDescN) ? __dadd_rn(ls, __dmul_rn(cur.vn, xl)) : ls;
+        ls = (cur.meta & kDescW) ? __dadd_rn(ls, __dmul_rn(cur.vw, xw)) : ls;
+        const double a = __dsub_rn(cur.b, ls);
+        Diag g;
+        g.d = cur.d;
+        g.r = cur.rc;
+        double q = g.cand(a);
+        const bool guard = Diag::in_range(a) && cur.rc != 0.0;
+        if (SAFE) {
+            const bool fix = act && !(guard && Diag::exact(a, cur.d, q));
+            if (__any_sync(FULL, fix)) {
+                if (fix) q = Diag::slow_div(a, cur.d);
+            }
+        } else {
+            // outside the guard (a zero numerator, extreme magnitudes): the full division, in-loop;
+            // inside it the candidate's proof runs off the chain and a failure fails the solve
+            const bool fix = act && !guard;
+            if (__any_sync(FULL, fix)) {
+                if (fix) q = Diag::slow_div(a, cur.d);
+            }
+            bad |= act && guard && !Diag::exact(a, cur.d, q);
+        }
+        // ---- publish (Alg.5 l.13-16); GRID records are read by GRID warps only (no shared-memory
+        // sentinel to avoid)
+        const int ri = act ? r : 0;
+#ifdef SPTRSV_GRID_M_NOSTORE  // measurement builds only (tools/)
+        if (false) {
+#else
+        if (PROTO == PROTO_FUSED) {
+#endif
+            const unsigned long long bits = (unsigned long long)__double_as_longlong(q);
+            grid_st_rec_if(act, p.rec + 2 * (size_t)ri, ep | (bits & 0xffffffffull), ep | (bits >> 32));
+            grid_st_x_if(act, reinterpret_cast<unsigned long long *>(p.x) + ri, bits);
+        } else if (act) {
+            p.x[r] = q;
+            st_release_u32(p.flags + r, epoch);
+        }
+        xl = act ? q : xl;
+        return true;
+    };
+    Row ra, rb;
+    int wbase = 0;  // (kGridBlk * b) mod kGridDesc: s_west slot of the block's first step
+    static_assert(kGridDesc % kGridBlk == 0 && kGridBlk % 2 == 0, "block steps tile the west ring");
     for (int b = 0; b < nblocks; ++b) {
         if (lane == 0) st_volatile_s32(&s_cons, kGridBlk * b);
         bar_sync_cp();
         if (stop) continue;
-        if (b == 0) fetch(cur);
-        const int s_end = min(steps, kGridBlk * (b + 1));
-        for (int s = kGridBlk * b; s < s_end; ++s) {
-            fetch(nxt);  // the next step's row (its lines were produced before this block)
-            const int r = cur.r;
-            const bool act = r >= 0;
-            const bool pend = (cur.meta & kDescFar) != 0;
-            double xf = 0.0;
-            // lane 0's west (line s) from the ring warp; pending far entries (rare)
-            if (ring_have <= s && s < lines) ring_have = ld_volatile_s32(&s_ring);
-            if (__any_sync(FULL, (ring_have <= s && s < lines) || pend)) {
-                if (!wait_for(s < lines ? s : -1, pend, cur.fc, xf)) {
-                    stop = true;
-                    break;
-                }
-            }
-            const double wv = s_west[(s < lines ? s : 0) % kGridDesc];
-            double xw = __shfl_up_sync(FULL, xl, 1);
-            xw = lane == 0 ? wv : xw;
-            // ---- Alg.1's row: far (ls0), north, west (column order), then the division
-            double ls = pend ? __dadd_rn(0.0, __dmul_rn(cur.ls0, xf)) : cur.ls0;
-            ls = (cur.meta & kDescN) ? __dadd_rn(ls, __dmul_rn(cur.vn, xl)) : ls;
-            ls = (cur.meta & kDescW) ? __dadd_rn(ls, __dmul_rn(cur.vw, xw)) : ls;
-            const double a = __dsub_rn(cur.b, ls);
-            Diag g;
-            g.d = cur.d;
-            g.r = cur.rc;
-            double q = g.cand(a);
-            const bool guard = Diag::in_range(a) && cur.rc != 0.0;
-            if (SAFE) {
-                const bool fix = act && !(guard && Diag::exact(a, cur.d, q));
-                if (__any_sync(FULL, fix)) {
-                    if (fix) q = Diag::slow_div(a, cur.d);
-                }
-            } else {
-                // outside the guard (a zero numerator, extreme magnitudes): the full division, in-loop;
-                // inside it the candidate's proof runs off the chain and a failure fails the solve
-                const bool fix = act && !guard;
-                if (__any_sync(FULL, fix)) {
-                    if (fix) q = Diag::slow_div(a, cur.d);
-                }
-                bad |= act && guard && !Diag::exact(a, cur.d, q);
-            }
-            // ---- publish (Alg.5 l.13-16); GRID records are read by GRID warps only (no shared-
-            // memory sentinel to avoid)
-            const int ri = act ? r : 0;
-            if (PROTO == PROTO_FUSED) {
-                const unsigned long long bits = (unsigned long long)__double_as_longlong(q);
-                st_relaxed_v2_u64_if(act, p.rec + 2 * (size_t)ri, ep | (bits & 0xffffffffull), ep | (bits >> 32));
-                st_u64_if(act, reinterpret_cast<unsigned long long *>(p.x) + ri, bits);
-            } else if (act) {
-                p.x[r] = q;
-                st_release_u32(p.flags + r, epoch);
-            }
-            xl = act ? q : xl;
-            cur = nxt;
+        if (b == 0) fetch(ra);
+        const int s0 = kGridBlk * b;
+        const int s_end = min(steps, s0 + kGridBlk);
+        // lane 0's west values of the whole block: one check per block (the ring warp stores lines in
+        // chunks), waiting only when the ring is behind
+        const int need = min(s_end, lines) - 1;
+        if (ring_have <= need) ring_have = ld_volatile_s32_nc(&s_ring);
+        if (ring_have <= need) {
+            double dummy;
+            if (!wait_for(need, false, 0, dummy)) stop = true;
         }
+        if (!stop) {
+            if (s_end - s0 == kGridBlk) {
+#pragma unroll
+                for (int k = 0; k < kGridBlk; k += 2) {
+                    if (!step(ra, rb, s0 + k, wbase + k) || !step(rb, ra, s0 + k + 1, wbase + k + 1)) {
+                        stop = true;
+                        break;
+                    }
+                }
+            } else {  // the last, partial block
+                for (int k = 0; k < s_end - s0; ++k) {
+                    Row &c = (k & 1) ? rb : ra;
+                    Row &nx = (k & 1) ? ra : rb;
+                    if (!step(c, nx, s0 + k, wbase + k)) {
+                        stop = true;
+                        break;
+                    }
+                }
+            }
+        }
+        wbase = wbase + kGridBlk == kGridDesc ? 0 : wbase + kGridBlk;
         if (stop && lane == 0) st_volatile_s32((int *)&s_stop, 1);  // producers and ring skip the rest
     }
     if (lane == 0) st_volatile_s32(&s_cons, 0x3fffffff);

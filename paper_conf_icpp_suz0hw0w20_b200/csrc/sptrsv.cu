@@ -1053,6 +1053,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.grid_m = h->grid_m;
     p.grid_lines = h->grid_m > 0 ? (int32_t)(((long long)h->n + h->grid_m - 1) / h->grid_m) : 0;
     p.grid_ecap = 32 * std::max(1, h->max_row);
+    p.grid_far = h->grid_far > 0 ? 1 : 0;
     p.x_host = x_host;
     p.bflag = bflag;
     p.bseq = bseq;
