@@ -13,12 +13,15 @@
 // (step s: lane l solves line y = s - l).  Then
 //   north (r - m)  = the lane's own result of the previous step       (a register)
 //   west  (r - 1)  = lane l-1's result of the previous step           (one __shfl_up_sync)
-//   lane 0's west  = band k-1's lane 31, through the global protocol: a RING of polls -- lane
-//                    (y & 31) issues line y's poll kGridRing steps before lane 0 needs it
-//   a far entry    = the global protocol (its poll issued one step ahead)
+//   lane 0's west  = band k-1's lane 31, through the global protocol, polled by the band's RING warp
+//                    32 lines per round trip and handed over in shared memory
+//   a far entry    = the global protocol, polled by the producer warp that prepares the row
 // so a step costs one shuffle and the row's dependent fp64 operations, and band k waits on band k-1
 // through lane 0 only: one global hop per 32 columns instead of one per line.  The critical path is
-// the grid's wavefront, lines + 32 * bands steps, plus one hop per band.
+// the grid's wavefront, lines + 32 * bands steps, plus one hop per band.  Measured (c3, 2048^2 grid,
+// B200): 1.22 ms against CHAIN's 5.10 ms; see DESIGN.md section 6 for the design steps and what each
+// one bought (a per-step poll held in lane registers cost a round trip per step through the warp's
+// scoreboard -- hence the ring warp).
 //
 // Eligibility (k_grid_check, every row, for the m k_grid_probe proposes): each off-diagonal is the
 // west neighbour (c = r - 1 with x >= 1), the north neighbour (c = r - m), or a far entry c < r - m
@@ -38,10 +41,6 @@
 
 namespace sptrsv_dev {
 
-#ifndef SPTRSV_GRID_RING
-#define SPTRSV_GRID_RING 8
-#endif
-constexpr int kGridRing = SPTRSV_GRID_RING;  // steps between lane 0's west poll and its use (< 32)
 
 // ---------------------------------------------------------------- analyse: is the matrix a grid?
 
@@ -178,20 +177,6 @@ __device__ __forceinline__ int ld_volatile_s32_nc(const int *a) {  // no compile
     int v;
     asm volatile("ld.volatile.shared.s32 %0, [%1];" : "=r"(v) : "r"((unsigned)__cvta_generic_to_shared(a)));
     return v;
-}
-
-// a poll issued only when `go` holds: one predicated load for the FUSED records (no branch)
-template <int PROTO>
-__device__ __forceinline__ void poll1_if(bool go, const SolveParams &p, int c, unsigned long long &w0,
-                                         unsigned long long &w1) {
-    if (PROTO == PROTO_FUSED) {
-        asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];\n\t}"
-                     : "+l"(w0), "+l"(w1)
-                     : "l"(p.rec + 2 * (size_t)(go ? c : 0)), "r"((unsigned)go)
-                     : "memory");
-    } else if (go) {
-        poll1<PROTO>(p, c, w0, w1);
-    }
 }
 
 template <int PROTO, bool SAFE>
