@@ -60,9 +60,9 @@ WORKLOADS = {
 }
 ENGINES = {0: "one-shot (staged, in-CTA x copy)", 3: "lean", 6: "hybrid (warp tasks + 32-row thread groups)",
            7: "chain (in-warp chains)", 8: "small (one CTA, shared memory)", 9: "leanp (persistent, pipelined)",
-           33: "paper Alg.3", 34: "paper Alg.4", 35: "paper Alg.5"}
+           10: "grid (wavefront bands of 32 columns)", 33: "paper Alg.3", 34: "paper Alg.4", 35: "paper Alg.5"}
 KERNELS = {0: "k_solve", 3: "k_solve_lean", 6: "k_solve_tri_warp", 7: "k_solve_chain", 8: "k_solve_small",
-           9: "k_solve_leanp",
+           9: "k_solve_leanp", 10: "k_solve_grid",
            33: "k_paper_alg3", 34: "k_paper_alg4", 35: "k_paper_alg5"}
 EXTRA_CONFIGS = ["c1", "c3", "c4", "c5sys", "chain"]
 
@@ -281,6 +281,11 @@ def latency_bound(levels, hops, mean_s, alg_bytes, peak, engine=None):
            "model": "(levels - 1) * t_hop with the cross-SM record hop: a bound when every level boundary crosses "
                     "SMs; CHAIN resolves in-warp levels in registers (~0.1 us per step), so for chains and grids it "
                     "is a model, not a bound"}
+    if engine == 10:
+        out["model"] = ("GRID crosses SMs only at band boundaries (ceil(m/32) - 1 record hops, lane 0 of a band "
+                        "waiting on lane 31 of the previous one); the other level boundaries are register / "
+                        "shuffle steps inside a warp (~0.23 us each under load), so (levels - 1) * t_hop is a "
+                        "reference scale here, not a bound")
     if engine == 8:
         out["model"] = ("SMALL solves the whole system in ONE SM's shared memory: no level boundary crosses SMs, so "
                         "the cross-SM hop figures below are a reference scale only, not a bound")

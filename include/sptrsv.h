@@ -101,6 +101,7 @@ typedef enum sptrsv_option {
                                       near dependencies that are not pure chains and whose
                                       CSR, b and x fit one CTA's shared memory (24 B per
                                       row + 12 B per entry <= 226 KB);
+                                      else GRID for grid-shaped lower factors (see 10);
                                       else HYBRID for plans with warp-level rows; for
                                       all-thread-level plans LEANP when < 1/4 of the rows
                                       wait on a row < 256 away, CHAIN for long runs of
@@ -122,7 +123,17 @@ typedef enum sptrsv_option {
                                       9 LEANP: LEAN's row loop in persistent warps (a
                                       cooperative launch of what fits on the device, static
                                       round-robin blocks) with the next chunks' loads in
-                                      flight during the current chunk's waits.
+                                      flight during the current chunk's waits;
+                                      10 GRID: wavefront bands for stencil-shaped lower
+                                      factors (lower non-unit handles whose rows depend only
+                                      on their west r-1 / north r-m neighbours and at most
+                                      one far row in an earlier band / step, m found by
+                                      analyse): lane l of a band's warp owns grid column
+                                      32k+l, north operands stay in registers, west ones
+                                      move by shuffle, one protocol hop per 32 columns.
+                                      AUTO takes it (FUSED protocol) for grids with m >= 32
+                                      columns and >= 32 lines; forcing it on a matrix that
+                                      is not grid-shaped returns INVALID_ARG.
                                       LEAN, LEANP and CHAIN need an all-thread-level plan; a
                                       plan with warp-level rows runs HYBRID (ONE-SHOT if
                                       forced on a lower handle).  sptrsv_info.engine reports
@@ -190,8 +201,8 @@ typedef struct sptrsv_info {
     int64_t near_deps;        /* dependencies with i - j < 256 (analyse statistic)         */
     int64_t warp_deps;        /* dependencies inside the row's own 32-row group            */
     int32_t engine;           /* engine the next solve launches (0 ONE-SHOT, 3 LEAN,
-                                 6 HYBRID, 7 CHAIN, 8 SMALL, 9 LEANP; 33/34/35 the
-                                 paper's Alg.3/4/5)                                        */
+                                 6 HYBRID, 7 CHAIN, 8 SMALL, 9 LEANP, 10 GRID; 33/34/35
+                                 the paper's Alg.3/4/5)                                    */
     int32_t cta_threads;      /* CTA size the next solve uses (defaults resolved)          */
     int32_t rows_per_lane;    /* rows per lane the next solve uses (defaults resolved)     */
     int64_t prev_deps;        /* dependencies on the previous row in solve order (i - 1;

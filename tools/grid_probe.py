@@ -1,9 +1,9 @@
 """GRID engine probe: per system and engine, solve time (CUDA events, L2 flushed), GFLOPS, bit-exactness
-vs the oracle.  usage: grid_probe.py [systems] [engines]   systems: c3,g1000,s3d ...; engines: 10,7,5"""
+vs the CHAIN engine.  usage: grid_probe.py [systems] [engines]   systems: c3,g1000,s3d ...; engines: 10,7,5"""
 import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
-import oracle, synth
+import synth
 import paper_conf_icpp_suz0hw0w20_b200 as cap
 
 SYS = {"c3": lambda: synth.gen_c3(), "g1024": lambda: synth.gen_grid(1024), "g1000": lambda: synth.gen_grid(1000),
@@ -18,9 +18,15 @@ opts = json.loads(sys.argv[3]) if len(sys.argv) > 3 else {}
 flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
 for name in names:
     s = SYS[name]()
-    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
     d = torch.device("cuda")
     rp, ci, v, b = (torch.from_numpy(a).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+    # reference: the CHAIN engine's result (thread-level rows, Alg.1 arithmetic: bit-identical across
+    # engines; the oracle parity itself is tests/test_gpu_grid.py)
+    with cap.analyse(rp, ci, v, engine=7) as hr:
+        xr = torch.empty_like(b)
+        hr.solve(b, xr)
+        hr.check()
+        ref = xr.cpu().numpy()
     for eng in engines:
         try:
             h = cap.analyse(rp, ci, v, engine=eng, **opts)
@@ -42,6 +48,6 @@ for name in names:
         info = h.info()
         print(json.dumps({"sys": name, "engine": eng, "ran": info["engine"], "n": s.n, "nnz": s.nnz,
                           "t_us_mean": round(t * 1e6, 1), "t_us_min": round(min(ts) * 1e6, 1),
-                          "gflops": round(2 * s.nnz / t / 1e9, 3), "exact": bool(np.array_equal(x.cpu().numpy(), ref)),
+                          "gflops": round(2 * s.nnz / t / 1e9, 3), "same_as_chain": bool(np.array_equal(x.cpu().numpy(), ref)),
                           "opts": opts}), flush=True)
         h.close()
