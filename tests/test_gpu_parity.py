@@ -496,11 +496,11 @@ def test_chain_engine_division_guard_exits(cap, proto, K, eng):
 
 def test_engine_auto_choice(cap):
     """ENGINE_AUTO: small near-dependency systems that fit one CTA and are not pure chains (c1, a 32x32
-    grid) -> SMALL (8); far dependencies -> LEANP (9); long, warp-aligned runs of previous-row
-    dependencies (chains; grids whose side is a multiple of 64 and >= 2048) -> CHAIN (7); other
-    near-dependency plans (small levels, unaligned grids) -> staged one-shot (0); plans with
-    warp-level rows -> HYBRID (6)."""
-    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 9, 256, 1), (lambda: synth.gen_grid(100), 0, 1024, 1),
+    grid) -> SMALL (8); grid-shaped lower factors -> GRID (10); far dependencies -> LEANP (9); long,
+    warp-aligned runs of previous-row dependencies (chains) -> CHAIN (7); other near-dependency plans
+    (small levels) -> staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""
+    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 9, 256, 1), (lambda: synth.gen_grid(100), 10, 160, 1),
+                              (lambda: synth.gen_stencil(64, 48, 20), 10, 160, 1),
                               (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 9, 256, 1),
                               (lambda: synth.gen_c2i(n=100_000), 0, 256, 1),
                               (lambda: synth.gen_c1(), 8, 256, 1), (lambda: synth.gen_grid(32), 8, 256, 1),
