@@ -179,7 +179,9 @@ __device__ __forceinline__ int ld_volatile_s32_nc(const int *a) {  // no compile
     return v;
 }
 
-template <int PROTO, bool SAFE>
+// FAR: the matrix has far entries (7-point-like stencils); without them the step carries no far-entry
+// code at all (one basic block less per step for the scheduler)
+template <int PROTO, bool SAFE, bool FAR>
 __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p) {
     extern __shared__ __align__(16) unsigned char gsm[];
     __shared__ uint32_t s_blk, s_epoch, s_stop;
@@ -430,7 +432,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             }
         }
     };
-    const bool has_far = p.grid_far != 0;
+    constexpr bool has_far = FAR;
     // one step (line s - lane; lane 0's west value in s_west slot ws): Alg.1's row, the division, the
     // publish.  `cur` is this step's row, `nxt` receives the next one (two register sets alternate)
     auto step = [&](Row &cur, Row &nxt, int s, int ws) -> bool {

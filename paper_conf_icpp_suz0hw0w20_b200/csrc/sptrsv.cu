@@ -855,12 +855,16 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         }
     }
     if (engine == ENG_GRID) {  // wavefront bands of 32 columns, one CTA per band (solve_grid.cuh)
-        static const lean_fn tab[2][2] = {{k_solve_grid<PROTO_FLAGS, false>, k_solve_grid<PROTO_FUSED, false>},
-                                          {k_solve_grid<PROTO_FLAGS, true>, k_solve_grid<PROTO_FUSED, true>}};
-        L->fn = (const void *)tab[h->chain_div == 1 ? 1 : 0][h->proto ? 1 : 0];
+        static const lean_fn tab[2][2][2] = {
+            {{k_solve_grid<PROTO_FLAGS, false, false>, k_solve_grid<PROTO_FUSED, false, false>},
+             {k_solve_grid<PROTO_FLAGS, true, false>, k_solve_grid<PROTO_FUSED, true, false>}},
+            {{k_solve_grid<PROTO_FLAGS, false, true>, k_solve_grid<PROTO_FUSED, false, true>},
+             {k_solve_grid<PROTO_FLAGS, true, true>, k_solve_grid<PROTO_FUSED, true, true>}}};
+        const int fv = h->grid_far > 0 ? 1 : 0;
+        L->fn = (const void *)tab[fv][h->chain_div == 1 ? 1 : 0][h->proto ? 1 : 0];
         L->smem = grid_smem_bytes(32 * std::max(1, h->max_row));
-        static size_t attr_set[64][4] = {};  // per device and kernel: the dynamic smem limit raised so far
-        size_t &cur = attr_set[h->device & 63][(h->chain_div == 1 ? 2 : 0) + (h->proto ? 1 : 0)];
+        static size_t attr_set[64][8] = {};  // per device and kernel: the dynamic smem limit raised so far
+        size_t &cur = attr_set[h->device & 63][fv * 4 + (h->chain_div == 1 ? 2 : 0) + (h->proto ? 1 : 0)];
         if (cur < L->smem) {
             if (cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess) {
                 (void)cudaGetLastError();
