@@ -149,6 +149,12 @@ template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 
+// the rare in-loop division outside the guard (zero numerators, extreme magnitudes): out of line, so the
+// step's hot path carries no divergent branch
+__device__ __noinline__ double grid_fix_div(bool fix, double a, double d, double q) {
+    return fix ? __ddiv_rn(a, d) : q;
+}
+
 // the consumer / producer barrier (named barrier 1, warps 0 .. kGridProd; the ring warp runs free)
 __device__ __forceinline__ void bar_sync_cp() {
     asm volatile("bar.sync 1, %0;" ::"n"(32 * (1 + kGridProd)) : "memory");
@@ -459,16 +465,12 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         const bool guard = Diag::in_range(a) && cur.rc != 0.0;
         if (SAFE) {
             const bool fix = act && !(guard && Diag::exact(a, cur.d, q));
-            if (__any_sync(FULL, fix)) {
-                if (fix) q = Diag::slow_div(a, cur.d);
-            }
+            if (__builtin_expect(__any_sync(FULL, fix), 0)) q = grid_fix_div(fix, a, cur.d, q);
         } else {
             // outside the guard (a zero numerator, extreme magnitudes): the full division, in-loop;
             // inside it the candidate's proof runs off the chain and a failure fails the solve
             const bool fix = act && !guard;
-            if (__any_sync(FULL, fix)) {
-                if (fix) q = Diag::slow_div(a, cur.d);
-            }
+            if (__builtin_expect(__any_sync(FULL, fix), 0)) q = grid_fix_div(fix, a, cur.d, q);
             bad |= act && guard && !Diag::exact(a, cur.d, q);
         }
         // ---- publish (Alg.5 l.13-16); GRID records are read by GRID warps only (no shared-memory
