@@ -471,7 +471,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             // inside it the candidate's proof runs off the chain and a failure fails the solve
             const bool fix = act && !guard;
             if (__builtin_expect(__any_sync(FULL, fix), 0)) q = grid_fix_div(fix, a, cur.d, q);
-            bad |= act && guard && !Diag::exact(a, cur.d, q);
+            // (bitwise: the proof runs unconditionally, no branch around it in the step)
+            const bool ex = Diag::exact(a, cur.d, q);
+            bad = bad | (act & guard & !ex);
         }
         // ---- publish (Alg.5 l.13-16); GRID records are read by GRID warps only (no shared-memory
         // sentinel to avoid)
