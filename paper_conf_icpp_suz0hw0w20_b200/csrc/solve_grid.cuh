@@ -133,7 +133,7 @@ static_assert(kGridBlk * (kGridA1 + 1) <= kGridRaw, "raw ring too small");
 enum : int { kDescN = 2, kDescW = 4, kDescFar = 8 /* far entry not folded: poll it */ };
 
 __host__ __device__ constexpr size_t grid_smem_bytes(int ecap) {
-    return (size_t)kGridDesc * 32 * (6 * 8 + 3 * 4) + (size_t)kGridDesc * 8 +
+    return (size_t)kGridDesc * 32 * 64 + (size_t)kGridDesc * 8 +
            (size_t)kGridRaw * (64 * 4 + 32 * 8 + (size_t)ecap * 12);
 }
 
@@ -210,12 +210,12 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
     const int steps = lines + nl - 1;
     const int nblocks = (steps + kGridBlk - 1) / kGridBlk;
     // ---- shared memory: descriptor ring, then raw ring
-    double *d_ls0 = reinterpret_cast<double *>(gsm);  // [desc][32]: far product summed (or vf if pending)
-    double *d_vn = d_ls0 + kGridDesc * 32, *d_vw = d_vn + kGridDesc * 32, *d_b = d_vw + kGridDesc * 32;
-    double *d_d = d_b + kGridDesc * 32, *d_rc = d_d + kGridDesc * 32;
-    int32_t *d_meta = reinterpret_cast<int32_t *>(d_rc + kGridDesc * 32), *d_fc = d_meta + kGridDesc * 32;
-    int32_t *d_row = d_fc + kGridDesc * 32;                                  // [desc][32]: row, -1 = none
-    double *s_west = reinterpret_cast<double *>(d_row + kGridDesc * 32);     // [desc]: lane 0's west x
+    // descriptors, [desc][32] 16-byte pairs (one 128-bit shared load each): {ls0 (far product summed, or
+    // vf if pending), vn}, {vw, b}, {d, RN(1/d)}, {meta, far column, row (-1 = none), 0}
+    double2 *d_a = reinterpret_cast<double2 *>(gsm);
+    double2 *d_bw = d_a + kGridDesc * 32, *d_dr = d_bw + kGridDesc * 32;
+    int4 *d_m = reinterpret_cast<int4 *>(d_dr + kGridDesc * 32);
+    double *s_west = reinterpret_cast<double *>(d_m + kGridDesc * 32);     // [desc]: lane 0's west x
     int32_t *s_rp = reinterpret_cast<int32_t *>(s_west + kGridDesc);        // [raw][64]
     double *s_b = reinterpret_cast<double *>(s_rp + kGridRaw * 64);          // [raw][32]
     double *s_val = s_b + kGridRaw * 32;                                     // [raw][E]
@@ -340,15 +340,10 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
                 dv = g.d;
                 rc = g.r;
             }
-            d_ls0[ds] = ls0;
-            d_vn[ds] = vn;
-            d_vw[ds] = vw;
-            d_b[ds] = bv;
-            d_d[ds] = dv;
-            d_rc[ds] = rc;
-            d_meta[ds] = meta;
-            d_fc[ds] = fc;
-            d_row[ds] = act ? r : -1;
+            d_a[ds] = make_double2(ls0, vn);
+            d_bw[ds] = make_double2(vw, bv);
+            d_dr[ds] = make_double2(dv, rc);
+            d_m[ds] = make_int4(meta, fc, act ? r : -1, 0);
         };
         // prologue: the raw rows of the first lines, then the descriptors of lines [0, kGridBlk]
         for (int y = w; y < kGridBlk + 1 + kGridBlk * kGridA1; y += kGridProd) stage_rp(y);
@@ -387,16 +382,18 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
     };
     auto fetch = [&](Row &o) {
         const int ds = fsl * 32 + lane;
-        const int row = d_row[ds];
+        const int4 mm = d_m[ds];
+        const double2 a2 = d_a[ds], bw = d_bw[ds], dr = d_dr[ds];
+        const int row = mm.z;
         o.r = (unsigned)fy < (unsigned)lines ? row : -1;
-        o.meta = d_meta[ds];
-        o.ls0 = d_ls0[ds];
-        o.vn = d_vn[ds];
-        o.vw = d_vw[ds];
-        o.b = d_b[ds];
-        o.d = d_d[ds];
-        o.rc = d_rc[ds];
-        o.fc = d_fc[ds];
+        o.meta = mm.x;
+        o.ls0 = a2.x;
+        o.vn = a2.y;
+        o.vw = bw.x;
+        o.b = bw.y;
+        o.d = dr.x;
+        o.rc = dr.y;
+        o.fc = mm.y;
         o.meta = o.r >= 0 ? o.meta : 0;
         ++fy;
         fsl = fsl == kGridDesc - 1 ? 0 : fsl + 1;
