@@ -11,7 +11,8 @@ SYS = {"c3": lambda: synth.gen_c3(), "g1024": lambda: synth.gen_grid(1024), "g10
        "r8192x512": lambda: synth.gen_stencil(8192, 512), "r512x8192": lambda: synth.gen_stencil(512, 8192),
        "s3d": lambda: synth.gen_stencil(128, 128, 128), "s3d64": lambda: synth.gen_stencil(64, 64, 256),
        "b1": lambda: synth.gen_stencil(32, 65536), "b2": lambda: synth.gen_stencil(64, 32768),
-       "b8": lambda: synth.gen_stencil(256, 8192), "b1f": lambda: synth.gen_stencil(32, 64, 1024)}
+       "b8": lambda: synth.gen_stencil(256, 8192), "w16k": lambda: synth.gen_stencil(16384, 64),
+       "w4k": lambda: synth.gen_stencil(4096, 256), "b1f": lambda: synth.gen_stencil(32, 64, 1024)}
 names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["c3", "g1000", "s3d"]
 engines = [int(e) for e in sys.argv[2].split(",")] if len(sys.argv) > 2 else [10, 7, 5]
 opts = json.loads(sys.argv[3]) if len(sys.argv) > 3 else {}
