@@ -120,12 +120,12 @@ __global__ void __launch_bounds__(256) k_grid_check(const int32_t *__restrict__ 
 // produces the descriptors of lines [B*b + B + 1, B*b + 2B] (B = kGridBlk), so the consumer always
 // finds the next B + 1 lines ready and its step is one shuffle, the row's dependent fp64 operations,
 // two stores and one-step-ahead shared-memory loads.
-constexpr int kGridProd = 3;              // producer warps (one per remaining SM sub-partition)
+constexpr int kGridProd = 4;              // producer warps
 constexpr int kGridBlk = 2 * kGridProd;   // consumer steps per block (each producer: 2 lines per block)
 constexpr int kGridDesc = 48;             // descriptor ring (lines): line y is read until step y + 30
 constexpr int kGridRaw = 64;              // raw CSR ring (lines)
-constexpr int kGridA1 = 8;                // rowptr / b staged this many blocks before production
-constexpr int kGridA2 = 4;                // entries staged this many blocks before production
+constexpr int kGridA1 = 6;                // rowptr / b staged this many blocks before production
+constexpr int kGridA2 = 3;                // entries staged this many blocks before production
 constexpr int kGridWarps = 2 + kGridProd;  // consumer, producers, ring
 static_assert(kGridA1 == 2 * kGridA2, "one cp.async wait covers both staging distances");
 static_assert(kGridBlk * (kGridA1 + 1) <= kGridRaw, "raw ring too small");
