@@ -131,9 +131,10 @@ typedef enum sptrsv_option {
                                       analyse): lane l of a band's warp owns grid column
                                       32k+l, north operands stay in registers, west ones
                                       move by shuffle, one protocol hop per 32 columns.
-                                      AUTO takes it (FUSED protocol) for grids with m >= 32
-                                      columns and >= 32 lines; forcing it on a matrix that
-                                      is not grid-shaped returns INVALID_ARG.
+                                      AUTO takes it (FUSED protocol) for 2D grids (<= 1/8 far
+                                      entries) with m >= 32 columns and >= 32 lines; forcing
+                                      it on a matrix that is not grid-shaped returns
+                                      INVALID_ARG.
                                       LEAN, LEANP and CHAIN need an all-thread-level plan; a
                                       plan with warp-level rows runs HYBRID (ONE-SHOT if
                                       forced on a lower handle).  sptrsv_info.engine reports

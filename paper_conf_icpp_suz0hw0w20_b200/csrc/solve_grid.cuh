@@ -108,8 +108,8 @@ __global__ void __launch_bounds__(256) k_grid_check(const int32_t *__restrict__ 
 
 // ---------------------------------------------------------------- the solve
 //
-// One band per CTA of four warps: warp 0, the CONSUMER, runs the band's chain (the skewed steps
-// above) and nothing else; warps 1..3, the PRODUCERS, keep it fed:
+// One band per CTA of six warps: warp 0, the CONSUMER, runs the band's chain (the skewed steps
+// above) and nothing else; warps 1..kGridProd, the PRODUCERS, keep it fed (the last warp is the RING):
 //   - raw CSR staging: the rows of one line of a band are contiguous, so rowptr / b / entries of a
 //     line are copied into a shared-memory ring (kGridRaw lines) by cp.async, coalesced, kGridA1 /
 //     kGridA2 blocks before they are needed;

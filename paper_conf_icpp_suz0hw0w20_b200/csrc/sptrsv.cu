@@ -687,9 +687,9 @@ bool small_fits(const sptrsv_handle_s *h) {
 }
 
 // ENGINE_GRID (solve_grid.cuh): usable when analyse found a line length m under which every row
-// keeps the band order (lower non-unit handles); AUTO takes it for grid-shaped factors -- m >= 32
+// keeps the band order (lower non-unit handles); AUTO takes it for 2D grid-shaped factors -- m >= 32
 // columns, >= 32 lines, >= 1/2 of the off-diagonals north / west neighbours, >= 1/4 west (the
-// wavefront runs along the lines).
+// wavefront runs along the lines), <= 1/8 far entries.
 bool grid_ok(const sptrsv_handle_s *h) {
     return h->tri == 0 && h->n > 0 && h->grid_m >= 2 && h->grid_viol == 0 && h->nnz > h->n;
 }
@@ -697,7 +697,11 @@ bool grid_auto(const sptrsv_handle_s *h) {
     if (!grid_ok(h) || h->proto != PROTO_FUSED) return false;
     const long long offdiag = h->nnz - h->n;
     const long long lines = ((long long)h->n + h->grid_m - 1) / h->grid_m;
-    return h->grid_m >= 32 && lines >= 32 && 2 * h->grid_fast >= offdiag && 4 * h->prev_deps >= offdiag;
+    // ... and no (or few) far entries: a 3D grid's wavefront is far shorter than its line count (levels
+    // ~ nx + ny + nz, lines ny * nz), so the level-parallel engines win there (64x48x20: ONE-SHOT 145 us,
+    // GRID 283 us; 128^3: CHAIN 1.8 ms, GRID 4.5 ms), while 2D grids are GRID's (100^2: 57 vs 142 us)
+    return h->grid_m >= 32 && lines >= 32 && 2 * h->grid_fast >= offdiag && 4 * h->prev_deps >= offdiag &&
+           8 * h->grid_far <= offdiag;
 }
 
 int resolve_engine(const sptrsv_handle_s *h) {

@@ -84,11 +84,11 @@ def test_c2_full_default_launch(proto):
 
 
 def test_c3_full_default_launch():
-    """c3 in the bench.py configuration: AUTO -> GRID (wavefront bands; 160-thread CTAs: consumer,
-    three producers, ring warp)."""
+    """c3 in the bench.py configuration: AUTO -> GRID (wavefront bands; 192-thread CTAs: consumer,
+    four producers, ring warp)."""
     s = synth.gen_c3(ones=True)
     x1, x2, info = _run(s)
-    assert (info["engine"], info["cta_threads"]) == (10, 160), info
+    assert (info["engine"], info["cta_threads"]) == (10, 192), info
     assert np.array_equal(x1, np.ones(s.n)) and np.array_equal(x2, np.ones(s.n))
     s = synth.gen_c3()
     ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)

@@ -499,9 +499,9 @@ def test_engine_auto_choice(cap):
     grid) -> SMALL (8); grid-shaped lower factors -> GRID (10); far dependencies -> LEANP (9); long,
     warp-aligned runs of previous-row dependencies (chains) -> CHAIN (7); other near-dependency plans
     (small levels) -> staged one-shot (0); plans with warp-level rows -> HYBRID (6)."""
-    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 9, 256, 1), (lambda: synth.gen_grid(100), 10, 160, 1),
-                              (lambda: synth.gen_stencil(64, 48, 20), 10, 160, 1),
-                              (lambda: synth.gen_stencil(8192, 64), 10, 160, 1),  # wide grids too (GRID 4.0 vs CHAIN 5.2 ms at 16384 x 64)
+    for gen, want, cta, K in ((lambda: synth.gen_c2(n=100_000), 9, 256, 1), (lambda: synth.gen_grid(100), 10, 192, 1),
+                              (lambda: synth.gen_stencil(64, 48, 20), 0, 256, 1),  # 3D: level-parallel engines
+                              (lambda: synth.gen_stencil(8192, 64), 10, 192, 1),  # wide grids too (GRID 4.0 vs CHAIN 5.2 ms at 16384 x 64)
                               (lambda: synth.gen_chain(3000), 7, 128, 2), (lambda: synth.gen_diag(5000), 9, 256, 1),
                               (lambda: synth.gen_c2i(n=100_000), 0, 256, 1),
                               (lambda: synth.gen_c1(), 8, 256, 1), (lambda: synth.gen_grid(32), 8, 256, 1),

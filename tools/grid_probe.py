@@ -12,7 +12,8 @@ SYS = {"c3": lambda: synth.gen_c3(), "g1024": lambda: synth.gen_grid(1024), "g10
        "s3d": lambda: synth.gen_stencil(128, 128, 128), "s3d64": lambda: synth.gen_stencil(64, 64, 256),
        "b1": lambda: synth.gen_stencil(32, 65536), "b2": lambda: synth.gen_stencil(64, 32768),
        "b8": lambda: synth.gen_stencil(256, 8192), "w16k": lambda: synth.gen_stencil(16384, 64),
-       "w4k": lambda: synth.gen_stencil(4096, 256), "b1f": lambda: synth.gen_stencil(32, 64, 1024)}
+       "w4k": lambda: synth.gen_stencil(4096, 256), "g100": lambda: synth.gen_grid(100),
+       "g300": lambda: synth.gen_grid(300), "g64x48x20": lambda: synth.gen_stencil(64, 48, 20), "b1f": lambda: synth.gen_stencil(32, 64, 1024)}
 names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["c3", "g1000", "s3d"]
 engines = [int(e) for e in sys.argv[2].split(",")] if len(sys.argv) > 2 else [10, 7, 5]
 opts = json.loads(sys.argv[3]) if len(sys.argv) > 3 else {}
