@@ -322,7 +322,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
                 meta = (hn ? kDescN : 0) | (hw ? kDescW : 0);
                 vw = hw ? v[hi - 2] : 0.0;
                 vn = hn ? v[jn] : 0.0;
-                if (jf >= lo) {  // the far entry (at most one: k_grid_check)
+                if (FAR && jf >= lo) {  // the far entry (at most one: k_grid_check)
                     fc = c[jf];
                     const double vf = v[jf];
                     unsigned long long f0, f1;
