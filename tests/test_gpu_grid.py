@@ -182,3 +182,45 @@ def test_c3_full_grid(cap, proto):
     assert info["engine"] == GRID
     for x in xs:
         assert np.array_equal(x, ref)
+
+
+def test_grid_solve_host_and_multi_rhs(cap):
+    """A GRID handle through sptrsv_solve_host (pinned host b / x) and sptrsv_solve_multi (the multi-RHS
+    kernel, engine-independent): bit-exact per column."""
+    s = synth.gen_stencil(200, 90, seed=13)
+    ref = oracle.solve(s.rowptr, s.colidx, s.val, s.b)
+    rp, ci, v, b = dev(s)
+    with cap.analyse(rp, ci, v) as h:
+        assert h.info()["engine"] == GRID
+        bh = torch.from_numpy(s.b).pin_memory()
+        xh = torch.full((s.n,), float("nan"), dtype=torch.float64).pin_memory()
+        h.solve_host(bh, xh)
+        assert np.array_equal(xh.numpy(), ref)
+        rng = np.random.default_rng(7)
+        B = rng.uniform(-1, 1, (s.n, 5))
+        X = h.solve_multi(torch.from_numpy(B).cuda())
+        h.check()
+        assert np.array_equal(X.cpu().numpy(), oracle.solve_multi(s.rowptr, s.colidx, s.val, B))
+        x = torch.full_like(b, float("nan"))  # and a device solve after the host / multi paths
+        h.solve(b, x)
+        h.check()
+        assert np.array_equal(x.cpu().numpy(), ref)
+
+
+def test_grid_batch_of_grids(cap):
+    """Independent grids of one line length as one block-diagonal batch handle: still grid-shaped (each
+    system starts on a line boundary), solved by GRID in one launch, every block bit-exact."""
+    systems = [synth.gen_stencil(96, 40, seed=21), synth.gen_stencil(96, 70, seed=22), synth.gen_stencil(96, 33, seed=23)]
+    d = torch.device("cuda:0")
+    devs = [tuple(torch.from_numpy(a).to(d) for a in (t.rowptr, t.colidx, t.val)) for t in systems]
+    refs = [oracle.solve(t.rowptr, t.colidx, t.val, t.b) for t in systems]
+    b = torch.from_numpy(np.concatenate([t.b for t in systems])).to(d)
+    with cap.analyse_batch(devs, engine=GRID) as h:
+        assert h.info()["engine"] == GRID
+        x = torch.full_like(b, float("nan"))
+        h.solve(b, x)
+        h.check()
+        got = x.cpu().numpy()
+        off = h.offsets
+        for k, ref in enumerate(refs):
+            assert np.array_equal(got[off[k]:off[k + 1]], ref), k
