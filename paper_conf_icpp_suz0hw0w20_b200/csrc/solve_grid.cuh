@@ -488,6 +488,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             st_release_u32(p.flags + r, epoch);
         }
         xl = act ? q : xl;
+#ifdef SPTRSV_GRID_TRACE  // measurement builds only (tools/grid_trace.py): publish time of every row
+        if (p.trace && act) p.trace[r] = globaltimer_ns();
+#endif
         return true;
     };
     Row ra, rb;
