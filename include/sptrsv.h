@@ -124,11 +124,11 @@ typedef enum sptrsv_option {
                                       cooperative launch of what fits on the device, static
                                       round-robin blocks) with the next chunks' loads in
                                       flight during the current chunk's waits;
-                                      10 GRID: wavefront bands for stencil-shaped lower
-                                      factors (lower non-unit handles whose rows depend only
-                                      on their west r-1 / north r-m neighbours and at most
-                                      one far row in an earlier band / step, m found by
-                                      analyse): lane l of a band's warp owns grid column
+                                      10 GRID: wavefront bands for stencil-shaped factors
+                                      (any triangular form, in logical rows: rows depending
+                                      only on their west r-1 / north r-m neighbours and at
+                                      most one far row in an earlier band / step, m found by
+                                      analyse; upper handles need n % m == 0): lane l of a band's warp owns grid column
                                       32k+l, north operands stay in registers, west ones
                                       move by shuffle, one protocol hop per 32 columns.
                                       AUTO takes it (FUSED protocol) for 2D grids (<= 1/8 far

@@ -44,20 +44,40 @@ namespace sptrsv_dev {
 
 // ---------------------------------------------------------------- analyse: is the matrix a grid?
 
-// One warp proposes the line length m: each lane samples one row and takes the distance to its
+// The triangular forms (G25) in LOGICAL rows: an upper handle solves logical row
+// r = n-1-i (physical row i), so its dependencies are logical columns n-1-c < r and the whole analysis
+// (and the engine) runs on the logical lower matrix; the off-diagonals of physical row [s, e):
+//   lower: [s, e-1) (diagonal last), unit lower: [s, e); upper: [s+1, e) (diagonal first), unit upper: [s, e)
+// and in logical column order they run ascending (lower) or descending (upper).
+struct GridForm {
+    bool up, unit;
+    int32_t n;
+    __device__ int logical(int i) const { return up ? n - 1 - i : i; }
+    __device__ void offdiag(int s, int e, int &lo, int &hi) const {
+        lo = (up && !unit) ? s + 1 : s;
+        hi = (!up && !unit) ? e - 1 : e;
+    }
+    // position of the t-th off-diagonal counted from the logically LAST one (t = 0: nearest dependency)
+    __device__ int from_last(int lo, int hi, int t) const { return up ? lo + t : hi - 1 - t; }
+};
+
+// One warp proposes the line length m: each lane samples one logical row and takes the distance to its
 // nearest off-diagonal that is not the previous row (the north neighbour of a grid row); the most
-// frequent candidate (>= 2 votes) wins.  Lower non-unit handles only (tri == 0).
+// frequent candidate (>= 2 votes) wins.  Upper handles need n to be a multiple of m (whole lines).
 __global__ void k_grid_probe(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ colidx, int32_t n,
                              AnalyseOut *out, int tri) {
     const int lane = threadIdx.x;
+    const GridForm f{(tri & 1) != 0, (tri & 2) != 0, n};
     int cand = 0;
-    const bool valid = out->status == ~0ull && tri == 0 && n >= 2;
+    const bool valid = out->status == ~0ull && n >= 2;
     if (valid) {
-        const int r = (int)((long long)(lane + 1) * n / 33);
-        const int s = rowptr[r], e = rowptr[r + 1];
-        int j = e - 2;  // the last off-diagonal (the diagonal is last)
-        if (j >= s && colidx[j] == r - 1) --j;
-        if (j >= s) cand = r - colidx[j];
+        const int rl = (int)((long long)(lane + 1) * n / 33);
+        const int i = f.logical(rl);
+        int lo, hi;
+        f.offdiag(rowptr[i], rowptr[i + 1], lo, hi);
+        int t = 0;
+        if (hi > lo && f.logical(colidx[f.from_last(lo, hi, 0)]) == rl - 1) t = 1;
+        if (hi - lo > t) cand = rl - f.logical(colidx[f.from_last(lo, hi, t)]);
     }
     const unsigned same = __match_any_sync(0xffffffffu, cand);
     const unsigned cnt = cand > 1 ? (unsigned)__popc(same) : 0u;
@@ -66,22 +86,30 @@ __global__ void k_grid_probe(const int32_t *__restrict__ rowptr, const int32_t *
         const unsigned long long o = __shfl_xor_sync(0xffffffffu, key, off);
         key = o > key ? o : key;
     }
-    if (lane == 0) out->grid_m = (valid && (key >> 32) >= 2) ? (int)(key & 0xffffffffu) : 0;
+    if (lane == 0) {
+        int m = (valid && (key >> 32) >= 2) ? (int)(key & 0xffffffffu) : 0;
+        if (f.up && m > 0 && n % m != 0) m = 0;
+        out->grid_m = m;
+    }
 }
 
 // Every row against the m of k_grid_probe: violations of the band order (see the header), fast
-// entries (north / west) and far entries.
+// entries (north / west) and far entries, in logical rows and columns.
 __global__ void __launch_bounds__(256) k_grid_check(const int32_t *__restrict__ rowptr,
-                                                    const int32_t *__restrict__ colidx, int32_t n, AnalyseOut *out) {
+                                                    const int32_t *__restrict__ colidx, int32_t n, AnalyseOut *out,
+                                                    int tri) {
     const int m = out->grid_m;
     if (m < 2 || out->status != ~0ull) return;
-    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    const GridForm f{(tri & 1) != 0, (tri & 2) != 0, n};
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
     unsigned viol = 0, fast = 0, far = 0;
-    if (r < n) {
+    if (i < n) {
+        const int r = f.logical(i);
         const int y = r / m, x = r - y * m, k = x >> 5, l = x & 31;
-        const int s = rowptr[r], e = rowptr[r + 1] - 1;  // off-diagonals [s, e)
-        for (int j = s; j < e; ++j) {
-            const int c = colidx[j];
+        int lo, hi;
+        f.offdiag(rowptr[i], rowptr[i + 1], lo, hi);
+        for (int j = lo; j < hi; ++j) {
+            const int c = f.logical(colidx[j]);
             if ((c == r - 1 && x >= 1) || c == r - m) {
                 ++fast;
             } else if (c < r - m) {
@@ -187,7 +215,10 @@ __device__ __forceinline__ int ld_volatile_s32_nc(const int *a) {  // no compile
 
 // FAR: the matrix has far entries (7-point-like stencils); without them the step carries no far-entry
 // code at all (one basic block less per step for the scheduler)
-template <int PROTO, bool SAFE, bool FAR>
+// UPPER / UNIT: the triangular forms (GridForm above): bands, lines and columns are logical; the CSR
+// slice of a band's logical line is a contiguous run of physical rows (reversed for upper handles,
+// which analyse admits only when n is a multiple of m); b, x and the records are physical.
+template <int PROTO, bool SAFE, bool FAR, bool UPPER = false, bool UNIT = false>
 __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p) {
     extern __shared__ __align__(16) unsigned char gsm[];
     __shared__ uint32_t s_blk, s_epoch, s_stop;
@@ -233,8 +264,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         uint32_t bo = p.backoff_min, idl = 0;
         while (base < lines) {
             const int y = base + lane;
-            const unsigned wr = (unsigned)y * (unsigned)m + (unsigned)x0 - 1u;
-            const bool need = y < lines && wr < n;
+            const unsigned wl = (unsigned)y * (unsigned)m + (unsigned)x0 - 1u;  // logical west row
+            const bool need = y < lines && wl < n;
+            const unsigned wr = UPPER ? n - 1u - wl : wl;                       // its physical row
             const bool room = y < ld_volatile_s32(&s_cons) + kGridDesc - 8;
             unsigned long long w0 = 0, w1 = 0;
             if (need && room) poll1<PROTO>(p, (int)wr, w0, w1);
@@ -275,10 +307,14 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
     if (warp > 0) {
         // ================================================================ producers
         const int w = warp - 1;
-        auto line_rows = [&](int y, unsigned &row0) -> int {  // rows of line y in this band (0: none)
-            row0 = (unsigned)y * (unsigned)m + (unsigned)x0;
-            if (y < 0 || y >= lines || row0 >= n) return 0;
-            return min(nl, (int)(n - row0));
+        // rows of logical line y in this band (0: none); row0 = the first PHYSICAL row of its CSR slice
+        // (upper: logical row y*m + x0 + j is physical n-1-(y*m + x0 + j), so the slice runs backwards)
+        auto line_rows = [&](int y, unsigned &row0) -> int {
+            const unsigned l0 = (unsigned)y * (unsigned)m + (unsigned)x0;
+            if (y < 0 || y >= lines || l0 >= n) return 0;
+            const int k = min(nl, (int)(n - l0));
+            row0 = UPPER ? n - l0 - (unsigned)k : l0;
+            return k;
         };
         auto stage_rp = [&](int y) {  // rowptr[row0 .. row0 + k] and b[row0 .. row0 + k)
             unsigned row0;
@@ -306,24 +342,31 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             if (y >= lines) return;
             const int sl = y & (kGridRaw - 1), ds = (y % kGridDesc) * 32 + lane;
             const bool act = lane < k;
-            const int r = (int)(row0 + lane);
+            const int pj = UPPER ? k - 1 - lane : lane;  // this lane's row in the (physical) slice
+            const int r = (int)(row0 + pj);              // physical row
+            const int rl = (int)((unsigned)y * (unsigned)m + (unsigned)x0) + lane;  // logical row
+            const GridForm gf{UPPER, UNIT, (int32_t)n};
             int meta = 0, fc = 0;
             double ls0 = 0.0, vn = 0.0, vw = 0.0, bv = 0.0, dv = 1.0, rc = 1.0;
             if (act) {
                 const int base = s_rp[sl * 64];
-                const int lo = s_rp[sl * 64 + lane] - base, hi = s_rp[sl * 64 + lane + 1] - base;
+                int lo, hi;
+                gf.offdiag(s_rp[sl * 64 + pj] - base, s_rp[sl * 64 + pj + 1] - base, lo, hi);
                 const double *v = s_val + (size_t)sl * E;
                 const int32_t *c = s_col + (size_t)sl * E;
-                const int len = hi - lo;
-                const bool hw = len > 1 && c[hi - 2] == r - 1;  // (row 0 has no west: no -1 sentinel)
-                const int jn = hi - 2 - (int)hw;
-                const bool hn = jn >= lo && c[jn] == r - m;
-                const int jf = jn - (int)hn;
+                const int cnt = hi - lo;
+                // off-diagonals counted from the logically last one: west (rl - 1), north (rl - m), far
+                const int jw = gf.from_last(lo, hi, 0);
+                const bool hw = cnt > 0 && gf.logical(c[jw]) == rl - 1;  // (row 0 has no west)
+                const int jn = gf.from_last(lo, hi, (int)hw);
+                const bool hn = cnt > (int)hw && gf.logical(c[jn]) == rl - m;
+                const int tf = (int)hw + (int)hn;
+                const int jf = gf.from_last(lo, hi, tf);
                 meta = (hn ? kDescN : 0) | (hw ? kDescW : 0);
-                vw = hw ? v[hi - 2] : 0.0;
+                vw = hw ? v[jw] : 0.0;
                 vn = hn ? v[jn] : 0.0;
-                if (FAR && jf >= lo) {  // the far entry (at most one: k_grid_check)
-                    fc = c[jf];
+                if (FAR && cnt > tf) {  // the far entry (at most one: k_grid_check)
+                    fc = c[jf];  // physical: the records are indexed by physical row
                     const double vf = v[jf];
                     unsigned long long f0, f1;
                     poll1<PROTO>(p, fc, f0, f1);
@@ -334,9 +377,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
                         meta |= kDescFar;
                     }
                 }
-                bv = s_b[sl * 32 + lane];
+                bv = s_b[sl * 32 + pj];
                 Diag g;
-                g.init(v[hi - 1]);
+                g.init(UNIT ? 1.0 : v[UPPER ? s_rp[sl * 64 + pj] - base : s_rp[sl * 64 + pj + 1] - base - 1]);
                 dv = g.d;
                 rc = g.r;
             }

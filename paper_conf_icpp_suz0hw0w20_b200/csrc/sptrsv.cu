@@ -575,7 +575,7 @@ int sptrsv_analyse_csr_ex(int32_t n, const int32_t *rowptr, const int32_t *colid
         if (n > 0) {
             k_validate<<<(n + 255) / 256, 256>>>(rowptr, colidx, val, n, h->ws.indeg, h->ws.aout, tri_flags);
             k_grid_probe<<<1, 32>>>(rowptr, colidx, n, h->ws.aout, tri_flags);
-            k_grid_check<<<(n + 255) / 256, 256>>>(rowptr, colidx, n, h->ws.aout);
+            k_grid_check<<<(n + 255) / 256, 256>>>(rowptr, colidx, n, h->ws.aout, tri_flags);
             if (cudaGetLastError() != cudaSuccess) {
                 rc = SPTRSV_ERR_CUDA;
                 break;
@@ -687,15 +687,16 @@ bool small_fits(const sptrsv_handle_s *h) {
 }
 
 // ENGINE_GRID (solve_grid.cuh): usable when analyse found a line length m under which every row
-// keeps the band order (lower non-unit handles); AUTO takes it for 2D grid-shaped factors -- m >= 32
+// keeps the band order (any triangular form, in logical rows); AUTO takes it for 2D grid-shaped factors -- m >= 32
 // columns, >= 32 lines, >= 1/2 of the off-diagonals north / west neighbours, >= 1/4 west (the
 // wavefront runs along the lines), <= 1/8 far entries.
 bool grid_ok(const sptrsv_handle_s *h) {
-    return h->tri == 0 && h->n > 0 && h->grid_m >= 2 && h->grid_viol == 0 && h->nnz > h->n;
+    const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;  // unit handles store no diagonal
+    return h->n > 0 && h->grid_m >= 2 && h->grid_viol == 0 && offdiag > 0;
 }
 bool grid_auto(const sptrsv_handle_s *h) {
     if (!grid_ok(h) || h->proto != PROTO_FUSED) return false;
-    const long long offdiag = h->nnz - h->n;
+    const long long offdiag = (h->tri & 2) ? h->nnz : h->nnz - h->n;
     const long long lines = ((long long)h->n + h->grid_m - 1) / h->grid_m;
     // ... and no (or few) far entries: a 3D grid's wavefront is far shorter than its line count (levels
     // ~ nx + ny + nz, lines ny * nz), so the level-parallel engines win there (64x48x20: ONE-SHOT 145 us,
@@ -859,16 +860,20 @@ int plan_launch(sptrsv_handle_s *h, Launch *L) {
         }
     }
     if (engine == ENG_GRID) {  // wavefront bands of 32 columns, one CTA per band (solve_grid.cuh)
-        static const lean_fn tab[2][2][2] = {
-            {{k_solve_grid<PROTO_FLAGS, false, false>, k_solve_grid<PROTO_FUSED, false, false>},
-             {k_solve_grid<PROTO_FLAGS, true, false>, k_solve_grid<PROTO_FUSED, true, false>}},
-            {{k_solve_grid<PROTO_FLAGS, false, true>, k_solve_grid<PROTO_FUSED, false, true>},
-             {k_solve_grid<PROTO_FLAGS, true, true>, k_solve_grid<PROTO_FUSED, true, true>}}};
+#define GRID_ROW(F_, U_, N_)                                                                               \
+    {{k_solve_grid<PROTO_FLAGS, false, F_, U_, N_>, k_solve_grid<PROTO_FUSED, false, F_, U_, N_>},            \
+     {k_solve_grid<PROTO_FLAGS, true, F_, U_, N_>, k_solve_grid<PROTO_FUSED, true, F_, U_, N_>}}
+        static const lean_fn tab[2][4][2][2] = {
+            {GRID_ROW(false, false, false), GRID_ROW(false, true, false), GRID_ROW(false, false, true),
+             GRID_ROW(false, true, true)},
+            {GRID_ROW(true, false, false), GRID_ROW(true, true, false), GRID_ROW(true, false, true),
+             GRID_ROW(true, true, true)}};
+#undef GRID_ROW
         const int fv = h->grid_far > 0 ? 1 : 0;
-        L->fn = (const void *)tab[fv][h->chain_div == 1 ? 1 : 0][h->proto ? 1 : 0];
+        L->fn = (const void *)tab[fv][h->tri & 3][h->chain_div == 1 ? 1 : 0][h->proto ? 1 : 0];
         L->smem = grid_smem_bytes(32 * std::max(1, h->max_row));
-        static size_t attr_set[64][8] = {};  // per device and kernel: the dynamic smem limit raised so far
-        size_t &cur = attr_set[h->device & 63][fv * 4 + (h->chain_div == 1 ? 2 : 0) + (h->proto ? 1 : 0)];
+        static size_t attr_set[64][32] = {};  // per device and kernel: the dynamic smem limit raised so far
+        size_t &cur = attr_set[h->device & 63][fv * 16 + (h->tri & 3) * 4 + (h->chain_div == 1 ? 2 : 0) + (h->proto ? 1 : 0)];
         if (cur < L->smem) {
             if (cudaFuncSetAttribute(L->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L->smem) != cudaSuccess) {
                 (void)cudaGetLastError();
@@ -1059,7 +1064,7 @@ static int solve_impl(sptrsv_handle_t h, const double *b, double *x, double *x_h
     p.split_last = h->split_last;
     p.chain_div = h->chain_div;
     p.grid_m = h->grid_m;
-    p.grid_lines = h->grid_m > 0 ? (int32_t)(((long long)h->n + h->grid_m - 1) / h->grid_m) : 0;
+    p.grid_lines = h->grid_m > 0 ? (int32_t)(((long long)h->n + h->grid_m - 1) / h->grid_m) : 0;  // (upper: n % m == 0)
     p.grid_ecap = 32 * std::max(1, h->max_row);
     p.grid_far = h->grid_far > 0 ? 1 : 0;
     p.x_host = x_host;

@@ -224,3 +224,47 @@ def test_grid_batch_of_grids(cap):
         off = h.offsets
         for k, ref in enumerate(refs):
             assert np.array_equal(got[off[k]:off[k + 1]], ref), k
+
+
+F4_SHAPES = [(64, 64, 1), (100, 37, 1), (33, 70, 1), (257, 9, 1), (40, 6, 5), (32, 4, 9)]
+
+
+@pytest.mark.parametrize("shape", F4_SHAPES, ids=lambda t: "x".join(str(v) for v in t))
+@pytest.mark.parametrize("flags", [1, 2, 3])
+@pytest.mark.parametrize("proto", [0, 1])
+def test_grid_triangular_forms(cap, shape, flags, proto):
+    """SURVEY f4 on GRID: upper (backward substitution in logical rows), unit lower, unit upper --
+    bit-exact vs oracle.solve_tri (the same order of operations: Alg.1 under the reversal, DESIGN G25)."""
+    nx, ny, nz = shape
+    s = synth.gen_stencil(nx, ny, nz, seed=nx + 3 * ny + flags)
+    if flags & 1:
+        s = synth.to_upper(s)
+    if flags & 2:
+        s = synth.to_unit(s, upper=bool(flags & 1))
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags)
+    d = torch.device("cuda:0")
+    rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+    with cap.analyse(rp, ci, v, upper=bool(flags & 1), unit_diag=bool(flags & 2), engine=GRID, protocol=proto) as h:
+        assert h.info()["engine"] == GRID
+        for _ in range(2):
+            x = torch.full_like(b, float("nan"))
+            h.solve(b, x)
+            h.check()
+            assert np.array_equal(x.cpu().numpy(), ref)
+
+
+def test_grid_upper_needs_whole_lines(cap):
+    """An upper handle whose last grid line is ragged is not grid-shaped (GRID needs n % m == 0 there):
+    forcing GRID is refused, AUTO runs another engine, the result is exact."""
+    s = synth.to_upper(synth.gen_stencil(96, 50, rows=96 * 50 - 17, seed=4))
+    ref = oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, 1)
+    d = torch.device("cuda:0")
+    rp, ci, v, b = (torch.from_numpy(np.ascontiguousarray(a)).to(d) for a in (s.rowptr, s.colidx, s.val, s.b))
+    with cap.analyse(rp, ci, v, upper=True) as h:
+        assert h.info()["engine"] != GRID
+        with pytest.raises(cap.SptrsvError):
+            h.set_option(cap._lib.OPT_ENGINE, GRID)
+        x = torch.full_like(b, float("nan"))
+        h.solve(b, x)
+        h.check()
+        assert np.array_equal(x.cpu().numpy(), ref)
