@@ -310,11 +310,11 @@ def test_tri_chain_engine_bit_exact(cap, which, flags, proto, K, cta):
 
 @pytest.mark.parametrize("flags", FORMS)
 def test_tri_chain_auto_choice_and_closed_forms(cap, flags):
-    """AUTO sends f4 chains to CHAIN (a 200^2 grid, whose lines do not align with CHAIN's 64-row
-    warps, to LEANP); the f4 bidiagonal closed forms stay exact."""
+    """AUTO sends f4 grids to GRID (a 200^2 grid factor in every form) and f4 chains to CHAIN; the f4
+    bidiagonal closed forms stay exact."""
     s = form(synth.gen_grid(200), flags)
     x, info = gpu_solve(cap, s, flags)
-    assert info["engine"] == 9, info
+    assert info["engine"] == 10, info
     assert np.array_equal(x, oracle.solve_tri(s.rowptr, s.colidx, s.val, s.b, flags))
     s = form(synth.gen_c2(n=100_000), flags)
     _, info = gpu_solve(cap, s, flags)
