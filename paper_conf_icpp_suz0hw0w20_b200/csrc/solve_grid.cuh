@@ -274,6 +274,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             const unsigned mask = __ballot_sync(FULL, rdy);
             const int L = __ffs(~mask) - 1 < 0 ? 32 : __ffs(~mask) - 1;  // ready prefix
             if (lane < L && need) s_west[y % kGridDesc] = value1<PROTO>(p, (int)wr, w0, w1);
+#ifdef SPTRSV_GRID_TRACE  // measurement builds only: when the ring warp stored line y's west value
+            if (p.trace && lane < L && need) p.trace[(size_t)n + (size_t)y * ((m + 31) / 32) + band] = globaltimer_ns();
+#endif
             __syncwarp();
             if (L > 0) {
                 __threadfence_block();

@@ -30,3 +30,15 @@ hand = first[:, 1:] - last[:, :-1]  # band k lane 0 line y - band k-1 lane 31 li
 print("hand-over ns (pub k-1 lane 31 -> pub k lane 0, same line): p10 %.0f p50 %.0f p90 %.0f" % tuple(np.percentile(hand, [10, 50, 90])))
 skew = last - first  # within a band: lane 31 line y - lane 0 line y
 print("in-band skew (lane 31 - lane 0, same line) us p50 %.2f" % (np.median(skew) / 1e3))
+
+# the ring warp: when band k stored line y's west value (trace[n + y * nb + k]) vs band k-1's lane 31 publish
+ring = tr[s.n: s.n + m * nb].cpu().numpy().astype(np.int64).reshape(m, nb)
+t0 = tr[: s.n].cpu().numpy().astype(np.int64)
+base = t0[t0 > 0].min()
+ring = ring - base
+pub31 = (tr[: s.n].cpu().numpy().astype(np.int64).reshape(m, m)[:, 31::32] - base)  # band k lane 31, line y
+det = ring[:, 1:] - pub31[:, :-1]
+print("ring detection ns (band k-1 lane 31 publish -> band k ring stored): p10 %.0f p50 %.0f p90 %.0f" % tuple(np.percentile(det, [10, 50, 90])))
+use = first[:, 1:] - ring[:, 1:] - base * 0  # band k lane 0 publish - ring store (same line)
+use = (t[:, 0::32][:, 1:]) - ring[:, 1:]
+print("ring store -> band k lane 0 publish ns: p10 %.0f p50 %.0f p90 %.0f" % tuple(np.percentile(use, [10, 50, 90])))
