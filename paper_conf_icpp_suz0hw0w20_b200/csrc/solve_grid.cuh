@@ -155,6 +155,10 @@ constexpr int kGridRaw = 64;              // raw CSR ring (lines)
 constexpr int kGridA1 = 6;                // rowptr / b staged this many blocks before production
 constexpr int kGridA2 = 3;                // entries staged this many blocks before production
 constexpr int kGridWarps = 2 + kGridProd;  // consumer, producers, ring
+#ifndef SPTRSV_GRID_RING_WARP
+#define SPTRSV_GRID_RING_WARP 4
+#endif
+constexpr int kGridRingWarp = SPTRSV_GRID_RING_WARP;  // (kGridWarps - 1 puts it on its own)
 static_assert(kGridA1 == 2 * kGridA2, "one cp.async wait covers both staging distances");
 static_assert(kGridBlk * (kGridA1 + 1) <= kGridRaw, "raw ring too small");
 
@@ -253,7 +257,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
     int32_t *s_col = reinterpret_cast<int32_t *>(s_val + (size_t)kGridRaw * E);  // [raw][E]
 
     const bool ring_on = band > 0;
-    if (warp == kGridWarps - 1) {
+    // warp roles: 0 consumer, kGridRingWarp the ring, the others producers (SM sub-partition = warp % 4:
+    // the ring warp, mostly waiting on its polls, shares the consumer's sub-partition)
+    if (warp == kGridRingWarp) {
         // ================================================================ the ring (band > 0)
         // Lane 0's west operand is band k-1's lane 31: this warp polls those records 32 lines at a
         // time (lane j: line base + j), stores the values of the ready prefix in s_west and advances
@@ -309,7 +315,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
     }
     if (warp > 0) {
         // ================================================================ producers
-        const int w = warp - 1;
+        const int w = warp < kGridRingWarp ? warp - 1 : warp - 2;
         // rows of logical line y in this band (0: none); row0 = the first PHYSICAL row of its CSR slice
         // (upper: logical row y*m + x0 + j is physical n-1-(y*m + x0 + j), so the slice runs backwards)
         auto line_rows = [&](int y, unsigned &row0) -> int {
