@@ -19,7 +19,7 @@
 // so a step costs one shuffle and the row's dependent fp64 operations, and band k waits on band k-1
 // through lane 0 only: one global hop per 32 columns instead of one per line.  The critical path is
 // the grid's wavefront, lines + 32 * bands steps, plus one hop per band.  Measured (c3, 2048^2 grid,
-// B200): 0.91 ms against CHAIN's 5.10 ms; see DESIGN.md section 6 for the design steps and what each
+// B200): 0.87 ms against CHAIN's 5.10 ms; see DESIGN.md section 6 for the design steps and what each
 // one bought (a per-step poll held in lane registers cost a round trip per step through the warp's
 // scoreboard -- hence the ring warp).
 //
