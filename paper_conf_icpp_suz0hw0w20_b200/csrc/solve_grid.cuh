@@ -450,7 +450,8 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         ++fy;
         fsl = fsl == kGridDesc - 1 ? 0 : fsl + 1;
     };
-    double xl = 0.0;  // this lane's latest x (the north operand of its next row)
+    double xl = 0.0;   // this lane's latest x (the north operand of its next row)
+    double xsh = 0.0;  // the west lane's latest x, shuffled as soon as it was computed (next step's west)
     bool bad = false, stop = false;
     int ring_have = ring_on ? 0 : 0x7fffffff;  // lines whose west value the ring warp has stored
     const unsigned long long ep = (unsigned long long)epoch << 32;
@@ -488,9 +489,9 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         }
     };
     constexpr bool has_far = FAR;
-    // one step (line s - lane; lane 0's west value in s_west slot ws): Alg.1's row, the division, the
-    // publish.  `cur` is this step's row, `nxt` receives the next one (two register sets alternate)
-    auto step = [&](Row &cur, Row &nxt, int s, int ws) -> bool {
+    // one step (line s - lane; lane 0's west value wv): Alg.1's row, the division, the publish.  `cur` is
+    // this step's row, `nxt` receives the next one (two register sets alternate)
+    auto step = [&](Row &cur, Row &nxt, int s, double wv) -> bool {
         fetch(nxt);  // the next step's row (its lines were produced before this block)
         const int r = cur.r;
         const bool act = r >= 0;
@@ -499,9 +500,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         if (has_far && __any_sync(FULL, pend)) {  // a far entry not published when its row was produced
             if (!wait_for(-1, pend, cur.fc, xf)) return false;
         }
-        const double wv = s_west[ws];
-        double xw = __shfl_up_sync(FULL, xl, 1);
-        xw = lane == 0 ? wv : xw;
+        const double xw = lane == 0 ? wv : xsh;
         // ---- Alg.1's row: far (ls0), north, west (column order), then the division
         double ls = pend ? __dadd_rn(0.0, __dmul_rn(cur.ls0, xf)) : cur.ls0;
         ls = (cur.meta & kDescN) ? __dadd_rn(ls, __dmul_rn(cur.vn, xl)) : ls;
@@ -515,11 +514,13 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         if (SAFE) {
             const bool fix = act && !(guard && Diag::exact(a, cur.d, q));
             if (__builtin_expect(__any_sync(FULL, fix), 0)) q = grid_fix_div(fix, a, cur.d, q);
+            xsh = __shfl_up_sync(FULL, q, 1);
         } else {
             // outside the guard (a zero numerator, extreme magnitudes): the full division, in-loop;
             // inside it the candidate's proof runs off the chain and a failure fails the solve
             const bool fix = act && !guard;
             if (__builtin_expect(__any_sync(FULL, fix), 0)) q = grid_fix_div(fix, a, cur.d, q);
+            xsh = __shfl_up_sync(FULL, q, 1);  // first: the next step's chain starts here
             // (bitwise: the proof runs unconditionally, no branch around it in the step)
             const bool ex = Diag::exact(a, cur.d, q);
             bad = bad | (act & guard & !ex);
@@ -539,7 +540,10 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             p.x[r] = q;
             st_release_u32(p.flags + r, epoch);
         }
-        xl = act ? q : xl;
+        // unconditionally: a lane's x is read (as its next row's north, or its east neighbour's west)
+        // only by active rows, and an active row's predecessor step on this lane / the west lane is active
+        // too (lines start and end on the skew: line s - l; rows past n, lanes past nl stay inactive)
+        xl = q;
 #ifdef SPTRSV_GRID_TRACE  // measurement builds only (tools/grid_trace.py): publish time of every row
         if (p.trace && act) p.trace[r] = globaltimer_ns();
 #endif
@@ -564,10 +568,19 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             if (!wait_for(need, false, 0, dummy)) stop = true;
         }
         if (!stop) {
+            asm volatile("" ::: "memory");  // the s_west loads stay after the s_ring check
             if (s_end - s0 == kGridBlk) {
+                // lane 0's west values of the block, loaded once (kGridBlk doubles, 16-byte aligned)
+                double wblk[kGridBlk];
 #pragma unroll
                 for (int k = 0; k < kGridBlk; k += 2) {
-                    if (!step(ra, rb, s0 + k, wbase + k) || !step(rb, ra, s0 + k + 1, wbase + k + 1)) {
+                    const double2 w2 = *reinterpret_cast<const double2 *>(s_west + wbase + k);
+                    wblk[k] = w2.x;
+                    wblk[k + 1] = w2.y;
+                }
+#pragma unroll
+                for (int k = 0; k < kGridBlk; k += 2) {
+                    if (!step(ra, rb, s0 + k, wblk[k]) || !step(rb, ra, s0 + k + 1, wblk[k + 1])) {
                         stop = true;
                         break;
                     }
@@ -576,7 +589,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
                 for (int k = 0; k < s_end - s0; ++k) {
                     Row &c = (k & 1) ? rb : ra;
                     Row &nx = (k & 1) ? ra : rb;
-                    if (!step(c, nx, s0 + k, wbase + k)) {
+                    if (!step(c, nx, s0 + k, s_west[wbase + k])) {
                         stop = true;
                         break;
                     }
