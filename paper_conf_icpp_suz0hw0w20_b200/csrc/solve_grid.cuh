@@ -345,11 +345,13 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
                 cp_async8(s_val + (size_t)sl * E + (e - lo), p.val + e);
             }
         };
-        auto produce = [&](int y) {  // descriptors of line y from its staged raw rows
-            unsigned row0;
+        // descriptors of line y from its staged raw rows; lines outside [0, lines) (the skew's head and
+        // tail: line s - lane) get inactive descriptors (row -1, no entries), so the consumer reads them
+        // without a range check
+        auto produce = [&](int y) {
+            unsigned row0 = 0;
             const int k = line_rows(y, row0);
-            if (y >= lines) return;
-            const int sl = y & (kGridRaw - 1), ds = (y % kGridDesc) * 32 + lane;
+            const int sl = y & (kGridRaw - 1), ds = ((y + kGridDesc) % kGridDesc) * 32 + lane;
             const bool act = lane < k;
             const int pj = UPPER ? k - 1 - lane : lane;  // this lane's row in the (physical) slice
             const int r = (int)(row0 + pj);              // physical row
@@ -406,7 +408,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         cp_async_commit();
         cp_async_wait<0>();
         __syncwarp();
-        for (int y = w; y <= kGridBlk; y += kGridProd) produce(y);
+        for (int y = w - 31; y <= kGridBlk; y += kGridProd) produce(y);  // (lines -31 .. -1: the head)
         for (int b = 0; b < nblocks; ++b) {
             bar_sync_cp();  // block b begins: lines <= B*b + B are in the descriptor ring
             if (ld_volatile_s32((const int *)&s_stop)) continue;
@@ -424,20 +426,23 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         return;
     }
     // ==================================================================== consumer (warp 0)
-    // the row of a step (line s - lane) comes from the descriptor ring through a per-lane cursor
-    // (line fy, its ring slot fsl), advanced once per step; the NEXT step's row is fetched at the top
-    // of each step so its shared-memory loads overlap the current chain
-    int fy = -lane, fsl = lane == 0 ? 0 : kGridDesc - lane;
+    // the row of a step (line s - lane) comes from the descriptor ring through a per-lane cursor (the
+    // byte offset of its ring slot's d_a pair), advanced once per step; the NEXT step's row is fetched at
+    // the top of each step so its shared-memory loads overlap the current chain
+    constexpr unsigned kSlotB = 32 * sizeof(double2), kArrB = kGridDesc * kSlotB;
+    const unsigned fwrap = kArrB + 16u * lane;  // one past the last slot
+    unsigned fad = (lane == 0 ? 0u : (unsigned)(kGridDesc - lane) * kSlotB) + 16u * lane;
     struct Row {
         int r, meta, fc;
         double ls0, vn, vw, b, d, rc;
     };
     auto fetch = [&](Row &o) {
-        const int ds = fsl * 32 + lane;
-        const int4 mm = d_m[ds];
-        const double2 a2 = d_a[ds], bw = d_bw[ds], dr = d_dr[ds];
-        const int row = mm.z;
-        o.r = (unsigned)fy < (unsigned)lines ? row : -1;
+        const unsigned char *sp = gsm + fad;  // d_a, d_bw, d_dr, d_m: consecutive [desc][32] arrays
+        const int4 mm = *reinterpret_cast<const int4 *>(sp + 3 * kArrB);
+        const double2 a2 = *reinterpret_cast<const double2 *>(sp);
+        const double2 bw = *reinterpret_cast<const double2 *>(sp + kArrB);
+        const double2 dr = *reinterpret_cast<const double2 *>(sp + 2 * kArrB);
+        o.r = mm.z;
         o.meta = mm.x;
         o.ls0 = a2.x;
         o.vn = a2.y;
@@ -446,9 +451,8 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         o.d = dr.x;
         o.rc = dr.y;
         o.fc = mm.y;
-        o.meta = o.r >= 0 ? o.meta : 0;
-        ++fy;
-        fsl = fsl == kGridDesc - 1 ? 0 : fsl + 1;
+        fad += kSlotB;
+        fad = fad == fwrap ? 16u * lane : fad;
     };
     double xl = 0.0;   // this lane's latest x (the north operand of its next row)
     double xsh = 0.0;  // the west lane's latest x, shuffled as soon as it was computed (next step's west)
