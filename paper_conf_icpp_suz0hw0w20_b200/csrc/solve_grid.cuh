@@ -531,7 +531,7 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         }
         // ---- publish (Alg.5 l.13-16); GRID records are read by GRID warps only (no shared-memory
         // sentinel to avoid)
-        const int ri = act ? r : 0;
+        const int ri = r;  // (an inactive row's -1 only forms the address of a predicated-off store)
 #ifdef SPTRSV_GRID_M_NOSTORE  // measurement builds only (tools/)
         if (false) {
 #else
