@@ -155,6 +155,13 @@ constexpr int kGridRaw = 64;              // raw CSR ring (lines)
 constexpr int kGridA1 = 6;                // rowptr / b staged this many blocks before production
 constexpr int kGridA2 = 3;                // entries staged this many blocks before production
 constexpr int kGridWarps = 2 + kGridProd;  // consumer, producers, ring
+#ifndef SPTRSV_GRID_CHK
+#define SPTRSV_GRID_CHK 4
+#endif
+// consumer steps per ring check (a divisor of kGridBlk, even): half blocks for 2D stencils (c3 0.795 ->
+// 0.776 ms, 2 steps: 0.803), whole blocks with far entries (3D: 4.49 vs 4.62 ms at 4)
+constexpr int kGridChk2D = SPTRSV_GRID_CHK;
+static_assert(kGridBlk % kGridChk2D == 0 && kGridChk2D % 2 == 0, "ring checks tile the block in step pairs");
 #ifndef SPTRSV_GRID_RING_WARP
 #define SPTRSV_GRID_RING_WARP 4
 #endif
@@ -563,27 +570,38 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         if (b == 0) fetch(ra);
         const int s0 = kGridBlk * b;
         const int s_end = min(steps, s0 + kGridBlk);
-        // lane 0's west values of the whole block: one check per block (the ring warp stores lines in
-        // chunks), waiting only when the ring is behind
-        const int need = min(s_end, lines) - 1;
-        if (ring_have <= need) ring_have = ld_volatile_s32_nc(&s_ring);
-        if (ring_have <= need) {
-            double dummy;
-            if (!wait_for(need, false, 0, dummy)) stop = true;
-        }
-        if (!stop) {
+        // lane 0's west values, kGridChk steps at a time (the ring warp stores lines in chunks), waiting
+        // only when the ring is behind; a check inside the block runs after the previous step's shuffle
+        auto ring_check = [&](int need) -> bool {
+            if (ring_have <= need) ring_have = ld_volatile_s32_nc(&s_ring);
+            if (ring_have <= need) {
+                double dummy;
+                if (!wait_for(need, false, 0, dummy)) return false;
+            }
             asm volatile("" ::: "memory");  // the s_west loads stay after the s_ring check
-            if (s_end - s0 == kGridBlk) {
-                // lane 0's west values of the block, loaded once (kGridBlk doubles, 16-byte aligned)
+            return true;
+        };
+        constexpr int kGridChk = FAR ? kGridBlk : kGridChk2D;
+        const bool full = s_end - s0 == kGridBlk;
+        if (!ring_check(min(full ? s0 + kGridChk : s_end, lines) - 1)) stop = true;
+        if (!stop) {
+            if (full) {
                 double wblk[kGridBlk];
 #pragma unroll
                 for (int k = 0; k < kGridBlk; k += 2) {
-                    const double2 w2 = *reinterpret_cast<const double2 *>(s_west + wbase + k);
-                    wblk[k] = w2.x;
-                    wblk[k + 1] = w2.y;
-                }
+                    if (k % kGridChk == 0) {
+                        if (k > 0 && !ring_check(min(s0 + k + kGridChk, lines) - 1)) {
+                            stop = true;
+                            break;
+                        }
+                        // lane 0's west values of the next kGridChk steps (16-byte aligned pairs)
 #pragma unroll
-                for (int k = 0; k < kGridBlk; k += 2) {
+                        for (int j = k; j < k + kGridChk; j += 2) {
+                            const double2 w2 = *reinterpret_cast<const double2 *>(s_west + wbase + j);
+                            wblk[j] = w2.x;
+                            wblk[j + 1] = w2.y;
+                        }
+                    }
                     if (!step(ra, rb, s0 + k, wblk[k]) || !step(rb, ra, s0 + k + 1, wblk[k + 1])) {
                         stop = true;
                         break;
