@@ -422,12 +422,15 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
             cp_async_wait<kGridA2 - 1>();
             __syncwarp();
             const int y0 = kGridBlk * b + kGridBlk + 1;
-            for (int y = y0 + w; y < y0 + kGridBlk; y += kGridProd) {
-                stage_rp(y + kGridBlk * kGridA1);
-                stage_ent(y + kGridBlk * kGridA2);
+            static_assert(kGridBlk % kGridProd == 0, "each producer: the same number of lines per block");
+#pragma unroll
+            for (int i = 0; i < kGridBlk / kGridProd; ++i) {
+                stage_rp(y0 + w + i * kGridProd + kGridBlk * kGridA1);
+                stage_ent(y0 + w + i * kGridProd + kGridBlk * kGridA2);
             }
             cp_async_commit();
-            for (int y = y0 + w; y < y0 + kGridBlk; y += kGridProd) produce(y);
+#pragma unroll
+            for (int i = 0; i < kGridBlk / kGridProd; ++i) produce(y0 + w + i * kGridProd);
         }
         cp_async_wait<0>();
         return;
