@@ -415,7 +415,11 @@ __global__ void __launch_bounds__(32 * kGridWarps, 1) k_solve_grid(SolveParams p
         cp_async_commit();
         cp_async_wait<0>();
         __syncwarp();
-        for (int y = w - 31; y <= kGridBlk; y += kGridProd) produce(y);  // (lines -31 .. -1: the head)
+        // lines -31 .. -1 (the head: inactive) and 0 .. kGridBlk; a line >= 0 is produced by the warp that
+        // staged it (y = w mod kGridProd: cp.async completion is per thread, no CTA barrier yet)
+        static_assert(32 % kGridProd == 0, "the head loop keeps each warp's staged lines");
+        for (int y = w - 32; y <= kGridBlk; y += kGridProd)
+            if (y > -32) produce(y);
         for (int b = 0; b < nblocks; ++b) {
             bar_sync_cp();  // block b begins: lines <= B*b + B are in the descriptor ring
             if (ld_volatile_s32((const int *)&s_stop)) continue;
